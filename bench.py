@@ -1,0 +1,321 @@
+#!/usr/bin/env python
+"""bench.py -- ACSR hot path on B200, one JSON line (driver contract).
+
+Step = one pass of the whole ACSR path over one synthetic matrix already resident in
+HBM: acsr_bin (row lengths -> bins -> work map, Alg. 1) + acsr_spmv (bin-specific
+kernels, Alg. 2-4).  Default workload = BASELINE.json configs[1]: R-MAT scale 20, edge
+factor 16, fp64 (C2).  `value` = GFLOP/s = 2*nnz per step / device time of the step
+(bin included: the per-update cost of the dynamic-graph setting).
+L2 is flushed (256 MiB write) between timed steps, outside the step's events.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl acsr|reference]
+                  [--workload rmat20|rmat20_f32|webgoogle|livejournal|pagerank|dynamic]
+
+With N > 1 (torchrun) every rank runs its own independent matrix (seed + rank): the
+units are independent problems, no data-path collective, scaling "weak"; the time is
+the max over ranks.  `--impl reference` times the CPU oracle (plain sequential C) on
+the same workload (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import synth  # noqa: E402
+
+FALLBACK_HBM = 6650.0
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return FALLBACK_HBM, "fallback"
+
+
+class Clocks:
+    """Sample nvidia-smi clocks + throttle reasons during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in self.lines:
+            f = [x.strip() for x in l.split(",")]
+            if len(f) < 6:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = max(mx, float(f[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx or None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------ workloads
+def make_workload(name, dev, rank):
+    seed_shift = 1000 * rank
+    dtype = torch.float32 if name.endswith("_f32") else torch.float64
+    if name.startswith("rmat20"):
+        rp, ci = synth.rmat_csr(20, seed=20 + seed_shift, device=dev)
+        label = f"rmat20_ef16_{'f32' if dtype == torch.float32 else 'f64'}"
+    elif name == "webgoogle":
+        rp, ci = synth.powerlaw_csr(seed=3 + seed_shift, device=dev, **synth.WEB_GOOGLE)
+        label = "webgoogle_like_f64"
+    elif name == "livejournal":
+        rp, ci = synth.powerlaw_csr(seed=4 + seed_shift, device=dev, **synth.LIVEJOURNAL)
+        label = "livejournal_like_f64"
+    else:
+        raise SystemExit(f"unknown workload {name}")
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 1014 + seed_shift, dtype, dev)
+    x = synth.vector(n, 2014 + seed_shift, dtype, dev)
+    return label, dtype, rp, ci, val, x
+
+
+def algorithmic_bytes(rp, ci, dtype):
+    """(s_v+4) nnz + 4(n+1) row_ptr + 4n bin_rows + s_v n_c x + s_v n y."""
+    n = rp.numel() - 1
+    nnz = ci.numel()
+    sv = 8 if dtype == torch.float64 else 4
+    n_c = int((torch.bincount(ci.long(), minlength=n) > 0).sum())
+    return (sv + 4) * nnz + 4 * (n + 1) + 4 * n + sv * n_c + sv * n, n_c
+
+
+def ncu_traffic(label):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        v = d.get(label)
+        if v:
+            return v
+    return None
+
+
+# ------------------------------------------------------------------------------ acsr arm
+def run_acsr(args, dev, rank, world):
+    import paper_conf_sc_ashariseps14_b200 as acsr
+
+    label, dtype, rp, ci, val, x = make_workload(args.workload, dev, rank)
+    n, nnz = rp.numel() - 1, ci.numel()
+    alg_bytes, n_c = algorithmic_bytes(rp, ci, dtype)
+    stream = torch.cuda.current_stream()
+    br = torch.empty(n, dtype=torch.int32, device=dev)
+    bo = torch.empty(33, dtype=torch.int32, device=dev)
+    ws = torch.empty(acsr.acsr_bin_workspace_bytes(n, nnz), dtype=torch.uint8, device=dev)
+    y = torch.empty(n, dtype=dtype, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def step():
+        acsr.acsr_bin(rp, None, nnz, br, bo, ws)
+        acsr.acsr_spmv(rp, ci, val, x, br, bo, ws, None, y)
+
+    for _ in range(args.warmup):
+        flush.zero_()
+        step()
+    torch.cuda.synchronize()
+    K = args.steps
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(K)]
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    with Clocks(torch.cuda.current_device()) as clk:
+        t0 = time.perf_counter()
+        for k in range(K):
+            flush.zero_()
+            ev[k][0].record(stream)
+            acsr.acsr_bin(rp, None, nnz, br, bo, ws)
+            ev[k][1].record(stream)
+            acsr.acsr_spmv(rp, ci, val, x, br, bo, ws, None, y)
+            ev[k][2].record(stream)
+        torch.cuda.synchronize()
+        wall = time.perf_counter() - t0
+    if world > 1:
+        torch.distributed.barrier()
+    t_bin = np.array([ev[k][0].elapsed_time(ev[k][1]) for k in range(K)])
+    t_spmv = np.array([ev[k][1].elapsed_time(ev[k][2]) for k in range(K)])
+    t_step = t_bin + t_spmv
+    tot = float(t_step.sum())
+    if world > 1:
+        tt = torch.tensor([tot], dtype=torch.float64, device=dev)
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        tot = float(tt.item())
+    # end-to-end through the public API with host buffers (pinned), copies inside
+    rp_h, ci_h, val_h, x_h = (t.cpu().pin_memory() for t in (rp, ci, val, x))
+    y_h = torch.empty(n, dtype=dtype).pin_memory()
+    for _ in range(2):
+        acsr.spmv_from_host(rp_h, ci_h, val_h, x_h, y_h, device=dev)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ke = max(3, min(K, 10))
+    e0.record(stream)
+    for _ in range(ke):
+        acsr.spmv_from_host(rp_h, ci_h, val_h, x_h, y_h, device=dev)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    t_e2e = e0.elapsed_time(e1) / ke
+    h2d = sum(t.numel() * t.element_size() for t in (rp_h, ci_h, val_h, x_h))
+    d2h = y_h.numel() * y_h.element_size()
+    if rank != 0:
+        return None
+    peak, peak_kind = peaks()
+    gflops = 2.0 * nnz * K * world / (tot * 1e-3) / 1e9
+    spmv_ms = float(t_spmv.mean())
+    achieved = alg_bytes / (spmv_ms * 1e-3) / 1e9
+    line = {
+        "metric": "SpMV GFLOP/s (bin+SpMV per step) & HBM GB/s vs peak",
+        "value": round(gflops, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K, "warmup": args.warmup,
+        "ms_per_step": round(tot / K, 5), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64" if dtype == torch.float64 else "f32", "data": "synthetic",
+        "config": {"workload": label, "n_rows": n, "nnz": nnz, "referenced_cols": n_c,
+                   "l2": "flushed: 256 MiB write between timed steps (outside the step events)",
+                   "parallelism": "independent matrix per rank (weak)" if world > 1 else "1 GPU"},
+        "breakdown": {"t_bin_ms": round(float(t_bin.mean()), 5), "t_spmv_ms": round(spmv_ms, 5),
+                      "pt_st": round(float(t_bin.mean()) / spmv_ms, 3),
+                      "spmv_gflops": round(2.0 * nnz / (spmv_ms * 1e-3) / 1e9, 2),
+                      "t_spmv_min_ms": round(float(t_spmv.min()), 5),
+                      "wall_s_timed_loop": round(wall, 4)},
+        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                     "frac": round(achieved / peak, 4), "traffic": ncu_traffic(label),
+                     "kernel": "acsr::spmv_kernel", "peak_kind": peak_kind,
+                     "algorithmic_bytes_per_launch": int(alg_bytes)},
+        "e2e": {"value": round(2.0 * nnz / (t_e2e * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
+                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+                "ms_per_step": round(t_e2e, 4)},
+        "gpu_launches": 4 * K,
+        "clocks": clk.summary(),
+    }
+    if not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(rp, ci, val, x, dtype)
+    return line
+
+
+def cpu_baseline(rp, ci, val, x, dtype, budget_s=12.0):
+    """The oracle's plain sequential SpMV (O4') on 1 host core, repeated over the whole
+    matrix for ~budget_s seconds; GFLOP/s with the same 2*nnz."""
+    import oracle
+
+    rph, cih = rp.cpu().numpy(), ci.cpu().numpy()
+    vh, xh = val.cpu().numpy(), x.cpu().numpy()
+    y = np.empty(rph.size - 1, vh.dtype)
+    oracle.spmv_plain(rph, cih, vh, xh, out=y)
+    reps, t0 = 0, time.perf_counter()
+    while time.perf_counter() - t0 < budget_s or reps < 2:
+        oracle.spmv_plain(rph, cih, vh, xh, out=y, threads=1)
+        reps += 1
+    dt = (time.perf_counter() - t0) / reps
+    return {"value": round(2.0 * cih.size / dt / 1e9, 4), "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+            "sample": f"whole matrix, plain sequential CSR SpMV (oracle O4'), {reps} reps, "
+                      f"{dt * 1e3:.1f} ms each; host has {os.cpu_count()} cores"}
+
+
+# ------------------------------------------------------------------------------ reference arm
+def run_reference(args, dev):
+    """The oracle as it stands (plain C, 1 core) on the same workload: bins (O3) + plain SpMV
+    (O4') per step."""
+    import oracle
+
+    label, dtype, rp, ci, val, x = make_workload(args.workload, dev, 0)
+    rph, cih = rp.cpu().numpy(), ci.cpu().numpy()
+    vh, xh = val.cpu().numpy(), x.cpu().numpy()
+    y = np.empty(rph.size - 1, vh.dtype)
+    for _ in range(min(args.warmup, 1)):
+        oracle.bins(rph)
+        oracle.spmv_plain(rph, cih, vh, xh, out=y)
+    K = args.steps
+    t0 = time.perf_counter()
+    for _ in range(K):
+        oracle.bins(rph)
+        oracle.spmv_plain(rph, cih, vh, xh, out=y)
+    dt = (time.perf_counter() - t0) / K
+    v = 2.0 * cih.size / dt / 1e9
+    return {"metric": "SpMV GFLOP/s (bin+SpMV per step) & HBM GB/s vs peak", "impl": "reference",
+            "value": round(v, 4), "unit": "GFLOP/s", "n_gpus": 1, "steps": K, "warmup": args.warmup,
+            "ms_per_step": round(dt * 1e3, 3), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64" if dtype == torch.float64 else "f32", "data": "synthetic",
+            "config": {"workload": label, "n_rows": int(rph.size - 1), "nnz": int(cih.size)},
+            "cpu_baseline": {"value": round(v, 4), "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+                             "sample": f"whole matrix per step: oracle bins (O3) + plain SpMV (O4'), {K} steps"},
+            "e2e": {"value": round(v, 4), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="acsr", choices=["acsr", "reference"])
+    ap.add_argument("--workload", default="rmat20")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        dev = torch.device("cuda", local) if torch.cuda.is_available() else torch.device("cpu")
+        print(json.dumps(run_reference(args, dev)), flush=True)
+        return
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        torch.distributed.init_process_group("nccl", device_id=dev)
+    line = run_acsr(args, dev, rank, world)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,180 @@
+/*
+ * acsr.h -- C ABI of libacsr.so: adaptive CSR SpMV (ACSR, Ashari et al., SC'14)
+ * for NVIDIA B200 (sm_100a).
+ *
+ * Citations "P:L" refer to line L of the paper text; "§8(x)" to
+ * SURVEY.md; "Qn" to the readings listed in DESIGN.md.
+ *
+ * Conventions (all entry points)
+ *  - Every pointer is a DEVICE pointer unless marked HOST.
+ *  - Every call is asynchronous on the caller's `stream` (a cudaStream_t; NULL =
+ *    legacy default stream).  Nothing is allocated inside the calls: scratch comes
+ *    from a caller-owned workspace sized by the matching *_workspace_bytes query.
+ *  - Argument errors detectable on the host (NULL where required, negative sizes,
+ *    workspace too small, unknown dtype) return synchronously and enqueue nothing.
+ *    Data-dependent errors (update batches) are reported in a DEVICE status word.
+ *    A failed kernel launch returns ACSR_ERR_CUDA; acsr_last_error() holds the text.
+ *  - Index arrays are int32, row lengths must fit int32, sum of lengths < 2^31.
+ *  - CSR may carry reserved slack after each row (§VII): row r occupies
+ *    [row_begin[r], row_end[r]).  Passing row_end == NULL means standard CSR
+ *    (§II: row r occupies [RowOffset[r], RowOffset[r+1]), i.e.
+ *    row_end = row_begin + 1 and row_begin has n_rows + 1 entries).
+ *  - There is no CPU fallback: on a machine without an sm_100 device every call
+ *    that would launch returns ACSR_ERR_CUDA.
+ */
+#ifndef ACSR_H
+#define ACSR_H
+
+#include <stddef.h>
+#include <stdint.h>
+#include <cuda_runtime_api.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    ACSR_OK = 0,
+    ACSR_ERR_INVALID_VALUE = 1, /* bad argument, or (device status) malformed change list */
+    ACSR_ERR_WORKSPACE = 2,     /* workspace pointer NULL or smaller than the query */
+    ACSR_ERR_CAPACITY = 3,      /* (device status) an updated row exceeds its reserved slack */
+    ACSR_ERR_CUDA = 4,          /* CUDA launch / runtime failure, see acsr_last_error() */
+    ACSR_ERR_NCCL = 5,          /* reserved for the NCCL exchange (multi-GPU) */
+    ACSR_ERR_UNSUPPORTED = 6    /* e.g. no sm_100 device */
+} acsr_status;
+
+typedef enum { ACSR_F32 = 0, ACSR_F64 = 1 } acsr_dtype;
+
+enum { ACSR_NBINS = 32 };
+
+/* ------------------------------------------------------------------------ */
+/* Binning (Alg. 1 "if (this is the first iteration) ... foreach row r do
+ * b_r <- b_r U {r}"; §III-A).
+ *
+ * Row r with len_r = row_end[r] - row_begin[r] non-zeros goes to bin
+ *     b = 0 if len_r == 0;  1 if len_r <= 2;  else ceil(log2(len_r))
+ * i.e. bin i holds [2^{i-1}+1 .. 2^i] non-zeros (reading Q1), bin 0 the
+ * empty rows (reading Q2).  Outputs:
+ *   bin_rows[n_rows]        row ids grouped by bin, ascending row id inside a bin
+ *                           (stable; reading Q3) -- the paper's BIN#N_Rows lists
+ *   bin_offsets[33]         bin b = bin_rows[bin_offsets[b] .. bin_offsets[b+1]),
+ *                           bin_offsets[32] = n_rows
+ *   plan_ws                 the SpMV work map (replaces Alg. 1's G1/G2 split and
+ *                           the dynamic-parallelism parent/child launches, P:61,
+ *                           P:68-105): per-warp work units in row-space order and
+ *                           the split plan for rows longer than 1024 non-zeros.
+ * nnz_max bounds the total number of stored entries (sum of row lengths) that
+ * any later acsr_bin on this workspace will see (for slack CSR: the capacity).
+ * The row-length array is read twice (count pass + stable scatter pass); no
+ * host synchronisation happens.  The result is deterministic and equals the
+ * oracle bit for bit. */
+size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t nnz_max);
+
+acsr_status acsr_bin(int64_t n_rows, int64_t nnz_max,
+                     const int32_t *row_begin, const int32_t *row_end /* NULL => standard CSR */,
+                     int32_t *bin_rows /* [n_rows] out */,
+                     int32_t *bin_offsets /* [ACSR_NBINS + 1] out */,
+                     void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream);
+
+/* ------------------------------------------------------------------------ */
+/* SpMV y = A x, computed directly on CSR with bin-specific mappings
+ * (Alg. 2): bins 1..6 use a sub-warp of 2^{b-1} lanes per row with
+ * shuffle reduction (exactly Alg. 2); bins 7..10 a warp per row; rows longer
+ * than 1024 non-zeros are cut into fixed chunks processed by different warps and
+ * combined in chunk order by the last-arriving warp (replaces the dynamic-
+ * parallelism parent/child kernels of Alg. 3/4; reading Q4/Q7/Q8).
+ *   dt          ACSR_F64: values/x/y are double; ACSR_F32: float (accumulated
+ *               in double, rounded once per row).
+ *   values      [nnz] or NULL => pattern matrix (all ones).
+ *   x           [n_cols];  y [n_rows] is overwritten, never read (reading Q5);
+ *               empty rows get +0.0 (reading Q2).
+ *   bin_rows, bin_offsets, plan_ws: produced by acsr_bin on the same row
+ *               lengths (re-bin after every acsr_update_edges).
+ * Deterministic: the summation order of every row depends only on the row's
+ * length and address alignment, never on scheduling. */
+acsr_status acsr_spmv(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
+                      const int32_t *row_begin, const int32_t *row_end /* NULL => standard */,
+                      const int32_t *col_idx, const void *values /* NULL => ones */,
+                      const void *x, void *y,
+                      const int32_t *bin_rows, const int32_t *bin_offsets,
+                      void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream);
+
+/* ------------------------------------------------------------------------ */
+/* PageRank step (Alg. 5; §VI-A) on one rank's rows.
+ *   PR^{k+1} = (1-d) PR^(0) + d (A^T PR^k),  A row-normalised.
+ * Storage (reading Q12): the IN-LINK pattern CSR (row v lists the sources u of
+ * the edges u -> v) and the scaled vector xs_u = PR_u / outdeg_u (0 when
+ * outdeg_u == 0, reading Q11).  One fused launch computes, for local row v,
+ *   y_v = sum_{u -> v} xs[u]
+ *   x_new[v]   = teleport + damping * y_v          (teleport = (1-d)/n, host)
+ *   xs_next[v] = outdeg[v] > 0 ? x_new[v] / outdeg[v] : 0
+ *   *delta2    = sum_v (x_new[v] - x[v])^2          (deterministic order)
+ * Multi-GPU (§VIII, reading Q19): each rank calls this on its contiguous
+ * row range and then all-gathers xs_next (caller side, torch.distributed/NCCL);
+ * col ids index the replicated xs. */
+typedef struct {
+    int64_t n_rows;               /* local rows */
+    int64_t n_cols;               /* length of xs (global, possibly padded) */
+    const int32_t *row_begin;     /* local in-link CSR */
+    const int32_t *row_end;       /* NULL => standard CSR */
+    const int32_t *col_idx;       /* source ids, index into xs */
+    const int32_t *bin_rows;      /* from acsr_bin on the local rows */
+    const int32_t *bin_offsets;
+    void *plan_ws;
+    size_t plan_ws_bytes;
+    const double *xs;             /* [n_cols] PR^k / outdeg, replicated */
+    const double *x;              /* [n_rows] PR^k of the local rows */
+    const int32_t *outdeg;        /* [n_rows] out-degree of the local vertices */
+    double *x_new;                /* [n_rows] PR^{k+1} */
+    double *xs_next;              /* [n_rows] PR^{k+1} / outdeg (the local slice) */
+    double damping;               /* d = 0.85 */
+    double teleport;              /* (1-d)/n_global, computed once on the host */
+    double *delta2;               /* [1] local sum of squared differences */
+} acsr_pr_args;
+
+acsr_status acsr_pagerank_step(const acsr_pr_args *args, cudaStream_t stream);
+
+/* xs[v] = outdeg[v] > 0 ? x[v] / outdeg[v] : 0 for v < n (IEEE division).
+ * Builds the first scaled vector of Alg. 5 (PR^(0) = 1/n) or of a warm
+ * start. */
+acsr_status acsr_pagerank_scale(int64_t n, const double *x, const int32_t *outdeg, double *xs,
+                                cudaStream_t stream);
+
+/* ------------------------------------------------------------------------ */
+/* Dynamic-graph update (§VII): for update i (row r = upd_rows[i],
+ * upd_rows strictly increasing) delete every entry whose column is in
+ * del_cols[del_ptr[i] .. del_ptr[i+1]) (sorted, non-decreasing), compact the
+ * row keeping order ("compresses (shifts columns) the row"), then append
+ * ins_cols[ins_ptr[i] .. ins_ptr[i+1]) in order (with ins_vals, or 1 for a
+ * pattern matrix).  outdeg (nullable, [n_cols]) gets -1 per removed and +1 per
+ * inserted entry.  Reading Q13: the batch is all-or-nothing -- it is first
+ * validated for every i in order:
+ *   (a) 0 <= upd_rows[i] < n_rows and upd_rows[i] > upd_rows[i-1]   INVALID_VALUE
+ *   (b) delete list non-decreasing                                   INVALID_VALUE
+ *   (c) 0 <= insert column < n_cols                                  INVALID_VALUE
+ *   (d) kept + inserted <= row_cap[r]                                CAPACITY
+ * status[0] = code of the smallest failing i (ACSR_OK if none), status[1] = that
+ * i (or -1).  On failure nothing is modified (bitwise).  del_ptr/del_cols may be
+ * NULL (insert-only batch).  Re-run acsr_bin afterwards. */
+size_t acsr_update_workspace_bytes(int64_t n_upd);
+
+acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
+                              const int32_t *row_begin, int32_t *row_end, const int32_t *row_cap,
+                              int32_t *col_idx, void *values /* NULL => pattern */,
+                              int64_t n_upd, const int32_t *upd_rows,
+                              const int32_t *del_ptr, const int32_t *del_cols,
+                              const int32_t *ins_ptr, const int32_t *ins_cols,
+                              const void *ins_vals /* NULL => ones */,
+                              int32_t *outdeg /* NULL or [n_cols] */,
+                              int32_t *status /* [2] out */,
+                              void *ws, size_t ws_bytes, cudaStream_t stream);
+
+/* ------------------------------------------------------------------------ */
+const char *acsr_status_string(acsr_status s);
+const char *acsr_last_error(void); /* thread-local detail of the last failure */
+int acsr_version(void);             /* 100 * major + minor */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ACSR_H */

@@ -1,0 +1,238 @@
+"""ACSR on B200: adaptive CSR SpMV (Ashari et al., SC'14), sm_100a.
+
+Thin ctypes binding over ``lib/libacsr.so`` (C ABI declared in ``include/acsr.h``).
+The functions carry the C names and only marshal arguments: every step of the path
+runs in the library's CUDA kernels.  PyTorch provides device memory
+(``tensor.data_ptr()``) and streams (``torch.cuda.current_stream()``); there is no
+CPU fallback -- importing this package fails loudly if the library is missing, and
+every call requires CUDA tensors.
+
+Entry points (same names as the C ABI):
+  acsr_bin            row binning + SpMV work map   (Alg. 1)
+  acsr_spmv           y = A x on CSR                (Alg. 2-4)
+  acsr_pagerank_step  one fused PageRank step       (Alg. 5)
+  acsr_pagerank_scale xs = x / outdeg
+  acsr_update_edges   dynamic-graph update          (§VII)
+Helpers: ``ACSRMatrix`` (owns CSR + plan), ``spmv_from_host`` (end-to-end path with
+host buffers), ``pagerank`` (single-GPU Alg. 5 loop) and
+``paper_conf_sc_ashariseps14_b200.dist`` (row-partitioned multi-GPU PageRank).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "lib", "libacsr.so")
+
+ACSR_OK = 0
+ACSR_ERR_INVALID_VALUE = 1
+ACSR_ERR_WORKSPACE = 2
+ACSR_ERR_CAPACITY = 3
+ACSR_ERR_CUDA = 4
+ACSR_F32 = 0
+ACSR_F64 = 1
+NBINS = 32
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"libacsr.so not built ({LIB_PATH}); run `python -c 'import __graft_entry__ as g; "
+                      f"g.build()'` -- there is no CPU fallback")
+
+_lib = ctypes.CDLL(LIB_PATH)
+_i64, _vp, _sz, _dbl = ctypes.c_int64, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_double
+_lib.acsr_bin_workspace_bytes.argtypes = [_i64, _i64]
+_lib.acsr_bin_workspace_bytes.restype = _sz
+_lib.acsr_bin.argtypes = [_i64, _i64, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
+_lib.acsr_bin.restype = ctypes.c_int
+_lib.acsr_spmv.argtypes = [ctypes.c_int, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _sz,
+                           _vp]
+_lib.acsr_spmv.restype = ctypes.c_int
+_lib.acsr_pagerank_scale.argtypes = [_i64, _vp, _vp, _vp, _vp]
+_lib.acsr_pagerank_scale.restype = ctypes.c_int
+_lib.acsr_update_workspace_bytes.argtypes = [_i64]
+_lib.acsr_update_workspace_bytes.restype = _sz
+_lib.acsr_update_edges.argtypes = [ctypes.c_int, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _i64, _vp, _vp,
+                                   _vp, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
+_lib.acsr_update_edges.restype = ctypes.c_int
+_lib.acsr_status_string.argtypes = [ctypes.c_int]
+_lib.acsr_status_string.restype = ctypes.c_char_p
+_lib.acsr_last_error.restype = ctypes.c_char_p
+_lib.acsr_version.restype = ctypes.c_int
+
+
+class PrArgs(ctypes.Structure):
+    """Mirror of ``acsr_pr_args`` (include/acsr.h)."""
+    _fields_ = [("n_rows", _i64), ("n_cols", _i64), ("row_begin", _vp), ("row_end", _vp),
+                ("col_idx", _vp), ("bin_rows", _vp), ("bin_offsets", _vp), ("plan_ws", _vp),
+                ("plan_ws_bytes", _sz), ("xs", _vp), ("x", _vp), ("outdeg", _vp), ("x_new", _vp),
+                ("xs_next", _vp), ("damping", _dbl), ("teleport", _dbl), ("delta2", _vp)]
+
+
+_lib.acsr_pagerank_step.argtypes = [ctypes.POINTER(PrArgs), _vp]
+_lib.acsr_pagerank_step.restype = ctypes.c_int
+
+EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_spmv", "acsr_pagerank_step",
+            "acsr_pagerank_scale", "acsr_update_workspace_bytes", "acsr_update_edges",
+            "acsr_status_string", "acsr_last_error", "acsr_version")
+
+
+class ACSRError(RuntimeError):
+    def __init__(self, code, what):
+        self.code = code
+        msg = _lib.acsr_status_string(code).decode()
+        detail = (_lib.acsr_last_error() or b"").decode()
+        super().__init__(f"{what}: {msg} {detail}")
+
+
+def _check(code, what):
+    if code != ACSR_OK:
+        raise ACSRError(code, what)
+
+
+def _dev(t, dtype, name, allow_none=False):
+    if t is None:
+        if allow_none:
+            return None
+        raise TypeError(f"{name} is required")
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA tensor (no CPU fallback)")
+    if dtype is not None and t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise TypeError(f"{name} must be contiguous")
+    return t.data_ptr()
+
+
+def _stream(stream):
+    s = torch.cuda.current_stream() if stream is None else stream
+    return s.cuda_stream
+
+
+def _dt(t):
+    if t.dtype == torch.float64:
+        return ACSR_F64
+    if t.dtype == torch.float32:
+        return ACSR_F32
+    raise TypeError(f"unsupported value dtype {t.dtype}")
+
+
+# --------------------------------------------------------------------------- binning
+def acsr_bin_workspace_bytes(n_rows: int, nnz_max: int) -> int:
+    return int(_lib.acsr_bin_workspace_bytes(int(n_rows), int(nnz_max)))
+
+
+def acsr_bin(row_begin, row_end=None, nnz_max=None, bin_rows=None, bin_offsets=None, plan_ws=None,
+             stream=None):
+    """Bin the rows.  Returns (bin_rows, bin_offsets, plan_ws)."""
+    n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
+    dev = row_begin.device
+    if nnz_max is None:
+        raise TypeError("nnz_max (bound on stored entries) is required")
+    if bin_rows is None:
+        bin_rows = torch.empty(max(n, 0), dtype=torch.int32, device=dev)
+    if bin_offsets is None:
+        bin_offsets = torch.empty(NBINS + 1, dtype=torch.int32, device=dev)
+    need = acsr_bin_workspace_bytes(n, nnz_max)
+    if plan_ws is None:
+        plan_ws = torch.empty(need, dtype=torch.uint8, device=dev)
+    _check(_lib.acsr_bin(n, int(nnz_max), _dev(row_begin, torch.int32, "row_begin"),
+                         _dev(row_end, torch.int32, "row_end", True),
+                         _dev(bin_rows, torch.int32, "bin_rows") if n > 0 else None,
+                         _dev(bin_offsets, torch.int32, "bin_offsets"),
+                         _dev(plan_ws, torch.uint8, "plan_ws"), plan_ws.numel(), _stream(stream)),
+           "acsr_bin")
+    return bin_rows, bin_offsets, plan_ws
+
+
+# --------------------------------------------------------------------------- SpMV
+def acsr_spmv(row_begin, col_idx, values, x, bin_rows, bin_offsets, plan_ws, row_end=None, y=None,
+              stream=None):
+    """y = A x with the bin-specific kernels.  values None => pattern matrix."""
+    n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
+    if y is None:
+        y = torch.empty(n, dtype=x.dtype, device=x.device)
+    if values is not None and values.dtype != x.dtype:
+        raise TypeError("values and x must have the same dtype")
+    _check(_lib.acsr_spmv(_dt(x), n, x.numel(), _dev(row_begin, torch.int32, "row_begin"),
+                          _dev(row_end, torch.int32, "row_end", True),
+                          _dev(col_idx, torch.int32, "col_idx") if col_idx.numel() else None,
+                          _dev(values, x.dtype, "values", True) if values is None or values.numel() else None,
+                          _dev(x, x.dtype, "x") if x.numel() else None,
+                          _dev(y, x.dtype, "y") if n else None,
+                          _dev(bin_rows, torch.int32, "bin_rows") if n else None,
+                          _dev(bin_offsets, torch.int32, "bin_offsets"),
+                          _dev(plan_ws, torch.uint8, "plan_ws"), plan_ws.numel(), _stream(stream)),
+           "acsr_spmv")
+    return y
+
+
+# --------------------------------------------------------------------------- PageRank
+def acsr_pagerank_scale(x, outdeg, xs=None, stream=None):
+    xs = torch.empty_like(x) if xs is None else xs
+    _check(_lib.acsr_pagerank_scale(x.numel(), _dev(x, torch.float64, "x"),
+                                    _dev(outdeg, torch.int32, "outdeg"), _dev(xs, torch.float64, "xs"),
+                                    _stream(stream)), "acsr_pagerank_scale")
+    return xs
+
+
+def acsr_pagerank_step(row_begin, col_idx, bin_rows, bin_offsets, plan_ws, xs, x, outdeg, x_new,
+                       xs_next, delta2, damping=0.85, teleport=None, n_global=None, row_end=None,
+                       stream=None):
+    """One fused PageRank step on the local rows (Alg. 5).  delta2: 1-element float64."""
+    n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
+    ng = xs.numel() if n_global is None else n_global
+    tel = (1.0 - damping) / ng if teleport is None else teleport
+    a = PrArgs(n, xs.numel(), _dev(row_begin, torch.int32, "row_begin"),
+               _dev(row_end, torch.int32, "row_end", True),
+               _dev(col_idx, torch.int32, "col_idx") if col_idx.numel() else None,
+               _dev(bin_rows, torch.int32, "bin_rows") if n else None,
+               _dev(bin_offsets, torch.int32, "bin_offsets"), _dev(plan_ws, torch.uint8, "plan_ws"),
+               plan_ws.numel(), _dev(xs, torch.float64, "xs") if xs.numel() else None,
+               _dev(x, torch.float64, "x") if n else None,
+               _dev(outdeg, torch.int32, "outdeg") if n else None,
+               _dev(x_new, torch.float64, "x_new") if n else None,
+               _dev(xs_next, torch.float64, "xs_next") if n else None, float(damping), float(tel),
+               _dev(delta2, torch.float64, "delta2"))
+    _check(_lib.acsr_pagerank_step(ctypes.byref(a), _stream(stream)), "acsr_pagerank_step")
+    return x_new, xs_next, delta2
+
+
+# --------------------------------------------------------------------------- update
+def acsr_update_workspace_bytes(n_upd: int) -> int:
+    return int(_lib.acsr_update_workspace_bytes(int(n_upd)))
+
+
+def acsr_update_edges(n_cols, row_begin, row_end, row_cap, col_idx, values, upd_rows, ins_ptr,
+                      ins_cols, ins_vals=None, del_ptr=None, del_cols=None, outdeg=None, status=None,
+                      ws=None, dtype=torch.float64, stream=None):
+    """Apply one change batch in place (§VII).  Returns the device status tensor [code, index]."""
+    n = row_begin.numel()
+    dev = row_begin.device
+    n_upd = upd_rows.numel()
+    if status is None:
+        status = torch.empty(2, dtype=torch.int32, device=dev)
+    if ws is None:
+        ws = torch.empty(acsr_update_workspace_bytes(n_upd), dtype=torch.uint8, device=dev)
+    vdt = values.dtype if values is not None else dtype
+    dt = ACSR_F64 if vdt == torch.float64 else ACSR_F32
+    opt = lambda t, d, nm: (_dev(t, d, nm) if t is not None and t.numel() else None)
+    _check(_lib.acsr_update_edges(dt, n, int(n_cols), _dev(row_begin, torch.int32, "row_begin"),
+                                  _dev(row_end, torch.int32, "row_end"), _dev(row_cap, torch.int32, "row_cap"),
+                                  _dev(col_idx, torch.int32, "col_idx"), opt(values, vdt, "values"), n_upd,
+                                  opt(upd_rows, torch.int32, "upd_rows"),
+                                  _dev(del_ptr, torch.int32, "del_ptr", True),
+                                  opt(del_cols, torch.int32, "del_cols") if del_ptr is not None else None,
+                                  opt(ins_ptr, torch.int32, "ins_ptr"), opt(ins_cols, torch.int32, "ins_cols"),
+                                  opt(ins_vals, vdt, "ins_vals"), _dev(outdeg, torch.int32, "outdeg", True),
+                                  _dev(status, torch.int32, "status"), _dev(ws, torch.uint8, "ws"), ws.numel(),
+                                  _stream(stream)), "acsr_update_edges")
+    return status
+
+
+def version() -> int:
+    return int(_lib.acsr_version())
+
+
+from .matrix import ACSRMatrix, pagerank, spmv_from_host  # noqa: E402

@@ -1,0 +1,292 @@
+// acsr_bin.cu -- row binning (Alg. 1 first-iteration preprocessing) and
+// the SpMV work map that replaces the G1/G2 split + dynamic parallelism.
+//
+// Three launches, no host synchronisation:
+//   1. bin_count   one CTA per TILE_ROWS-row tile: per-tile histogram of bin ids
+//                  (row lengths from the row offsets, P:47 / P:360 "scanning of
+//                  row-lengths"), plus per-tile light-unit and heavy-chunk counts.
+//   2. bin_scan    one CTA per scan row (32 bins + 2 unit rows): exclusive scan
+//                  over tiles; the last CTA turns the bin totals into
+//                  bin_offsets[0..32] and the unit totals into the plan header.
+//   3. bin_scatter one CTA per tile: stable ranks (warp __match_any_sync + per-warp
+//                  counts scanned across warps, 16 rounds of 256 rows in row
+//                  order) -> bin_rows; then writes the tile's work units.
+#include <cuda_runtime.h>
+
+#include "acsr_internal.cuh"
+
+namespace acsr {
+
+template <bool HAS_END>
+__device__ __forceinline__ int row_length(const int32_t *__restrict__ rb,
+                                          const int32_t *__restrict__ re, int64_t r)
+{
+    int b = __ldg(rb + r);
+    int e = HAS_END ? __ldg(re + r) : __ldg(rb + r + 1);
+    return e - b;
+}
+
+template <bool HAS_END>
+__global__ void __launch_bounds__(BIN_THREADS)
+bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
+                 int32_t *__restrict__ cnt, int n_tiles, PlanHeader *hdr)
+{
+    __shared__ int hist[NBINS];
+    __shared__ int heavy;
+    const int tid = threadIdx.x;
+    if (blockIdx.x == 0 && tid == 0) hdr->scan_ticket = 0;  // bin_scan runs after us
+    if (tid < NBINS) hist[tid] = 0;
+    if (tid == 0) heavy = 0;
+    __syncthreads();
+    const int64_t base = (int64_t)blockIdx.x * TILE_ROWS;
+    int my_heavy = 0;
+#pragma unroll 4
+    for (int k = 0; k < TILE_ROUNDS; k++) {
+        int64_t r = base + k * BIN_THREADS + tid;
+        if (r < n) {
+            int len = row_length<HAS_END>(rb, re, r);
+            int b = bin_of_len(len);
+            atomicAdd(&hist[b], 1);
+            if (b >= HEAVY_BIN) my_heavy += heavy_chunks(len);
+        }
+    }
+    // warp-reduce the heavy chunk count
+    for (int o = 16; o > 0; o >>= 1) my_heavy += __shfl_xor_sync(0xffffffffu, my_heavy, o);
+    if ((tid & 31) == 0 && my_heavy) atomicAdd(&heavy, my_heavy);
+    __syncthreads();
+    if (tid < NBINS) cnt[(int64_t)tid * n_tiles + blockIdx.x] = hist[tid];
+    if (tid == NBINS) {
+        int lu = 0;
+#pragma unroll
+        for (int b = 0; b <= LIGHT_MAX_BIN; b++) lu += (hist[b] + unit_rows(b) - 1) / unit_rows(b);
+        cnt[(int64_t)NBINS * n_tiles + blockIdx.x] = lu;
+        cnt[(int64_t)(NBINS + 1) * n_tiles + blockIdx.x] = heavy;
+    }
+}
+
+constexpr int SCAN_THREADS = 1024;
+
+__global__ void __launch_bounds__(SCAN_THREADS)
+bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int n_tiles,
+                PlanHeader *hdr, int32_t *__restrict__ bin_offsets, int64_t n_rows,
+                int64_t light_cap, int64_t heavy_cap, int64_t off_units, int64_t off_partial,
+                int64_t off_ticket, int64_t off_warp_part)
+{
+    __shared__ int warp_sums[SCAN_THREADS / 32];
+    __shared__ int is_last;
+    const int row = blockIdx.x;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int32_t *a = cnt + (int64_t)row * n_tiles;
+    int32_t *o = toff + (int64_t)row * n_tiles;
+    const int ipt = (n_tiles + SCAN_THREADS - 1) / SCAN_THREADS;
+    const int lo = min(tid * ipt, n_tiles), hi = min(lo + ipt, n_tiles);
+    int s = 0;
+    for (int i = lo; i < hi; i++) s += a[i];
+    // block exclusive scan of s
+    int incl = s;
+    for (int d = 1; d < 32; d <<= 1) {
+        int t = __shfl_up_sync(0xffffffffu, incl, d);
+        if (lane >= d) incl += t;
+    }
+    if (lane == 31) warp_sums[warp] = incl;
+    __syncthreads();
+    if (warp == 0) {
+        int w = warp_sums[lane];
+        int wi = w;
+        for (int d = 1; d < 32; d <<= 1) {
+            int t = __shfl_up_sync(0xffffffffu, wi, d);
+            if (lane >= d) wi += t;
+        }
+        warp_sums[lane] = wi - w;  // exclusive
+        if (lane == 31) hdr->totals[row] = wi;
+    }
+    __syncthreads();
+    int run = warp_sums[warp] + incl - s;
+    for (int i = lo; i < hi; i++) {
+        o[i] = run;
+        run += a[i];
+    }
+    // last CTA: bin offsets + unit totals
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) is_last = (atomicAdd(&hdr->scan_ticket, 1) == SCAN_ROWS - 1);
+    __syncthreads();
+    if (is_last && tid == 0) {
+        __threadfence();
+        volatile int32_t *tot = hdr->totals;
+        int acc = 0;
+        for (int b = 0; b < NBINS; b++) {
+            bin_offsets[b] = acc;
+            acc += tot[b];
+        }
+        bin_offsets[NBINS] = acc;  // == n_rows
+        int nl = tot[NBINS], nh = tot[NBINS + 1];
+        int ovf = (nl > light_cap) || (nh > heavy_cap);
+        hdr->overflow = ovf;
+        hdr->n_light_units = ovf ? 0 : nl;
+        hdr->n_heavy_units = ovf ? 0 : nh;
+        hdr->n_units = ovf ? 0 : nl + nh;
+        hdr->n_tiles = n_tiles;
+        hdr->off_units = off_units;
+        hdr->off_partial = off_partial;
+        hdr->off_ticket = off_ticket;
+        hdr->off_warp_part = off_warp_part;
+        hdr->done_ticket = 0;
+        hdr->scan_ticket = 0;
+        (void)n_rows;
+    }
+}
+
+template <bool HAS_END>
+__global__ void __launch_bounds__(BIN_THREADS)
+bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
+                   int32_t *__restrict__ bin_rows, const int32_t *__restrict__ bin_offsets,
+                   const int32_t *__restrict__ toff, int n_tiles, const PlanHeader *__restrict__ hdr,
+                   int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap)
+{
+    constexpr int NW = BIN_THREADS / 32;
+    __shared__ int run[NBINS];
+    __shared__ int wcnt[NW][NBINS];
+    __shared__ int wbase[NW][NBINS];
+    __shared__ int seg[NBINS];       // global start of this tile's segment of bin b
+    __shared__ int hw[NW];           // per-warp heavy chunk totals -> exclusive bases
+    __shared__ int heavy_run;
+    __shared__ int upre[LIGHT_MAX_BIN + 2];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int tile = blockIdx.x;
+    const int overflow = hdr->overflow;
+    const int n_heavy = hdr->n_heavy_units;
+    if (tid < NBINS) {
+        run[tid] = 0;
+        seg[tid] = bin_offsets[tid] + toff[(int64_t)tid * n_tiles + tile];
+    }
+    for (int i = tid; i < NW * NBINS; i += BIN_THREADS) (&wcnt[0][0])[i] = 0;
+    if (tid == 0) heavy_run = toff[(int64_t)(NBINS + 1) * n_tiles + tile];
+    __syncthreads();
+    const int64_t base = (int64_t)tile * TILE_ROWS;
+    const unsigned lt = (1u << lane) - 1u;
+    for (int k = 0; k < TILE_ROUNDS; k++) {
+        int64_t r = base + k * BIN_THREADS + tid;
+        bool valid = r < n;
+        int len = valid ? row_length<HAS_END>(rb, re, r) : 0;
+        int b = valid ? bin_of_len(len) : NBINS;  // NBINS = sentinel for past-the-end rows
+        unsigned mask = __match_any_sync(0xffffffffu, b);
+        int rank = __popc(mask & lt);
+        if (valid && rank == 0) wcnt[warp][b] = __popc(mask);
+        int hc = (valid && b >= HEAVY_BIN) ? heavy_chunks(len) : 0;
+        int hincl = hc;
+        for (int d = 1; d < 32; d <<= 1) {
+            int t = __shfl_up_sync(0xffffffffu, hincl, d);
+            if (lane >= d) hincl += t;
+        }
+        if (lane == 31) hw[warp] = hincl;
+        __syncthreads();
+        if (tid < NBINS) {
+            int acc = run[tid];
+#pragma unroll
+            for (int w = 0; w < NW; w++) {
+                wbase[w][tid] = acc;
+                acc += wcnt[w][tid];
+                wcnt[w][tid] = 0;
+            }
+            run[tid] = acc;
+        } else if (tid == NBINS) {
+            int acc = heavy_run;
+#pragma unroll
+            for (int w = 0; w < NW; w++) {
+                int t = hw[w];
+                hw[w] = acc;
+                acc += t;
+            }
+            heavy_run = acc;
+        }
+        __syncthreads();
+        if (valid) {
+            bin_rows[seg[b] + wbase[warp][b] + rank] = (int32_t)r;
+            if (hc > 0 && !overflow) {
+                int u0 = hw[warp] + hincl - hc;
+                for (int c = 0; c < hc; c++) {
+                    if (u0 + c < heavy_cap) units[u0 + c] = make_int2((int)r, (int)(HEAVY_FLAG | (uint32_t)c));
+                }
+                if (u0 < heavy_cap) tickets[u0] = 0;
+            }
+        }
+        __syncthreads();
+    }
+    if (overflow) return;
+    // light work units of this tile: bins 0..10, in bin order, row-contiguous
+    if (tid == 0) {
+        int acc = 0;
+        for (int b = 0; b <= LIGHT_MAX_BIN; b++) {
+            upre[b] = acc;
+            acc += (run[b] + unit_rows(b) - 1) / unit_rows(b);
+        }
+        upre[LIGHT_MAX_BIN + 1] = acc;
+    }
+    __syncthreads();
+    const int ubase = n_heavy + toff[(int64_t)NBINS * n_tiles + tile];
+    const int total = upre[LIGHT_MAX_BIN + 1];
+    for (int j = tid; j < total; j += BIN_THREADS) {
+        int b = 0;
+        while (upre[b + 1] <= j) b++;
+        int q = j - upre[b];
+        int K = unit_rows(b);
+        int c = min(K, run[b] - q * K);
+        units[ubase + j] = make_int2(seg[b] + q * K, (b << 24) | c);
+    }
+}
+
+}  // namespace acsr
+
+using namespace acsr;
+
+extern "C" size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t nnz_max)
+{
+    if (n_rows < 0 || nnz_max < 0) return 0;
+    return plan_layout(n_rows, nnz_max).total;
+}
+
+extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t nnz_max, const int32_t *row_begin,
+                                const int32_t *row_end, int32_t *bin_rows, int32_t *bin_offsets,
+                                void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream)
+{
+    if (n_rows < 0 || nnz_max < 0 || n_rows >= (int64_t)1 << 31 || !bin_offsets ||
+        (n_rows > 0 && (!row_begin || !bin_rows))) {
+        acsr_set_error("acsr_bin: invalid argument");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    PlanLayout L = plan_layout(n_rows, nnz_max);
+    if (!plan_ws || plan_ws_bytes < L.total) {
+        acsr_set_error("acsr_bin: workspace %zu < required %zu", plan_ws_bytes, L.total);
+        return ACSR_ERR_WORKSPACE;
+    }
+    char *ws = (char *)plan_ws;
+    PlanHeader *hdr = (PlanHeader *)ws;
+    if (n_rows == 0) {
+        cudaMemsetAsync(hdr, 0, sizeof(PlanHeader), stream);
+        cudaMemsetAsync(bin_offsets, 0, sizeof(int32_t) * (NBINS + 1), stream);
+        return acsr_check_launch("acsr_bin(empty)");
+    }
+    int32_t *cnt = (int32_t *)(ws + L.off_cnt);
+    int32_t *toff = (int32_t *)(ws + L.off_toff);
+    int2 *units = (int2 *)(ws + L.off_units);
+    int32_t *tickets = (int32_t *)(ws + L.off_ticket);
+    const int nt = (int)L.n_tiles;
+    if (row_end)
+        bin_count_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
+    else
+        bin_count_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
+    bin_scan_kernel<<<SCAN_ROWS, SCAN_THREADS, 0, stream>>>(cnt, toff, nt, hdr, bin_offsets, n_rows,
+                                                              L.light_cap, L.heavy_cap,
+                                                              (int64_t)L.off_units, (int64_t)L.off_partial,
+                                                              (int64_t)L.off_ticket, (int64_t)L.off_warp_part);
+    if (row_end)
+        bin_scatter_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, bin_rows,
+                                                                   bin_offsets, toff, nt, hdr, units,
+                                                                   tickets, L.heavy_cap);
+    else
+        bin_scatter_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, bin_rows,
+                                                                    bin_offsets, toff, nt, hdr, units,
+                                                                    tickets, L.heavy_cap);
+    return acsr_check_launch("acsr_bin");
+}

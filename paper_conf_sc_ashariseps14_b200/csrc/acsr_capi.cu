@@ -1,0 +1,58 @@
+// acsr_capi.cu -- status strings, thread-local error text, device queries.
+#include <cuda_runtime.h>
+#include <stdarg.h>
+#include <stdio.h>
+
+#include "acsr_internal.cuh"
+
+static thread_local char g_err[512] = "";
+
+void acsr_set_error(const char *fmt, ...)
+{
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+}
+
+acsr_status acsr_check_launch(const char *what)
+{
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+        acsr_set_error("%s: %s (%s)", what, cudaGetErrorString(e), cudaGetErrorName(e));
+        return ACSR_ERR_CUDA;
+    }
+    return ACSR_OK;
+}
+
+int acsr_num_sms()
+{
+    static int sms[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (!sms[dev]) {
+        int v = 0;
+        cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+        sms[dev] = v > 0 ? v : 148;
+    }
+    return sms[dev];
+}
+
+extern "C" const char *acsr_status_string(acsr_status s)
+{
+    switch (s) {
+        case ACSR_OK: return "ACSR_OK";
+        case ACSR_ERR_INVALID_VALUE: return "ACSR_ERR_INVALID_VALUE";
+        case ACSR_ERR_WORKSPACE: return "ACSR_ERR_WORKSPACE";
+        case ACSR_ERR_CAPACITY: return "ACSR_ERR_CAPACITY";
+        case ACSR_ERR_CUDA: return "ACSR_ERR_CUDA";
+        case ACSR_ERR_NCCL: return "ACSR_ERR_NCCL";
+        case ACSR_ERR_UNSUPPORTED: return "ACSR_ERR_UNSUPPORTED";
+    }
+    return "ACSR_UNKNOWN_STATUS";
+}
+
+extern "C" const char *acsr_last_error(void) { return g_err; }
+
+extern "C" int acsr_version(void) { return 100; }

@@ -1,0 +1,114 @@
+// acsr_internal.cuh -- constants, plan-workspace layout and small device helpers
+// shared by the libacsr.so translation units.  sm_100a only.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/acsr.h"
+
+namespace acsr {
+
+// ---------------------------------------------------------------- binning tiles
+// acsr_bin processes the rows in tiles of TILE_ROWS rows (one CTA per tile, 16
+// rounds of 256 rows).  The per-(bin, tile) counts double as the row-space
+// locality unit of the SpMV work map.
+constexpr int BIN_THREADS = 256;
+constexpr int TILE_ROWS = 4096;
+constexpr int TILE_ROUNDS = TILE_ROWS / BIN_THREADS;
+constexpr int NBINS = ACSR_NBINS;
+
+// ---------------------------------------------------------------- SpMV mapping
+// bins 1..6  : sub-warp of 2^{b-1} lanes per row, <= 2 nnz per lane (Alg. 2)
+// bins 7..10 : one warp per row
+// bins >= 11 : "heavy" rows (> 1024 nnz), cut into HEAVY_CHUNK-nnz chunks, one
+//              warp per chunk, deterministic last-arriver combine.
+constexpr int LIGHT_MAX_BIN = 10;
+constexpr int HEAVY_BIN = LIGHT_MAX_BIN + 1;
+constexpr int HEAVY_CHUNK = 1024;  // power of two
+
+// rows per light work unit, by bin (~8-12 KB of CSR traffic per unit)
+__host__ __device__ constexpr int unit_rows(int b)
+{
+    return b == 0 ? 1024 : b == 1 ? 256 : b == 2 ? 128 : b == 3 ? 128 : b == 4 ? 64
+         : b == 5 ? 32 : b == 6 ? 16 : b == 7 ? 8 : b == 8 ? 4 : b == 9 ? 2 : 1;
+}
+
+constexpr int SPMV_THREADS = 256;
+constexpr int SPMV_WARPS = SPMV_THREADS / 32;
+constexpr int MAX_WARPS = 160 * 64;  // >= SMs * resident warps on any sm_100 part
+
+// unit descriptor: light  x = first index into bin_rows, y = (bin << 24) | rows
+//                  heavy  x = row id,                     y = 0x80000000 | chunk
+constexpr uint32_t HEAVY_FLAG = 0x80000000u;
+
+// ---------------------------------------------------------------- plan header
+struct PlanHeader {
+    int32_t n_heavy_units;  // heavy units come first in the unit list
+    int32_t n_light_units;
+    int32_t n_units;
+    int32_t scan_ticket;    // last-CTA detection in the scan kernel
+    int32_t done_ticket;    // last-warp detection in the PageRank epilogue
+    int32_t overflow;       // 1 if the unit list exceeded the workspace bounds
+    int32_t n_tiles;
+    int32_t pad;
+    int64_t off_units, off_partial, off_ticket, off_warp_part;  // byte offsets from the header
+    int32_t totals[NBINS + 2 + 2];  // per scan row totals (bins, light units, heavy units)
+};
+
+struct PlanLayout {
+    int64_t n_tiles = 0, light_cap = 0, heavy_cap = 0;
+    size_t off_cnt = 0, off_toff = 0, off_tile_units = 0, off_units = 0, off_partial = 0,
+           off_ticket = 0, off_warp_part = 0, total = 0;
+};
+
+__host__ __device__ inline size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+// Tile-level arrays are [ (NBINS + 2) x n_tiles ]: rows 0..31 the per-bin counts,
+// row 32 light units per tile, row 33 heavy units per tile.
+constexpr int SCAN_ROWS = NBINS + 2;
+
+inline PlanLayout plan_layout(int64_t n_rows, int64_t nnz_max)
+{
+    PlanLayout L;
+    L.n_tiles = (n_rows + TILE_ROWS - 1) / TILE_ROWS;
+    L.light_cap = n_rows + (int64_t)(LIGHT_MAX_BIN + 1) * L.n_tiles + 1;
+    int64_t heavy_rows_max = nnz_max / (HEAVY_CHUNK + 1) + 1;
+    L.heavy_cap = nnz_max / HEAVY_CHUNK + heavy_rows_max + 1;
+    size_t o = align_up(sizeof(PlanHeader), 256);
+    L.off_cnt = o;
+    o = align_up(o + sizeof(int32_t) * SCAN_ROWS * (size_t)L.n_tiles, 256);
+    L.off_toff = o;
+    o = align_up(o + sizeof(int32_t) * SCAN_ROWS * (size_t)L.n_tiles, 256);
+    L.off_tile_units = o;  // (unused slot kept for layout stability)
+    o = align_up(o + 256, 256);
+    L.off_units = o;
+    o = align_up(o + sizeof(int2) * (size_t)(L.light_cap + L.heavy_cap), 256);
+    L.off_partial = o;
+    o = align_up(o + sizeof(double) * (size_t)L.heavy_cap, 256);
+    L.off_ticket = o;
+    o = align_up(o + sizeof(int32_t) * (size_t)L.heavy_cap, 256);
+    L.off_warp_part = o;
+    o = align_up(o + sizeof(double) * (size_t)MAX_WARPS, 256);
+    L.total = o;
+    return L;
+}
+
+// ---------------------------------------------------------------- device helpers
+__device__ __forceinline__ int bin_of_len(int len)
+{
+    // bin 0: empty; 1: {1,2}; b = ceil(log2 len) otherwise
+    return len <= 0 ? 0 : (len <= 2 ? 1 : 32 - __clz(len - 1));
+}
+
+__device__ __forceinline__ int heavy_chunks(int len) { return (len + HEAVY_CHUNK - 1) / HEAVY_CHUNK; }
+
+template <typename T>
+__device__ __forceinline__ T ldg_stream(const T *p) { return __ldcs(p); }
+
+}  // namespace acsr
+
+// error plumbing (acsr_capi.cu)
+void acsr_set_error(const char *fmt, ...);
+acsr_status acsr_check_launch(const char *what);
+int acsr_num_sms();

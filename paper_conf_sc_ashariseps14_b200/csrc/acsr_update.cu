@@ -1,0 +1,189 @@
+// acsr_update.cu -- dynamic-graph update on slack CSR (§VII).
+//
+// The paper uses one warp per updated row with only its first thread working
+// (P:335).  Here every lane works: pass 1 validates the whole batch (one warp per
+// update, deletes counted by binary search in the sorted delete list) and records
+// the smallest failing index with a 64-bit atomicMin; pass 2 (only if the batch is
+// valid -- all-or-nothing, reading Q13) compacts each row with a warp ballot
+// prefix (stable, in place: a lane's destination is never past its source) and
+// appends the inserts lane-parallel.  Out-degrees change by integer atomics, so
+// the result is exact and independent of scheduling.
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include "acsr_internal.cuh"
+
+namespace acsr {
+
+constexpr int UPD_THREADS = 256;
+constexpr unsigned long long NO_FAIL = ~0ull;
+
+__device__ __forceinline__ bool member(const int32_t *__restrict__ d, int lo, int hi, int c)
+{
+    int l = lo, h = hi;
+    while (l < h) {
+        int mid = (l + h) >> 1;
+        if (__ldg(d + mid) < c) l = mid + 1;
+        else h = mid;
+    }
+    return l < hi && __ldg(d + l) == c;
+}
+
+__global__ void __launch_bounds__(UPD_THREADS)
+update_validate_kernel(int64_t n_rows, int64_t n_cols, const int32_t *__restrict__ rb,
+                       const int32_t *__restrict__ re, const int32_t *__restrict__ cap,
+                       const int32_t *__restrict__ col, int64_t n_upd,
+                       const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
+                       const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
+                       const int32_t *__restrict__ icol, unsigned long long *key)
+{
+    const int lane = threadIdx.x & 31;
+    const int64_t i = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
+    if (i >= n_upd) return;
+    int code = ACSR_OK;
+    const int r = __ldg(upd + i);
+    if (r < 0 || r >= n_rows || (i > 0 && r <= __ldg(upd + i - 1))) code = ACSR_ERR_INVALID_VALUE;
+    int d0 = 0, d1 = 0;
+    if (dptr) {
+        d0 = __ldg(dptr + i);
+        d1 = __ldg(dptr + i + 1);
+    }
+    if (code == ACSR_OK && dptr) {
+        bool bad = false;
+        for (int j = d0 + 1 + lane; j < d1; j += 32) bad |= __ldg(dcol + j) < __ldg(dcol + j - 1);
+        if (__any_sync(0xffffffffu, bad)) code = ACSR_ERR_INVALID_VALUE;
+    }
+    const int i0 = __ldg(iptr + i), i1 = __ldg(iptr + i + 1);
+    if (code == ACSR_OK) {
+        bool bad = false;
+        for (int j = i0 + lane; j < i1; j += 32) {
+            int c = __ldg(icol + j);
+            bad |= (c < 0 || c >= n_cols);
+        }
+        if (__any_sync(0xffffffffu, bad)) code = ACSR_ERR_INVALID_VALUE;
+    }
+    if (code == ACSR_OK) {
+        const int b = __ldg(rb + r), e = __ldg(re + r);
+        int dels = 0;
+        if (d1 > d0)
+            for (int k = b + lane; k < e; k += 32) dels += member(dcol, d0, d1, __ldg(col + k)) ? 1 : 0;
+        for (int o = 16; o > 0; o >>= 1) dels += __shfl_xor_sync(0xffffffffu, dels, o);
+        long long new_len = (long long)(e - b) - dels + (i1 - i0);
+        if (new_len > __ldg(cap + r)) code = ACSR_ERR_CAPACITY;
+    }
+    if (code != ACSR_OK && lane == 0) atomicMin(key, ((unsigned long long)i << 3) | (unsigned)code);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(UPD_THREADS)
+update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
+                    int32_t *__restrict__ col, T *__restrict__ val, int64_t n_upd,
+                    const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
+                    const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
+                    const int32_t *__restrict__ icol, const T *__restrict__ ival, T one,
+                    int32_t *__restrict__ outdeg, const unsigned long long *key,
+                    int32_t *__restrict__ status)
+{
+    const unsigned long long k = *(volatile const unsigned long long *)key;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        status[0] = k == NO_FAIL ? ACSR_OK : (int32_t)(k & 7);
+        status[1] = k == NO_FAIL ? -1 : (int32_t)(k >> 3);
+    }
+    if (k != NO_FAIL) return;  // all-or-nothing
+    const int lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    const int64_t i = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
+    if (i >= n_upd) return;
+    const int r = __ldg(upd + i);
+    const int b = __ldg(rb + r), e = re[r];
+    int w = e;
+    const int d0 = dptr ? __ldg(dptr + i) : 0, d1 = dptr ? __ldg(dptr + i + 1) : 0;
+    if (d1 > d0) {
+        w = b;
+        for (int k0 = b; k0 < e; k0 += 32) {
+            int kk = k0 + lane;
+            bool valid = kk < e;
+            int c = valid ? col[kk] : 0;
+            T v = T();
+            if (val && valid) v = val[kk];
+            bool del = valid && member(dcol, d0, d1, c);
+            bool keep = valid && !del;
+            unsigned m = __ballot_sync(0xffffffffu, keep);
+            __syncwarp();  // every lane has read its source before anyone writes
+            if (keep) {
+                int dst = w + __popc(m & lt);
+                col[dst] = c;
+                if (val) val[dst] = v;
+            }
+            if (del && outdeg) atomicSub(outdeg + c, 1);
+            w += __popc(m);
+            __syncwarp();
+        }
+    }
+    const int i0 = __ldg(iptr + i), i1 = __ldg(iptr + i + 1);
+    for (int j = i0 + lane; j < i1; j += 32) {
+        int c = __ldg(icol + j);
+        col[w + (j - i0)] = c;
+        if (val) val[w + (j - i0)] = ival ? ival[j] : one;
+        if (outdeg) atomicAdd(outdeg + c, 1);
+    }
+    if (lane == 0) re[r] = w + (i1 - i0);
+}
+
+}  // namespace acsr
+
+using namespace acsr;
+
+extern "C" size_t acsr_update_workspace_bytes(int64_t n_upd)
+{
+    (void)n_upd;
+    return 256;
+}
+
+extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
+                                         const int32_t *row_begin, int32_t *row_end,
+                                         const int32_t *row_cap, int32_t *col_idx, void *values,
+                                         int64_t n_upd, const int32_t *upd_rows,
+                                         const int32_t *del_ptr, const int32_t *del_cols,
+                                         const int32_t *ins_ptr, const int32_t *ins_cols,
+                                         const void *ins_vals, int32_t *outdeg, int32_t *status,
+                                         void *ws, size_t ws_bytes, cudaStream_t stream)
+{
+    if (n_rows < 0 || n_cols < 0 || n_upd < 0 || !status || (dt != ACSR_F32 && dt != ACSR_F64) ||
+        (n_upd > 0 && (!row_begin || !row_end || !row_cap || !col_idx || !upd_rows || !ins_ptr)) ||
+        ((del_ptr == nullptr) != (del_cols == nullptr) && del_ptr != nullptr && n_upd > 0)) {
+        acsr_set_error("acsr_update_edges: invalid argument");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    if (!ws || ws_bytes < acsr_update_workspace_bytes(n_upd)) {
+        acsr_set_error("acsr_update_edges: workspace too small");
+        return ACSR_ERR_WORKSPACE;
+    }
+    unsigned long long *key = (unsigned long long *)ws;
+    cudaMemsetAsync(key, 0xff, sizeof(unsigned long long), stream);
+    const int wpb = UPD_THREADS / 32;
+    const int64_t blocks64 = n_upd > 0 ? (n_upd + wpb - 1) / wpb : 1;
+    if (blocks64 > 0x7fffffff) return ACSR_ERR_INVALID_VALUE;
+    const int blocks = (int)blocks64;
+    if (n_upd > 0)
+        update_validate_kernel<<<blocks, UPD_THREADS, 0, stream>>>(n_rows, n_cols, row_begin, row_end,
+                                                                   row_cap, col_idx, n_upd, upd_rows,
+                                                                   del_ptr, del_cols, ins_ptr, ins_cols,
+                                                                   key);
+    if (dt == ACSR_F64) {
+        uint64_t one;
+        double d1 = 1.0;
+        memcpy(&one, &d1, 8);
+        update_apply_kernel<uint64_t><<<blocks, UPD_THREADS, 0, stream>>>(
+            row_begin, row_end, col_idx, (uint64_t *)values, n_upd, upd_rows, del_ptr, del_cols, ins_ptr,
+            ins_cols, (const uint64_t *)ins_vals, one, outdeg, key, status);
+    } else {
+        uint32_t one;
+        float f1 = 1.0f;
+        memcpy(&one, &f1, 4);
+        update_apply_kernel<uint32_t><<<blocks, UPD_THREADS, 0, stream>>>(
+            row_begin, row_end, col_idx, (uint32_t *)values, n_upd, upd_rows, del_ptr, del_cols, ins_ptr,
+            ins_cols, (const uint32_t *)ins_vals, one, outdeg, key, status);
+    }
+    return acsr_check_launch("acsr_update_edges");
+}

@@ -1,0 +1,89 @@
+"""Convenience objects over the C ABI (argument marshalling only).
+
+``ACSRMatrix`` owns a (possibly slack) CSR on the device together with its bins and
+plan workspace; ``spmv_from_host`` is the end-to-end path a user with host arrays
+takes (pinned H2D copies, bin, SpMV, D2H); ``pagerank`` is the single-GPU Alg. 5 loop
+ with the convergence test of reading Q9.
+"""
+from __future__ import annotations
+
+import torch
+
+from . import (acsr_bin, acsr_bin_workspace_bytes, acsr_pagerank_scale, acsr_pagerank_step,
+               acsr_spmv, acsr_update_edges)
+
+
+class ACSRMatrix:
+    """Device CSR + ACSR bins.  row_end None => standard CSR (row_begin has n+1 entries)."""
+
+    def __init__(self, row_begin, col_idx, values=None, n_cols=None, row_end=None, row_cap=None,
+                 nnz_max=None):
+        self.row_begin = row_begin
+        self.row_end = row_end
+        self.row_cap = row_cap
+        self.col_idx = col_idx
+        self.values = values
+        self.n_rows = row_begin.numel() - 1 if row_end is None else row_begin.numel()
+        self.n_cols = self.n_rows if n_cols is None else n_cols
+        self.nnz_max = col_idx.numel() if nnz_max is None else nnz_max
+        dev = row_begin.device
+        self.bin_rows = torch.empty(self.n_rows, dtype=torch.int32, device=dev)
+        self.bin_offsets = torch.empty(33, dtype=torch.int32, device=dev)
+        self.plan_ws = torch.empty(acsr_bin_workspace_bytes(self.n_rows, self.nnz_max),
+                                   dtype=torch.uint8, device=dev)
+        self.rebin()
+
+    def rebin(self, stream=None):
+        acsr_bin(self.row_begin, self.row_end, self.nnz_max, self.bin_rows, self.bin_offsets,
+                 self.plan_ws, stream)
+
+    def spmv(self, x, y=None, stream=None):
+        return acsr_spmv(self.row_begin, self.col_idx, self.values, x, self.bin_rows,
+                         self.bin_offsets, self.plan_ws, self.row_end, y, stream)
+
+    def update(self, changes, outdeg=None, ins_vals=None, status=None, ws=None, stream=None):
+        """changes: dict of CUDA int32 tensors upd_rows, ins_ptr, ins_cols[, del_ptr, del_cols]."""
+        assert self.row_end is not None and self.row_cap is not None, "update needs slack CSR"
+        return acsr_update_edges(self.n_cols, self.row_begin, self.row_end, self.row_cap,
+                                 self.col_idx, self.values, changes["upd_rows"], changes["ins_ptr"],
+                                 changes["ins_cols"], ins_vals, changes.get("del_ptr"),
+                                 changes.get("del_cols"), outdeg, status, ws, stream=stream)
+
+
+def spmv_from_host(row_ptr_h, col_h, val_h, x_h, y_h=None, device="cuda", stream=None):
+    """End-to-end y = A x from (pinned) host arrays: H2D, acsr_bin, acsr_spmv, D2H."""
+    rp = row_ptr_h.to(device, non_blocking=True)
+    ci = col_h.to(device, non_blocking=True)
+    va = None if val_h is None else val_h.to(device, non_blocking=True)
+    x = x_h.to(device, non_blocking=True)
+    br, bo, ws = acsr_bin(rp, None, ci.numel(), stream=stream)
+    y = acsr_spmv(rp, ci, va, x, br, bo, ws, stream=stream)
+    if y_h is None:
+        return y.cpu()
+    y_h.copy_(y, non_blocking=True)
+    return y_h
+
+
+def pagerank(m: ACSRMatrix, outdeg, x0=None, damping=0.85, eps=1e-6, max_iter=1000, stream=None):
+    """Alg. 5 on one GPU over the in-link pattern matrix m.  Returns (x, iterations, delta2).
+    The convergence test reads one double per iteration (the paper's host loop)."""
+    n = m.n_rows
+    dev = m.row_begin.device
+    x = torch.full((n,), 1.0 / n, dtype=torch.float64, device=dev) if x0 is None else x0.clone()
+    xs = acsr_pagerank_scale(x, outdeg, stream=stream)
+    x_new = torch.empty_like(x)
+    xs_next = torch.empty_like(x)
+    d2 = torch.zeros(1, dtype=torch.float64, device=dev)
+    teleport = (1.0 - damping) / n
+    it = 0
+    delta2 = float("inf")
+    while it < max_iter:
+        acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xs, x,
+                           outdeg, x_new, xs_next, d2, damping, teleport, n, m.row_end, stream)
+        x, x_new = x_new, x
+        xs, xs_next = xs_next, xs
+        it += 1
+        delta2 = float(d2.item())
+        if delta2 ** 0.5 <= eps:
+            break
+    return x, it, delta2

@@ -1,0 +1,379 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bins and updates: bit-exact.  SpMV on integer-valued data: bit-exact (every summation
+order is exact).  SpMV on U(-1,1) data: |y - y_ref| <= 1e-12 * (|A||x|)_r in fp64 and
+1e-5 * (|A||x|)_r in fp32 (north_star; reading Q16); rows with den == 0 must match bitwise
+(+0.0 for empty rows).  PageRank: step-wise at the fp64 bar, loop iteration count within
++-1 of the oracle (reading Q18).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+TOL = {torch.float64: 1e-12, torch.float32: 1e-5}
+
+
+def check_spmv(y_gpu, y_ref, den, dtype, exact=False):
+    y_gpu = np.asarray(y_gpu, dtype=np.float64)
+    y_ref = np.asarray(y_ref, dtype=np.float64)
+    if exact:
+        assert np.array_equal(y_gpu, y_ref), np.flatnonzero(y_gpu != y_ref)[:10]
+        return
+    zero = den == 0
+    assert np.array_equal(y_gpu[zero], y_ref[zero])
+    assert not np.any(np.signbit(y_gpu[zero]) != np.signbit(y_ref[zero]))
+    err = np.abs(y_gpu - y_ref)
+    bad = err > TOL[dtype] * den
+    assert not bad.any(), (np.flatnonzero(bad)[:10], err[bad][:5], den[bad][:5])
+
+
+def run_csr(acsr, rp, ci, val, x, dev, row_end=None):
+    rbd = rp.to(dev)
+    red = None if row_end is None else row_end.to(dev)
+    m = acsr.ACSRMatrix(rbd, ci.to(dev), None if val is None else val.to(dev),
+                        n_cols=x.numel(), row_end=red, nnz_max=max(ci.numel(), 1))
+    y = m.spmv(x.to(dev))
+    torch.cuda.synchronize()
+    return m, y.cpu()
+
+
+# ------------------------------------------------------------------------------ bins
+@pytest.mark.parametrize("scale", [10, 14, 17])
+def test_bins_bitwise_rmat(acsr, cuda, scale):
+    rp, ci = synth.rmat_csr(scale)
+    m, _ = run_csr(acsr, rp, ci, None, torch.ones(rp.numel() - 1, dtype=torch.float64), cuda)
+    br, off = oracle.bins(rp.numpy())
+    assert np.array_equal(m.bin_offsets.cpu().numpy(), off)
+    assert np.array_equal(m.bin_rows.cpu().numpy(), br)
+
+
+def test_bins_boundary_and_slack(acsr, cuda):
+    lens = synth.boundary_lengths(17)
+    rp, ci = synth.boundary_csr(lens * 3, 1 << 18, 5)
+    rb, re, cap, c2, _ = synth.with_slack(rp, ci)
+    br, off = oracle.bins(rb.numpy(), re.numpy())
+    out = acsr.acsr_bin(rb.to(cuda), re.to(cuda), nnz_max=c2.numel())
+    torch.cuda.synchronize()
+    assert np.array_equal(out[1].cpu().numpy(), off)
+    assert np.array_equal(out[0].cpu().numpy(), br)
+
+
+@pytest.mark.parametrize("n", [0, 1, 4095, 4096, 4097, 70000])
+def test_bins_edge_sizes(acsr, cuda, n):
+    g = torch.Generator().manual_seed(n)
+    ln = torch.randint(0, 40, (n,), generator=g) * (torch.rand(n, generator=g) < 0.5)
+    if n:
+        ln[n // 2] = 5000  # one heavy row
+    rp = torch.zeros(n + 1, dtype=torch.int64)
+    rp[1:] = torch.cumsum(ln, 0)
+    rp = rp.to(torch.int32)
+    br, bo, ws = acsr.acsr_bin(rp.to(cuda), None, nnz_max=int(rp[-1]))
+    torch.cuda.synchronize()
+    br_ref, off_ref = oracle.bins(rp.numpy())
+    assert np.array_equal(bo.cpu().numpy(), off_ref)
+    assert np.array_equal(br.cpu().numpy(), br_ref)
+
+
+# ------------------------------------------------------------------------------ SpMV exact
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_spmv_integer_bitwise_rmat14(acsr, cuda, dtype):
+    rp, ci = synth.rmat_csr(14)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 1014, dtype, integer=True)
+    x = synth.vector(n, 2014, dtype, integer=True)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y.numpy(), y_ref, den, dtype, exact=True)
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_spmv_integer_bitwise_boundary(acsr, cuda, dtype):
+    # one row per bin edge up to 2^17+1 nnz: every mapping (sub-warp widths 1..32, warp,
+    # split rows with many chunks) is exercised; integer data makes every order exact.
+    lens = synth.boundary_lengths(17)
+    rp, ci = synth.boundary_csr(lens, 1 << 18, 3)
+    val = synth.values(ci.numel(), 7, dtype, integer=True)
+    x = synth.vector(1 << 18, 8, dtype, integer=True)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y.numpy(), y_ref, den, dtype, exact=True)
+
+
+def test_identity_permutation_pattern(acsr, cuda):
+    n = 100_000
+    x = synth.vector(n, 5)
+    rp = torch.arange(n + 1, dtype=torch.int32)
+    _, y = run_csr(acsr, rp, torch.arange(n, dtype=torch.int32), torch.ones(n, dtype=torch.float64), x, cuda)
+    assert torch.equal(y, x)
+    perm = torch.randperm(n, generator=torch.Generator().manual_seed(1)).to(torch.int32)
+    _, y = run_csr(acsr, rp, perm, None, x, cuda)
+    assert torch.equal(y, x[perm.long()])
+
+
+# ------------------------------------------------------------------------------ SpMV float
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+@pytest.mark.parametrize("scale", [14, 16])
+def test_spmv_float_rmat(acsr, cuda, dtype, scale):
+    rp, ci = synth.rmat_csr(scale)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 1014, dtype)
+    x = synth.vector(n, 2014, dtype)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y.numpy(), y_ref, den, dtype)
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_spmv_float_boundary(acsr, cuda, dtype):
+    lens = synth.boundary_lengths(17)
+    rp, ci = synth.boundary_csr(lens, 1 << 18, 9)
+    val = synth.values(ci.numel(), 10, dtype)
+    x = synth.vector(1 << 18, 11, dtype)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y.numpy(), y_ref, den, dtype)
+
+
+@pytest.mark.parametrize("dtype,L", [(torch.float64, 100_000), (torch.float32, 1_000_000)])
+def test_adversarial_long_equal_row(acsr, cuda, dtype, L):
+    # 0.1 repeated: sequential fp64 misses 1e-12 at 1e5 terms, sequential fp32 misses 1e-5
+    # at 1e6 terms; the chunked tree must not.
+    rp = torch.tensor([0, L, L], dtype=torch.int32)
+    ci = torch.zeros(L, dtype=torch.int32)
+    val = torch.full((L,), 0.1, dtype=dtype)
+    x = torch.ones(1, dtype=dtype)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y.numpy(), y_ref, den, dtype)
+
+
+def test_powerlaw_webgoogle_like(acsr, cuda):
+    rp, ci = synth.powerlaw_csr(seed=3, **dict(synth.WEB_GOOGLE, n=200_000))
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 4)
+    x = synth.vector(n, 5)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y.numpy(), y_ref, den, torch.float64)
+
+
+def test_slack_csr_equals_standard_and_determinism(acsr, cuda):
+    rp, ci = synth.rmat_csr(15)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 1)
+    x = synth.vector(n, 2)
+    m, y1 = run_csr(acsr, rp, ci, val, x, cuda)
+    y2 = m.spmv(x.to(cuda)).cpu()
+    assert torch.equal(y1, y2)  # run-to-run bitwise
+    rb, re, cap, c2, v2 = synth.with_slack(rp, ci, val)
+    _, y3 = run_csr(acsr, rb, c2, v2, x, cuda, row_end=re)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y3.numpy(), y_ref, den, torch.float64)
+
+
+def test_empty_and_all_empty(acsr, cuda):
+    rp = torch.zeros(1, dtype=torch.int32)
+    m, y = run_csr(acsr, rp, torch.zeros(0, dtype=torch.int32), torch.zeros(0, dtype=torch.float64),
+                   torch.ones(3, dtype=torch.float64), cuda)
+    assert y.numel() == 0
+    rp = torch.zeros(5001, dtype=torch.int32)
+    m, y = run_csr(acsr, rp, torch.zeros(0, dtype=torch.int32), torch.zeros(0, dtype=torch.float64),
+                   torch.ones(3, dtype=torch.float64), cuda)
+    assert torch.equal(y, torch.zeros(5000, dtype=torch.float64))
+    assert not torch.signbit(y).any()
+
+
+def test_full_size_rmat20_sampled(acsr, cuda):
+    """C2 at BASELINE size, in the launch configuration bench.py times: bins bitwise, and
+    sampled rows (every bin, the longest rows) against the oracle one by one."""
+    rp, ci = synth.rmat_csr(20, device=cuda)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 1014, device=cuda)
+    x = synth.vector(n, 2014, device=cuda)
+    m = acsr.ACSRMatrix(rp, ci, val)
+    y = m.spmv(x).cpu().numpy()
+    rph = rp.cpu().numpy()
+    br, off = oracle.bins(rph)
+    assert np.array_equal(m.bin_offsets.cpu().numpy(), off)
+    assert np.array_equal(m.bin_rows.cpu().numpy(), br)
+    ln = np.diff(rph)
+    rng = np.random.default_rng(0)
+    sample = set(rng.choice(n, 4000, replace=False).tolist()) | set(np.argsort(ln)[-50:].tolist())
+    for b in range(32):  # a few rows of every non-empty bin
+        sample |= set(br[off[b]:off[b + 1]][:20].tolist())
+    rows = np.array(sorted(sample))
+    sub_rp = np.zeros(rows.size + 1, np.int64)
+    sub_rp[1:] = np.cumsum(ln[rows])
+    cih, vh = ci.cpu().numpy(), val.cpu().numpy()
+    sub_ci = np.concatenate([cih[rph[r]:rph[r + 1]] for r in rows])
+    sub_v = np.concatenate([vh[rph[r]:rph[r + 1]] for r in rows])
+    y_ref, den = oracle.spmv(sub_rp.astype(np.int32), sub_ci, sub_v, x.cpu().numpy())
+    check_spmv(y[rows], y_ref, den, torch.float64)
+
+
+# ------------------------------------------------------------------------------ PageRank
+def _inlink(scale, dev):
+    rp, ci = synth.rmat_csr(scale, transpose=True)
+    n = rp.numel() - 1
+    od = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    return rp, ci, od, n
+
+
+def test_pagerank_step_parity(acsr, cuda):
+    rp, ci, od, n = _inlink(14, cuda)
+    x = synth.vector(n, 3).abs() / n
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda))
+    xs = acsr.acsr_pagerank_scale(x.to(cuda), od.to(cuda))
+    xn = torch.empty(n, dtype=torch.float64, device=cuda)
+    xsn = torch.empty_like(xn)
+    d2 = torch.zeros(1, dtype=torch.float64, device=cuda)
+    acsr.acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xs,
+                            x.to(cuda), od.to(cuda), xn, xsn, d2, 0.85, 0.15 / n)
+    xn_ref, d2_ref = oracle.pagerank_step(rp.numpy(), ci.numpy(), od.numpy(), x.numpy(), 0.15 / n, 0.85)
+    # den of the step = teleport + d * sum xs  (all terms >= 0)
+    xs_h = np.where(od.numpy() > 0, x.numpy() / np.maximum(od.numpy(), 1), 0.0)
+    _, den = oracle.spmv(rp.numpy(), ci.numpy(), None, xs_h)
+    bound = 1e-12 * (0.15 / n + 0.85 * den) + 2.3e-16 * np.abs(xn_ref)
+    assert np.all(np.abs(xn.cpu().numpy() - xn_ref) <= bound)
+    xsn_ref = np.where(od.numpy() > 0, xn_ref / np.maximum(od.numpy(), 1), 0.0)
+    assert np.allclose(xsn.cpu().numpy(), xsn_ref, rtol=1e-12, atol=0)
+    assert float(d2.item()) == pytest.approx(d2_ref, rel=1e-9)
+    # deterministic Delta^2 and x_new across runs
+    xn2 = torch.empty_like(xn)
+    d22 = torch.zeros_like(d2)
+    acsr.acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xs,
+                            x.to(cuda), od.to(cuda), xn2, xsn, d22, 0.85, 0.15 / n)
+    assert torch.equal(xn, xn2) and torch.equal(d2, d22)
+
+
+def test_pagerank_converged_parity(acsr, cuda):
+    rp, ci, od, n = _inlink(16, cuda)
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda))
+    x, it, d2 = acsr.pagerank(m, od.to(cuda), eps=1e-6)
+    x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)
+    assert abs(it - it_ref) <= 1
+    if it == it_ref:
+        xr = x_ref
+    else:
+        xr, _, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=0.0, max_iter=it)
+    assert np.all(np.abs(x.cpu().numpy() - xr) <= 1e-11 * xr + 1e-18)
+
+
+def test_pagerank_closed_forms(acsr, cuda):
+    # directed cycle -> uniform 1/n after one step
+    n = 10007
+    rp = torch.arange(n + 1, dtype=torch.int32)
+    ci = ((torch.arange(n) - 1) % n).to(torch.int32)  # in-link of v is v-1
+    od = torch.ones(n, dtype=torch.int32)
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda))
+    x, it, _ = acsr.pagerank(m, od.to(cuda))
+    assert it == 1 and torch.allclose(x.cpu(), torch.full((n,), 1.0 / n, dtype=torch.float64), rtol=2e-16, atol=0)
+    # a -> b (b dangling): (1-d)/2 and (1-d)(1+d)/2 (tests/golden/pagerank_two_vertex.txt)
+    m = acsr.ACSRMatrix(torch.tensor([0, 0, 1], dtype=torch.int32, device=cuda),
+                        torch.tensor([0], dtype=torch.int32, device=cuda))
+    x, it, _ = acsr.pagerank(m, torch.tensor([1, 0], dtype=torch.int32, device=cuda), eps=1e-15)
+    assert x[0].item() == pytest.approx(0.075, rel=1e-15)
+    assert x[1].item() == pytest.approx(0.13875, rel=1e-15)
+
+
+# ------------------------------------------------------------------------------ update
+def _slack_graph(scale, frac=4, dtype=torch.float64):
+    rp, ci = synth.rmat_csr(scale, transpose=True)
+    val = synth.values(ci.numel(), 5, dtype)
+    rb, re, cap, c2, v2 = synth.with_slack(rp, ci, val, frac=frac)
+    n = rp.numel() - 1
+    od = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    return n, rb, re, cap, c2, v2, od, rp, ci
+
+
+def _dev_changes(ch, dev):
+    return {k: torch.from_numpy(v).to(dev) for k, v in ch.items()}
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_update_insert_bitwise(acsr, cuda, dtype):
+    n, rb, re, cap, col, val, od, rp, ci = _slack_graph(14, dtype=dtype)
+    keys = np.sort(np.repeat(np.arange(n), np.diff(rp.numpy())).astype(np.int64) * n + ci.numpy())
+    ch, _ = next(synth.insert_batches(14, 1, 4096, keys))
+    iv = synth.values(ch["ins_cols"].size, 99, dtype)
+    # oracle on host copies
+    re_h, col_h, val_h, od_h = re.numpy().copy(), col.numpy().copy(), val.numpy().copy(), od.numpy().copy()
+    code, idx = oracle.update(n, rb.numpy(), re_h, cap.numpy(), col_h, val_h, ch["upd_rows"], None, None,
+                              ch["ins_ptr"], ch["ins_cols"], iv.numpy(), od_h)
+    assert code == 0
+    m = acsr.ACSRMatrix(rb.to(cuda), col.to(cuda), val.to(cuda), row_end=re.to(cuda), row_cap=cap.to(cuda),
+                        nnz_max=col.numel())
+    odd = od.to(cuda)
+    st = m.update(_dev_changes(ch, cuda), outdeg=odd, ins_vals=iv.to(cuda))
+    torch.cuda.synchronize()
+    assert st.cpu().tolist() == [0, -1]
+    re_g = m.row_end.cpu().numpy()
+    assert np.array_equal(re_g, re_h)
+    col_g, val_g = m.col_idx.cpu().numpy(), m.values.cpu().numpy()
+    live = np.concatenate([np.arange(b, e) for b, e in zip(rb.numpy(), re_h)])
+    assert np.array_equal(col_g[live], col_h[live])
+    assert np.array_equal(val_g[live].view(np.uint8), val_h[live].view(np.uint8))
+    assert np.array_equal(odd.cpu().numpy(), od_h)
+    # re-bin + SpMV on the updated slack CSR vs the oracle
+    m.rebin()
+    x = synth.vector(n, 6, dtype)
+    y = m.spmv(x.to(cuda)).cpu().numpy()
+    br, off = oracle.bins(rb.numpy(), re_h)
+    assert np.array_equal(m.bin_rows.cpu().numpy(), br)
+    y_ref, den = oracle.spmv(rb.numpy(), col_h, val_h, x.numpy(), row_end=re_h)
+    check_spmv(y, y_ref, den, dtype)
+
+
+def test_update_mixed_bitwise(acsr, cuda):
+    n, rb, re, cap, col, val, od, rp, ci = _slack_graph(12, frac=1)
+    ch = next(synth.mixed_batches(rp.numpy(), ci.numpy(), n, 0.1, 5, 1))
+    re_h, col_h, od_h = re.numpy().copy(), col.numpy().copy(), od.numpy().copy()
+    code, _ = oracle.update(n, rb.numpy(), re_h, cap.numpy(), col_h, None, ch["upd_rows"], ch["del_ptr"],
+                            ch["del_cols"], ch["ins_ptr"], ch["ins_cols"], None, od_h)
+    assert code == 0
+    m = acsr.ACSRMatrix(rb.to(cuda), col.to(cuda), None, row_end=re.to(cuda), row_cap=cap.to(cuda),
+                        nnz_max=col.numel())
+    odd = od.to(cuda)
+    st = m.update(_dev_changes(ch, cuda), outdeg=odd)
+    torch.cuda.synchronize()
+    assert st.cpu().tolist() == [0, -1]
+    assert np.array_equal(m.row_end.cpu().numpy(), re_h)
+    live = np.concatenate([np.arange(b, e) for b, e in zip(rb.numpy(), re_h)])
+    assert np.array_equal(m.col_idx.cpu().numpy()[live], col_h[live])
+    assert np.array_equal(odd.cpu().numpy(), od_h)
+
+
+def test_update_rejections_leave_matrix_unchanged(acsr, cuda):
+    n, rb, re, cap, col, val, od, rp, ci = _slack_graph(10)
+    m = acsr.ACSRMatrix(rb.to(cuda), col.to(cuda), val.to(cuda), row_end=re.to(cuda), row_cap=cap.to(cuda),
+                        nnz_max=col.numel())
+    odd = od.to(cuda)
+    snap = [t.clone() for t in (m.row_end, m.col_idx, m.values, odd)]
+    free7 = int(cap[7] - (re[7] - rb[7]))
+    cases = [
+        (dict(upd_rows=[3, 7], ins_ptr=[0, 1, free7 + 2], ins_cols=[1] + [2] * (free7 + 1)), [3, 1]),
+        (dict(upd_rows=[5, 5], ins_ptr=[0, 1, 2], ins_cols=[1, 2]), [1, 1]),
+        (dict(upd_rows=[5, 6], ins_ptr=[0, 1, 2], ins_cols=[1, n]), [1, 1]),
+        (dict(upd_rows=[5, 6], ins_ptr=[0, 1, 2], ins_cols=[1, 2], del_ptr=[0, 0, 2], del_cols=[9, 3]), [1, 1]),
+    ]
+    for ch, expect in cases:
+        chd = {k: torch.tensor(v, dtype=torch.int32, device=cuda) for k, v in ch.items()}
+        st = m.update(chd, outdeg=odd)
+        torch.cuda.synchronize()
+        assert st.cpu().tolist() == expect
+        for a, b in zip((m.row_end, m.col_idx, m.values, odd), snap):
+            assert torch.equal(a, b)
+
+
+def test_argument_errors(acsr, cuda):
+    with pytest.raises(TypeError):
+        acsr.acsr_bin(torch.zeros(3, dtype=torch.int32), None, nnz_max=0)  # CPU tensor
+    rp = torch.zeros(3, dtype=torch.int32, device=cuda)
+    with pytest.raises(acsr.ACSRError) as e:
+        acsr.acsr_bin(rp, None, nnz_max=0, plan_ws=torch.empty(8, dtype=torch.uint8, device=cuda))
+    assert e.value.code == acsr.ACSR_ERR_WORKSPACE

@@ -216,6 +216,8 @@ def acsr_update_edges(n_cols, row_begin, row_end, row_cap, col_idx, values, upd_
     if ws is None:
         ws = torch.empty(acsr_update_workspace_bytes(n_upd), dtype=torch.uint8, device=dev)
     vdt = values.dtype if values is not None else dtype
+    if del_ptr is not None and (del_cols is None or del_cols.numel() == 0):
+        del_ptr, del_cols = None, None  # insert-only batch
     dt = ACSR_F64 if vdt == torch.float64 else ACSR_F32
     opt = lambda t, d, nm: (_dev(t, d, nm) if t is not None and t.numel() else None)
     _check(_lib.acsr_update_edges(dt, n, int(n_cols), _dev(row_begin, torch.int32, "row_begin"),

@@ -325,7 +325,7 @@ extern "C" acsr_status acsr_spmv(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
 {
     if (n_rows < 0 || n_cols < 0 || n_rows >= ((int64_t)1 << 31) ||
         (dt != ACSR_F32 && dt != ACSR_F64) ||
-        (n_rows > 0 && (!row_begin || !y || (n_cols > 0 && (!x || !col_idx))))) {
+        (n_rows > 0 && (!row_begin || !y))) {
         acsr_set_error("acsr_spmv: invalid argument");
         return ACSR_ERR_INVALID_VALUE;
     }
@@ -353,8 +353,7 @@ extern "C" acsr_status acsr_spmv(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
 extern "C" acsr_status acsr_pagerank_step(const acsr_pr_args *p, cudaStream_t stream)
 {
     if (!p || p->n_rows < 0 || p->n_cols < 0 || p->n_rows >= ((int64_t)1 << 31) || !p->delta2 ||
-        (p->n_rows > 0 && (!p->row_begin || !p->x || !p->outdeg || !p->x_new || !p->xs_next ||
-                           (p->n_cols > 0 && (!p->xs || !p->col_idx))))) {
+        (p->n_rows > 0 && (!p->row_begin || !p->x || !p->outdeg || !p->x_new || !p->xs_next))) {
         acsr_set_error("acsr_pagerank_step: invalid argument");
         return ACSR_ERR_INVALID_VALUE;
     }

@@ -1,0 +1,136 @@
+"""Row-partitioned multi-GPU PageRank (§VIII P:343-348 "a simple division ... each GPU is
+thus responsible for computing half the results", generalised to P ranks; reading Q19).
+
+One process per GPU (torchrun); ``torch.distributed`` (NCCL over NVLink/NVSwitch) is the
+plumbing.  Per iteration each rank runs ONE fused ``acsr_pagerank_step`` launch on its
+contiguous row range (SpMV on the in-link pattern + teleport/damping epilogue + xs slice +
+Delta^2 partial), then
+
+  * all-gathers the xs slices (equal-size padded slices, in place -> NCCL ring/NVLS
+    all-gather; the only data-path exchange, A9 in SURVEY §8(a)),
+  * all-reduces the 8-byte Delta^2 (the convergence test of Alg. 5, reading Q9).
+
+Host logic here (partition, column renumbering into the padded layout, the loop) is
+device-agnostic so it is unit-tested with the gloo backend on CPU (tests/test_dist_gloo.py)
+by injecting a CPU step function; on GPUs the step is the CUDA kernel.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+
+def partition_rows(row_lengths: np.ndarray, P: int, b_nnz: int = 4, b_row: int = 36) -> np.ndarray:
+    """Contiguous split balanced on cost(r) = b_nnz*len_r + b_row (integer bytes; PageRank
+    pattern: 4 B per column index + 36 B per row).  splits[0] = 0, splits[P] = n and
+    splits[k] = min{r : sum_{r'<r} cost >= ceil(k*total/P)}."""
+    ln = np.asarray(row_lengths, dtype=np.int64)
+    n = ln.size
+    pref = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(b_nnz * ln + b_row, out=pref[1:])
+    total = int(pref[-1])
+    s = np.empty(P + 1, dtype=np.int64)
+    s[0], s[P] = 0, n
+    for k in range(1, P):
+        t = -(-k * total // P)
+        s[k] = int(np.searchsorted(pref, t, side="left"))
+    return s
+
+
+def padded_layout(splits: np.ndarray):
+    """Equal-size slices for the in-place all-gather: vertex v of rank k lives at
+    k*L + (v - splits[k]) with L = max slice length."""
+    sizes = np.diff(splits)
+    L = int(sizes.max()) if sizes.size else 0
+    return L
+
+
+def renumber_columns(col: torch.Tensor, splits: np.ndarray, L: int) -> torch.Tensor:
+    """Global vertex ids -> padded positions (setup, once per graph)."""
+    sp = torch.as_tensor(splits[1:-1], dtype=torch.int64, device=col.device)
+    c = col.to(torch.int64)
+    owner = torch.searchsorted(sp, c, right=True)
+    start = torch.as_tensor(splits[:-1], dtype=torch.int64, device=col.device)[owner]
+    return (owner * L + (c - start)).to(torch.int32)
+
+
+class DistPageRank:
+    """PageRank over P ranks.  Each rank passes its local in-link CSR rows
+    [splits[rank], splits[rank+1]) with GLOBAL column ids; the object renumbers the
+    columns once and owns the replicated padded xs buffers.
+
+    step_fn(local, xs, x, x_new, xs_next_slice, delta2) computes one local step; the
+    default runs the CUDA kernel (acsr_pagerank_step)."""
+
+    def __init__(self, row_ptr_local, col_local, outdeg_local, splits, n_global, damping=0.85,
+                 group=None, step_fn=None, scale_fn=None, device=None):
+        self.group = group
+        self.rank = dist.get_rank(group) if dist.is_initialized() else 0
+        self.world = dist.get_world_size(group) if dist.is_initialized() else 1
+        self.splits = np.asarray(splits, dtype=np.int64)
+        assert self.splits.size == self.world + 1
+        self.n_global = int(n_global)
+        self.n_local = int(self.splits[self.rank + 1] - self.splits[self.rank])
+        self.L = padded_layout(self.splits)
+        self.damping = float(damping)
+        self.teleport = (1.0 - self.damping) / self.n_global  # computed once, same bits on all ranks
+        self.device = row_ptr_local.device if device is None else device
+        self.row_ptr = row_ptr_local
+        self.col = renumber_columns(col_local, self.splits, self.L) if self.world > 1 else col_local
+        self.outdeg = outdeg_local
+        self.step_fn = step_fn or self._cuda_step
+        self.scale_fn = scale_fn or self._cuda_scale
+        dev = self.device
+        self.xs = torch.zeros(self.world * self.L, dtype=torch.float64, device=dev)
+        self.xs_next = torch.zeros_like(self.xs)
+        self.delta2 = torch.zeros(1, dtype=torch.float64, device=dev)
+        self._m = None
+        if self.step_fn is self._cuda_step:
+            from .matrix import ACSRMatrix
+            self._m = ACSRMatrix(self.row_ptr, self.col, None, n_cols=self.xs.numel())
+
+    def _slice(self, buf):
+        return buf[self.rank * self.L: self.rank * self.L + self.n_local]
+
+    def _cuda_step(self, xs, x, x_new, xs_next_slice, delta2):
+        from . import acsr_pagerank_step
+        m = self._m
+        acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xs, x,
+                           self.outdeg, x_new, xs_next_slice, delta2, self.damping, self.teleport,
+                           self.n_global)
+
+    def _cuda_scale(self, x, outdeg, out):
+        from . import acsr_pagerank_scale
+        acsr_pagerank_scale(x, outdeg, out)
+
+    def exchange(self, buf):
+        if self.world > 1:
+            chunk = buf[self.rank * self.L:(self.rank + 1) * self.L]  # padded: tail stays 0
+            dist.all_gather_into_tensor(buf, chunk.clone() if buf.device.type == "cpu" else chunk,
+                                        group=self.group)
+
+    def run(self, x0_local=None, eps=1e-6, max_iter=1000):
+        """Alg. 5 loop; returns (x_local, iterations, delta2_global)."""
+        dev = self.device
+        if x0_local is None:
+            x = torch.full((self.n_local,), 1.0 / self.n_global, dtype=torch.float64, device=dev)
+        else:
+            x = x0_local.clone()
+        # xs^0 slice = x^0 / outdeg (IEEE division), then gather
+        self.scale_fn(x, self.outdeg, self._slice(self.xs))
+        self.exchange(self.xs)
+        x_new = torch.empty_like(x)
+        it, d2 = 0, float("inf")
+        while it < max_iter:
+            self.step_fn(self.xs, x, x_new, self._slice(self.xs_next), self.delta2)
+            self.exchange(self.xs_next)
+            if self.world > 1:
+                dist.all_reduce(self.delta2, group=self.group)
+            x, x_new = x_new, x
+            self.xs, self.xs_next = self.xs_next, self.xs
+            it += 1
+            d2 = float(self.delta2.item())
+            if d2 ** 0.5 <= eps:
+                break
+        return x, it, d2

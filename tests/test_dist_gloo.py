@@ -1,0 +1,100 @@
+"""Multi-process (world_size 2, gloo, CPU) test of the row-partitioned PageRank host logic:
+partition, column renumbering into the padded all-gather layout, in-place all-gather of the
+xs slices, all-reduce of Delta^2 and the Alg. 5 loop.  The per-rank local step is injected
+(the CPU oracle on the local rows) -- the CUDA step itself is covered by tests -m gpu."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle
+import synth
+from paper_conf_sc_ashariseps14_b200 import dist as acsr_dist
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, scale, out):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    rp, ci = synth.rmat_csr(scale, transpose=True)
+    n = rp.numel() - 1
+    od = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    splits = acsr_dist.partition_rows(np.diff(rp.numpy()), world)
+    lo, hi = int(splits[rank]), int(splits[rank + 1])
+    rpl = (rp[lo:hi + 1] - rp[lo]).contiguous()
+    cil = ci[int(rp[lo]):int(rp[hi])].contiguous()
+    odl = od[lo:hi].contiguous()
+
+    def step(xs, x, x_new, xs_next_slice, delta2):
+        xn, d2 = oracle.pagerank_step(rpl.numpy(), pr.col.numpy(), np.ones(xs.numel(), np.int32),
+                                      xs.numpy(), pr.teleport, pr.damping)
+        # oracle with outdeg = 1 gathers xs itself: y_v = sum xs_u  (xs already scaled)
+        x_new.copy_(torch.from_numpy(xn))
+        xs_next_slice.copy_(torch.where(odl > 0, x_new / odl.clamp(min=1).double(), torch.zeros_like(x_new)))
+        delta2.fill_(float(((x_new - x) ** 2).sum()))
+
+    def scale(x, outdeg, outv):
+        outv.copy_(torch.where(outdeg > 0, x / outdeg.clamp(min=1).double(), torch.zeros_like(x)))
+
+    pr = acsr_dist.DistPageRank(rpl, cil, odl, splits, n, step_fn=step, scale_fn=scale,
+                                device=torch.device("cpu"))
+    x, it, d2 = pr.run(eps=1e-8)
+    xs_all = [torch.zeros(pr.L, dtype=torch.float64) for _ in range(world)]
+    xp = torch.zeros(pr.L, dtype=torch.float64)
+    xp[: x.numel()] = x
+    dist.all_gather(xs_all, xp)
+    if rank == 0:
+        full = torch.cat([xs_all[k][: int(splits[k + 1] - splits[k])] for k in range(world)])
+        out.put((full.numpy(), it, d2, splits))
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2])
+def test_partitioned_pagerank_matches_single(world):
+    scale = 11
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, scale, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    full, it, d2, splits = q.get(timeout=240)
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    rp, ci = synth.rmat_csr(scale, transpose=True)
+    n = rp.numel() - 1
+    od = torch.bincount(ci.long(), minlength=n).to(torch.int32).numpy()
+    x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od, eps=1e-8)
+    assert abs(it - it_ref) <= 1
+    assert np.allclose(full, x_ref, rtol=1e-11, atol=1e-18)
+    assert splits[0] == 0 and splits[-1] == n and np.all(np.diff(splits) > 0)
+
+
+def test_partition_matches_oracle_rule():
+    rp, _ = synth.rmat_csr(12)
+    for P in (1, 2, 4, 8):
+        s = acsr_dist.partition_rows(np.diff(rp.numpy()), P)
+        assert np.array_equal(s, oracle.partition(rp.numpy(), P, 4, 36))
+
+
+def test_renumber_roundtrip():
+    splits = np.array([0, 5, 12, 20])
+    L = acsr_dist.padded_layout(splits)
+    col = torch.arange(20, dtype=torch.int32)
+    c2 = acsr_dist.renumber_columns(col, splits, L)
+    owner = c2 // L
+    assert torch.equal(owner, torch.tensor([0] * 5 + [1] * 7 + [2] * 8))
+    back = torch.tensor(splits[:-1])[owner.long()] + c2 % L
+    assert torch.equal(back.to(torch.int32), col)

@@ -49,7 +49,8 @@ enum { ACSR_NBINS = 32 };
 
 /* ------------------------------------------------------------------------ */
 /* Binning (Alg. 1 "if (this is the first iteration) ... foreach row r do
- * b_r <- b_r U {r}"; §III-A).
+ * b_r <- b_r U {r}"; §III-A).  Inputs are those of
+ * Alg. 1: the CSR matrix (row offsets, col_idx).
  *
  * Row r with len_r = row_end[r] - row_begin[r] non-zeros goes to bin
  *     b = 0 if len_r == 0;  1 if len_r <= 2;  else ceil(log2(len_r))
@@ -61,17 +62,23 @@ enum { ACSR_NBINS = 32 };
  *                           bin_offsets[32] = n_rows
  *   plan_ws                 the SpMV work map (replaces Alg. 1's G1/G2 split and
  *                           the dynamic-parallelism parent/child launches, P:61,
- *                           P:68-105): per-warp work units in row-space order and
- *                           the split plan for rows longer than 1024 non-zeros.
- * nnz_max bounds the total number of stored entries (sum of row lengths) that
- * any later acsr_bin on this workspace will see (for slack CSR: the capacity).
+ *                           P:68-105): warp work units in row-space order, the
+ *                           split plan for rows longer than 1024 non-zeros, and
+ *                           (if col_idx != NULL) the hot-column vote table of the
+ *                           SpMV's shared-memory x cache (the B200 stand-in for the
+ *                           paper's texture-bound x; a sample of about 2^18
+ *                           entries -- a performance hint only, never a result).
+ * n_cols is the length of x (column ids outside [0, n_cols) are ignored by the
+ * sampler).  nnz_max bounds the number of stored entries (sum of row lengths)
+ * that any later acsr_bin on this workspace will see (slack CSR: the capacity).
  * The row-length array is read twice (count pass + stable scatter pass); no
- * host synchronisation happens.  The result is deterministic and equals the
- * oracle bit for bit. */
+ * host synchronisation happens.  bin_rows/bin_offsets are deterministic and
+ * equal the oracle bit for bit.  plan_ws must not be shared by concurrent calls. */
 size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t nnz_max);
 
-acsr_status acsr_bin(int64_t n_rows, int64_t nnz_max,
+acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
                      const int32_t *row_begin, const int32_t *row_end /* NULL => standard CSR */,
+                     const int32_t *col_idx /* NULL => no x cache */,
                      int32_t *bin_rows /* [n_rows] out */,
                      int32_t *bin_offsets /* [ACSR_NBINS + 1] out */,
                      void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream);

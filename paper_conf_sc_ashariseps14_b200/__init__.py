@@ -44,7 +44,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 _i64, _vp, _sz, _dbl = ctypes.c_int64, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_double
 _lib.acsr_bin_workspace_bytes.argtypes = [_i64, _i64]
 _lib.acsr_bin_workspace_bytes.restype = _sz
-_lib.acsr_bin.argtypes = [_i64, _i64, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
+_lib.acsr_bin.argtypes = [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
 _lib.acsr_bin.restype = ctypes.c_int
 _lib.acsr_spmv.argtypes = [ctypes.c_int, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _sz,
                            _vp]
@@ -124,8 +124,9 @@ def acsr_bin_workspace_bytes(n_rows: int, nnz_max: int) -> int:
 
 
 def acsr_bin(row_begin, row_end=None, nnz_max=None, bin_rows=None, bin_offsets=None, plan_ws=None,
-             stream=None):
-    """Bin the rows.  Returns (bin_rows, bin_offsets, plan_ws)."""
+             stream=None, col_idx=None, n_cols=0):
+    """Bin the rows.  Returns (bin_rows, bin_offsets, plan_ws).  col_idx (with
+    n_cols) additionally builds the hot-column table of the SpMV x cache."""
     n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
     dev = row_begin.device
     if nnz_max is None:
@@ -137,8 +138,9 @@ def acsr_bin(row_begin, row_end=None, nnz_max=None, bin_rows=None, bin_offsets=N
     need = acsr_bin_workspace_bytes(n, nnz_max)
     if plan_ws is None:
         plan_ws = torch.empty(need, dtype=torch.uint8, device=dev)
-    _check(_lib.acsr_bin(n, int(nnz_max), _dev(row_begin, torch.int32, "row_begin"),
+    _check(_lib.acsr_bin(n, int(n_cols), int(nnz_max), _dev(row_begin, torch.int32, "row_begin"),
                          _dev(row_end, torch.int32, "row_end", True),
+                         _dev(col_idx, torch.int32, "col_idx") if col_idx is not None and col_idx.numel() else None,
                          _dev(bin_rows, torch.int32, "bin_rows") if n > 0 else None,
                          _dev(bin_offsets, torch.int32, "bin_offsets"),
                          _dev(plan_ws, torch.uint8, "plan_ws"), plan_ws.numel(), _stream(stream)),

@@ -68,13 +68,19 @@ constexpr int SCAN_THREADS = 1024;
 
 __global__ void __launch_bounds__(SCAN_THREADS)
 bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int n_tiles,
-                PlanHeader *hdr, int32_t *__restrict__ bin_offsets, int64_t n_rows,
-                int64_t light_cap, int64_t heavy_cap, int64_t off_units, int64_t off_partial,
-                int64_t off_ticket, int64_t off_warp_part)
+                PlanHeader *hdr, int32_t *__restrict__ bin_offsets, int64_t n_rows, int64_t n_cols,
+                int64_t light_cap, int64_t heavy_cap, PlanLayout L, int xc_valid, int xc_stride)
 {
     __shared__ int warp_sums[SCAN_THREADS / 32];
     __shared__ int is_last;
     const int row = blockIdx.x;
+    if (row >= SCAN_ROWS) {  // helper CTAs: clear the x-cache vote table
+        uint32_t *vote = (uint32_t *)((char *)hdr + L.off_xc_vote);
+        for (int i = (row - SCAN_ROWS) * SCAN_THREADS + threadIdx.x; i < XC_SLOTS;
+             i += (gridDim.x - SCAN_ROWS) * SCAN_THREADS)
+            vote[i] = 0u;
+        return;
+    }
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int32_t *a = cnt + (int64_t)row * n_tiles;
     int32_t *o = toff + (int64_t)row * n_tiles;
@@ -127,14 +133,52 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
         hdr->n_heavy_units = ovf ? 0 : nh;
         hdr->n_units = ovf ? 0 : nl + nh;
         hdr->n_tiles = n_tiles;
-        hdr->off_units = off_units;
-        hdr->off_partial = off_partial;
-        hdr->off_ticket = off_ticket;
-        hdr->off_warp_part = off_warp_part;
-        hdr->done_ticket = 0;
+        hdr->off_units = (int64_t)L.off_units;
+        hdr->off_partial = (int64_t)L.off_partial;
+        hdr->off_ticket = (int64_t)L.off_ticket;
+        hdr->off_xc_vote = (int64_t)L.off_xc_vote;
+        hdr->off_xc_tag = (int64_t)L.off_xc_tag;
+        hdr->off_xc_val = (int64_t)L.off_xc_val;
+        hdr->xc_valid = xc_valid;
+        hdr->xc_stride = xc_stride;
+        hdr->n_cols = n_cols;
+        hdr->work_ctr = 0;
+        hdr->exit_ticket = 0;
+        hdr->d2_hi = 0;
+        hdr->d2_lo = 0;
         hdr->scan_ticket = 0;
         (void)n_rows;
     }
+}
+
+// x-cache vote: Boyer-Moore majority per slot over a strided sample of the row's
+// entries (one CAS on a packed (tag16 << 16 | votes16) word per sampled entry).
+__device__ __forceinline__ void xc_vote(uint32_t *vote, int c, int64_t n_cols)
+{
+    if (c < 0 || c >= n_cols) return;  // slack garbage or bad ids: ignore (hint only)
+    const uint32_t s = (uint32_t)c & (XC_SLOTS - 1);
+    const uint32_t t = (uint32_t)c >> XC_BITS;
+    if (t >= XC_NOTAG) return;
+    uint32_t old = vote[s];
+    while (true) {
+        uint32_t ot = old >> 16, ov = old & 0xFFFFu, nw;
+        if (ov == 0) nw = (t << 16) | 1u;
+        else if (ot == t) nw = ov < 0xFFFFu ? old + 1u : old;
+        else nw = old - 1u;
+        if (nw == old) return;
+        uint32_t prev = atomicCAS(vote + s, old, nw);
+        if (prev == old) return;
+        old = prev;
+    }
+}
+
+__device__ __forceinline__ void xc_sample(const int32_t *__restrict__ rb, int64_t r, int len,
+                                          const int32_t *__restrict__ col, uint32_t *vote,
+                                          int64_t n_cols, int stride)
+{
+    const int beg = __ldg(rb + r);
+    for (int k = (int)(mix32((uint32_t)r) % (uint32_t)stride); k < len; k += stride)
+        xc_vote(vote, __ldg(col + beg + k), n_cols);
 }
 
 template <bool HAS_END>
@@ -142,7 +186,9 @@ __global__ void __launch_bounds__(BIN_THREADS)
 bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
                    int32_t *__restrict__ bin_rows, const int32_t *__restrict__ bin_offsets,
                    const int32_t *__restrict__ toff, int n_tiles, const PlanHeader *__restrict__ hdr,
-                   int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap)
+                   int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap,
+                   const int32_t *__restrict__ col, uint32_t *__restrict__ vote, int64_t n_cols,
+                   int xc_stride)
 {
     constexpr int NW = BIN_THREADS / 32;
     __shared__ int run[NBINS];
@@ -201,6 +247,7 @@ bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__r
             heavy_run = acc;
         }
         __syncthreads();
+        if (valid && col && len > 0) xc_sample(rb, r, len, col, vote, n_cols, xc_stride);
         if (valid) {
             bin_rows[seg[b] + wbase[warp][b] + rank] = (int32_t)r;
             if (hc > 0 && !overflow) {
@@ -246,11 +293,12 @@ extern "C" size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t nnz_max)
     return plan_layout(n_rows, nnz_max).total;
 }
 
-extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t nnz_max, const int32_t *row_begin,
-                                const int32_t *row_end, int32_t *bin_rows, int32_t *bin_offsets,
+extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
+                                const int32_t *row_begin, const int32_t *row_end,
+                                const int32_t *col_idx, int32_t *bin_rows, int32_t *bin_offsets,
                                 void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream)
 {
-    if (n_rows < 0 || nnz_max < 0 || n_rows >= (int64_t)1 << 31 || !bin_offsets ||
+    if (n_rows < 0 || n_cols < 0 || nnz_max < 0 || n_rows >= (int64_t)1 << 31 || !bin_offsets ||
         (n_rows > 0 && (!row_begin || !bin_rows))) {
         acsr_set_error("acsr_bin: invalid argument");
         return ACSR_ERR_INVALID_VALUE;
@@ -276,17 +324,24 @@ extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t nnz_max, const int32_t *
         bin_count_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
     else
         bin_count_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
-    bin_scan_kernel<<<SCAN_ROWS, SCAN_THREADS, 0, stream>>>(cnt, toff, nt, hdr, bin_offsets, n_rows,
-                                                              L.light_cap, L.heavy_cap,
-                                                              (int64_t)L.off_units, (int64_t)L.off_partial,
-                                                              (int64_t)L.off_ticket, (int64_t)L.off_warp_part);
+    const int xc_valid = col_idx != nullptr && n_cols > 0 && n_cols < ((int64_t)XC_NOTAG << XC_BITS);
+    int64_t stride64 = nnz_max >> XC_SAMPLE_LOG2;
+    const int xc_stride = (int)(stride64 < 1 ? 1 : (stride64 > (1 << 30) ? (1 << 30) : stride64));
+    uint32_t *vote = (uint32_t *)(ws + L.off_xc_vote);
+    const int zero_ctas = (XC_SLOTS + SCAN_THREADS - 1) / SCAN_THREADS;
+    bin_scan_kernel<<<SCAN_ROWS + zero_ctas, SCAN_THREADS, 0, stream>>>(
+        cnt, toff, nt, hdr, bin_offsets, n_rows, n_cols, L.light_cap, L.heavy_cap, L, xc_valid, xc_stride);
     if (row_end)
         bin_scatter_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, bin_rows,
                                                                    bin_offsets, toff, nt, hdr, units,
-                                                                   tickets, L.heavy_cap);
+                                                                   tickets, L.heavy_cap,
+                                                                   xc_valid ? col_idx : nullptr, vote,
+                                                                   n_cols, xc_stride);
     else
         bin_scatter_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, bin_rows,
                                                                     bin_offsets, toff, nt, hdr, units,
-                                                                    tickets, L.heavy_cap);
+                                                                    tickets, L.heavy_cap,
+                                                                    xc_valid ? col_idx : nullptr, vote,
+                                                                    n_cols, xc_stride);
     return acsr_check_launch("acsr_bin");
 }

@@ -10,11 +10,11 @@
 namespace acsr {
 
 // ---------------------------------------------------------------- binning tiles
-// acsr_bin processes the rows in tiles of TILE_ROWS rows (one CTA per tile, 16
-// rounds of 256 rows).  The per-(bin, tile) counts double as the row-space
+// acsr_bin processes the rows in tiles of TILE_ROWS rows (one CTA per tile, rounds
+// of 256 rows in row order).  The per-(bin, tile) counts double as the row-space
 // locality unit of the SpMV work map.
 constexpr int BIN_THREADS = 256;
-constexpr int TILE_ROWS = 4096;
+constexpr int TILE_ROWS = 1024;
 constexpr int TILE_ROUNDS = TILE_ROWS / BIN_THREADS;
 constexpr int NBINS = ACSR_NBINS;
 
@@ -27,16 +27,27 @@ constexpr int LIGHT_MAX_BIN = 10;
 constexpr int HEAVY_BIN = LIGHT_MAX_BIN + 1;
 constexpr int HEAVY_CHUNK = 1024;  // power of two
 
-// rows per light work unit, by bin (~8-12 KB of CSR traffic per unit)
+// rows per light work unit, by bin (~6-12 KB of CSR traffic per unit)
 __host__ __device__ constexpr int unit_rows(int b)
 {
     return b == 0 ? 1024 : b == 1 ? 256 : b == 2 ? 128 : b == 3 ? 128 : b == 4 ? 64
          : b == 5 ? 32 : b == 6 ? 16 : b == 7 ? 8 : b == 8 ? 4 : b == 9 ? 2 : 1;
 }
 
-constexpr int SPMV_THREADS = 256;
+// One persistent CTA of 1024 threads per SM: the whole SM shares one x cache.
+constexpr int SPMV_THREADS = 1024;
 constexpr int SPMV_WARPS = SPMV_THREADS / 32;
-constexpr int MAX_WARPS = 160 * 64;  // >= SMs * resident warps on any sm_100 part
+
+// ---------------------------------------------------------------- x cache
+// Direct-mapped cache of "hot" x entries in shared memory: slot s = c mod XC_SLOTS
+// holds x[c] for the column c chosen for that slot at bin time (Boyer-Moore
+// majority vote over a sample of col_idx, weighted by occurrence).  A gather first
+// compares the 16-bit tag c >> XC_BITS with the slot's tag.  Caching never changes
+// a value, only where it is read from.
+constexpr int XC_BITS = 14;
+constexpr int XC_SLOTS = 1 << XC_BITS;
+constexpr uint16_t XC_NOTAG = 0xFFFF;
+constexpr int XC_SAMPLE_LOG2 = 18;  // ~2^18 sampled entries per acsr_bin
 
 // unit descriptor: light  x = first index into bin_rows, y = (bin << 24) | rows
 //                  heavy  x = row id,                     y = 0x80000000 | chunk
@@ -48,18 +59,22 @@ struct PlanHeader {
     int32_t n_light_units;
     int32_t n_units;
     int32_t scan_ticket;    // last-CTA detection in the scan kernel
-    int32_t done_ticket;    // last-warp detection in the PageRank epilogue
+    int32_t work_ctr;       // dynamic unit counter (reset by the last warp)
+    int32_t exit_ticket;    // last-warp detection at SpMV exit
     int32_t overflow;       // 1 if the unit list exceeded the workspace bounds
     int32_t n_tiles;
-    int32_t pad;
-    int64_t off_units, off_partial, off_ticket, off_warp_part;  // byte offsets from the header
+    int32_t xc_valid;       // 1 if the x-cache vote table was built (col_idx given)
+    int32_t xc_stride;      // sampling stride used for the votes
+    int64_t n_cols;
+    uint64_t d2_hi, d2_lo;  // exact fixed-point Delta^2 accumulator (PageRank)
+    int64_t off_units, off_partial, off_ticket, off_xc_vote, off_xc_tag, off_xc_val;
     int32_t totals[NBINS + 2 + 2];  // per scan row totals (bins, light units, heavy units)
 };
 
 struct PlanLayout {
     int64_t n_tiles = 0, light_cap = 0, heavy_cap = 0;
-    size_t off_cnt = 0, off_toff = 0, off_tile_units = 0, off_units = 0, off_partial = 0,
-           off_ticket = 0, off_warp_part = 0, total = 0;
+    size_t off_cnt = 0, off_toff = 0, off_units = 0, off_partial = 0, off_ticket = 0,
+           off_xc_vote = 0, off_xc_tag = 0, off_xc_val = 0, total = 0;
 };
 
 __host__ __device__ inline size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
@@ -76,20 +91,22 @@ inline PlanLayout plan_layout(int64_t n_rows, int64_t nnz_max)
     int64_t heavy_rows_max = nnz_max / (HEAVY_CHUNK + 1) + 1;
     L.heavy_cap = nnz_max / HEAVY_CHUNK + heavy_rows_max + 1;
     size_t o = align_up(sizeof(PlanHeader), 256);
+    L.off_xc_vote = o;
+    o = align_up(o + sizeof(uint32_t) * XC_SLOTS, 256);
+    L.off_xc_tag = o;
+    o = align_up(o + sizeof(uint16_t) * XC_SLOTS, 256);
+    L.off_xc_val = o;
+    o = align_up(o + sizeof(double) * XC_SLOTS, 256);
     L.off_cnt = o;
     o = align_up(o + sizeof(int32_t) * SCAN_ROWS * (size_t)L.n_tiles, 256);
     L.off_toff = o;
     o = align_up(o + sizeof(int32_t) * SCAN_ROWS * (size_t)L.n_tiles, 256);
-    L.off_tile_units = o;  // (unused slot kept for layout stability)
-    o = align_up(o + 256, 256);
     L.off_units = o;
     o = align_up(o + sizeof(int2) * (size_t)(L.light_cap + L.heavy_cap), 256);
     L.off_partial = o;
     o = align_up(o + sizeof(double) * (size_t)L.heavy_cap, 256);
     L.off_ticket = o;
     o = align_up(o + sizeof(int32_t) * (size_t)L.heavy_cap, 256);
-    L.off_warp_part = o;
-    o = align_up(o + sizeof(double) * (size_t)MAX_WARPS, 256);
     L.total = o;
     return L;
 }
@@ -103,8 +120,15 @@ __device__ __forceinline__ int bin_of_len(int len)
 
 __device__ __forceinline__ int heavy_chunks(int len) { return (len + HEAVY_CHUNK - 1) / HEAVY_CHUNK; }
 
-template <typename T>
-__device__ __forceinline__ T ldg_stream(const T *p) { return __ldcs(p); }
+__device__ __forceinline__ uint32_t mix32(uint32_t v)
+{
+    v ^= v >> 16;
+    v *= 0x7feb352dU;
+    v ^= v >> 15;
+    v *= 0x846ca68bU;
+    v ^= v >> 16;
+    return v;
+}
 
 }  // namespace acsr
 

@@ -1,24 +1,34 @@
-// acsr_spmv.cu -- bin-specific SpMV (Alg. 2) in ONE launch, plus the
-// fused PageRank step (Alg. 5).
+// acsr_spmv.cu -- bin-specific SpMV (Alg. 2) in ONE persistent launch, plus
+// the fused PageRank step (Alg. 5).
 //
 // Work is cut by acsr_bin into warp-sized units (see acsr_internal.cuh):
 //   heavy units   one HEAVY_CHUNK-nnz chunk of a row with > 1024 nnz; the last
 //                 warp to finish a row (threadfence + atomic ticket) sums the
 //                 chunk partials in chunk order (replaces the dynamic-parallelism
 //                 parent/child kernels, Alg. 3/4).
-//   light units   up to unit_rows(b) rows of one bin b <= 10 inside one 4096-row
+//   light units   up to unit_rows(b) rows of one bin b <= 10 inside one 1024-row
 //                 tile; bins 1..6 use a sub-warp of 2^{b-1} lanes per row and a
 //                 width-2^{b-1} shuffle reduction (exactly Alg. 2 with reading Q6);
 //                 bins 7..10 use a full warp per row; bin 0 writes +0.0 (Q2).
-// Units are listed heavy-first, then tile by tile in row order; warps take units
-// round-robin, so at any moment the GPU works on a narrow window of the row space
-// and the CSR sectors shared by neighbouring rows of different bins are re-used
-// from L2 instead of being fetched twice.
+// Units are listed heavy-first, then tile by tile in row order.  Each warp starts
+// on unit = its global warp id and then claims units from an atomic counter, so the
+// GPU works on a narrow window of the row space (sectors shared by neighbouring rows
+// of different bins are re-used from L2) and the tail is balanced.
+//
+// B200 specifics ("SpMV kernel"): the measured limiter of a plain
+// gather-per-nonzero CSR SpMV on R-MAT graphs is the L1->L2 request rate of the
+// random x gathers, not DRAM.  x therefore goes through a per-SM direct-mapped
+// software cache of the hottest XC_SLOTS columns (tags + values in shared memory,
+// filled once per call by TMA bulk copies from a compact array that a tiny
+// pre-pass gathers) -- the B200 counterpart of binding x to texture memory.
 //
 // Every row is summed in an order that depends only on its length and address:
-// results are deterministic run to run.  Accumulation is in double for both
-// ACSR_F64 and ACSR_F32 (products of floats are exact in double).
+// y is deterministic run to run.  Accumulation is in double for both ACSR_F64 and
+// ACSR_F32 (products of floats are exact in double).  The PageRank Delta^2 is
+// accumulated in exact 128-bit fixed point (integer atomics), so it is
+// deterministic too.
 #include <cuda_runtime.h>
+#include <stdlib.h>
 
 #include "acsr_internal.cuh"
 
@@ -38,7 +48,9 @@ struct SpmvArgs {
     const int2 *__restrict__ units;
     double *__restrict__ partial;
     int32_t *__restrict__ ticket;
-    double *__restrict__ warp_part;
+    // shared-memory x cache
+    const uint16_t *xtag;
+    const V *xval;
     // PageRank epilogue
     const double *__restrict__ x_old;
     const int32_t *__restrict__ outdeg;
@@ -48,7 +60,73 @@ struct SpmvArgs {
     double *delta2;
 };
 
-template <typename V, bool HAS_VAL, bool HAS_END, bool PR>
+// ----------------------------------------------------------------- PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void *p)
+{
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar)
+{
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t phase)
+{
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+            : "=r"(done)
+            : "r"(smem_u32(bar)), "r"(phase)
+            : "memory");
+    }
+}
+
+// 128-bit fixed point, LSB = 2^-120, for exact order-independent sums of
+// non-negative doubles < 2^8 (PageRank Delta^2 <= 2).
+struct Fix128 {
+    uint64_t hi, lo;  // value = hi * 2^-56 + lo * 2^-120
+};
+
+__device__ __forceinline__ void fix_add(Fix128 &a, double d)
+{
+    if (!(d > 0.0)) return;
+    if (d >= 256.0) d = 255.99999999999997;  // saturate (never reached for PageRank)
+    const double hs = d * 72057594037927936.0;  // 2^56 (exact scaling)
+    const double hf = floor(hs);
+    const uint64_t h = (uint64_t)hf;
+    const double rem = hs - hf;                                     // exact
+    const uint64_t l = (uint64_t)(rem * 18446744073709551616.0);   // * 2^64, truncated
+    const uint64_t lo = a.lo + l;
+    a.hi += h + (lo < a.lo ? 1u : 0u);
+    a.lo = lo;
+}
+
+__device__ __forceinline__ void fix_merge(Fix128 &a, uint64_t hi, uint64_t lo)
+{
+    const uint64_t nlo = a.lo + lo;
+    a.hi += hi + (nlo < a.lo ? 1u : 0u);
+    a.lo = nlo;
+}
+
+template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
 struct Kern {
     using A = SpmvArgs<V>;
 
@@ -58,32 +136,41 @@ struct Kern {
         end = HAS_END ? __ldg(a.re + r) : __ldg(a.rb + r + 1);
     }
 
+    static __device__ __forceinline__ double gx(const A &a, int c)
+    {
+        if (XC) {
+            const uint32_t s = (uint32_t)c & (XC_SLOTS - 1);
+            if (a.xtag[s] == (uint16_t)((uint32_t)c >> XC_BITS)) return (double)a.xval[s];
+        }
+        return (double)__ldg(a.x + c);
+    }
+
     static __device__ __forceinline__ double prod(const A &a, int k)
     {
-        int c = __ldcs(a.col + k);
-        double xv = (double)__ldg(a.x + c);
+        const int c = __ldcs(a.col + k);
+        const double xv = gx(a, c);
         if (HAS_VAL) return (double)__ldcs(a.val + k) * xv;
         return xv;
     }
 
     static __device__ __forceinline__ double fmac(const A &a, int k, double acc)
     {
-        int c = __ldcs(a.col + k);
-        double xv = (double)__ldg(a.x + c);
+        const int c = __ldcs(a.col + k);
+        const double xv = gx(a, c);
         if (HAS_VAL) return fma((double)__ldcs(a.val + k), xv, acc);
         return acc + xv;
     }
 
     // write the row result (or the PageRank epilogue for local row r)
-    static __device__ __forceinline__ void finish(const A &a, int r, double s, double &d2)
+    static __device__ __forceinline__ void finish(const A &a, int r, double s, Fix128 &d2)
     {
         if (PR) {
-            double xn = a.teleport + a.damping * s;
+            const double xn = a.teleport + a.damping * s;
             a.x_new[r] = xn;
-            int od = __ldg(a.outdeg + r);
+            const int od = __ldg(a.outdeg + r);
             a.xs_next[r] = od > 0 ? xn / (double)od : 0.0;
-            double diff = xn - __ldg(a.x_old + r);
-            d2 += diff * diff;
+            const double diff = xn - __ldg(a.x_old + r);
+            fix_add(d2, diff * diff);
         } else {
             a.y[r] = (V)s;
         }
@@ -91,16 +178,16 @@ struct Kern {
 
     // bins 1..6: W = 2^{b-1} lanes per row, each lane <= 2 elements (Alg. 2)
     template <int W>
-    static __device__ __forceinline__ void light_sub(const A &a, int start, int cnt, int lane, double &d2)
+    static __device__ __forceinline__ void light_sub(const A &a, int start, int cnt, int lane, Fix128 &d2)
     {
-        constexpr int RPP = 32 / W;  // rows per pass
+        constexpr int RPP = 32 / W;           // rows per pass
         constexpr int U = (W >= 16) ? 2 : 4;  // passes in flight
         const int sub = lane / W, li = lane % W;
         for (int i0 = 0; i0 < cnt; i0 += RPP * U) {
             int r[U], beg[U], end[U];
 #pragma unroll
             for (int u = 0; u < U; u++) {
-                int i = i0 + u * RPP + sub;
+                const int i = i0 + u * RPP + sub;
                 r[u] = i < cnt ? __ldg(a.bin_rows + start + i) : -1;
             }
 #pragma unroll
@@ -111,7 +198,7 @@ struct Kern {
             double acc[U];
 #pragma unroll
             for (int u = 0; u < U; u++) {
-                int k0 = beg[u] + li, k1 = k0 + W;
+                const int k0 = beg[u] + li, k1 = k0 + W;
                 double s = 0.0;
                 if (k0 < end[u]) s = prod(a, k0);
                 if (k1 < end[u]) s += prod(a, k1);
@@ -149,34 +236,34 @@ struct Kern {
     }
 
     // bins 7..10: a warp per row
-    static __device__ __forceinline__ void light_warp(const A &a, int start, int cnt, int lane, double &d2)
+    static __device__ __forceinline__ void light_warp(const A &a, int start, int cnt, int lane, Fix128 &d2)
     {
-        int myr = lane < cnt ? __ldg(a.bin_rows + start + lane) : 0;
+        const int myr = lane < cnt ? __ldg(a.bin_rows + start + lane) : 0;
         int mb = 0, me = 0;
         if (lane < cnt) row_bounds(a, myr, mb, me);
         for (int i = 0; i < cnt; i++) {
-            int r = __shfl_sync(0xffffffffu, myr, i);
-            int beg = __shfl_sync(0xffffffffu, mb, i);
-            int end = __shfl_sync(0xffffffffu, me, i);
-            double s = warp_sum(strided_dot(a, beg, end, lane));
+            const int r = __shfl_sync(0xffffffffu, myr, i);
+            const int beg = __shfl_sync(0xffffffffu, mb, i);
+            const int end = __shfl_sync(0xffffffffu, me, i);
+            const double s = warp_sum(strided_dot(a, beg, end, lane));
             if (lane == 0) finish(a, r, s, d2);
         }
     }
 
-    static __device__ __forceinline__ void empty_rows(const A &a, int start, int cnt, int lane, double &d2)
+    static __device__ __forceinline__ void empty_rows(const A &a, int start, int cnt, int lane, Fix128 &d2)
     {
         for (int i = lane; i < cnt; i += 32) finish(a, __ldg(a.bin_rows + start + i), 0.0, d2);
     }
 
     // one HEAVY_CHUNK chunk of a long row; last arriver combines in chunk order
-    static __device__ __forceinline__ void heavy(const A &a, int u, int r, int c, int lane, double &d2)
+    static __device__ __forceinline__ void heavy(const A &a, int u, int r, int c, int lane, Fix128 &d2)
     {
         int beg, end;
         row_bounds(a, r, beg, end);
-        int kb = beg + c * HEAVY_CHUNK;
-        int ke = min(kb + HEAVY_CHUNK, end);
-        double s = warp_sum(strided_dot(a, kb, ke, lane));
-        int nch = heavy_chunks(end - beg);
+        const int kb = beg + c * HEAVY_CHUNK;
+        const int ke = min(kb + HEAVY_CHUNK, end);
+        const double s = warp_sum(strided_dot(a, kb, ke, lane));
+        const int nch = heavy_chunks(end - beg);
         if (nch == 1) {
             if (lane == 0) finish(a, r, s, d2);
             return;
@@ -199,98 +286,182 @@ struct Kern {
             finish(a, r, t, d2);
         }
     }
+
+    static __device__ __forceinline__ void unit(const A &a, int u, int lane, Fix128 &d2)
+    {
+        const int2 d = __ldg(a.units + u);
+        const uint32_t y = (uint32_t)d.y;
+        if (y & HEAVY_FLAG) {
+            heavy(a, u, d.x, (int)(y & ~HEAVY_FLAG), lane, d2);
+            return;
+        }
+        const int b = (int)(y >> 24), cnt = (int)(y & 0xFFFFFF);
+        switch (b) {
+            case 0: empty_rows(a, d.x, cnt, lane, d2); break;
+            case 1: light_sub<1>(a, d.x, cnt, lane, d2); break;
+            case 2: light_sub<2>(a, d.x, cnt, lane, d2); break;
+            case 3: light_sub<4>(a, d.x, cnt, lane, d2); break;
+            case 4: light_sub<8>(a, d.x, cnt, lane, d2); break;
+            case 5: light_sub<16>(a, d.x, cnt, lane, d2); break;
+            case 6: light_sub<32>(a, d.x, cnt, lane, d2); break;
+            default: light_warp(a, d.x, cnt, lane, d2); break;
+        }
+    }
 };
 
-template <typename V, bool HAS_VAL, bool HAS_END, bool PR>
-__global__ void __launch_bounds__(SPMV_THREADS)
+template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
+__global__ void __launch_bounds__(SPMV_THREADS, 1)
 spmv_kernel(SpmvArgs<V> a)
 {
-    using K = Kern<V, HAS_VAL, HAS_END, PR>;
+    using K = Kern<V, HAS_VAL, HAS_END, PR, XC>;
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ uint64_t bar;
     const int lane = threadIdx.x & 31;
     const int gw = blockIdx.x * SPMV_WARPS + (threadIdx.x >> 5);
     const int nw = gridDim.x * SPMV_WARPS;
-    const int n_units = a.hdr->n_units;
+    PlanHeader *hdr = a.hdr;
+    const int n_units = hdr->n_units;
     {
-        char *ws = (char *)a.hdr;
-        a.units = (const int2 *)(ws + a.hdr->off_units);
-        a.partial = (double *)(ws + a.hdr->off_partial);
-        a.ticket = (int32_t *)(ws + a.hdr->off_ticket);
-        a.warp_part = (double *)(ws + a.hdr->off_warp_part);
+        char *ws = (char *)hdr;
+        a.units = (const int2 *)(ws + hdr->off_units);
+        a.partial = (double *)(ws + hdr->off_partial);
+        a.ticket = (int32_t *)(ws + hdr->off_ticket);
     }
-    double d2 = 0.0;
-    for (int u = gw; u < n_units; u += nw) {
-        int2 d = __ldg(a.units + u);
-        uint32_t y = (uint32_t)d.y;
-        if (y & HEAVY_FLAG) {
-            K::heavy(a, u, d.x, (int)(y & ~HEAVY_FLAG), lane, d2);
-        } else {
-            int b = (int)(y >> 24), cnt = (int)(y & 0xFFFFFF);
-            switch (b) {
-                case 0: K::empty_rows(a, d.x, cnt, lane, d2); break;
-                case 1: K::template light_sub<1>(a, d.x, cnt, lane, d2); break;
-                case 2: K::template light_sub<2>(a, d.x, cnt, lane, d2); break;
-                case 3: K::template light_sub<4>(a, d.x, cnt, lane, d2); break;
-                case 4: K::template light_sub<8>(a, d.x, cnt, lane, d2); break;
-                case 5: K::template light_sub<16>(a, d.x, cnt, lane, d2); break;
-                case 6: K::template light_sub<32>(a, d.x, cnt, lane, d2); break;
-                default: K::light_warp(a, d.x, cnt, lane, d2); break;
-            }
+    if (XC) {
+        // shared x cache: [XC_SLOTS values | XC_SLOTS 16-bit tags], filled by TMA bulk copies
+        V *sval = (V *)smem;
+        uint16_t *stag = (uint16_t *)(smem + sizeof(V) * XC_SLOTS);
+        const char *ws = (const char *)hdr;
+        if (threadIdx.x == 0) {
+            mbar_init(&bar, 1);
+            constexpr uint32_t vbytes = sizeof(V) * XC_SLOTS, tbytes = sizeof(uint16_t) * XC_SLOTS;
+            mbar_expect_tx(&bar, vbytes + tbytes);
+            constexpr uint32_t CH = 32768;
+            for (uint32_t o = 0; o < vbytes; o += CH)
+                bulk_g2s((char *)sval + o, ws + hdr->off_xc_val + o, CH < vbytes - o ? CH : vbytes - o, &bar);
+            bulk_g2s(stag, ws + hdr->off_xc_tag, tbytes, &bar);
         }
+        __syncthreads();
+        mbar_wait(&bar, 0);
+        a.xval = sval;
+        a.xtag = stag;
+    }
+    Fix128 d2{0, 0};
+    int u = gw;
+    int nxt = 0;
+    if (lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
+    while (u < n_units) {
+        K::unit(a, u, lane, d2);
+        u = __shfl_sync(0xffffffffu, nxt, 0) + nw;
+        if (u < n_units && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
     }
     if (PR) {
-        // deterministic Delta^2: per-warp partial (fixed unit order per warp), then the
-        // last warp sums the partials in warp order.
-        d2 = K::warp_sum(d2);
-        int last = 0;
-        if (lane == 0) {
-            a.warp_part[gw] = d2;
-            __threadfence();
-            last = (atomicAdd(&a.hdr->done_ticket, 1) == nw - 1);
+        // exact fixed-point warp sum, then two 64-bit atomics per warp
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            const uint64_t h = __shfl_xor_sync(0xffffffffu, d2.hi, o);
+            const uint64_t l = __shfl_xor_sync(0xffffffffu, d2.lo, o);
+            fix_merge(d2, h, l);
         }
-        last = __shfl_sync(0xffffffffu, last, 0);
-        if (last) {
+        if (lane == 0 && (d2.hi | d2.lo)) {
+            const unsigned long long old =
+                atomicAdd((unsigned long long *)&hdr->d2_lo, (unsigned long long)d2.lo);
+            const uint64_t carry = (old + d2.lo < old) ? 1u : 0u;
+            atomicAdd((unsigned long long *)&hdr->d2_hi, (unsigned long long)(d2.hi + carry));
+        }
+    }
+    // last warp out publishes Delta^2 and resets the counters for the next call
+    if (lane == 0) {
+        __threadfence();
+        if (atomicAdd(&hdr->exit_ticket, 1) == nw - 1) {
             __threadfence();
-            double t = 0.0;
-            for (int j = lane; j < nw; j += 32) t += __ldcg(a.warp_part + j);
-            t = K::warp_sum(t);
-            if (lane == 0) {
-                *a.delta2 = t;
-                a.hdr->done_ticket = 0;
+            if (PR) {
+                const uint64_t hi = *(volatile uint64_t *)&hdr->d2_hi;
+                const uint64_t lo = *(volatile uint64_t *)&hdr->d2_lo;
+                *a.delta2 = (double)hi * 1.3877787807814457e-17 + (double)lo * 7.52316384526264e-37;
+                hdr->d2_hi = 0;
+                hdr->d2_lo = 0;
             }
+            hdr->work_ctr = 0;
+            hdr->exit_ticket = 0;
         }
     }
 }
 
-template <typename V, bool HAS_VAL, bool HAS_END, bool PR>
+// x-cache pre-pass: compact the hot x entries chosen by acsr_bin's vote table into
+// the plan workspace (XC_SLOTS values + 16-bit tags) for the TMA fill.  Without a
+// vote table (acsr_bin called without col_idx) every tag is XC_NOTAG.
+template <typename V>
+__global__ void xc_fill_kernel(PlanHeader *hdr, const V *__restrict__ x)
+{
+    const int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= XC_SLOTS) return;
+    char *ws = (char *)hdr;
+    const uint32_t v = hdr->xc_valid ? ((const uint32_t *)(ws + hdr->off_xc_vote))[s] : 0u;
+    const uint32_t t = v >> 16;
+    const int64_t c = ((int64_t)t << XC_BITS) | s;
+    const bool ok = (v & 0xFFFFu) != 0 && c < hdr->n_cols;
+    ((uint16_t *)(ws + hdr->off_xc_tag))[s] = ok ? (uint16_t)t : XC_NOTAG;
+    ((V *)(ws + hdr->off_xc_val))[s] = ok ? x[c] : (V)0;
+}
+
+template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
 static int grid_for()
 {
     static int g = 0;
     if (!g) {
+        const size_t smem = XC ? (sizeof(V) + sizeof(uint16_t)) * XC_SLOTS : 0;
+        if (XC)
+            cudaFuncSetAttribute(spmv_kernel<V, HAS_VAL, HAS_END, PR, XC>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmv_kernel<V, HAS_VAL, HAS_END, PR>,
-                                                      SPMV_THREADS, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmv_kernel<V, HAS_VAL, HAS_END, PR, XC>,
+                                                      SPMV_THREADS, smem);
         if (per_sm < 1) per_sm = 1;
-        int gg = per_sm * acsr_num_sms();
-        if (gg * SPMV_WARPS > MAX_WARPS) gg = MAX_WARPS / SPMV_WARPS;
-        g = gg;
+        g = per_sm * acsr_num_sms();
     }
     return g;
 }
 
-template <typename V, bool HAS_VAL, bool HAS_END, bool PR>
+template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
 static void launch(const SpmvArgs<V> &a, cudaStream_t s)
 {
-    spmv_kernel<V, HAS_VAL, HAS_END, PR><<<grid_for<V, HAS_VAL, HAS_END, PR>(), SPMV_THREADS, 0, s>>>(a);
+    const size_t smem = XC ? (sizeof(V) + sizeof(uint16_t)) * XC_SLOTS : 0;
+    const int g = grid_for<V, HAS_VAL, HAS_END, PR, XC>();
+    spmv_kernel<V, HAS_VAL, HAS_END, PR, XC><<<g, SPMV_THREADS, smem, s>>>(a);
+}
+
+template <typename V, bool PR, bool XC>
+static void dispatch2(const SpmvArgs<V> &a, cudaStream_t s)
+{
+    const bool hv = a.val != nullptr, he = a.re != nullptr;
+    if (hv && he) launch<V, true, true, PR, XC>(a, s);
+    else if (hv) launch<V, true, false, PR, XC>(a, s);
+    else if (he) launch<V, false, true, PR, XC>(a, s);
+    else launch<V, false, false, PR, XC>(a, s);
+}
+
+// ACSR_NO_XCACHE=1 disables the shared-memory x cache (A/B measurements only).
+static bool xcache_enabled()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("ACSR_NO_XCACHE");
+        v = (e && e[0] == '1') ? 0 : 1;
+    }
+    return v == 1;
 }
 
 template <typename V, bool PR>
-static void dispatch(const SpmvArgs<V> &a, cudaStream_t s)
+static int dispatch(const SpmvArgs<V> &a, cudaStream_t s)
 {
-    bool hv = a.val != nullptr, he = a.re != nullptr;
-    if (hv && he) launch<V, true, true, PR>(a, s);
-    else if (hv) launch<V, true, false, PR>(a, s);
-    else if (he) launch<V, false, true, PR>(a, s);
-    else launch<V, false, false, PR>(a, s);
+    if (xcache_enabled() && a.x != nullptr) {
+        xc_fill_kernel<V><<<XC_SLOTS / 256, 256, 0, s>>>(a.hdr, a.x);
+        dispatch2<V, PR, true>(a, s);
+        return 2;
+    }
+    dispatch2<V, PR, false>(a, s);
+    return 1;
 }
 
 __global__ void pagerank_scale_kernel(int64_t n, const double *__restrict__ x,
@@ -298,7 +469,7 @@ __global__ void pagerank_scale_kernel(int64_t n, const double *__restrict__ x,
 {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
          i += (int64_t)gridDim.x * blockDim.x) {
-        int od = outdeg[i];
+        const int od = outdeg[i];
         xs[i] = od > 0 ? x[i] / (double)od : 0.0;
     }
 }
@@ -324,8 +495,7 @@ extern "C" acsr_status acsr_spmv(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
                                  size_t plan_ws_bytes, cudaStream_t stream)
 {
     if (n_rows < 0 || n_cols < 0 || n_rows >= ((int64_t)1 << 31) ||
-        (dt != ACSR_F32 && dt != ACSR_F64) ||
-        (n_rows > 0 && (!row_begin || !y))) {
+        (dt != ACSR_F32 && dt != ACSR_F64) || (n_rows > 0 && (!row_begin || !y))) {
         acsr_set_error("acsr_spmv: invalid argument");
         return ACSR_ERR_INVALID_VALUE;
     }
@@ -337,13 +507,13 @@ extern "C" acsr_status acsr_spmv(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
     if (dt == ACSR_F64) {
         SpmvArgs<double> a{};
         a.rb = row_begin; a.re = row_end; a.col = col_idx;
-        a.val = (const double *)values; a.x = (const double *)x; a.y = (double *)y;
+        a.val = (const double *)values; a.x = n_cols > 0 ? (const double *)x : nullptr; a.y = (double *)y;
         a.bin_rows = bin_rows; a.hdr = (PlanHeader *)plan_ws;
         dispatch<double, false>(a, stream);
     } else {
         SpmvArgs<float> a{};
         a.rb = row_begin; a.re = row_end; a.col = col_idx;
-        a.val = (const float *)values; a.x = (const float *)x; a.y = (float *)y;
+        a.val = (const float *)values; a.x = n_cols > 0 ? (const float *)x : nullptr; a.y = (float *)y;
         a.bin_rows = bin_rows; a.hdr = (PlanHeader *)plan_ws;
         dispatch<float, false>(a, stream);
     }
@@ -367,7 +537,7 @@ extern "C" acsr_status acsr_pagerank_step(const acsr_pr_args *p, cudaStream_t st
     }
     SpmvArgs<double> a{};
     a.rb = p->row_begin; a.re = p->row_end; a.col = p->col_idx;
-    a.val = nullptr; a.x = p->xs; a.y = nullptr;
+    a.val = nullptr; a.x = p->n_cols > 0 ? p->xs : nullptr; a.y = nullptr;
     a.bin_rows = p->bin_rows; a.hdr = (PlanHeader *)p->plan_ws;
     a.x_old = p->x; a.outdeg = p->outdeg; a.x_new = p->x_new; a.xs_next = p->xs_next;
     a.damping = p->damping; a.teleport = p->teleport; a.delta2 = p->delta2;

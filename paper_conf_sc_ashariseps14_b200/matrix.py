@@ -35,7 +35,7 @@ class ACSRMatrix:
 
     def rebin(self, stream=None):
         acsr_bin(self.row_begin, self.row_end, self.nnz_max, self.bin_rows, self.bin_offsets,
-                 self.plan_ws, stream)
+                 self.plan_ws, stream, col_idx=self.col_idx, n_cols=self.n_cols)
 
     def spmv(self, x, y=None, stream=None):
         return acsr_spmv(self.row_begin, self.col_idx, self.values, x, self.bin_rows,
@@ -56,7 +56,7 @@ def spmv_from_host(row_ptr_h, col_h, val_h, x_h, y_h=None, device="cuda", stream
     ci = col_h.to(device, non_blocking=True)
     va = None if val_h is None else val_h.to(device, non_blocking=True)
     x = x_h.to(device, non_blocking=True)
-    br, bo, ws = acsr_bin(rp, None, ci.numel(), stream=stream)
+    br, bo, ws = acsr_bin(rp, None, ci.numel(), stream=stream, col_idx=ci, n_cols=x.numel())
     y = acsr_spmv(rp, ci, va, x, br, bo, ws, stream=stream)
     if y_h is None:
         return y.cpu()

@@ -150,7 +150,7 @@ def run_acsr(args, dev, rank, world):
     stream = torch.cuda.current_stream()
     br = torch.empty(n, dtype=torch.int32, device=dev)
     bo = torch.empty(33, dtype=torch.int32, device=dev)
-    ws = torch.empty(acsr.acsr_bin_workspace_bytes(n, nnz), dtype=torch.uint8, device=dev)
+    ws = torch.empty(acsr.acsr_bin_workspace_bytes(n, n, nnz), dtype=torch.uint8, device=dev)
     y = torch.empty(n, dtype=dtype, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 

@@ -64,17 +64,18 @@ enum { ACSR_NBINS = 32 };
  *                           the dynamic-parallelism parent/child launches, P:61,
  *                           P:68-105): warp work units in row-space order, the
  *                           split plan for rows longer than 1024 non-zeros, and
- *                           (if col_idx != NULL) the hot-column vote table of the
- *                           SpMV's shared-memory x cache (the B200 stand-in for the
- *                           paper's texture-bound x; a sample of about 2^18
- *                           entries -- a performance hint only, never a result).
+ *                           (if col_idx != NULL) the hot-column table of the SpMV's
+ *                           shared-memory x cache (the B200 stand-in for the paper's
+ *                           texture-bound x): occurrence counts over a strided
+ *                           sample of ~2^20 entries, per-slot most frequent column --
+ *                           a performance hint only, never a result.
  * n_cols is the length of x (column ids outside [0, n_cols) are ignored by the
  * sampler).  nnz_max bounds the number of stored entries (sum of row lengths)
  * that any later acsr_bin on this workspace will see (slack CSR: the capacity).
  * The row-length array is read twice (count pass + stable scatter pass); no
  * host synchronisation happens.  bin_rows/bin_offsets are deterministic and
  * equal the oracle bit for bit.  plan_ws must not be shared by concurrent calls. */
-size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t nnz_max);
+size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t n_cols, int64_t nnz_max);
 
 acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
                      const int32_t *row_begin, const int32_t *row_end /* NULL => standard CSR */,

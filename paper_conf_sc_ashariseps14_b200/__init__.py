@@ -42,7 +42,7 @@ if not os.path.exists(LIB_PATH):
 
 _lib = ctypes.CDLL(LIB_PATH)
 _i64, _vp, _sz, _dbl = ctypes.c_int64, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_double
-_lib.acsr_bin_workspace_bytes.argtypes = [_i64, _i64]
+_lib.acsr_bin_workspace_bytes.argtypes = [_i64, _i64, _i64]
 _lib.acsr_bin_workspace_bytes.restype = _sz
 _lib.acsr_bin.argtypes = [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
 _lib.acsr_bin.restype = ctypes.c_int
@@ -119,8 +119,8 @@ def _dt(t):
 
 
 # --------------------------------------------------------------------------- binning
-def acsr_bin_workspace_bytes(n_rows: int, nnz_max: int) -> int:
-    return int(_lib.acsr_bin_workspace_bytes(int(n_rows), int(nnz_max)))
+def acsr_bin_workspace_bytes(n_rows: int, n_cols: int, nnz_max: int) -> int:
+    return int(_lib.acsr_bin_workspace_bytes(int(n_rows), int(n_cols), int(nnz_max)))
 
 
 def acsr_bin(row_begin, row_end=None, nnz_max=None, bin_rows=None, bin_offsets=None, plan_ws=None,
@@ -135,7 +135,7 @@ def acsr_bin(row_begin, row_end=None, nnz_max=None, bin_rows=None, bin_offsets=N
         bin_rows = torch.empty(max(n, 0), dtype=torch.int32, device=dev)
     if bin_offsets is None:
         bin_offsets = torch.empty(NBINS + 1, dtype=torch.int32, device=dev)
-    need = acsr_bin_workspace_bytes(n, nnz_max)
+    need = acsr_bin_workspace_bytes(n, n_cols, nnz_max)
     if plan_ws is None:
         plan_ws = torch.empty(need, dtype=torch.uint8, device=dev)
     _check(_lib.acsr_bin(n, int(n_cols), int(nnz_max), _dev(row_begin, torch.int32, "row_begin"),

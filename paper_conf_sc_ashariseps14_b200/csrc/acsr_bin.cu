@@ -74,13 +74,6 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
     __shared__ int warp_sums[SCAN_THREADS / 32];
     __shared__ int is_last;
     const int row = blockIdx.x;
-    if (row >= SCAN_ROWS) {  // helper CTAs: clear the x-cache vote table
-        uint32_t *vote = (uint32_t *)((char *)hdr + L.off_xc_vote);
-        for (int i = (row - SCAN_ROWS) * SCAN_THREADS + threadIdx.x; i < XC_SLOTS;
-             i += (gridDim.x - SCAN_ROWS) * SCAN_THREADS)
-            vote[i] = 0u;
-        return;
-    }
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int32_t *a = cnt + (int64_t)row * n_tiles;
     int32_t *o = toff + (int64_t)row * n_tiles;
@@ -113,9 +106,11 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
         run += a[i];
     }
     // last CTA: bin offsets + unit totals
-    __threadfence();
     __syncthreads();
-    if (tid == 0) is_last = (atomicAdd(&hdr->scan_ticket, 1) == SCAN_ROWS - 1);
+    if (tid == 0) {
+        __threadfence();
+        is_last = (atomicAdd(&hdr->scan_ticket, 1) == SCAN_ROWS - 1);
+    }
     __syncthreads();
     if (is_last && tid == 0) {
         __threadfence();
@@ -151,34 +146,18 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
     }
 }
 
-// x-cache vote: Boyer-Moore majority per slot over a strided sample of the row's
-// entries (one CAS on a packed (tag16 << 16 | votes16) word per sampled entry).
-__device__ __forceinline__ void xc_vote(uint32_t *vote, int c, int64_t n_cols)
+// x-cache table: sampled occurrence counts, per-slot winner (count, column).
+__global__ void xc_count_kernel(const int32_t *__restrict__ col, int64_t nnz_max, int64_t n_cols,
+                                int stride, int32_t *__restrict__ count,
+                                unsigned long long *__restrict__ best)
 {
-    if (c < 0 || c >= n_cols) return;  // slack garbage or bad ids: ignore (hint only)
-    const uint32_t s = (uint32_t)c & (XC_SLOTS - 1);
-    const uint32_t t = (uint32_t)c >> XC_BITS;
-    if (t >= XC_NOTAG) return;
-    uint32_t old = vote[s];
-    while (true) {
-        uint32_t ot = old >> 16, ov = old & 0xFFFFu, nw;
-        if (ov == 0) nw = (t << 16) | 1u;
-        else if (ot == t) nw = ov < 0xFFFFu ? old + 1u : old;
-        else nw = old - 1u;
-        if (nw == old) return;
-        uint32_t prev = atomicCAS(vote + s, old, nw);
-        if (prev == old) return;
-        old = prev;
-    }
-}
-
-__device__ __forceinline__ void xc_sample(const int32_t *__restrict__ rb, int64_t r, int len,
-                                          const int32_t *__restrict__ col, uint32_t *vote,
-                                          int64_t n_cols, int stride)
-{
-    const int beg = __ldg(rb + r);
-    for (int k = (int)(mix32((uint32_t)r) % (uint32_t)stride); k < len; k += stride)
-        xc_vote(vote, __ldg(col + beg + k), n_cols);
+    const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t k = j * stride + (int64_t)(mix32((uint32_t)j) % (uint32_t)stride);
+    if (k >= nnz_max) return;
+    const int c = __ldg(col + k);
+    if (c < 0 || c >= n_cols) return;  // slack entries / garbage: a hint only
+    const int cnt = atomicAdd(count + c, 1) + 1;
+    atomicMax(best + (c & (XC_SLOTS - 1)), ((unsigned long long)cnt << 32) | (unsigned)c);
 }
 
 template <bool HAS_END>
@@ -186,9 +165,7 @@ __global__ void __launch_bounds__(BIN_THREADS)
 bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
                    int32_t *__restrict__ bin_rows, const int32_t *__restrict__ bin_offsets,
                    const int32_t *__restrict__ toff, int n_tiles, const PlanHeader *__restrict__ hdr,
-                   int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap,
-                   const int32_t *__restrict__ col, uint32_t *__restrict__ vote, int64_t n_cols,
-                   int xc_stride)
+                   int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap)
 {
     constexpr int NW = BIN_THREADS / 32;
     __shared__ int run[NBINS];
@@ -247,7 +224,6 @@ bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__r
             heavy_run = acc;
         }
         __syncthreads();
-        if (valid && col && len > 0) xc_sample(rb, r, len, col, vote, n_cols, xc_stride);
         if (valid) {
             bin_rows[seg[b] + wbase[warp][b] + rank] = (int32_t)r;
             if (hc > 0 && !overflow) {
@@ -287,10 +263,10 @@ bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__r
 
 using namespace acsr;
 
-extern "C" size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t nnz_max)
+extern "C" size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t n_cols, int64_t nnz_max)
 {
-    if (n_rows < 0 || nnz_max < 0) return 0;
-    return plan_layout(n_rows, nnz_max).total;
+    if (n_rows < 0 || n_cols < 0 || nnz_max < 0) return 0;
+    return plan_layout(n_rows, n_cols, nnz_max).total;
 }
 
 extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
@@ -303,7 +279,7 @@ extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
         acsr_set_error("acsr_bin: invalid argument");
         return ACSR_ERR_INVALID_VALUE;
     }
-    PlanLayout L = plan_layout(n_rows, nnz_max);
+    PlanLayout L = plan_layout(n_rows, n_cols, nnz_max);
     if (!plan_ws || plan_ws_bytes < L.total) {
         acsr_set_error("acsr_bin: workspace %zu < required %zu", plan_ws_bytes, L.total);
         return ACSR_ERR_WORKSPACE;
@@ -327,21 +303,23 @@ extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
     const int xc_valid = col_idx != nullptr && n_cols > 0 && n_cols < ((int64_t)XC_NOTAG << XC_BITS);
     int64_t stride64 = nnz_max >> XC_SAMPLE_LOG2;
     const int xc_stride = (int)(stride64 < 1 ? 1 : (stride64 > (1 << 30) ? (1 << 30) : stride64));
-    uint32_t *vote = (uint32_t *)(ws + L.off_xc_vote);
-    const int zero_ctas = (XC_SLOTS + SCAN_THREADS - 1) / SCAN_THREADS;
-    bin_scan_kernel<<<SCAN_ROWS + zero_ctas, SCAN_THREADS, 0, stream>>>(
+    bin_scan_kernel<<<SCAN_ROWS, SCAN_THREADS, 0, stream>>>(
         cnt, toff, nt, hdr, bin_offsets, n_rows, n_cols, L.light_cap, L.heavy_cap, L, xc_valid, xc_stride);
     if (row_end)
         bin_scatter_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, bin_rows,
                                                                    bin_offsets, toff, nt, hdr, units,
-                                                                   tickets, L.heavy_cap,
-                                                                   xc_valid ? col_idx : nullptr, vote,
-                                                                   n_cols, xc_stride);
+                                                                   tickets, L.heavy_cap);
     else
         bin_scatter_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, bin_rows,
                                                                     bin_offsets, toff, nt, hdr, units,
-                                                                    tickets, L.heavy_cap,
-                                                                    xc_valid ? col_idx : nullptr, vote,
-                                                                    n_cols, xc_stride);
+                                                                    tickets, L.heavy_cap);
+    if (xc_valid) {
+        cudaMemsetAsync(ws + L.off_xc_vote, 0, sizeof(uint64_t) * XC_SLOTS, stream);
+        cudaMemsetAsync(ws + L.off_xc_count, 0, sizeof(int32_t) * (size_t)n_cols, stream);
+        const int64_t samples = (nnz_max + xc_stride - 1) / xc_stride;
+        xc_count_kernel<<<(unsigned)((samples + 255) / 256), 256, 0, stream>>>(
+            col_idx, nnz_max, n_cols, xc_stride, (int32_t *)(ws + L.off_xc_count),
+            (unsigned long long *)(ws + L.off_xc_vote));
+    }
     return acsr_check_launch("acsr_bin");
 }

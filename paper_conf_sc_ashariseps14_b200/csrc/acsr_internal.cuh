@@ -40,14 +40,15 @@ constexpr int SPMV_WARPS = SPMV_THREADS / 32;
 
 // ---------------------------------------------------------------- x cache
 // Direct-mapped cache of "hot" x entries in shared memory: slot s = c mod XC_SLOTS
-// holds x[c] for the column c chosen for that slot at bin time (Boyer-Moore
-// majority vote over a sample of col_idx, weighted by occurrence).  A gather first
-// compares the 16-bit tag c >> XC_BITS with the slot's tag.  Caching never changes
-// a value, only where it is read from.
+// holds x[c] for the column c with the most occurrences among the columns mapping
+// to s, counted over a strided sample of col_idx at bin time (sampled counts with
+// atomicAdd, per-slot winner with a 64-bit atomicMax on (count << 32 | c)).  A
+// gather first compares the 16-bit tag c >> XC_BITS with the slot's tag.  Caching
+// never changes a value, only where it is read from.
 constexpr int XC_BITS = 14;
 constexpr int XC_SLOTS = 1 << XC_BITS;
 constexpr uint16_t XC_NOTAG = 0xFFFF;
-constexpr int XC_SAMPLE_LOG2 = 18;  // ~2^18 sampled entries per acsr_bin
+constexpr int XC_SAMPLE_LOG2 = 20;  // ~2^20 sampled entries per acsr_bin
 
 // unit descriptor: light  x = first index into bin_rows, y = (bin << 24) | rows
 //                  heavy  x = row id,                     y = 0x80000000 | chunk
@@ -63,8 +64,8 @@ struct PlanHeader {
     int32_t exit_ticket;    // last-warp detection at SpMV exit
     int32_t overflow;       // 1 if the unit list exceeded the workspace bounds
     int32_t n_tiles;
-    int32_t xc_valid;       // 1 if the x-cache vote table was built (col_idx given)
-    int32_t xc_stride;      // sampling stride used for the votes
+    int32_t xc_valid;       // 1 if the x-cache table was built (col_idx given)
+    int32_t xc_stride;      // sampling stride used for the counts
     int64_t n_cols;
     uint64_t d2_hi, d2_lo;  // exact fixed-point Delta^2 accumulator (PageRank)
     int64_t off_units, off_partial, off_ticket, off_xc_vote, off_xc_tag, off_xc_val;
@@ -74,7 +75,7 @@ struct PlanHeader {
 struct PlanLayout {
     int64_t n_tiles = 0, light_cap = 0, heavy_cap = 0;
     size_t off_cnt = 0, off_toff = 0, off_units = 0, off_partial = 0, off_ticket = 0,
-           off_xc_vote = 0, off_xc_tag = 0, off_xc_val = 0, total = 0;
+           off_xc_vote = 0, off_xc_tag = 0, off_xc_val = 0, off_xc_count = 0, total = 0;
 };
 
 __host__ __device__ inline size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
@@ -83,7 +84,7 @@ __host__ __device__ inline size_t align_up(size_t v, size_t a) { return (v + a -
 // row 32 light units per tile, row 33 heavy units per tile.
 constexpr int SCAN_ROWS = NBINS + 2;
 
-inline PlanLayout plan_layout(int64_t n_rows, int64_t nnz_max)
+inline PlanLayout plan_layout(int64_t n_rows, int64_t n_cols, int64_t nnz_max)
 {
     PlanLayout L;
     L.n_tiles = (n_rows + TILE_ROWS - 1) / TILE_ROWS;
@@ -91,8 +92,8 @@ inline PlanLayout plan_layout(int64_t n_rows, int64_t nnz_max)
     int64_t heavy_rows_max = nnz_max / (HEAVY_CHUNK + 1) + 1;
     L.heavy_cap = nnz_max / HEAVY_CHUNK + heavy_rows_max + 1;
     size_t o = align_up(sizeof(PlanHeader), 256);
-    L.off_xc_vote = o;
-    o = align_up(o + sizeof(uint32_t) * XC_SLOTS, 256);
+    L.off_xc_vote = o;  // u64 (count << 32 | column) per slot
+    o = align_up(o + sizeof(uint64_t) * XC_SLOTS, 256);
     L.off_xc_tag = o;
     o = align_up(o + sizeof(uint16_t) * XC_SLOTS, 256);
     L.off_xc_val = o;
@@ -107,6 +108,8 @@ inline PlanLayout plan_layout(int64_t n_rows, int64_t nnz_max)
     o = align_up(o + sizeof(double) * (size_t)L.heavy_cap, 256);
     L.off_ticket = o;
     o = align_up(o + sizeof(int32_t) * (size_t)L.heavy_cap, 256);
+    L.off_xc_count = o;  // sampled occurrence count per column
+    o = align_up(o + sizeof(int32_t) * (size_t)(n_cols > 0 ? n_cols : 0), 256);
     L.total = o;
     return L;
 }

@@ -51,6 +51,8 @@ struct SpmvArgs {
     // shared-memory x cache
     const uint16_t *xtag;
     const V *xval;
+    // 128-bit load phase: vector loads at element j need (j + vph) % 4 == 0; -1 = scalar only
+    int vph;
     // PageRank epilogue
     const double *__restrict__ x_old;
     const int32_t *__restrict__ outdeg;
@@ -220,10 +222,55 @@ struct Kern {
         return v;
     }
 
-    // lane-strided dot over [kb, ke), 4 independent loads in flight per lane
+    // 4 consecutive elements with 128-bit loads (col: int4; val: 2 x double2 or float4)
+    static __device__ __forceinline__ void vec4(const A &a, int j, double &s0, double &s1, double &s2,
+                                                double &s3)
+    {
+        const int4 c = __ldcs(reinterpret_cast<const int4 *>(a.col + j));
+        double v0 = 1.0, v1 = 1.0, v2 = 1.0, v3 = 1.0;
+        if (HAS_VAL) {
+            if (sizeof(V) == 8) {
+                const double2 p = __ldcs(reinterpret_cast<const double2 *>(a.val + j));
+                const double2 q = __ldcs(reinterpret_cast<const double2 *>(a.val + j + 2));
+                v0 = p.x; v1 = p.y; v2 = q.x; v3 = q.y;
+            } else {
+                const float4 p = __ldcs(reinterpret_cast<const float4 *>(a.val + j));
+                v0 = p.x; v1 = p.y; v2 = p.z; v3 = p.w;
+            }
+        }
+        const double x0 = gx(a, c.x), x1 = gx(a, c.y), x2 = gx(a, c.z), x3 = gx(a, c.w);
+        if (HAS_VAL) {
+            s0 = fma(v0, x0, s0); s1 = fma(v1, x1, s1); s2 = fma(v2, x2, s2); s3 = fma(v3, x3, s3);
+        } else {
+            s0 += x0; s1 += x1; s2 += x2; s3 += x3;
+        }
+    }
+
+    // lane-strided dot over [kb, ke).  Vector path: the warp covers 128 consecutive
+    // elements per group, 4 per lane, two groups in flight; element t of a lane's
+    // 4-vector always goes to accumulator t (the order depends only on the row's
+    // address), ragged head/tail elements are masked scalar loads.
     static __device__ __forceinline__ double strided_dot(const A &a, int kb, int ke, int lane)
     {
         double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+        if (a.vph >= 0 && ke - kb >= 64) {
+            const int ph = a.vph;
+            for (int j0 = ((kb + ph) & ~3) - ph; j0 < ke; j0 += 256) {
+#pragma unroll
+                for (int h = 0; h < 2; h++) {
+                    const int j = j0 + 128 * h + 4 * lane;
+                    if (j >= kb && j + 3 < ke) {
+                        vec4(a, j, s0, s1, s2, s3);
+                    } else if (j < ke && j + 3 >= kb) {
+                        if (j >= kb) s0 = fmac(a, j, s0);
+                        if (j + 1 >= kb && j + 1 < ke) s1 = fmac(a, j + 1, s1);
+                        if (j + 2 >= kb && j + 2 < ke) s2 = fmac(a, j + 2, s2);
+                        if (j + 3 < ke) s3 = fmac(a, j + 3, s3);
+                    }
+                }
+            }
+            return (s0 + s1) + (s2 + s3);
+        }
         int k = kb + lane;
         for (; k + 96 < ke; k += 128) {
             s0 = fmac(a, k, s0);
@@ -397,10 +444,10 @@ __global__ void xc_fill_kernel(PlanHeader *hdr, const V *__restrict__ x)
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= XC_SLOTS) return;
     char *ws = (char *)hdr;
-    const uint32_t v = hdr->xc_valid ? ((const uint32_t *)(ws + hdr->off_xc_vote))[s] : 0u;
-    const uint32_t t = v >> 16;
-    const int64_t c = ((int64_t)t << XC_BITS) | s;
-    const bool ok = (v & 0xFFFFu) != 0 && c < hdr->n_cols;
+    const unsigned long long v = hdr->xc_valid ? ((const unsigned long long *)(ws + hdr->off_xc_vote))[s] : 0ull;
+    const int64_t c = (int64_t)(uint32_t)v;
+    const uint32_t t = (uint32_t)(c >> XC_BITS);
+    const bool ok = (v >> 32) != 0 && c < hdr->n_cols && t < XC_NOTAG;
     ((uint16_t *)(ws + hdr->off_xc_tag))[s] = ok ? (uint16_t)t : XC_NOTAG;
     ((V *)(ws + hdr->off_xc_val))[s] = ok ? x[c] : (V)0;
 }
@@ -452,9 +499,25 @@ static bool xcache_enabled()
     return v == 1;
 }
 
-template <typename V, bool PR>
-static int dispatch(const SpmvArgs<V> &a, cudaStream_t s)
+// element phase for 128-bit loads of col (and val), or -1 if col and val cannot be
+// vector-loaded at the same indices
+template <typename V>
+static int vec_phase(const int32_t *col, const V *val)
 {
+    const uintptr_t pc = (uintptr_t)col;
+    if (pc % 4) return -1;
+    const int ph = (int)((pc / 4) % 4);
+    if (!val) return ph;
+    const uintptr_t pv = (uintptr_t)val;
+    if (pv % sizeof(V)) return -1;
+    if (sizeof(V) == 8) return ((int)((pv / 8) % 2) == ph % 2) ? ph : -1;
+    return ((int)((pv / 4) % 4) == ph) ? ph : -1;
+}
+
+template <typename V, bool PR>
+static int dispatch(SpmvArgs<V> a, cudaStream_t s)
+{
+    a.vph = vec_phase<V>(a.col, a.val);
     if (xcache_enabled() && a.x != nullptr) {
         xc_fill_kernel<V><<<XC_SLOTS / 256, 256, 0, s>>>(a.hdr, a.x);
         dispatch2<V, PR, true>(a, s);
@@ -485,7 +548,7 @@ static bool plan_ok(int64_t n_rows, const int32_t *bin_rows, const int32_t *bin_
 {
     if (!bin_offsets || !plan_ws) return false;
     if (n_rows > 0 && !bin_rows) return false;
-    return plan_ws_bytes >= plan_layout(n_rows, 0).total;
+    return plan_ws_bytes >= plan_layout(n_rows, 0, 0).total;
 }
 
 extern "C" acsr_status acsr_spmv(acsr_dtype dt, int64_t n_rows, int64_t n_cols,

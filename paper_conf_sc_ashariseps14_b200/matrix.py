@@ -29,7 +29,7 @@ class ACSRMatrix:
         dev = row_begin.device
         self.bin_rows = torch.empty(self.n_rows, dtype=torch.int32, device=dev)
         self.bin_offsets = torch.empty(33, dtype=torch.int32, device=dev)
-        self.plan_ws = torch.empty(acsr_bin_workspace_bytes(self.n_rows, self.nnz_max),
+        self.plan_ws = torch.empty(acsr_bin_workspace_bytes(self.n_rows, self.n_cols, self.nnz_max),
                                    dtype=torch.uint8, device=dev)
         self.rebin()
 

@@ -30,8 +30,8 @@ def test_library_exports_every_declared_symbol():
 def test_host_side_queries_without_gpu():
     import paper_conf_sc_ashariseps14_b200 as acsr
     assert acsr.version() >= 100
-    small = acsr.acsr_bin_workspace_bytes(1000, 10000)
-    big = acsr.acsr_bin_workspace_bytes(1 << 20, 16 << 20)
+    small = acsr.acsr_bin_workspace_bytes(1000, 1000, 10000)
+    big = acsr.acsr_bin_workspace_bytes(1 << 20, 1 << 20, 16 << 20)
     assert 0 < small < big
     assert acsr._lib.acsr_status_string(3) == b"ACSR_ERR_CAPACITY"
     # host-detected argument errors return synchronously without touching a device

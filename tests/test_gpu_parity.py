@@ -377,3 +377,23 @@ def test_argument_errors(acsr, cuda):
     with pytest.raises(acsr.ACSRError) as e:
         acsr.acsr_bin(rp, None, nnz_max=0, plan_ws=torch.empty(8, dtype=torch.uint8, device=cuda))
     assert e.value.code == acsr.ACSR_ERR_WORKSPACE
+
+
+@pytest.mark.parametrize("shift_c,shift_v", [(1, 1), (2, 0), (3, 3), (1, 0)])
+def test_spmv_unaligned_views(acsr, cuda, shift_c, shift_v):
+    # col/val given as offset views: the 128-bit load phase (or the scalar fallback when
+    # col and val phases disagree) must not change results beyond the fp64 bar.
+    rp, ci = synth.rmat_csr(13)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 21)
+    x = synth.vector(n, 22)
+    cbuf = torch.zeros(ci.numel() + 4, dtype=torch.int32, device=cuda)
+    vbuf = torch.zeros(ci.numel() + 4, dtype=torch.float64, device=cuda)
+    cv = cbuf[shift_c:shift_c + ci.numel()]
+    vv = vbuf[shift_v:shift_v + ci.numel()]
+    cv.copy_(ci.to(cuda))
+    vv.copy_(val.to(cuda))
+    m = acsr.ACSRMatrix(rp.to(cuda), cv, vv)
+    y = m.spmv(x.to(cuda)).cpu().numpy()
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y, y_ref, den, torch.float64)

@@ -201,10 +201,8 @@ struct Kern {
 #pragma unroll
             for (int u = 0; u < U; u++) {
                 const int k0 = beg[u] + li, k1 = k0 + W;
-                double s = 0.0;
-                if (k0 < end[u]) s = prod(a, k0);
-                if (k1 < end[u]) s += prod(a, k1);
-                acc[u] = s;
+                acc[u] = fmacp(a, k0 < end[u], k0, 0.0);
+                acc[u] = fmacp(a, k1 < end[u], k1, acc[u]);
             }
 #pragma unroll
             for (int u = 0; u < U; u++) {
@@ -222,63 +220,88 @@ struct Kern {
         return v;
     }
 
-    // 4 consecutive elements with 128-bit loads (col: int4; val: 2 x double2 or float4)
-    static __device__ __forceinline__ void vec4(const A &a, int j, double &s0, double &s1, double &s2,
-                                                double &s3)
+    // predicated gather: p false => 0 without touching memory
+    static __device__ __forceinline__ double gxp(const A &a, bool p, int c)
     {
-        const int4 c = __ldcs(reinterpret_cast<const int4 *>(a.col + j));
-        double v0 = 1.0, v1 = 1.0, v2 = 1.0, v3 = 1.0;
-        if (HAS_VAL) {
-            if (sizeof(V) == 8) {
-                const double2 p = __ldcs(reinterpret_cast<const double2 *>(a.val + j));
-                const double2 q = __ldcs(reinterpret_cast<const double2 *>(a.val + j + 2));
-                v0 = p.x; v1 = p.y; v2 = q.x; v3 = q.y;
-            } else {
-                const float4 p = __ldcs(reinterpret_cast<const float4 *>(a.val + j));
-                v0 = p.x; v1 = p.y; v2 = p.z; v3 = p.w;
-            }
-        }
-        const double x0 = gx(a, c.x), x1 = gx(a, c.y), x2 = gx(a, c.z), x3 = gx(a, c.w);
-        if (HAS_VAL) {
-            s0 = fma(v0, x0, s0); s1 = fma(v1, x1, s1); s2 = fma(v2, x2, s2); s3 = fma(v3, x3, s3);
+        double v = 0.0;
+        if (XC) {
+            const uint32_t s = (uint32_t)c & (XC_SLOTS - 1);
+            const bool hit = p && a.xtag[s] == (uint16_t)((uint32_t)c >> XC_BITS);
+            if (hit) v = (double)a.xval[s];
+            if (p && !hit) v = (double)__ldg(a.x + c);
         } else {
-            s0 += x0; s1 += x1; s2 += x2; s3 += x3;
+            if (p) v = (double)__ldg(a.x + c);
         }
+        return v;
     }
 
-    // lane-strided dot over [kb, ke).  Vector path: the warp covers 128 consecutive
-    // elements per group, 4 per lane, two groups in flight; element t of a lane's
-    // 4-vector always goes to accumulator t (the order depends only on the row's
-    // address), ragged head/tail elements are masked scalar loads.
+    // masked scalar element: contributes val[k] * x[col[k]] only when p
+    static __device__ __forceinline__ double fmacp(const A &a, bool p, int k, double acc)
+    {
+        const int c = p ? __ldcs(a.col + k) : 0;
+        const double xv = gxp(a, p, c);
+        if (HAS_VAL) {
+            const double v = p ? (double)__ldcs(a.val + k) : 0.0;
+            return fma(v, xv, acc);
+        }
+        return acc + xv;
+    }
+
+    // lane-strided dot over [kb, ke).
+    // Vector path (rows >= 64 nnz): a scalar head of <= 3 elements up to the first index
+    // j_a with (j_a + vph) % 4 == 0, then groups of 128 consecutive elements with one
+    // 128-bit col load (int4) and 128-bit val loads per lane, TWO groups per iteration
+    // issued back to back (8 gathers in flight per lane, no branches in the body), then
+    // a lane-strided masked tail.  Element t of a lane's 4-vector always feeds
+    // accumulator t: the summation order depends only on (kb, ke, vph).
     static __device__ __forceinline__ double strided_dot(const A &a, int kb, int ke, int lane)
     {
         double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+        int k;
         if (a.vph >= 0 && ke - kb >= 64) {
-            const int ph = a.vph;
-            for (int j0 = ((kb + ph) & ~3) - ph; j0 < ke; j0 += 256) {
-#pragma unroll
-                for (int h = 0; h < 2; h++) {
-                    const int j = j0 + 128 * h + 4 * lane;
-                    if (j >= kb && j + 3 < ke) {
-                        vec4(a, j, s0, s1, s2, s3);
-                    } else if (j < ke && j + 3 >= kb) {
-                        if (j >= kb) s0 = fmac(a, j, s0);
-                        if (j + 1 >= kb && j + 1 < ke) s1 = fmac(a, j + 1, s1);
-                        if (j + 2 >= kb && j + 2 < ke) s2 = fmac(a, j + 2, s2);
-                        if (j + 3 < ke) s3 = fmac(a, j + 3, s3);
+            const int ja = ((kb + a.vph + 3) & ~3) - a.vph;  // first aligned index >= kb
+            s0 = fmacp(a, lane < ja - kb, kb + lane, s0);
+            int j = ja;
+            for (; j + 256 <= ke; j += 256) {
+                const int e0 = j + 4 * lane, e1 = e0 + 128;
+                const int4 c0 = __ldcs(reinterpret_cast<const int4 *>(a.col + e0));
+                const int4 c1 = __ldcs(reinterpret_cast<const int4 *>(a.col + e1));
+                double v[8];
+                if (HAS_VAL) {
+                    if (sizeof(V) == 8) {
+                        const double2 p0 = __ldcs(reinterpret_cast<const double2 *>(a.val + e0));
+                        const double2 p1 = __ldcs(reinterpret_cast<const double2 *>(a.val + e0 + 2));
+                        const double2 p2 = __ldcs(reinterpret_cast<const double2 *>(a.val + e1));
+                        const double2 p3 = __ldcs(reinterpret_cast<const double2 *>(a.val + e1 + 2));
+                        v[0] = p0.x; v[1] = p0.y; v[2] = p1.x; v[3] = p1.y;
+                        v[4] = p2.x; v[5] = p2.y; v[6] = p3.x; v[7] = p3.y;
+                    } else {
+                        const float4 p0 = __ldcs(reinterpret_cast<const float4 *>(a.val + e0));
+                        const float4 p1 = __ldcs(reinterpret_cast<const float4 *>(a.val + e1));
+                        v[0] = p0.x; v[1] = p0.y; v[2] = p0.z; v[3] = p0.w;
+                        v[4] = p1.x; v[5] = p1.y; v[6] = p1.z; v[7] = p1.w;
                     }
                 }
+                const double x0 = gx(a, c0.x), x1 = gx(a, c0.y), x2 = gx(a, c0.z), x3 = gx(a, c0.w);
+                const double x4 = gx(a, c1.x), x5 = gx(a, c1.y), x6 = gx(a, c1.z), x7 = gx(a, c1.w);
+                if (HAS_VAL) {
+                    s0 = fma(v[0], x0, s0); s1 = fma(v[1], x1, s1); s2 = fma(v[2], x2, s2); s3 = fma(v[3], x3, s3);
+                    s0 = fma(v[4], x4, s0); s1 = fma(v[5], x5, s1); s2 = fma(v[6], x6, s2); s3 = fma(v[7], x7, s3);
+                } else {
+                    s0 += x0; s1 += x1; s2 += x2; s3 += x3;
+                    s0 += x4; s1 += x5; s2 += x6; s3 += x7;
+                }
             }
-            return (s0 + s1) + (s2 + s3);
+            k = j + lane;  // tail (< 256 elements), lane-strided, masked, 4 in flight
+        } else {
+            k = kb + lane;
         }
-        int k = kb + lane;
-        for (; k + 96 < ke; k += 128) {
-            s0 = fmac(a, k, s0);
-            s1 = fmac(a, k + 32, s1);
-            s2 = fmac(a, k + 64, s2);
-            s3 = fmac(a, k + 96, s3);
+        for (; k < ke; k += 128) {
+            s0 = fmacp(a, true, k, s0);
+            s1 = fmacp(a, k + 32 < ke, k + 32, s1);
+            s2 = fmacp(a, k + 64 < ke, k + 64, s2);
+            s3 = fmacp(a, k + 96 < ke, k + 96, s3);
         }
-        for (; k < ke; k += 32) s0 = fmac(a, k, s0);
         return (s0 + s1) + (s2 + s3);
     }
 

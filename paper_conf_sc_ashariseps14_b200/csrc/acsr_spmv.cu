@@ -462,12 +462,13 @@ spmv_kernel(SpmvArgs<V> a)
 // the plan workspace (XC_SLOTS values + 16-bit tags) for the TMA fill.  Without a
 // vote table (acsr_bin called without col_idx) every tag is XC_NOTAG.
 template <typename V>
-__global__ void xc_fill_kernel(PlanHeader *hdr, const V *__restrict__ x)
+__global__ void xc_fill_kernel(PlanHeader *hdr, const V *__restrict__ x, int force_miss)
 {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= XC_SLOTS) return;
     char *ws = (char *)hdr;
-    const unsigned long long v = hdr->xc_valid ? ((const unsigned long long *)(ws + hdr->off_xc_vote))[s] : 0ull;
+    const unsigned long long v =
+        (hdr->xc_valid && !force_miss) ? ((const unsigned long long *)(ws + hdr->off_xc_vote))[s] : 0ull;
     const int64_t c = (int64_t)(uint32_t)v;
     const uint32_t t = (uint32_t)(c >> XC_BITS);
     const bool ok = (v >> 32) != 0 && c < hdr->n_cols && t < XC_NOTAG;
@@ -511,15 +512,25 @@ static void dispatch2(const SpmvArgs<V> &a, cudaStream_t s)
     else launch<V, false, false, PR, XC>(a, s);
 }
 
-// ACSR_NO_XCACHE=1 disables the shared-memory x cache (A/B measurements only).
+// A/B knobs for measurements only (read once):
+//   ACSR_NO_XCACHE=1   plain gathers, no shared-memory x cache
+//   ACSR_XC_MISS=1     cache path with every tag invalid (lookup cost without hits)
+static int env_flag(const char *name)
+{
+    const char *e = getenv(name);
+    return (e && e[0] == '1') ? 1 : 0;
+}
 static bool xcache_enabled()
 {
     static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("ACSR_NO_XCACHE");
-        v = (e && e[0] == '1') ? 0 : 1;
-    }
+    if (v < 0) v = env_flag("ACSR_NO_XCACHE") ? 0 : 1;
     return v == 1;
+}
+static int xcache_force_miss()
+{
+    static int v = -1;
+    if (v < 0) v = env_flag("ACSR_XC_MISS");
+    return v;
 }
 
 // element phase for 128-bit loads of col (and val), or -1 if col and val cannot be
@@ -542,7 +553,7 @@ static int dispatch(SpmvArgs<V> a, cudaStream_t s)
 {
     a.vph = vec_phase<V>(a.col, a.val);
     if (xcache_enabled() && a.x != nullptr) {
-        xc_fill_kernel<V><<<XC_SLOTS / 256, 256, 0, s>>>(a.hdr, a.x);
+        xc_fill_kernel<V><<<XC_SLOTS / 256, 256, 0, s>>>(a.hdr, a.x, xcache_force_miss());
         dispatch2<V, PR, true>(a, s);
         return 2;
     }

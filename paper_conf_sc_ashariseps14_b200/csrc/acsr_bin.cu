@@ -43,12 +43,13 @@ bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__res
 #pragma unroll 4
     for (int k = 0; k < TILE_ROUNDS; k++) {
         int64_t r = base + k * BIN_THREADS + tid;
-        if (r < n) {
-            int len = row_length<HAS_END>(rb, re, r);
-            int b = bin_of_len(len);
-            atomicAdd(&hist[b], 1);
-            if (b >= HEAVY_BIN) my_heavy += heavy_chunks(len);
-        }
+        const bool valid = r < n;
+        const int len = valid ? row_length<HAS_END>(rb, re, r) : 0;
+        const int b = valid ? bin_of_len(len) : NBINS;
+        // warp-aggregated histogram update: one shared atomic per distinct bin
+        const unsigned m = __match_any_sync(0xffffffffu, b);
+        if (valid && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&hist[b], __popc(m));
+        if (b >= HEAVY_BIN && valid) my_heavy += heavy_chunks(len);
     }
     // warp-reduce the heavy chunk count
     for (int o = 16; o > 0; o >>= 1) my_heavy += __shfl_xor_sync(0xffffffffu, my_heavy, o);
@@ -112,16 +113,20 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
         is_last = (atomicAdd(&hdr->scan_ticket, 1) == SCAN_ROWS - 1);
     }
     __syncthreads();
-    if (is_last && tid == 0) {
+    if (is_last && warp == 0) {
+        // one parallel load per lane (not a serial chain of L2 round trips)
         __threadfence();
-        volatile int32_t *tot = hdr->totals;
-        int acc = 0;
-        for (int b = 0; b < NBINS; b++) {
-            bin_offsets[b] = acc;
-            acc += tot[b];
+        const int t = __ldcg(hdr->totals + lane);
+        int incl = t;
+        for (int d = 1; d < 32; d <<= 1) {
+            const int v = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += v;
         }
-        bin_offsets[NBINS] = acc;  // == n_rows
-        int nl = tot[NBINS], nh = tot[NBINS + 1];
+        bin_offsets[lane] = incl - t;
+        if (lane == 31) bin_offsets[NBINS] = incl;  // == n_rows
+    }
+    if (is_last && tid == 0) {
+        const int nl = __ldcg(hdr->totals + NBINS), nh = __ldcg(hdr->totals + NBINS + 1);
         int ovf = (nl > light_cap) || (nh > heavy_cap);
         hdr->overflow = ovf;
         hdr->n_light_units = ovf ? 0 : nl;

@@ -48,9 +48,10 @@ struct SpmvArgs {
     const int2 *__restrict__ units;
     double *__restrict__ partial;
     int32_t *__restrict__ ticket;
-    // shared-memory x cache
+    // shared-memory x cache (2^xc_bits slots)
     const uint16_t *xtag;
     const V *xval;
+    int xc_bits;
     // 128-bit load phase: vector loads at element j need (j + vph) % 4 == 0; -1 = scalar only
     int vph;
     // PageRank epilogue
@@ -141,8 +142,8 @@ struct Kern {
     static __device__ __forceinline__ double gx(const A &a, int c)
     {
         if (XC) {
-            const uint32_t s = (uint32_t)c & (XC_SLOTS - 1);
-            if (a.xtag[s] == (uint16_t)((uint32_t)c >> XC_BITS)) return (double)a.xval[s];
+            const uint32_t s = (uint32_t)c & ((1u << a.xc_bits) - 1u);
+            if (a.xtag[s] == (uint16_t)((uint32_t)c >> a.xc_bits)) return (double)a.xval[s];
         }
         return (double)__ldg(a.x + c);
     }
@@ -225,8 +226,8 @@ struct Kern {
     {
         double v = 0.0;
         if (XC) {
-            const uint32_t s = (uint32_t)c & (XC_SLOTS - 1);
-            const bool hit = p && a.xtag[s] == (uint16_t)((uint32_t)c >> XC_BITS);
+            const uint32_t s = (uint32_t)c & ((1u << a.xc_bits) - 1u);
+            const bool hit = p && a.xtag[s] == (uint16_t)((uint32_t)c >> a.xc_bits);
             if (hit) v = (double)a.xval[s];
             if (p && !hit) v = (double)__ldg(a.x + c);
         } else {
@@ -399,12 +400,13 @@ spmv_kernel(SpmvArgs<V> a)
     }
     if (XC) {
         // shared x cache: [XC_SLOTS values | XC_SLOTS 16-bit tags], filled by TMA bulk copies
+        const uint32_t slots = 1u << a.xc_bits;
         V *sval = (V *)smem;
-        uint16_t *stag = (uint16_t *)(smem + sizeof(V) * XC_SLOTS);
+        uint16_t *stag = (uint16_t *)(smem + sizeof(V) * slots);
         const char *ws = (const char *)hdr;
         if (threadIdx.x == 0) {
             mbar_init(&bar, 1);
-            constexpr uint32_t vbytes = sizeof(V) * XC_SLOTS, tbytes = sizeof(uint16_t) * XC_SLOTS;
+            const uint32_t vbytes = sizeof(V) * slots, tbytes = sizeof(uint16_t) * slots;
             mbar_expect_tx(&bar, vbytes + tbytes);
             constexpr uint32_t CH = 32768;
             for (uint32_t o = 0; o < vbytes; o += CH)
@@ -462,44 +464,51 @@ spmv_kernel(SpmvArgs<V> a)
 // the plan workspace (XC_SLOTS values + 16-bit tags) for the TMA fill.  Without a
 // vote table (acsr_bin called without col_idx) every tag is XC_NOTAG.
 template <typename V>
-__global__ void xc_fill_kernel(PlanHeader *hdr, const V *__restrict__ x, int force_miss)
+__global__ void xc_fill_kernel(PlanHeader *hdr, const V *__restrict__ x, int bits, int force_miss)
 {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
-    if (s >= XC_SLOTS) return;
+    const int slots = 1 << bits;
+    if (s >= slots) return;
     char *ws = (char *)hdr;
-    const unsigned long long v =
-        (hdr->xc_valid && !force_miss) ? ((const unsigned long long *)(ws + hdr->off_xc_vote))[s] : 0ull;
+    unsigned long long v = 0ull;
+    if (hdr->xc_valid && !force_miss) {
+        const unsigned long long *best = (const unsigned long long *)(ws + hdr->off_xc_vote);
+        for (int j = s; j < XC_SLOTS; j += slots) v = max(v, best[j]);  // counts compare first
+    }
     const int64_t c = (int64_t)(uint32_t)v;
-    const uint32_t t = (uint32_t)(c >> XC_BITS);
+    const uint32_t t = (uint32_t)(c >> bits);
     const bool ok = (v >> 32) != 0 && c < hdr->n_cols && t < XC_NOTAG;
     ((uint16_t *)(ws + hdr->off_xc_tag))[s] = ok ? (uint16_t)t : XC_NOTAG;
     ((V *)(ws + hdr->off_xc_val))[s] = ok ? x[c] : (V)0;
 }
 
-template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
-static int grid_for()
+static int env_int(const char *name, int dflt)
 {
-    static int g = 0;
-    if (!g) {
-        const size_t smem = XC ? (sizeof(V) + sizeof(uint16_t)) * XC_SLOTS : 0;
-        if (XC)
-            cudaFuncSetAttribute(spmv_kernel<V, HAS_VAL, HAS_END, PR, XC>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmv_kernel<V, HAS_VAL, HAS_END, PR, XC>,
-                                                      SPMV_THREADS, smem);
-        if (per_sm < 1) per_sm = 1;
-        g = per_sm * acsr_num_sms();
-    }
-    return g;
+    const char *e = getenv(name);
+    return (e && e[0]) ? atoi(e) : dflt;
+}
+
+// dynamic shared memory of the SpMV launch: the x cache plus an optional reserve
+// (ACSR_SMEM_RESERVE, bytes; measurements only -- it shrinks L1)
+template <typename V, bool XC>
+static size_t spmv_smem(int bits)
+{
+    static int reserve = -1;
+    if (reserve < 0) reserve = env_int("ACSR_SMEM_RESERVE", 0);
+    return (XC ? (sizeof(V) + sizeof(uint16_t)) * ((size_t)1 << bits) : 0) + (size_t)reserve;
 }
 
 template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
 static void launch(const SpmvArgs<V> &a, cudaStream_t s)
 {
-    const size_t smem = XC ? (sizeof(V) + sizeof(uint16_t)) * XC_SLOTS : 0;
-    const int g = grid_for<V, HAS_VAL, HAS_END, PR, XC>();
-    spmv_kernel<V, HAS_VAL, HAS_END, PR, XC><<<g, SPMV_THREADS, smem, s>>>(a);
+    static size_t configured = 0;
+    const size_t smem = spmv_smem<V, XC>(a.xc_bits);
+    if (smem > configured) {
+        cudaFuncSetAttribute(spmv_kernel<V, HAS_VAL, HAS_END, PR, XC>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        configured = smem;
+    }
+    spmv_kernel<V, HAS_VAL, HAS_END, PR, XC><<<acsr_num_sms(), SPMV_THREADS, smem, s>>>(a);
 }
 
 template <typename V, bool PR, bool XC>
@@ -548,12 +557,25 @@ static int vec_phase(const int32_t *col, const V *val)
     return ((int)((pv / 4) % 4) == ph) ? ph : -1;
 }
 
+static int xcache_bits()
+{
+    static int v = -1;
+    if (v < 0) {
+        v = env_int("ACSR_XC_BITS", XC_BITS);
+        if (v < 8) v = 8;
+        if (v > XC_BITS) v = XC_BITS;
+    }
+    return v;
+}
+
 template <typename V, bool PR>
 static int dispatch(SpmvArgs<V> a, cudaStream_t s)
 {
     a.vph = vec_phase<V>(a.col, a.val);
+    a.xc_bits = xcache_bits();
     if (xcache_enabled() && a.x != nullptr) {
-        xc_fill_kernel<V><<<XC_SLOTS / 256, 256, 0, s>>>(a.hdr, a.x, xcache_force_miss());
+        xc_fill_kernel<V><<<((1 << a.xc_bits) + 255) / 256, 256, 0, s>>>(a.hdr, a.x, a.xc_bits,
+                                                                          xcache_force_miss());
         dispatch2<V, PR, true>(a, s);
         return 2;
     }

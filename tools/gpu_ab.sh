@@ -2,9 +2,8 @@
 TAG=${1:-ab}; shift; WLS=${@:-rmat20}
 mkdir -p gpurun_out
 for wl in $WLS; do
-  timeout 120 python tools/spmv_ab.py $wl >> gpurun_out/ab_$TAG.jsonl 2>&1
-  ACSR_NO_XCACHE=1 timeout 120 python tools/spmv_ab.py $wl >> gpurun_out/ab_$TAG.jsonl 2>&1
-  ACSR_XC_MISS=1 timeout 120 python tools/spmv_ab.py $wl >> gpurun_out/ab_$TAG.jsonl 2>&1
+  for v in "ACSR_NO_XCACHE=1" "ACSR_NO_XCACHE=1 ACSR_SMEM_RESERVE=163840" "ACSR_NO_XCACHE=1 ACSR_SMEM_RESERVE=65536" "ACSR_XC_BITS=14" "ACSR_XC_BITS=13" "ACSR_XC_BITS=12" "ACSR_XC_BITS=11" "ACSR_XC_BITS=12 ACSR_XC_MISS=1"; do
+    env $v timeout 120 python tools/spmv_ab.py $wl >> gpurun_out/ab_$TAG.jsonl 2>&1
+  done
 done
 cat gpurun_out/ab_$TAG.jsonl
-timeout 300 ncu --metrics gpu__time_duration.sum --cache-control none --clock-control none -k regex:"spmv_kernel|bin_|xc_" --csv --log-file gpurun_out/launches_nc_$TAG.csv python tools/spmv_ab.py rmat20 3 > /dev/null 2>&1

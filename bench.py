@@ -257,6 +257,146 @@ def cpu_baseline(rp, ci, val, x, dtype, budget_s=12.0):
                       f"{dt * 1e3:.1f} ms each; host has {os.cpu_count()} cores"}
 
 
+# ------------------------------------------------------------------------------ PageRank (C4)
+def run_pagerank(args, dev, rank, world):
+    """C4 on one GPU per rank (independent replicas when N > 1): in-link pattern CSR of
+    R-MAT scale S (default 24 on one GPU; 26 with --scale 26), one fused
+    acsr_pagerank_step per iteration (SpMV + epilogue + Delta^2).  value = GTEPS
+    (nnz per iteration / iteration time); also the cold-start iteration count."""
+    import paper_conf_sc_ashariseps14_b200 as acsr
+
+    S = args.scale or 24
+    rp, ci = synth.rmat_csr(S, seed=S + 1000 * rank, device=dev, transpose=True)
+    n, nnz = rp.numel() - 1, ci.numel()
+    outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    n_nd = int((outdeg > 0).sum())
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    m = acsr.ACSRMatrix(rp, ci)
+    e1.record()
+    torch.cuda.synchronize()
+    t_bin = e0.elapsed_time(e1)
+    x = torch.full((n,), 1.0 / n, dtype=torch.float64, device=dev)
+    xs = acsr.acsr_pagerank_scale(x, outdeg)
+    xn, xsn = torch.empty_like(x), torch.empty_like(x)
+    d2 = torch.zeros(1, dtype=torch.float64, device=dev)
+    tel = 0.15 / n
+
+    def step():
+        acsr.acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xs, x,
+                                outdeg, xn, xsn, d2, 0.85, tel, n)
+
+    for _ in range(args.warmup):
+        step()
+    K = args.steps
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(K + 1)]
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    with Clocks(torch.cuda.current_device()) as clk:
+        ev[0].record()
+        for k in range(K):
+            step()
+            ev[k + 1].record()
+        torch.cuda.synchronize()
+    ts = np.array([ev[k].elapsed_time(ev[k + 1]) for k in range(K)])
+    tot = float(ts.sum())
+    if world > 1:
+        tt = torch.tensor([tot], dtype=torch.float64, device=dev)
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        tot = float(tt.item())
+    x2, it, dd = acsr.pagerank(m, outdeg, eps=1e-6)
+    torch.cuda.synchronize()
+    if rank != 0:
+        return None
+    peak, kind = peaks()
+    alg = 4 * nnz + 36 * n + 8 * n_nd
+    ms = tot / K
+    return {"metric": "PageRank iteration GTEPS (in-link pattern SpMV + fused epilogue)",
+            "value": round(nnz * world / (ms * 1e-3) / 1e9, 3), "unit": "GTEPS", "n_gpus": world, "steps": K,
+            "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"pagerank_rmat{S}_inlink", "n_rows": n, "nnz": nnz, "non_dangling": n_nd,
+                       "l2": "not flushed (iterative use); x = %d MB" % (8 * n >> 20),
+                       "parallelism": "independent replica per rank" if world > 1 else "1 GPU"},
+            "breakdown": {"t_bin_ms": round(t_bin, 4), "cold_iterations": it, "final_delta": dd ** 0.5,
+                          "gflops_equiv": round(nnz / (ms * 1e-3) / 1e9, 2)},
+            "roofline": {"bound": "hbm", "achieved": round(alg / (ms * 1e-3) / 1e9, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(alg / (ms * 1e-3) / 1e9 / peak, 4), "traffic": None,
+                         "kernel": "acsr::spmv_kernel<PR>", "peak_kind": kind,
+                         "algorithmic_bytes_per_launch": int(alg)},
+            "gpu_launches": K, "clocks": clk.summary()}
+
+
+# ------------------------------------------------------------------------------ dynamic graph (C5)
+def run_dynamic(args, dev, rank, world):
+    """C5: R-MAT s20 in-link pattern with slack (cap = len + max(4, len/4)); per batch of
+    16,384 inserted edges: H2D of the change lists, acsr_update_edges, acsr_bin, one SpMV
+    (timed) and a warm-started PageRank to eps = 1e-6."""
+    import paper_conf_sc_ashariseps14_b200 as acsr
+
+    S = args.scale or 20
+    B = args.batches or (args.warmup + args.steps)
+    rp, ci = synth.rmat_csr(S, device=dev, transpose=True)
+    n = rp.numel() - 1
+    keys = np.sort((torch.repeat_interleave(torch.arange(n, device=dev), (rp[1:] - rp[:-1]).long()) * n
+                    + ci.long()).cpu().numpy())
+    rb, re, cap, col, _ = synth.with_slack(rp, ci)
+    outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    m = acsr.ACSRMatrix(rb, col, None, row_end=re, row_cap=cap, nnz_max=col.numel())
+    x, it0, _ = acsr.pagerank(m, outdeg, eps=1e-6)
+    t_gen = time.perf_counter()
+    batches = [(ch, k) for ch, k in synth.insert_batches(S, B, 16384, keys, device=dev)]
+    t_gen = time.perf_counter() - t_gen
+    st = torch.empty(2, dtype=torch.int32, device=dev)
+    uws = torch.empty(acsr.acsr_update_workspace_bytes(1 << 20), dtype=torch.uint8, device=dev)
+    xs_tmp = torch.empty(n, dtype=torch.float64, device=dev)
+    y = torch.empty(n, dtype=torch.float64, device=dev)
+    rec = []
+    for b, (ch, k) in enumerate(batches):
+        pinned = {kk: torch.from_numpy(v).pin_memory() for kk, v in ch.items()}
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(5)]
+        torch.cuda.synchronize()
+        ev[0].record()
+        chd = {kk: v.to(dev, non_blocking=True) for kk, v in pinned.items()}
+        ev[1].record()
+        m.update(chd, outdeg=outdeg, status=st, ws=uws)
+        ev[2].record()
+        m.rebin()
+        ev[3].record()
+        acsr.acsr_pagerank_scale(x, outdeg, xs_tmp)
+        m.spmv(xs_tmp, y)
+        ev[4].record()
+        torch.cuda.synchronize()
+        assert st.cpu().tolist() == [0, -1], st
+        t0 = time.perf_counter()
+        x, it, _ = acsr.pagerank(m, outdeg, x0=x, eps=1e-6)
+        torch.cuda.synchronize()
+        t_pr = time.perf_counter() - t0
+        if b >= args.warmup:
+            rec.append([ev[i].elapsed_time(ev[i + 1]) for i in range(4)] + [t_pr * 1e3, it, k])
+    r = np.array(rec)
+    if rank != 0:
+        return None
+    t_h2d, t_upd, t_bin, t_spmv = (float(r[:, i].mean()) for i in range(4))
+    return {"metric": "bin+SpMV ms per dynamic-graph update (C5)", "value": round(t_bin + t_spmv, 5),
+            "unit": "ms", "n_gpus": world, "steps": len(rec), "warmup": args.warmup,
+            "ms_per_step": round(t_h2d + t_upd + t_bin + t_spmv, 5), "higher_is_better": False,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"dynamic_rmat{S}_inlink_16384_insert_batches", "n_rows": n,
+                       "batches_timed": len(rec), "cold_iterations": it0},
+            "breakdown": {"t_h2d_ms": round(t_h2d, 5), "t_update_ms": round(t_upd, 5), "t_bin_ms": round(t_bin, 5),
+                          "t_spmv_ms": round(t_spmv, 5), "bin_lt_spmv": bool(t_bin < t_spmv),
+                          "pt_st": round(t_bin / t_spmv, 3),
+                          "rebuild_plus_spmv_ms": round(t_upd + t_bin + t_spmv, 5),
+                          "pagerank_warm_ms": round(float(r[:, 4].mean()), 4),
+                          "warm_iterations_mean": round(float(r[:, 5].mean()), 2),
+                          "inserted_edges_mean": round(float(r[:, 6].mean()), 1),
+                          "batch_encode_s_total": round(t_gen, 2)},
+            "gpu_launches": None}
+
+
 # ------------------------------------------------------------------------------ reference arm
 def run_reference(args, dev):
     """The oracle as it stands (plain C, 1 core) on the same workload: bins (O3) + plain SpMV
@@ -295,6 +435,8 @@ def main():
     ap.add_argument("--impl", default="acsr", choices=["acsr", "reference"])
     ap.add_argument("--workload", default="rmat20")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--scale", type=int, default=None, help="R-MAT scale for pagerank/dynamic")
+    ap.add_argument("--batches", type=int, default=None, help="dynamic: number of insertion batches")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -310,7 +452,12 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         torch.distributed.init_process_group("nccl", device_id=dev)
-    line = run_acsr(args, dev, rank, world)
+    if args.workload == "pagerank":
+        line = run_pagerank(args, dev, rank, world)
+    elif args.workload == "dynamic":
+        line = run_dynamic(args, dev, rank, world)
+    else:
+        line = run_acsr(args, dev, rank, world)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -12,6 +12,7 @@
 //                  counts scanned across warps, 16 rounds of 256 rows in row
 //                  order) -> bin_rows; then writes the tile's work units.
 #include <cuda_runtime.h>
+#include <stdlib.h>
 
 #include "acsr_internal.cuh"
 
@@ -305,7 +306,10 @@ extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
         bin_count_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
     else
         bin_count_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
-    const int xc_valid = col_idx != nullptr && n_cols > 0 && n_cols < ((int64_t)XC_NOTAG << XC_BITS);
+    // the x-cache table is built only when the (experimental, default-off) cache is enabled
+    const char *xe = getenv("ACSR_XCACHE");
+    const int xc_valid = xe && xe[0] == '1' && col_idx != nullptr && n_cols > 0 &&
+                         n_cols < ((int64_t)XC_NOTAG << XC_BITS);
     int64_t stride64 = nnz_max >> XC_SAMPLE_LOG2;
     const int xc_stride = (int)(stride64 < 1 ? 1 : (stride64 > (1 << 30) ? (1 << 30) : stride64));
     bin_scan_kernel<<<SCAN_ROWS, SCAN_THREADS, 0, stream>>>(

@@ -521,9 +521,13 @@ static void dispatch2(const SpmvArgs<V> &a, cudaStream_t s)
     else launch<V, false, false, PR, XC>(a, s);
 }
 
-// A/B knobs for measurements only (read once):
-//   ACSR_NO_XCACHE=1   plain gathers, no shared-memory x cache
+// The shared-memory x cache is OFF by default: measured on B200 its
+// tag lookups sit in the same L1TEX queue as the outstanding gathers, so they add a
+// full queue latency to every gather and the kernel got slower (C2: 93 -> 116 us)
+// even though L2 requests fell.  Knobs (read once; measurements only):
+//   ACSR_XCACHE=1      enable the cache (acsr_bin must also see ACSR_XCACHE=1)
 //   ACSR_XC_MISS=1     cache path with every tag invalid (lookup cost without hits)
+//   ACSR_XC_BITS=k     2^k slots (k <= 14)
 static int env_flag(const char *name)
 {
     const char *e = getenv(name);
@@ -532,7 +536,7 @@ static int env_flag(const char *name)
 static bool xcache_enabled()
 {
     static int v = -1;
-    if (v < 0) v = env_flag("ACSR_NO_XCACHE") ? 0 : 1;
+    if (v < 0) v = env_flag("ACSR_XCACHE");
     return v == 1;
 }
 static int xcache_force_miss()

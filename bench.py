@@ -270,10 +270,11 @@ def run_pagerank(args, dev, rank, world):
     n, nnz = rp.numel() - 1, ci.numel()
     outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
     n_nd = int((outdeg > 0).sum())
+    m = acsr.ACSRMatrix(rp, ci)
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record()
-    m = acsr.ACSRMatrix(rp, ci)
+    m.rebin()
     e1.record()
     torch.cuda.synchronize()
     t_bin = e0.elapsed_time(e1)
@@ -329,6 +330,59 @@ def run_pagerank(args, dev, rank, world):
             "gpu_launches": K, "clocks": clk.summary()}
 
 
+def run_pagerank_dist(args, dev, rank, world):
+    """C4 row-partitioned across the ranks (reading Q19): every rank builds the
+    in-link graph, keeps its nnz-balanced contiguous row range, and per iteration runs
+    one fused acsr_pagerank_step + NCCL all-gather of the xs slices + all-reduce of
+    Delta^2 (paper_conf_sc_ashariseps14_b200.dist).  Strong scaling (fixed graph)."""
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+
+    S = args.scale or 24
+    rp, ci = synth.rmat_csr(S, device=dev, transpose=True)
+    n = rp.numel() - 1
+    outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    splits = pdist.partition_rows((rp[1:] - rp[:-1]).cpu().numpy(), world)
+    lo, hi = int(splits[rank]), int(splits[rank + 1])
+    rpl = (rp[lo:hi + 1] - rp[lo]).contiguous()
+    cil = ci[int(rp[lo]):int(rp[hi])].clone()
+    odl = outdeg[lo:hi].clone()
+    nnz_local = cil.numel()
+    del rp, ci
+    torch.cuda.empty_cache()
+    pr = pdist.DistPageRank(rpl, cil, odl, splits, n)
+    for _ in range(args.warmup):
+        pr.run(max_iter=1)
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    K = args.steps
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with Clocks(torch.cuda.current_device()) as clk:
+        e0.record()
+        x, it, d2 = pr.run(eps=0.0, max_iter=K)
+        e1.record()
+        torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / K
+    if world > 1:
+        tt = torch.tensor([ms], dtype=torch.float64, device=dev)
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        ms = float(tt.item())
+        nz = torch.tensor([nnz_local], dtype=torch.int64, device=dev)
+        torch.distributed.all_reduce(nz)
+        nnz = int(nz.item())
+    else:
+        nnz = nnz_local
+    if rank != 0:
+        return None
+    return {"metric": "PageRank iteration GTEPS, row-partitioned (NCCL all-gather of xs)",
+            "value": round(nnz / (ms * 1e-3) / 1e9, 3), "unit": "GTEPS", "n_gpus": world, "steps": K,
+            "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"pagerank_rmat{S}_inlink_partitioned", "n_rows": n, "nnz": nnz,
+                       "parallelism": f"row-partitioned x{world}", "padded_slice": pr.L},
+            "gpu_launches": K, "clocks": clk.summary()}
+
+
 # ------------------------------------------------------------------------------ dynamic graph (C5)
 def run_dynamic(args, dev, rank, world):
     """C5: R-MAT s20 in-link pattern with slack (cap = len + max(4, len/4)); per batch of
@@ -354,6 +408,7 @@ def run_dynamic(args, dev, rank, world):
     xs_tmp = torch.empty(n, dtype=torch.float64, device=dev)
     y = torch.empty(n, dtype=torch.float64, device=dev)
     rec = []
+    relayouts = 0
     for b, (ch, k) in enumerate(batches):
         pinned = {kk: torch.from_numpy(v).pin_memory() for kk, v in ch.items()}
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(5)]
@@ -369,7 +424,15 @@ def run_dynamic(args, dev, rank, world):
         m.spmv(xs_tmp, y)
         ev[4].record()
         torch.cuda.synchronize()
-        assert st.cpu().tolist() == [0, -1], st
+        regrow = 0
+        while st.cpu().tolist() != [0, -1]:  # CAPACITY: nothing was applied (all-or-nothing)
+            assert int(st[0]) == acsr.ACSR_ERR_CAPACITY and regrow < 4, st
+            m.grow()
+            m.update(chd, outdeg=outdeg, status=st, ws=uws)
+            m.rebin()
+            torch.cuda.synchronize()
+            regrow += 1
+        relayouts += regrow
         t0 = time.perf_counter()
         x, it, _ = acsr.pagerank(m, outdeg, x0=x, eps=1e-6)
         torch.cuda.synchronize()
@@ -393,7 +456,8 @@ def run_dynamic(args, dev, rank, world):
                           "pagerank_warm_ms": round(float(r[:, 4].mean()), 4),
                           "warm_iterations_mean": round(float(r[:, 5].mean()), 2),
                           "inserted_edges_mean": round(float(r[:, 6].mean()), 1),
-                          "batch_encode_s_total": round(t_gen, 2)},
+                          "batch_encode_s_total": round(t_gen, 2),
+                          "relayouts": relayouts},
             "gpu_launches": None}
 
 
@@ -454,6 +518,8 @@ def main():
         torch.distributed.init_process_group("nccl", device_id=dev)
     if args.workload == "pagerank":
         line = run_pagerank(args, dev, rank, world)
+    elif args.workload == "pagerank_dist":
+        line = run_pagerank_dist(args, dev, rank, world)
     elif args.workload == "dynamic":
         line = run_dynamic(args, dev, rank, world)
     else:

@@ -177,6 +177,20 @@ acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
                               int32_t *status /* [2] out */,
                               void *ws, size_t ws_bytes, cudaStream_t stream);
 
+/* Re-layout of a slack CSR (§VII keeps "some additional memory ... at the end of
+ * each CSR row"; what happens when a row outgrows it is unstated -- reading
+ * R4 in DESIGN.md: after a CAPACITY rejection the caller re-lays the matrix out with
+ * larger capacities and re-submits the batch).  Row r is copied, in order, from
+ * [old_begin[r], old_end[r]) to [new_begin[r], new_begin[r] + len); new_end[r] is
+ * set.  new_begin (with the capacities it implies) is chosen by the caller; the
+ * new arrays must not overlap the old ones.  Values are moved as opaque 4/8-byte
+ * items (NULL/NULL = pattern). */
+acsr_status acsr_relayout(acsr_dtype dt, int64_t n_rows,
+                          const int32_t *old_begin, const int32_t *old_end,
+                          const int32_t *old_col, const void *old_val,
+                          const int32_t *new_begin, int32_t *new_end,
+                          int32_t *new_col, void *new_val, cudaStream_t stream);
+
 /* ------------------------------------------------------------------------ */
 const char *acsr_status_string(acsr_status s);
 const char *acsr_last_error(void); /* thread-local detail of the last failure */

@@ -56,6 +56,8 @@ _lib.acsr_update_workspace_bytes.restype = _sz
 _lib.acsr_update_edges.argtypes = [ctypes.c_int, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _i64, _vp, _vp,
                                    _vp, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
 _lib.acsr_update_edges.restype = ctypes.c_int
+_lib.acsr_relayout.argtypes = [ctypes.c_int, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp]
+_lib.acsr_relayout.restype = ctypes.c_int
 _lib.acsr_status_string.argtypes = [ctypes.c_int]
 _lib.acsr_status_string.restype = ctypes.c_char_p
 _lib.acsr_last_error.restype = ctypes.c_char_p
@@ -74,7 +76,7 @@ _lib.acsr_pagerank_step.argtypes = [ctypes.POINTER(PrArgs), _vp]
 _lib.acsr_pagerank_step.restype = ctypes.c_int
 
 EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_spmv", "acsr_pagerank_step",
-            "acsr_pagerank_scale", "acsr_update_workspace_bytes", "acsr_update_edges",
+            "acsr_pagerank_scale", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_relayout",
             "acsr_status_string", "acsr_last_error", "acsr_version")
 
 
@@ -233,6 +235,20 @@ def acsr_update_edges(n_cols, row_begin, row_end, row_cap, col_idx, values, upd_
                                   _dev(status, torch.int32, "status"), _dev(ws, torch.uint8, "ws"), ws.numel(),
                                   _stream(stream)), "acsr_update_edges")
     return status
+
+
+def acsr_relayout(old_begin, old_end, old_col, old_val, new_begin, new_end, new_col, new_val,
+                  dtype=torch.float64, stream=None):
+    """Copy every row of a slack CSR into a new layout (after a CAPACITY rejection)."""
+    n = old_begin.numel()
+    vdt = old_val.dtype if old_val is not None else dtype
+    dt = ACSR_F64 if vdt == torch.float64 else ACSR_F32
+    _check(_lib.acsr_relayout(dt, n, _dev(old_begin, torch.int32, "old_begin"),
+                              _dev(old_end, torch.int32, "old_end"), _dev(old_col, torch.int32, "old_col"),
+                              _dev(old_val, vdt, "old_val", True), _dev(new_begin, torch.int32, "new_begin"),
+                              _dev(new_end, torch.int32, "new_end"), _dev(new_col, torch.int32, "new_col"),
+                              _dev(new_val, vdt, "new_val", True), _stream(stream)), "acsr_relayout")
+    return new_end
 
 
 def version() -> int:

@@ -41,11 +41,16 @@ bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__res
     __syncthreads();
     const int64_t base = (int64_t)blockIdx.x * TILE_ROWS;
     int my_heavy = 0;
-#pragma unroll 4
+    int lens[TILE_ROUNDS];
+#pragma unroll
+    for (int k = 0; k < TILE_ROUNDS; k++) {  // all row-length loads in flight at once
+        const int64_t r = base + k * BIN_THREADS + tid;
+        lens[k] = r < n ? row_length<HAS_END>(rb, re, r) : -1;
+    }
+#pragma unroll
     for (int k = 0; k < TILE_ROUNDS; k++) {
-        int64_t r = base + k * BIN_THREADS + tid;
-        const bool valid = r < n;
-        const int len = valid ? row_length<HAS_END>(rb, re, r) : 0;
+        const bool valid = lens[k] >= 0;
+        const int len = valid ? lens[k] : 0;
         const int b = valid ? bin_of_len(len) : NBINS;
         // warp-aggregated histogram update: one shared atomic per distinct bin
         const unsigned m = __match_any_sync(0xffffffffu, b);
@@ -79,34 +84,37 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int32_t *a = cnt + (int64_t)row * n_tiles;
     int32_t *o = toff + (int64_t)row * n_tiles;
-    const int ipt = (n_tiles + SCAN_THREADS - 1) / SCAN_THREADS;
-    const int lo = min(tid * ipt, n_tiles), hi = min(lo + ipt, n_tiles);
-    int s = 0;
-    for (int i = lo; i < hi; i++) s += a[i];
-    // block exclusive scan of s
-    int incl = s;
-    for (int d = 1; d < 32; d <<= 1) {
-        int t = __shfl_up_sync(0xffffffffu, incl, d);
-        if (lane >= d) incl += t;
-    }
-    if (lane == 31) warp_sums[warp] = incl;
+    // coalesced block scan over chunks of SCAN_THREADS elements with a running carry
+    __shared__ int carry;
+    if (tid == 0) carry = 0;
     __syncthreads();
-    if (warp == 0) {
-        int w = warp_sums[lane];
-        int wi = w;
+    for (int c0 = 0; c0 < n_tiles; c0 += SCAN_THREADS) {
+        const int i = c0 + tid;
+        const int s = i < n_tiles ? a[i] : 0;
+        int incl = s;
         for (int d = 1; d < 32; d <<= 1) {
-            int t = __shfl_up_sync(0xffffffffu, wi, d);
-            if (lane >= d) wi += t;
+            const int t = __shfl_up_sync(0xffffffffu, incl, d);
+            if (lane >= d) incl += t;
         }
-        warp_sums[lane] = wi - w;  // exclusive
-        if (lane == 31) hdr->totals[row] = wi;
+        if (lane == 31) warp_sums[warp] = incl;
+        __syncthreads();
+        if (warp == 0) {
+            const int w = warp_sums[lane];
+            int wi = w;
+            for (int d = 1; d < 32; d <<= 1) {
+                const int t = __shfl_up_sync(0xffffffffu, wi, d);
+                if (lane >= d) wi += t;
+            }
+            warp_sums[lane] = wi - w;  // exclusive
+        }
+        __syncthreads();
+        const int base_c = carry;
+        if (i < n_tiles) o[i] = base_c + warp_sums[warp] + incl - s;
+        __syncthreads();
+        if (tid == SCAN_THREADS - 1) carry = base_c + warp_sums[warp] + incl;
+        __syncthreads();
     }
-    __syncthreads();
-    int run = warp_sums[warp] + incl - s;
-    for (int i = lo; i < hi; i++) {
-        o[i] = run;
-        run += a[i];
-    }
+    if (tid == 0) hdr->totals[row] = carry;
     // last CTA: bin offsets + unit totals
     __syncthreads();
     if (tid == 0) {
@@ -194,10 +202,17 @@ bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__r
     __syncthreads();
     const int64_t base = (int64_t)tile * TILE_ROWS;
     const unsigned lt = (1u << lane) - 1u;
+    int lens[TILE_ROUNDS];
+#pragma unroll
+    for (int k = 0; k < TILE_ROUNDS; k++) {  // all row-length loads in flight at once
+        const int64_t r = base + k * BIN_THREADS + tid;
+        lens[k] = r < n ? row_length<HAS_END>(rb, re, r) : 0;
+    }
+#pragma unroll
     for (int k = 0; k < TILE_ROUNDS; k++) {
         int64_t r = base + k * BIN_THREADS + tid;
         bool valid = r < n;
-        int len = valid ? row_length<HAS_END>(rb, re, r) : 0;
+        int len = lens[k];
         int b = valid ? bin_of_len(len) : NBINS;  // NBINS = sentinel for past-the-end rows
         unsigned mask = __match_any_sync(0xffffffffu, b);
         int rank = __popc(mask & lt);

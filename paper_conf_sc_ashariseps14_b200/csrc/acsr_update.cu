@@ -130,9 +130,53 @@ update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
     if (lane == 0) re[r] = w + (i1 - i0);
 }
 
+// re-layout: copy row r from [ob[r], oe[r]) to [nb[r], nb[r] + len) (warp per row)
+template <typename T>
+__global__ void __launch_bounds__(UPD_THREADS)
+relayout_kernel(int64_t n_rows, const int32_t *__restrict__ ob, const int32_t *__restrict__ oe,
+                const int32_t *__restrict__ ocol, const T *__restrict__ oval,
+                const int32_t *__restrict__ nb, int32_t *__restrict__ ne, int32_t *__restrict__ ncol,
+                T *__restrict__ nval)
+{
+    const int lane = threadIdx.x & 31;
+    const int64_t r = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
+    if (r >= n_rows) return;
+    const int b = __ldg(ob + r), e = __ldg(oe + r), d = __ldg(nb + r);
+    for (int k = lane; k < e - b; k += 32) {
+        ncol[d + k] = __ldg(ocol + b + k);
+        if (oval) nval[d + k] = __ldg(oval + b + k);
+    }
+    if (lane == 0) ne[r] = d + (e - b);
+}
+
 }  // namespace acsr
 
 using namespace acsr;
+
+extern "C" acsr_status acsr_relayout(acsr_dtype dt, int64_t n_rows, const int32_t *old_begin,
+                                     const int32_t *old_end, const int32_t *old_col,
+                                     const void *old_val, const int32_t *new_begin, int32_t *new_end,
+                                     int32_t *new_col, void *new_val, cudaStream_t stream)
+{
+    if (n_rows < 0 || (dt != ACSR_F32 && dt != ACSR_F64) ||
+        (n_rows > 0 && (!old_begin || !old_end || !new_begin || !new_end)) ||
+        ((old_val == nullptr) != (new_val == nullptr))) {
+        acsr_set_error("acsr_relayout: invalid argument");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    if (n_rows == 0) return ACSR_OK;
+    const int wpb = UPD_THREADS / 32;
+    const int64_t blocks = (n_rows + wpb - 1) / wpb;
+    if (dt == ACSR_F64)
+        relayout_kernel<uint64_t><<<(unsigned)blocks, UPD_THREADS, 0, stream>>>(
+            n_rows, old_begin, old_end, old_col, (const uint64_t *)old_val, new_begin, new_end, new_col,
+            (uint64_t *)new_val);
+    else
+        relayout_kernel<uint32_t><<<(unsigned)blocks, UPD_THREADS, 0, stream>>>(
+            n_rows, old_begin, old_end, old_col, (const uint32_t *)old_val, new_begin, new_end, new_col,
+            (uint32_t *)new_val);
+    return acsr_check_launch("acsr_relayout");
+}
 
 extern "C" size_t acsr_update_workspace_bytes(int64_t n_upd)
 {

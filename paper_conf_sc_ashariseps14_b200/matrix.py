@@ -10,7 +10,7 @@ from __future__ import annotations
 import torch
 
 from . import (acsr_bin, acsr_bin_workspace_bytes, acsr_pagerank_scale, acsr_pagerank_step,
-               acsr_spmv, acsr_update_edges)
+               acsr_relayout, acsr_spmv, acsr_update_edges)
 
 
 class ACSRMatrix:
@@ -48,6 +48,33 @@ class ACSRMatrix:
                                  self.col_idx, self.values, changes["upd_rows"], changes["ins_ptr"],
                                  changes["ins_cols"], ins_vals, changes.get("del_ptr"),
                                  changes.get("del_cols"), outdeg, status, ws, stream=stream)
+
+    def grow(self, min_slack=8, frac=2, stream=None):
+        """Re-lay the slack CSR out with cap_r = len_r + max(min_slack, ceil(len_r / frac))
+        (reading R4: after a CAPACITY rejection), then re-bin."""
+        assert self.row_end is not None
+        ln = (self.row_end - self.row_begin).to(torch.int64)
+        cap = torch.maximum(self.row_cap.to(torch.int64),
+                            ln + torch.clamp((ln + frac - 1) // frac, min=min_slack))
+        nb = torch.zeros_like(cap)
+        nb[1:] = torch.cumsum(cap, 0)[:-1]
+        total = int(nb[-1] + cap[-1]) if cap.numel() else 0
+        assert total < 2 ** 31
+        dev = self.row_begin.device
+        new_begin = nb.to(torch.int32)
+        new_end = torch.empty_like(new_begin)
+        new_col = torch.full((max(total, 1),), -1, dtype=torch.int32, device=dev)
+        new_val = None if self.values is None else torch.zeros(max(total, 1), dtype=self.values.dtype,
+                                                               device=dev)
+        acsr_relayout(self.row_begin, self.row_end, self.col_idx, self.values, new_begin, new_end, new_col,
+                      new_val, stream=stream)
+        self.row_begin, self.row_end, self.row_cap = new_begin, new_end, cap.to(torch.int32)
+        self.col_idx, self.values = new_col, new_val
+        if total > self.nnz_max:
+            self.nnz_max = total
+            self.plan_ws = torch.empty(acsr_bin_workspace_bytes(self.n_rows, self.n_cols, self.nnz_max),
+                                       dtype=torch.uint8, device=dev)
+        self.rebin(stream)
 
 
 def spmv_from_host(row_ptr_h, col_h, val_h, x_h, y_h=None, device="cuda", stream=None):

@@ -397,3 +397,52 @@ def test_spmv_unaligned_views(acsr, cuda, shift_c, shift_v):
     y = m.spmv(x.to(cuda)).cpu().numpy()
     y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
     check_spmv(y, y_ref, den, torch.float64)
+
+
+def test_dist_pagerank_single_rank_cuda(acsr, cuda):
+    # the partitioned driver (dist.py) on one rank runs the same fused CUDA step: it must
+    # reproduce the single-GPU loop bitwise and the oracle within the converged bar
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+    rp, ci, od, n = _inlink(14, cuda)
+    splits = pdist.partition_rows(np.diff(rp.numpy()), 1)
+    pr = pdist.DistPageRank(rp.to(cuda), ci.to(cuda), od.to(cuda), splits, n)
+    x, it, d2 = pr.run(eps=1e-6)
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda))
+    x1, it1, d21 = acsr.pagerank(m, od.to(cuda), eps=1e-6)
+    assert it == it1 and torch.equal(x, x1)
+    x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)
+    assert abs(it - it_ref) <= 1
+
+
+def test_capacity_reject_then_grow_and_retry(acsr, cuda):
+    # reading R4: a CAPACITY rejection leaves the matrix unchanged; acsr_relayout (via
+    # ACSRMatrix.grow) adds slack; the same batch then applies bit-for-bit like the oracle
+    n, rb, re, cap, col, val, od, rp, ci = _slack_graph(11)
+    m = acsr.ACSRMatrix(rb.to(cuda), col.to(cuda), val.to(cuda), row_end=re.to(cuda), row_cap=cap.to(cuda),
+                        nnz_max=col.numel())
+    odd = od.to(cuda)
+    r = 9
+    free = int(cap[r] - (re[r] - rb[r]))
+    ins = np.arange(free + 3, dtype=np.int32) % n
+    ch = {"upd_rows": torch.tensor([r], dtype=torch.int32, device=cuda),
+          "ins_ptr": torch.tensor([0, ins.size], dtype=torch.int32, device=cuda),
+          "ins_cols": torch.from_numpy(ins).to(cuda)}
+    st = m.update(ch, outdeg=odd)
+    assert st.cpu().tolist() == [3, 0]
+    live_before = [m.col_idx[m.row_begin[i]:m.row_end[i]].cpu() for i in range(0, n, 97)]
+    m.grow()
+    live_after = [m.col_idx[m.row_begin[i]:m.row_end[i]].cpu() for i in range(0, n, 97)]
+    assert all(torch.equal(a, b) for a, b in zip(live_before, live_after))
+    st = m.update(ch, outdeg=odd)
+    torch.cuda.synchronize()
+    assert st.cpu().tolist() == [0, -1]
+    got = m.col_idx[m.row_begin[r]:m.row_end[r]].cpu().numpy()
+    exp = np.concatenate([col.numpy()[rb[r]:re[r]], ins])
+    assert np.array_equal(got, exp)
+    assert int(odd.sum()) == int(od.sum()) + ins.size
+    m.rebin()
+    x = synth.vector(n, 3)
+    y = m.spmv(x.to(cuda)).cpu().numpy()
+    y_ref, den = oracle.spmv(m.row_begin.cpu().numpy(), m.col_idx.cpu().numpy(), m.values.cpu().numpy(),
+                             x.numpy(), row_end=m.row_end.cpu().numpy())
+    check_spmv(y, y_ref, den, torch.float64)

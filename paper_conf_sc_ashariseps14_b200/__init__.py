@@ -25,7 +25,10 @@ import os
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "lib", "libacsr.so")
+# ACSR_LIB_VARIANT=<name> loads lib/libacsr_<name>.so (compile-time A/B variants built by
+# tools/build_variants.sh; measurements only).
+_VARIANT = os.environ.get("ACSR_LIB_VARIANT", "")
+LIB_PATH = os.path.join(_HERE, "lib", f"libacsr_{_VARIANT}.so" if _VARIANT else "libacsr.so")
 
 ACSR_OK = 0
 ACSR_ERR_INVALID_VALUE = 1

@@ -129,6 +129,104 @@ __device__ __forceinline__ void fix_merge(Fix128 &a, uint64_t hi, uint64_t lo)
     a.lo = nlo;
 }
 
+// ----------------------------------------------------------------- load flavours
+// Streamed CSR arrays (col, val) and the gathered x use separate cache policies.
+// Compile-time choice (ACSR_STREAM_LD / ACSR_X_LD) so variants can be A/B-measured:
+//   ACSR_STREAM_LD 0: ld.global.cs (evict-first)   1: ld.global.nc.L1::no_allocate
+//   ACSR_X_LD      0: ld.global.nc                 1: ld.global.nc.L1::evict_last
+#ifndef ACSR_STREAM_LD
+#define ACSR_STREAM_LD 0
+#endif
+#ifndef ACSR_X_LD
+#define ACSR_X_LD 0
+#endif
+
+__device__ __forceinline__ int lds_i(const int *p)
+{
+#if ACSR_STREAM_LD == 1
+    int v;
+    asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+#else
+    return __ldcs(p);
+#endif
+}
+__device__ __forceinline__ double lds_d(const double *p)
+{
+#if ACSR_STREAM_LD == 1
+    double v;
+    asm volatile("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(p));
+    return v;
+#else
+    return __ldcs(p);
+#endif
+}
+__device__ __forceinline__ float lds_f(const float *p)
+{
+#if ACSR_STREAM_LD == 1
+    float v;
+    asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+#else
+    return __ldcs(p);
+#endif
+}
+__device__ __forceinline__ int4 lds_i4(const int *p)
+{
+#if ACSR_STREAM_LD == 1
+    int4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+#else
+    return __ldcs(reinterpret_cast<const int4 *>(p));
+#endif
+}
+__device__ __forceinline__ double2 lds_d2(const double *p)
+{
+#if ACSR_STREAM_LD == 1
+    double2 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0,%1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
+    return v;
+#else
+    return __ldcs(reinterpret_cast<const double2 *>(p));
+#endif
+}
+__device__ __forceinline__ float4 lds_f4(const float *p)
+{
+#if ACSR_STREAM_LD == 1
+    float4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+    return v;
+#else
+    return __ldcs(reinterpret_cast<const float4 *>(p));
+#endif
+}
+__device__ __forceinline__ double lds_v(const double *p) { return lds_d(p); }
+__device__ __forceinline__ double lds_v(const float *p) { return (double)lds_f(p); }
+
+__device__ __forceinline__ double ldx(const double *p)
+{
+#if ACSR_X_LD == 1
+    double v;
+    asm volatile("ld.global.nc.L1::evict_last.f64 %0, [%1];" : "=d"(v) : "l"(p));
+    return v;
+#else
+    return __ldg(p);
+#endif
+}
+__device__ __forceinline__ double ldx(const float *p)
+{
+#if ACSR_X_LD == 1
+    float v;
+    asm volatile("ld.global.nc.L1::evict_last.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return (double)v;
+#else
+    return (double)__ldg(p);
+#endif
+}
+
 template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
 struct Kern {
     using A = SpmvArgs<V>;
@@ -145,22 +243,22 @@ struct Kern {
             const uint32_t s = (uint32_t)c & ((1u << a.xc_bits) - 1u);
             if (a.xtag[s] == (uint16_t)((uint32_t)c >> a.xc_bits)) return (double)a.xval[s];
         }
-        return (double)__ldg(a.x + c);
+        return ldx(a.x + c);
     }
 
     static __device__ __forceinline__ double prod(const A &a, int k)
     {
-        const int c = __ldcs(a.col + k);
+        const int c = lds_i(a.col + k);
         const double xv = gx(a, c);
-        if (HAS_VAL) return (double)__ldcs(a.val + k) * xv;
+        if (HAS_VAL) return lds_v(a.val + k) * xv;
         return xv;
     }
 
     static __device__ __forceinline__ double fmac(const A &a, int k, double acc)
     {
-        const int c = __ldcs(a.col + k);
+        const int c = lds_i(a.col + k);
         const double xv = gx(a, c);
-        if (HAS_VAL) return fma((double)__ldcs(a.val + k), xv, acc);
+        if (HAS_VAL) return fma(lds_v(a.val + k), xv, acc);
         return acc + xv;
     }
 
@@ -229,9 +327,9 @@ struct Kern {
             const uint32_t s = (uint32_t)c & ((1u << a.xc_bits) - 1u);
             const bool hit = p && a.xtag[s] == (uint16_t)((uint32_t)c >> a.xc_bits);
             if (hit) v = (double)a.xval[s];
-            if (p && !hit) v = (double)__ldg(a.x + c);
+            if (p && !hit) v = ldx(a.x + c);
         } else {
-            if (p) v = (double)__ldg(a.x + c);
+            if (p) v = ldx(a.x + c);
         }
         return v;
     }
@@ -239,10 +337,10 @@ struct Kern {
     // masked scalar element: contributes val[k] * x[col[k]] only when p
     static __device__ __forceinline__ double fmacp(const A &a, bool p, int k, double acc)
     {
-        const int c = p ? __ldcs(a.col + k) : 0;
+        const int c = p ? lds_i(a.col + k) : 0;
         const double xv = gxp(a, p, c);
         if (HAS_VAL) {
-            const double v = p ? (double)__ldcs(a.val + k) : 0.0;
+            const double v = p ? lds_v(a.val + k) : 0.0;
             return fma(v, xv, acc);
         }
         return acc + xv;
@@ -265,20 +363,20 @@ struct Kern {
             int j = ja;
             for (; j + 256 <= ke; j += 256) {
                 const int e0 = j + 4 * lane, e1 = e0 + 128;
-                const int4 c0 = __ldcs(reinterpret_cast<const int4 *>(a.col + e0));
-                const int4 c1 = __ldcs(reinterpret_cast<const int4 *>(a.col + e1));
+                const int4 c0 = lds_i4(a.col + e0);
+                const int4 c1 = lds_i4(a.col + e1);
                 double v[8];
                 if (HAS_VAL) {
                     if (sizeof(V) == 8) {
-                        const double2 p0 = __ldcs(reinterpret_cast<const double2 *>(a.val + e0));
-                        const double2 p1 = __ldcs(reinterpret_cast<const double2 *>(a.val + e0 + 2));
-                        const double2 p2 = __ldcs(reinterpret_cast<const double2 *>(a.val + e1));
-                        const double2 p3 = __ldcs(reinterpret_cast<const double2 *>(a.val + e1 + 2));
+                        const double2 p0 = lds_d2((const double *)(a.val + e0));
+                        const double2 p1 = lds_d2((const double *)(a.val + e0 + 2));
+                        const double2 p2 = lds_d2((const double *)(a.val + e1));
+                        const double2 p3 = lds_d2((const double *)(a.val + e1 + 2));
                         v[0] = p0.x; v[1] = p0.y; v[2] = p1.x; v[3] = p1.y;
                         v[4] = p2.x; v[5] = p2.y; v[6] = p3.x; v[7] = p3.y;
                     } else {
-                        const float4 p0 = __ldcs(reinterpret_cast<const float4 *>(a.val + e0));
-                        const float4 p1 = __ldcs(reinterpret_cast<const float4 *>(a.val + e1));
+                        const float4 p0 = lds_f4((const float *)(a.val + e0));
+                        const float4 p1 = lds_f4((const float *)(a.val + e1));
                         v[0] = p0.x; v[1] = p0.y; v[2] = p0.z; v[3] = p0.w;
                         v[4] = p1.x; v[5] = p1.y; v[6] = p1.z; v[7] = p1.w;
                     }

@@ -79,6 +79,7 @@ class DistPageRank:
         self.row_ptr = row_ptr_local
         self.col = renumber_columns(col_local, self.splits, self.L) if self.world > 1 else col_local
         self.outdeg = outdeg_local
+        use_cuda = step_fn is None
         self.step_fn = step_fn or self._cuda_step
         self.scale_fn = scale_fn or self._cuda_scale
         dev = self.device
@@ -86,7 +87,7 @@ class DistPageRank:
         self.xs_next = torch.zeros_like(self.xs)
         self.delta2 = torch.zeros(1, dtype=torch.float64, device=dev)
         self._m = None
-        if self.step_fn is self._cuda_step:
+        if use_cuda:
             from .matrix import ACSRMatrix
             self._m = ACSRMatrix(self.row_ptr, self.col, None, n_cols=self.xs.numel())
 

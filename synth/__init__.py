@@ -276,28 +276,31 @@ def encode_changes(n_rows: int, ins_rows: np.ndarray, ins_cols: np.ndarray,
                 del_cols=del_cols.astype(np.int32))
 
 
-def insert_batches(scale: int, n_batches: int, batch_edges: int, existing_keys: np.ndarray,
-                   base_seed: int = 3000, graph_seed: int | None = None, device=None):
+def insert_batches(scale: int, n_batches: int, batch_edges: int, existing_keys, base_seed: int = 3000,
+                   graph_seed: int | None = None, device=None):
     """C5: batch b draws ``batch_edges`` R-MAT edges (same generator and vertex permutation as the
-    base graph, edge seed base_seed + b), keeps in-link orientation (row = destination), drops
+    base graph, edge seed base_seed + 1 + b), keeps in-link orientation (row = destination), drops
     edges already present (base graph or earlier batches) and in-batch duplicates, and encodes
     the survivors as insert-only change lists.  existing_keys: sorted int64 row*n+col keys of
-    the base in-link graph.  Yields (changes dict, n_inserted)."""
+    the base in-link graph (numpy or tensor).  Filtering runs on ``device``.  Yields
+    (changes dict of host int32 numpy arrays, n_inserted)."""
     graph_seed = scale if graph_seed is None else graph_seed
+    dev = _dev(device)
     n = 1 << scale
-    new_id = rmat_perm(scale, graph_seed, device)
-    keys = np.asarray(existing_keys, np.int64)
+    new_id = rmat_perm(scale, graph_seed, dev)
+    keys = torch.as_tensor(existing_keys, dtype=torch.int64).to(dev)
     for b in range(n_batches):
-        src, dst = rmat_edges(scale, 16, base_seed + 1 + b, device, n_edges=batch_edges,
-                              new_id=new_id)
-        k = (dst.to(torch.int64) * n + src.to(torch.int64)).cpu().numpy()
-        k = np.unique(k)
-        pos = np.searchsorted(keys, k)
-        present = (pos < keys.size) & (keys[np.minimum(pos, keys.size - 1)] == k)
+        src, dst = rmat_edges(scale, 16, base_seed + 1 + b, dev, n_edges=batch_edges, new_id=new_id)
+        k = torch.unique(dst.to(torch.int64) * n + src.to(torch.int64), sorted=True)
+        pos = torch.searchsorted(keys, k)
+        present = keys[torch.clamp(pos, max=max(keys.numel() - 1, 0))] == k if keys.numel() else \
+            torch.zeros_like(k, dtype=torch.bool)
+        present &= pos < keys.numel()
         k = k[~present]
-        keys = np.union1d(keys, k)
-        ch = encode_changes(n, k // n, k % n)
-        yield ch, int(k.size)
+        keys = torch.sort(torch.cat([keys, k])).values
+        kh = k.cpu().numpy()
+        ch = encode_changes(n, kh // n, kh % n)
+        yield ch, int(kh.size)
 
 
 def mixed_batches(row_ptr: np.ndarray, col: np.ndarray, n_cols: int, frac_rows: float,

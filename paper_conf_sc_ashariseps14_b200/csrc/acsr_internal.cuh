@@ -34,8 +34,12 @@ __host__ __device__ constexpr int unit_rows(int b)
          : b == 5 ? 32 : b == 6 ? 16 : b == 7 ? 8 : b == 8 ? 4 : b == 9 ? 2 : 1;
 }
 
-// One persistent CTA of 1024 threads per SM: the whole SM shares one x cache.
-constexpr int SPMV_THREADS = 1024;
+// Persistent CTAs (grid = resident CTAs per SM x SMs).  1024 threads: the whole SM
+// shares one (optional) x cache.  Overridable for A/B builds.
+#ifndef ACSR_SPMV_THREADS
+#define ACSR_SPMV_THREADS 1024
+#endif
+constexpr int SPMV_THREADS = ACSR_SPMV_THREADS;
 constexpr int SPMV_WARPS = SPMV_THREADS / 32;
 
 // ---------------------------------------------------------------- x cache

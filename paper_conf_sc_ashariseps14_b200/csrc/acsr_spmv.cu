@@ -133,7 +133,9 @@ __device__ __forceinline__ void fix_merge(Fix128 &a, uint64_t hi, uint64_t lo)
 // Streamed CSR arrays (col, val) and the gathered x use separate cache policies.
 // Compile-time choice (ACSR_STREAM_LD / ACSR_X_LD) so variants can be A/B-measured:
 //   ACSR_STREAM_LD 0: ld.global.cs (evict-first)   1: ld.global.nc.L1::no_allocate
+//                  2: ld.global.nc.L1::no_allocate + L2 evict_first cache policy
 //   ACSR_X_LD      0: ld.global.nc                 1: ld.global.nc.L1::evict_last
+//                  2: ld.global.nc + L2 evict_last cache policy (createpolicy)
 #ifndef ACSR_STREAM_LD
 #define ACSR_STREAM_LD 0
 #endif
@@ -141,9 +143,26 @@ __device__ __forceinline__ void fix_merge(Fix128 &a, uint64_t hi, uint64_t lo)
 #define ACSR_X_LD 0
 #endif
 
+__device__ __forceinline__ uint64_t pol_evict_first()
+{
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t pol_evict_last()
+{
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
 __device__ __forceinline__ int lds_i(const int *p)
 {
-#if ACSR_STREAM_LD == 1
+#if ACSR_STREAM_LD == 2
+    int v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol_evict_first()));
+    return v;
+#elif ACSR_STREAM_LD == 1
     int v;
     asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));
     return v;
@@ -153,7 +172,11 @@ __device__ __forceinline__ int lds_i(const int *p)
 }
 __device__ __forceinline__ double lds_d(const double *p)
 {
-#if ACSR_STREAM_LD == 1
+#if ACSR_STREAM_LD == 2
+    double v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(pol_evict_first()));
+    return v;
+#elif ACSR_STREAM_LD == 1
     double v;
     asm volatile("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(p));
     return v;
@@ -163,7 +186,11 @@ __device__ __forceinline__ double lds_d(const double *p)
 }
 __device__ __forceinline__ float lds_f(const float *p)
 {
-#if ACSR_STREAM_LD == 1
+#if ACSR_STREAM_LD == 2
+    float v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol_evict_first()));
+    return v;
+#elif ACSR_STREAM_LD == 1
     float v;
     asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v) : "l"(p));
     return v;
@@ -173,7 +200,12 @@ __device__ __forceinline__ float lds_f(const float *p)
 }
 __device__ __forceinline__ int4 lds_i4(const int *p)
 {
-#if ACSR_STREAM_LD == 1
+#if ACSR_STREAM_LD == 2
+    int4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol_evict_first()));
+    return v;
+#elif ACSR_STREAM_LD == 1
     int4 v;
     asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
@@ -184,7 +216,11 @@ __device__ __forceinline__ int4 lds_i4(const int *p)
 }
 __device__ __forceinline__ double2 lds_d2(const double *p)
 {
-#if ACSR_STREAM_LD == 1
+#if ACSR_STREAM_LD == 2
+    double2 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0,%1}, [%2], %3;" : "=d"(v.x), "=d"(v.y) : "l"(p), "l"(pol_evict_first()));
+    return v;
+#elif ACSR_STREAM_LD == 1
     double2 v;
     asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0,%1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
     return v;
@@ -194,7 +230,12 @@ __device__ __forceinline__ double2 lds_d2(const double *p)
 }
 __device__ __forceinline__ float4 lds_f4(const float *p)
 {
-#if ACSR_STREAM_LD == 1
+#if ACSR_STREAM_LD == 2
+    float4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pol_evict_first()));
+    return v;
+#elif ACSR_STREAM_LD == 1
     float4 v;
     asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
                  : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
@@ -208,7 +249,11 @@ __device__ __forceinline__ double lds_v(const float *p) { return (double)lds_f(p
 
 __device__ __forceinline__ double ldx(const double *p)
 {
-#if ACSR_X_LD == 1
+#if ACSR_X_LD == 2
+    double v;
+    asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(pol_evict_last()));
+    return v;
+#elif ACSR_X_LD == 1
     double v;
     asm volatile("ld.global.nc.L1::evict_last.f64 %0, [%1];" : "=d"(v) : "l"(p));
     return v;
@@ -218,7 +263,11 @@ __device__ __forceinline__ double ldx(const double *p)
 }
 __device__ __forceinline__ double ldx(const float *p)
 {
-#if ACSR_X_LD == 1
+#if ACSR_X_LD == 2
+    float v;
+    asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol_evict_last()));
+    return (double)v;
+#elif ACSR_X_LD == 1
     float v;
     asm volatile("ld.global.nc.L1::evict_last.f32 %0, [%1];" : "=f"(v) : "l"(p));
     return (double)v;
@@ -478,8 +527,12 @@ struct Kern {
     }
 };
 
+#ifndef ACSR_SCHED_STATIC
+#define ACSR_SCHED_STATIC 0  // 1: static round-robin units (A/B builds)
+#endif
+
 template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
-__global__ void __launch_bounds__(SPMV_THREADS, 1)
+__global__ void __launch_bounds__(SPMV_THREADS, 1024 / SPMV_THREADS)
 spmv_kernel(SpmvArgs<V> a)
 {
     using K = Kern<V, HAS_VAL, HAS_END, PR, XC>;
@@ -517,6 +570,9 @@ spmv_kernel(SpmvArgs<V> a)
         a.xtag = stag;
     }
     Fix128 d2{0, 0};
+#if ACSR_SCHED_STATIC
+    for (int u = gw; u < n_units; u += nw) K::unit(a, u, lane, d2);
+#else
     int u = gw;
     int nxt = 0;
     if (lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
@@ -525,6 +581,7 @@ spmv_kernel(SpmvArgs<V> a)
         u = __shfl_sync(0xffffffffu, nxt, 0) + nw;
         if (u < n_units && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
     }
+#endif
     if (PR) {
         // exact fixed-point warp sum, then two 64-bit atomics per warp
 #pragma unroll
@@ -606,7 +663,13 @@ static void launch(const SpmvArgs<V> &a, cudaStream_t s)
                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         configured = smem;
     }
-    spmv_kernel<V, HAS_VAL, HAS_END, PR, XC><<<acsr_num_sms(), SPMV_THREADS, smem, s>>>(a);
+    static int per_sm = 0;
+    if (!per_sm) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmv_kernel<V, HAS_VAL, HAS_END, PR, XC>,
+                                                      SPMV_THREADS, smem);
+        if (per_sm < 1) per_sm = 1;
+    }
+    spmv_kernel<V, HAS_VAL, HAS_END, PR, XC><<<per_sm * acsr_num_sms(), SPMV_THREADS, smem, s>>>(a);
 }
 
 template <typename V, bool PR, bool XC>

@@ -4,8 +4,19 @@ set -e
 cd "$(dirname "$0")/.."
 L=paper_conf_sc_ashariseps14_b200/lib
 F="-O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo -Xcompiler -fPIC -shared -cudart shared"
-build() { name=$1; shift; nvcc $F "$@" -o $L/libacsr_$name.so paper_conf_sc_ashariseps14_b200/csrc/*.cu; }
-build s1 -DACSR_STREAM_LD=1
-build x1 -DACSR_X_LD=1
-build s1x1 -DACSR_STREAM_LD=1 -DACSR_X_LD=1
+build() { name=$1; shift; nvcc $F "$@" -o $L/libacsr_$name.so paper_conf_sc_ashariseps14_b200/csrc/*.cu & }
+for v in "$@"; do
+  case $v in
+    s1) build s1 -DACSR_STREAM_LD=1 ;;
+    x1) build x1 -DACSR_X_LD=1 ;;
+    s2) build s2 -DACSR_STREAM_LD=2 ;;
+    x2) build x2 -DACSR_X_LD=2 ;;
+    s2x2) build s2x2 -DACSR_STREAM_LD=2 -DACSR_X_LD=2 ;;
+    st) build st -DACSR_SCHED_STATIC=1 ;;
+    t256) build t256 -DACSR_SPMV_THREADS=256 ;;
+    t512) build t512 -DACSR_SPMV_THREADS=512 ;;
+    t256st) build t256st -DACSR_SPMV_THREADS=256 -DACSR_SCHED_STATIC=1 ;;
+  esac
+done
+wait
 ls $L

@@ -6,3 +6,4 @@ for v in "" s1 x1 s1x1; do
   done
 done
 cat gpurun_out/ab_$TAG.jsonl
+timeout 300 python -m pytest tests/test_gpu_parity.py -q -k "dist or grow" 2>&1 | tail -3

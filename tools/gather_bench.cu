@@ -72,13 +72,14 @@ int main(int argc, char **argv)
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
     const long n = 16L << 20;
-    std::vector<long> ncols_list = {1L << 20, 1L << 17, 1L << 14};
+    std::vector<long> ncols_list = {1L << 20, 1L << 17, 1L << 14, 1L << 26, 1L << 24};
+    if (argc > 1) ncols_list = {1L << 26, 1L << 24, 1L << 22};
     int *idx;
     double *x, *y;
     CK(cudaMalloc(&idx, n * 4));
     CK(cudaMalloc(&y, n * 8));
-    CK(cudaMalloc(&x, (1L << 20) * 8));
-    CK(cudaMemset(x, 0, (1L << 20) * 8));
+    CK(cudaMalloc(&x, (1L << 26) * 8));
+    CK(cudaMemset(x, 0, (1L << 26) * 8));
     std::vector<int> h(n);
     for (long ncols : ncols_list) {
         uint64_t s = 88172645463325252ull;

@@ -188,24 +188,18 @@ def test_empty_and_all_empty(acsr, cuda):
     assert not torch.signbit(y).any()
 
 
-def test_full_size_rmat20_sampled(acsr, cuda):
-    """C2 at BASELINE size, in the launch configuration bench.py times: bins bitwise, and
-    sampled rows (every bin, the longest rows) against the oracle one by one."""
-    rp, ci = synth.rmat_csr(20, device=cuda)
-    n = rp.numel() - 1
-    val = synth.values(ci.numel(), 1014, device=cuda)
-    x = synth.vector(n, 2014, device=cuda)
-    m = acsr.ACSRMatrix(rp, ci, val)
-    y = m.spmv(x).cpu().numpy()
+def sampled_parity(rp, ci, val, x, y, bins_check=None, n_random=4000, seed=0):
+    """Check y (host numpy) on a sample of rows -- random rows, the longest rows and the
+    first rows of every bin -- against the oracle computed row by row on the sample."""
     rph = rp.cpu().numpy()
-    br, off = oracle.bins(rph)
-    assert np.array_equal(m.bin_offsets.cpu().numpy(), off)
-    assert np.array_equal(m.bin_rows.cpu().numpy(), br)
+    n = rph.size - 1
     ln = np.diff(rph)
-    rng = np.random.default_rng(0)
-    sample = set(rng.choice(n, 4000, replace=False).tolist()) | set(np.argsort(ln)[-50:].tolist())
-    for b in range(32):  # a few rows of every non-empty bin
-        sample |= set(br[off[b]:off[b + 1]][:20].tolist())
+    rng = np.random.default_rng(seed)
+    sample = set(rng.choice(n, min(n_random, n), replace=False).tolist()) | set(np.argsort(ln)[-50:].tolist())
+    if bins_check is not None:
+        br, off = bins_check
+        for b in range(32):
+            sample |= set(br[off[b]:off[b + 1]][:20].tolist())
     rows = np.array(sorted(sample))
     sub_rp = np.zeros(rows.size + 1, np.int64)
     sub_rp[1:] = np.cumsum(ln[rows])
@@ -213,7 +207,49 @@ def test_full_size_rmat20_sampled(acsr, cuda):
     sub_ci = np.concatenate([cih[rph[r]:rph[r + 1]] for r in rows])
     sub_v = np.concatenate([vh[rph[r]:rph[r + 1]] for r in rows])
     y_ref, den = oracle.spmv(sub_rp.astype(np.int32), sub_ci, sub_v, x.cpu().numpy())
-    check_spmv(y[rows], y_ref, den, torch.float64)
+    check_spmv(y[rows], y_ref, den, val.dtype)
+
+
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_full_size_rmat20_sampled(acsr, cuda, dtype):
+    """C2 at BASELINE size, in the launch configuration bench.py times: bins bitwise, and
+    sampled rows (every bin, the longest rows) against the oracle one by one."""
+    rp, ci = synth.rmat_csr(20, device=cuda)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 1014, dtype, device=cuda)
+    x = synth.vector(n, 2014, dtype, device=cuda)
+    m = acsr.ACSRMatrix(rp, ci, val)
+    y = m.spmv(x).cpu().numpy()
+    br, off = oracle.bins(rp.cpu().numpy())
+    assert np.array_equal(m.bin_offsets.cpu().numpy(), off)
+    assert np.array_equal(m.bin_rows.cpu().numpy(), br)
+    sampled_parity(rp, ci, val, x, y, (br, off))
+
+
+@pytest.mark.parametrize("shape", ["WEB_GOOGLE", "LIVEJOURNAL"])
+def test_full_size_powerlaw_sampled(acsr, cuda, shape):
+    """C3 shapes at full size (0.9 M / 4.85 M rows): bins bitwise + sampled rows."""
+    rp, ci = synth.powerlaw_csr(seed=3, device=cuda, **getattr(synth, shape))
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 4, device=cuda)
+    x = synth.vector(n, 5, device=cuda)
+    m = acsr.ACSRMatrix(rp, ci, val)
+    y = m.spmv(x).cpu().numpy()
+    br, off = oracle.bins(rp.cpu().numpy())
+    assert np.array_equal(m.bin_rows.cpu().numpy(), br)
+    sampled_parity(rp, ci, val, x, y, (br, off), n_random=3000)
+
+
+def test_c1_rmat14_single_spmv(acsr, cuda):
+    """C1 exactly as BASELINE.json configs[0] names it: R-MAT s14 fp64, one SpMV, every
+    row against the oracle."""
+    rp, ci = synth.rmat_csr(14)
+    val = synth.values(ci.numel(), 1014)
+    x = synth.vector(rp.numel() - 1, 2014)
+    br, bo, ws = acsr.acsr_bin(rp.to(cuda), None, nnz_max=ci.numel(), col_idx=ci.to(cuda), n_cols=x.numel())
+    y = acsr.acsr_spmv(rp.to(cuda), ci.to(cuda), val.to(cuda), x.to(cuda), br, bo, ws).cpu().numpy()
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y, y_ref, den, torch.float64)
 
 
 # ------------------------------------------------------------------------------ PageRank
@@ -251,8 +287,9 @@ def test_pagerank_step_parity(acsr, cuda):
     assert torch.equal(xn, xn2) and torch.equal(d2, d22)
 
 
-def test_pagerank_converged_parity(acsr, cuda):
-    rp, ci, od, n = _inlink(16, cuda)
+@pytest.mark.parametrize("scale", [16, 20])
+def test_pagerank_converged_parity(acsr, cuda, scale):
+    rp, ci, od, n = _inlink(scale, cuda)
     m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda))
     x, it, d2 = acsr.pagerank(m, od.to(cuda), eps=1e-6)
     x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)

@@ -204,6 +204,7 @@ def run_acsr(args, dev, rank, world):
     t_e2e = e0.elapsed_time(e1) / ke
     h2d = sum(t.numel() * t.element_size() for t in (rp_h, ci_h, val_h, x_h))
     d2h = y_h.numel() * y_h.element_size()
+    ctx = cusparse_context(rp, ci, val, x, n)
     if rank != 0:
         return None
     peak, peak_kind = peaks()
@@ -222,7 +223,11 @@ def run_acsr(args, dev, rank, world):
                       "pt_st": round(float(t_bin.mean()) / spmv_ms, 3),
                       "spmv_gflops": round(2.0 * nnz / (spmv_ms * 1e-3) / 1e9, 2),
                       "t_spmv_min_ms": round(float(t_spmv.min()), 5),
-                      "wall_s_timed_loop": round(wall, 4)},
+                      "wall_s_timed_loop": round(wall, 4),
+                      "gather_roofline_ms": round(nnz / 197e9 * 1e3, 5),
+                      "gather_roofline_note": "pure random 8-byte gathers from an L2-resident x run at ~197 G/s "
+                                              "on this B200 (profiles/r1_gather_bench.jsonl); one gather per nnz"},
+        "context": ctx,
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": ncu_traffic(label),
                      "kernel": "acsr::spmv_kernel", "peak_kind": peak_kind,
@@ -236,6 +241,31 @@ def run_acsr(args, dev, rank, world):
     if not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(rp, ci, val, x, dtype)
     return line
+
+
+def cusparse_context(rp, ci, val, x, n):
+    """Context only (not our path): cuSPARSE CSR SpMV through torch.sparse_csr on the same
+    matrix, same L2 flush protocol.  Returns ms and GFLOP/s, or the error text."""
+    try:
+        A = torch.sparse_csr_tensor(rp.to(torch.int64), ci.to(torch.int64), val, size=(n, x.numel()))
+        flush = torch.empty(256 << 20, dtype=torch.uint8, device=x.device)
+        xs = x.view(-1, 1)
+        for _ in range(3):
+            (A @ xs)
+        ts = []
+        for _ in range(10):
+            flush.zero_()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            (A @ xs)
+            e1.record()
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        ms = float(np.median(ts))
+        return {"cusparse_csr_spmv_ms": round(ms, 5), "cusparse_gflops": round(2.0 * ci.numel() / (ms * 1e-3) / 1e9, 2),
+                "note": "torch.sparse_csr @ dense (cuSPARSE), context only; no binning cost"}
+    except Exception as e:  # pragma: no cover - context only
+        return {"cusparse_error": str(e)[:200]}
 
 
 def cpu_baseline(rp, ci, val, x, dtype, budget_s=12.0):

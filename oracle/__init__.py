@@ -14,6 +14,8 @@ arrays (host memory).  Function-level citations are in the C file:
 * ``spmv_plain``        O4', the timed plain sequential SpMV (cpu_baseline)
 * ``pagerank_step``     O6, P:279-291 (Alg. 5) with readings Q11/Q12
 * ``pagerank``          O6', P:285-289, P:297, P:326 with reading Q9
+* ``rwr_step``/``rwr``   Eq. 8, P:318-324 (RWR) with reading R5
+* ``hits_step``/``hits`` Eq. 5-7, P:299-317 (HITS) with reading R6
 * ``update``            O7, P:334-335 (§VII) with reading Q13
 * ``partition``         O8, replaces P:345 (reading Q19)
 * ``csr_build``         O1, P:30 (§II)
@@ -65,6 +67,13 @@ def _L():
         _lib.oracle_pagerank.argtypes = [i64, i32p, i32p, i32p, i32p, vp, dp, dp, dp, ctypes.c_int,
                                          vp, vp]
         _lib.oracle_pagerank.restype = ctypes.c_int
+        _lib.oracle_rwr_step.argtypes = [i64, i32p, i32p, i32p, i32p, vp, dp, i64, vp]
+        _lib.oracle_rwr_step.restype = ctypes.c_double
+        _lib.oracle_rwr.argtypes = [i64, i32p, i32p, i32p, i32p, vp, dp, i64, dp, ctypes.c_int, vp, vp]
+        _lib.oracle_rwr.restype = ctypes.c_int
+        _lib.oracle_hits_step.argtypes = [i64, i32p, i32p, i32p, i32p, vp, vp, vp, vp, vp]
+        _lib.oracle_hits.argtypes = [i64, i32p, i32p, i32p, i32p, vp, vp, dp, ctypes.c_int, vp]
+        _lib.oracle_hits.restype = ctypes.c_int
         _lib.oracle_update.argtypes = [i64, i64, i32p, i32p, i32p, i32p, vp, ctypes.c_int, i64,
                                        i32p, i32p, i32p, i32p, i32p, vp, i32p, i32p]
         _lib.oracle_update.restype = ctypes.c_int
@@ -160,6 +169,55 @@ def pagerank(row_begin, col, outdeg, x0=None, d=0.85, eps=1e-6, max_iter=1000, r
     it = _L().oracle_pagerank(n, _p(rb), _p(re), _p(c), _p(od), _p(x), float(teleport), float(d),
                               float(eps), int(max_iter), _p(work), _p(d2))
     return x, int(it), float(d2[0])
+
+
+def rwr_step(row_begin, col, outdeg, r, c, restart, row_end=None):
+    """Eq. 8 step (reading R5).  Returns (r_new, delta2)."""
+    rb, re, cc, od = _i32(row_begin), _i32(row_end), _i32(col), _i32(outdeg)
+    n = _n_rows(rb, re)
+    r = np.ascontiguousarray(r, np.float64)
+    rn = np.empty(n, np.float64)
+    d2 = _L().oracle_rwr_step(n, _p(rb), _p(re), _p(cc), _p(od), _p(r), float(c), int(restart), _p(rn))
+    return rn, float(d2)
+
+
+def rwr(row_begin, col, outdeg, restart, c=0.85, eps=1e-6, max_iter=1000, row_end=None, r0=None):
+    """Eq. 8 loop from r^0 = e_i.  Returns (r, iterations, last_delta2)."""
+    rb, re, cc, od = _i32(row_begin), _i32(row_end), _i32(col), _i32(outdeg)
+    n = _n_rows(rb, re)
+    if r0 is None:
+        r = np.zeros(n, np.float64)
+        r[restart] = 1.0
+    else:
+        r = np.array(r0, np.float64, copy=True)
+    work = np.empty(n, np.float64)
+    d2 = np.zeros(1, np.float64)
+    it = _L().oracle_rwr(n, _p(rb), _p(re), _p(cc), _p(od), _p(r), float(c), int(restart), float(eps),
+                         int(max_iter), _p(work), _p(d2))
+    return r, int(it), float(d2[0])
+
+
+def hits_step(out_ptr, out_col, in_ptr, in_col, a, h):
+    """Eq. 5-7 step with reading R6 (unit L2 norm).  Returns (a', h', [da2, dh2])."""
+    op, oc, ip, ic = (_i32(t) for t in (out_ptr, out_col, in_ptr, in_col))
+    n = op.size - 1
+    a = np.ascontiguousarray(a, np.float64)
+    h = np.ascontiguousarray(h, np.float64)
+    an, hn, d2 = np.empty(n), np.empty(n), np.empty(2)
+    _L().oracle_hits_step(n, _p(op), _p(oc), _p(ip), _p(ic), _p(a), _p(h), _p(an), _p(hn), _p(d2))
+    return an, hn, d2
+
+
+def hits(out_ptr, out_col, in_ptr, in_col, eps=1e-6, max_iter=1000):
+    """Eq. 5-7 loop from a = h = 1/|V|.  Returns (a, h, iterations)."""
+    op, oc, ip, ic = (_i32(t) for t in (out_ptr, out_col, in_ptr, in_col))
+    n = op.size - 1
+    a = np.full(n, 1.0 / n)
+    h = np.full(n, 1.0 / n)
+    work = np.empty(2 * n)
+    it = _L().oracle_hits(n, _p(op), _p(oc), _p(ip), _p(ic), _p(a), _p(h), float(eps), int(max_iter),
+                          _p(work))
+    return a, h, int(it)
 
 
 def update(n_cols, row_begin, row_end, row_cap, col, val, upd_rows, del_ptr, del_cols, ins_ptr,

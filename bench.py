@@ -413,6 +413,43 @@ def run_pagerank_dist(args, dev, rank, world):
             "gpu_launches": K, "clocks": clk.summary()}
 
 
+def run_hits_rwr(args, dev, rank, world):
+    """HITS (Eq. 5-7) or RWR (Eq. 8) on R-MAT scale S (default 20) to eps = 1e-6:
+    value = GTEPS (nnz per iteration / mean iteration time, host loop included)."""
+    import paper_conf_sc_ashariseps14_b200 as acsr
+
+    S = args.scale or 20
+    if args.workload == "hits":
+        rp, ci = synth.rmat_csr(S, device=dev)
+        nnz_it = 2 * ci.numel()
+        run = lambda: acsr.hits(rp, ci, eps=1e-6)
+    else:
+        rp, ci = synth.rmat_csr(S, device=dev, transpose=True)
+        n = rp.numel() - 1
+        od = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+        m = acsr.ACSRMatrix(rp, ci)
+        hub = int(torch.argmax(od))
+        nnz_it = ci.numel()
+        run = lambda: acsr.rwr(m, od, hub, c=0.85, eps=1e-6)
+    for _ in range(max(1, args.warmup // 3)):
+        run()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    out = run()
+    torch.cuda.synchronize()
+    dt = time.perf_counter() - t0
+    it = out[2] if args.workload == "hits" else out[1]
+    if rank != 0:
+        return None
+    ms = dt * 1e3 / it
+    return {"metric": f"{args.workload.upper()} iteration GTEPS (to eps=1e-6, host convergence loop included)",
+            "value": round(nnz_it / (ms * 1e-3) / 1e9, 3), "unit": "GTEPS", "n_gpus": world, "steps": it,
+            "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{args.workload}_rmat{S}", "nnz_per_iteration": nnz_it, "iterations": it,
+                       "total_ms": round(dt * 1e3, 3)}}
+
+
 # ------------------------------------------------------------------------------ dynamic graph (C5)
 def run_dynamic(args, dev, rank, world):
     """C5: R-MAT s20 in-link pattern with slack (cap = len + max(4, len/4)); per batch of
@@ -552,6 +589,8 @@ def main():
         line = run_pagerank_dist(args, dev, rank, world)
     elif args.workload == "dynamic":
         line = run_dynamic(args, dev, rank, world)
+    elif args.workload in ("hits", "rwr"):
+        line = run_hits_rwr(args, dev, rank, world)
     else:
         line = run_acsr(args, dev, rank, world)
     if rank == 0:

@@ -135,18 +135,36 @@ typedef struct {
     const int32_t *outdeg;        /* [n_rows] out-degree of the local vertices */
     double *x_new;                /* [n_rows] PR^{k+1} */
     double *xs_next;              /* [n_rows] PR^{k+1} / outdeg (the local slice) */
-    double damping;               /* d = 0.85 */
-    double teleport;              /* (1-d)/n_global, computed once on the host */
+    double damping;               /* d = 0.85; c for RWR */
+    double teleport;              /* (1-d)/n_global, computed once on the host; 0 for RWR */
     double *delta2;               /* [1] local sum of squared differences */
+    int64_t restart;              /* RWR restart row (local index) or -1 */
+    double restart_weight;        /* added to x_new[restart]: (1-c) for RWR */
 } acsr_pr_args;
 
 acsr_status acsr_pagerank_step(const acsr_pr_args *args, cudaStream_t stream);
+
+/* The same fused step is Random Walk with Restart (Eq. 8):
+ *   r' = c (W r) + (1 - c) e_i,  W_{vu} = 1/outdeg_u on every edge u -> v (reading R5)
+ * with damping = c, teleport = 0, restart = i, restart_weight = 1 - c. */
 
 /* xs[v] = outdeg[v] > 0 ? x[v] / outdeg[v] : 0 for v < n (IEEE division).
  * Builds the first scaled vector of Alg. 5 (PR^(0) = 1/n) or of a warm
  * start. */
 acsr_status acsr_pagerank_scale(int64_t n, const double *x, const int32_t *outdeg, double *xs,
                                 cudaStream_t stream);
+
+/* ------------------------------------------------------------------------ */
+/* HITS normalisation (Eq. 5-7).  The HITS step is one acsr_spmv on the
+ * 2n x 2n pattern matrix [[0, A^T], [A, 0]] applied to v = [a; h] (Eq. 7); this call
+ * then scales each half of y = [A^T h; A a] to unit Euclidean norm (reading R6; a zero
+ * half stays zero) into v_next and writes dist2[0] = ||a' - a||^2, dist2[1] =
+ * ||h' - h||^2 (the convergence test "until both ... converge", with the
+ * Euclidean distance of P:326).  Deterministic (fixed reduction order).
+ * y, v, v_next: [2n] device doubles; dist2: [2] device. */
+size_t acsr_hits_workspace_bytes(int64_t n);
+acsr_status acsr_hits_normalize(int64_t n, const double *y, const double *v, double *v_next,
+                                double *dist2, void *ws, size_t ws_bytes, cudaStream_t stream);
 
 /* ------------------------------------------------------------------------ */
 /* Dynamic-graph update (§VII): for update i (row r = upd_rows[i],

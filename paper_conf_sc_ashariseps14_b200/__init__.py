@@ -72,14 +72,20 @@ class PrArgs(ctypes.Structure):
     _fields_ = [("n_rows", _i64), ("n_cols", _i64), ("row_begin", _vp), ("row_end", _vp),
                 ("col_idx", _vp), ("bin_rows", _vp), ("bin_offsets", _vp), ("plan_ws", _vp),
                 ("plan_ws_bytes", _sz), ("xs", _vp), ("x", _vp), ("outdeg", _vp), ("x_new", _vp),
-                ("xs_next", _vp), ("damping", _dbl), ("teleport", _dbl), ("delta2", _vp)]
+                ("xs_next", _vp), ("damping", _dbl), ("teleport", _dbl), ("delta2", _vp),
+                ("restart", _i64), ("restart_weight", _dbl)]
 
 
 _lib.acsr_pagerank_step.argtypes = [ctypes.POINTER(PrArgs), _vp]
 _lib.acsr_pagerank_step.restype = ctypes.c_int
+_lib.acsr_hits_workspace_bytes.argtypes = [_i64]
+_lib.acsr_hits_workspace_bytes.restype = _sz
+_lib.acsr_hits_normalize.argtypes = [_i64, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
+_lib.acsr_hits_normalize.restype = ctypes.c_int
 
 EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_spmv", "acsr_pagerank_step",
             "acsr_pagerank_scale", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_relayout",
+            "acsr_hits_workspace_bytes", "acsr_hits_normalize",
             "acsr_status_string", "acsr_last_error", "acsr_version")
 
 
@@ -186,8 +192,9 @@ def acsr_pagerank_scale(x, outdeg, xs=None, stream=None):
 
 def acsr_pagerank_step(row_begin, col_idx, bin_rows, bin_offsets, plan_ws, xs, x, outdeg, x_new,
                        xs_next, delta2, damping=0.85, teleport=None, n_global=None, row_end=None,
-                       stream=None):
-    """One fused PageRank step on the local rows (Alg. 5).  delta2: 1-element float64."""
+                       stream=None, restart=-1, restart_weight=0.0):
+    """One fused PageRank step on the local rows (Alg. 5).  delta2: 1-element float64.
+    With teleport=0, damping=c, restart=i, restart_weight=1-c it is an RWR step (Eq. 8)."""
     n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
     ng = xs.numel() if n_global is None else n_global
     tel = (1.0 - damping) / ng if teleport is None else teleport
@@ -201,7 +208,7 @@ def acsr_pagerank_step(row_begin, col_idx, bin_rows, bin_offsets, plan_ws, xs, x
                _dev(outdeg, torch.int32, "outdeg") if n else None,
                _dev(x_new, torch.float64, "x_new") if n else None,
                _dev(xs_next, torch.float64, "xs_next") if n else None, float(damping), float(tel),
-               _dev(delta2, torch.float64, "delta2"))
+               _dev(delta2, torch.float64, "delta2"), int(restart), float(restart_weight))
     _check(_lib.acsr_pagerank_step(ctypes.byref(a), _stream(stream)), "acsr_pagerank_step")
     return x_new, xs_next, delta2
 
@@ -254,8 +261,24 @@ def acsr_relayout(old_begin, old_end, old_col, old_val, new_begin, new_end, new_
     return new_end
 
 
+def acsr_hits_workspace_bytes(n: int) -> int:
+    return int(_lib.acsr_hits_workspace_bytes(int(n)))
+
+
+def acsr_hits_normalize(y, v, v_next, dist2, ws=None, stream=None):
+    """HITS normalisation of y = [A^T h; A a] into v_next (Eq. 5-7, reading R6)."""
+    n = y.numel() // 2
+    if ws is None:
+        ws = torch.empty(acsr_hits_workspace_bytes(n), dtype=torch.uint8, device=y.device)
+    _check(_lib.acsr_hits_normalize(n, _dev(y, torch.float64, "y"), _dev(v, torch.float64, "v"),
+                                    _dev(v_next, torch.float64, "v_next"), _dev(dist2, torch.float64, "dist2"),
+                                    _dev(ws, torch.uint8, "ws"), ws.numel(), _stream(stream)),
+           "acsr_hits_normalize")
+    return v_next, dist2
+
+
 def version() -> int:
     return int(_lib.acsr_version())
 
 
-from .matrix import ACSRMatrix, pagerank, spmv_from_host  # noqa: E402
+from .matrix import ACSRMatrix, hits, hits_matrix, pagerank, rwr, spmv_from_host  # noqa: E402

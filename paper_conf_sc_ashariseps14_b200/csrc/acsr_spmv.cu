@@ -61,6 +61,8 @@ struct SpmvArgs {
     double *__restrict__ xs_next;
     double damping, teleport;
     double *delta2;
+    int64_t restart;
+    double restart_weight;
 };
 
 // ----------------------------------------------------------------- PTX helpers
@@ -315,7 +317,7 @@ struct Kern {
     static __device__ __forceinline__ void finish(const A &a, int r, double s, Fix128 &d2)
     {
         if (PR) {
-            const double xn = a.teleport + a.damping * s;
+            const double xn = a.teleport + a.damping * s + (r == a.restart ? a.restart_weight : 0.0);
             a.x_new[r] = xn;
             const int od = __ldg(a.outdeg + r);
             a.xs_next[r] = od > 0 ? xn / (double)od : 0.0;
@@ -825,6 +827,7 @@ extern "C" acsr_status acsr_pagerank_step(const acsr_pr_args *p, cudaStream_t st
     a.bin_rows = p->bin_rows; a.hdr = (PlanHeader *)p->plan_ws;
     a.x_old = p->x; a.outdeg = p->outdeg; a.x_new = p->x_new; a.xs_next = p->xs_next;
     a.damping = p->damping; a.teleport = p->teleport; a.delta2 = p->delta2;
+    a.restart = p->restart; a.restart_weight = p->restart_weight;
     dispatch<double, true>(a, stream);
     return acsr_check_launch("acsr_pagerank_step");
 }

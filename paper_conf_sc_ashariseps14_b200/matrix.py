@@ -9,8 +9,8 @@ from __future__ import annotations
 
 import torch
 
-from . import (acsr_bin, acsr_bin_workspace_bytes, acsr_pagerank_scale, acsr_pagerank_step,
-               acsr_relayout, acsr_spmv, acsr_update_edges)
+from . import (acsr_bin, acsr_bin_workspace_bytes, acsr_hits_normalize, acsr_hits_workspace_bytes,
+               acsr_pagerank_scale, acsr_pagerank_step, acsr_relayout, acsr_spmv, acsr_update_edges)
 
 
 class ACSRMatrix:
@@ -114,3 +114,72 @@ def pagerank(m: ACSRMatrix, outdeg, x0=None, damping=0.85, eps=1e-6, max_iter=10
         if delta2 ** 0.5 <= eps:
             break
     return x, it, delta2
+
+
+def rwr(m: ACSRMatrix, outdeg, restart: int, c=0.85, eps=1e-6, max_iter=1000, r0=None, stream=None):
+    """Random Walk with Restart (Eq. 8; reading R5) on the in-link pattern m:
+    r' = c (W r) + (1-c) e_restart, r^0 = e_restart.  One fused acsr_pagerank_step per
+    iteration (teleport 0, restart weight 1-c).  Returns (r, iterations, delta2)."""
+    n = m.n_rows
+    dev = m.row_begin.device
+    if r0 is None:
+        r = torch.zeros(n, dtype=torch.float64, device=dev)
+        r[restart] = 1.0
+    else:
+        r = r0.clone()
+    rs = acsr_pagerank_scale(r, outdeg, stream=stream)
+    r_new, rs_next = torch.empty_like(r), torch.empty_like(r)
+    d2 = torch.zeros(1, dtype=torch.float64, device=dev)
+    it, delta2 = 0, float("inf")
+    while it < max_iter:
+        acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, rs, r, outdeg,
+                           r_new, rs_next, d2, c, 0.0, n, m.row_end, stream, restart=restart,
+                           restart_weight=1.0 - c)
+        r, r_new = r_new, r
+        rs, rs_next = rs_next, rs
+        it += 1
+        delta2 = float(d2.item())
+        if delta2 ** 0.5 <= eps:
+            break
+    return r, it, delta2
+
+
+def hits_matrix(out_ptr, out_col, n=None):
+    """The 2n x 2n pattern CSR [[0, A^T], [A, 0]] of Eq. 7 from the out-link CSR of A
+    (input construction: torch sort/scan on the device)."""
+    n = out_ptr.numel() - 1 if n is None else n
+    dev = out_ptr.device
+    ln = (out_ptr[1:] - out_ptr[:-1]).long()
+    src = torch.repeat_interleave(torch.arange(n, device=dev), ln)
+    dst = out_col.long()
+    order = torch.sort(dst * n + src).indices  # A^T rows = targets, sorted by source
+    in_ptr = torch.zeros(n + 1, dtype=torch.int64, device=dev)
+    in_ptr[1:] = torch.cumsum(torch.bincount(dst, minlength=n), 0)
+    in_col = src[order]
+    nnz = out_col.numel()
+    row_ptr = torch.cat([in_ptr, out_ptr[1:].long() + nnz]).to(torch.int32)
+    col = torch.cat([in_col + n, out_col.long()]).to(torch.int32)
+    return row_ptr, col
+
+
+def hits(out_ptr, out_col, eps=1e-6, max_iter=1000, stream=None):
+    """HITS (Eq. 5-7; reading R6): one acsr_spmv on [[0, A^T], [A, 0]] per
+    iteration plus acsr_hits_normalize.  a^0 = h^0 = 1/|V|.  Returns (a, h, iters)."""
+    n = out_ptr.numel() - 1
+    dev = out_ptr.device
+    rp, col = hits_matrix(out_ptr, out_col, n)
+    B = ACSRMatrix(rp, col, None, n_cols=2 * n)
+    v = torch.full((2 * n,), 1.0 / n, dtype=torch.float64, device=dev)
+    y, vn = torch.empty_like(v), torch.empty_like(v)
+    d2 = torch.zeros(2, dtype=torch.float64, device=dev)
+    ws = torch.empty(acsr_hits_workspace_bytes(n), dtype=torch.uint8, device=dev)
+    it = 0
+    while it < max_iter:
+        B.spmv(v, y, stream)
+        acsr_hits_normalize(y, v, vn, d2, ws, stream)
+        v, vn = vn, v
+        it += 1
+        da, dh = (float(t) for t in d2.cpu())
+        if da ** 0.5 <= eps and dh ** 0.5 <= eps:
+            break
+    return v[:n], v[n:], it

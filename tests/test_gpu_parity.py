@@ -483,3 +483,42 @@ def test_capacity_reject_then_grow_and_retry(acsr, cuda):
     y_ref, den = oracle.spmv(m.row_begin.cpu().numpy(), m.col_idx.cpu().numpy(), m.values.cpu().numpy(),
                              x.numpy(), row_end=m.row_end.cpu().numpy())
     check_spmv(y, y_ref, den, torch.float64)
+
+
+# ------------------------------------------------------------------------------ RWR / HITS
+def test_rwr_parity(acsr, cuda):
+    rp, ci, od, n = _inlink(14, cuda)
+    i = int(np.argmax(od.numpy()))  # restart at a hub
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda))
+    r, it, d2 = acsr.rwr(m, od.to(cuda), i, c=0.85, eps=1e-6)
+    r_ref, it_ref, _ = oracle.rwr(rp.numpy(), ci.numpy(), od.numpy(), i, c=0.85, eps=1e-6)
+    assert abs(it - it_ref) <= 1
+    if it != it_ref:
+        r_ref, _, _ = oracle.rwr(rp.numpy(), ci.numpy(), od.numpy(), i, c=0.85, eps=0.0, max_iter=it)
+    assert np.all(np.abs(r.cpu().numpy() - r_ref) <= 1e-11 * r_ref + 1e-18)
+    # one step from the same iterate meets the fp64 step bar
+    rr = synth.vector(n, 9).abs().numpy()
+    rs = torch.where(od > 0, torch.from_numpy(rr) / od.clamp(min=1), torch.zeros(n, dtype=torch.float64))
+    rn, rsn = torch.empty(n, dtype=torch.float64, device=cuda), torch.empty(n, dtype=torch.float64, device=cuda)
+    d2 = torch.zeros(1, dtype=torch.float64, device=cuda)
+    acsr.acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, rs.to(cuda),
+                            torch.from_numpy(rr).to(cuda), od.to(cuda), rn, rsn, d2, 0.85, 0.0, n,
+                            restart=i, restart_weight=0.15)
+    rn_ref, d2_ref = oracle.rwr_step(rp.numpy(), ci.numpy(), od.numpy(), rr, 0.85, i)
+    _, den = oracle.spmv(rp.numpy(), ci.numpy(), None, rs.numpy())
+    assert np.all(np.abs(rn.cpu().numpy() - rn_ref) <= 1e-12 * 0.85 * den + 2.3e-16 * np.abs(rn_ref))
+    assert float(d2.item()) == pytest.approx(d2_ref, rel=1e-9)
+
+
+@pytest.mark.parametrize("scale", [12, 16])
+def test_hits_parity(acsr, cuda, scale):
+    rp, ci = synth.rmat_csr(scale)  # rows = sources: the adjacency A of Eq. 5-6
+    n = rp.numel() - 1
+    a, h, it = acsr.hits(rp.to(cuda), ci.to(cuda), eps=1e-6)
+    rpT, ciT = synth.rmat_csr(scale, transpose=True)
+    a_ref, h_ref, it_ref = oracle.hits(rp.numpy(), ci.numpy(), rpT.numpy(), ciT.numpy(), eps=1e-6)
+    assert abs(it - it_ref) <= 1
+    if it != it_ref:
+        a_ref, h_ref, _ = oracle.hits(rp.numpy(), ci.numpy(), rpT.numpy(), ciT.numpy(), eps=0.0, max_iter=it)
+    assert np.allclose(a.cpu().numpy(), a_ref, rtol=1e-9, atol=1e-15)
+    assert np.allclose(h.cpu().numpy(), h_ref, rtol=1e-9, atol=1e-15)

@@ -299,6 +299,13 @@ def run_pagerank(args, dev, rank, world):
     rp, ci = synth.rmat_csr(S, seed=S + 1000 * rank, device=dev, transpose=True)
     n, nnz = rp.numel() - 1, ci.numel()
     outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    t_relabel = None
+    if args.relabel:
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        rp, ci, outdeg, _ = acsr.degree_relabel(rp, ci, outdeg)
+        torch.cuda.synchronize()
+        t_relabel = time.perf_counter() - t0
     n_nd = int((outdeg > 0).sum())
     m = acsr.ACSRMatrix(rp, ci)
     torch.cuda.synchronize()
@@ -348,7 +355,9 @@ def run_pagerank(args, dev, rank, world):
             "value": round(nnz * world / (ms * 1e-3) / 1e9, 3), "unit": "GTEPS", "n_gpus": world, "steps": K,
             "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"pagerank_rmat{S}_inlink", "n_rows": n, "nnz": nnz, "non_dangling": n_nd,
+            "config": {"workload": f"pagerank_rmat{S}_inlink" + ("_degree_relabelled" if args.relabel else ""),
+                       "n_rows": n, "nnz": nnz, "non_dangling": n_nd,
+                       "relabel_s": None if t_relabel is None else round(t_relabel, 3),
                        "l2": "not flushed (iterative use); x = %d MB" % (8 * n >> 20),
                        "parallelism": "independent replica per rank" if world > 1 else "1 GPU"},
             "breakdown": {"t_bin_ms": round(t_bin, 4), "cold_iterations": it, "final_delta": dd ** 0.5,
@@ -528,6 +537,71 @@ def run_dynamic(args, dev, rank, world):
             "gpu_launches": None}
 
 
+def run_dynamic_mixed(args, dev, rank, world):
+    """The paper's dynamic experiment: PageRank converges, then per
+    epoch 10 % of the rows change (each column deleted or another added with probability
+    1/2), only the change list goes to the device, the matrix is updated in place and
+    re-binned, PageRank warm-starts from the previous vector; 10 epochs."""
+    import paper_conf_sc_ashariseps14_b200 as acsr
+
+    S = args.scale or 20
+    E = args.batches or 10
+    rp, ci = synth.rmat_csr(S, device=dev, transpose=True)
+    n = rp.numel() - 1
+    rb, re, cap, col, _ = synth.with_slack(rp, ci, frac=1)  # about 2x slack (reading R3)
+    outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    m = acsr.ACSRMatrix(rb, col, None, row_end=re, row_cap=cap, nnz_max=col.numel())
+    t0 = time.perf_counter()
+    x, it0, _ = acsr.pagerank(m, outdeg, eps=1e-6)
+    torch.cuda.synchronize()
+    t_cold = time.perf_counter() - t0
+    st = torch.empty(2, dtype=torch.int32, device=dev)
+    uws = torch.empty(acsr.acsr_update_workspace_bytes(1 << 22), dtype=torch.uint8, device=dev)
+    rec, relayouts = [], 0
+    for ep in range(E):
+        ch = synth.mixed_epoch(m.row_begin, m.row_end, m.col_idx, n, 0.10, 5000 + ep)
+        pinned = {k: torch.from_numpy(v).pin_memory() for k, v in ch.items()}
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+        torch.cuda.synchronize()
+        ev[0].record()
+        chd = {k: v.to(dev, non_blocking=True) for k, v in pinned.items()}
+        ev[1].record()
+        m.update(chd, outdeg=outdeg, status=st, ws=uws)
+        ev[2].record()
+        m.rebin()
+        ev[3].record()
+        torch.cuda.synchronize()
+        while st.cpu().tolist() != [0, -1]:
+            assert int(st[0]) == acsr.ACSR_ERR_CAPACITY and relayouts < 20, st
+            m.grow()
+            m.update(chd, outdeg=outdeg, status=st, ws=uws)
+            m.rebin()
+            torch.cuda.synchronize()
+            relayouts += 1
+        t1 = time.perf_counter()
+        x, it, _ = acsr.pagerank(m, outdeg, x0=x, eps=1e-6)
+        torch.cuda.synchronize()
+        t_pr = time.perf_counter() - t1
+        rec.append([ev[0].elapsed_time(ev[1]), ev[1].elapsed_time(ev[2]), ev[2].elapsed_time(ev[3]),
+                    t_pr * 1e3, it, int(ch["del_cols"].size), int(ch["ins_cols"].size)])
+    r = np.array(rec)
+    if rank != 0:
+        return None
+    return {"metric": "dynamic PageRank epoch (paper §VII): update + re-bin ms, warm iterations",
+            "value": round(float((r[:, 1] + r[:, 2]).mean()), 5), "unit": "ms", "n_gpus": world,
+            "steps": E, "warmup": 0, "ms_per_step": round(float(r[:, :4].sum(1).mean()), 4),
+            "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": f"dynamic_mixed_rmat{S}_10pct_rows_{E}_epochs", "n_rows": n,
+                       "cold_iterations": it0, "cold_pagerank_ms": round(t_cold * 1e3, 3)},
+            "breakdown": {"t_h2d_ms": round(float(r[:, 0].mean()), 5), "t_update_ms": round(float(r[:, 1].mean()), 5),
+                          "t_bin_ms": round(float(r[:, 2].mean()), 5),
+                          "pagerank_warm_ms": round(float(r[:, 3].mean()), 4),
+                          "warm_iterations": [int(v) for v in r[:, 4]],
+                          "deleted_per_epoch": round(float(r[:, 5].mean()), 1),
+                          "inserted_per_epoch": round(float(r[:, 6].mean()), 1), "relayouts": relayouts}}
+
+
 # ------------------------------------------------------------------------------ reference arm
 def run_reference(args, dev):
     """The oracle as it stands (plain C, 1 core) on the same workload: bins (O3) + plain SpMV
@@ -568,6 +642,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--scale", type=int, default=None, help="R-MAT scale for pagerank/dynamic")
     ap.add_argument("--batches", type=int, default=None, help="dynamic: number of insertion batches")
+    ap.add_argument("--relabel", action="store_true", help="pagerank: degree-ordered vertex relabelling")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -589,6 +664,8 @@ def main():
         line = run_pagerank_dist(args, dev, rank, world)
     elif args.workload == "dynamic":
         line = run_dynamic(args, dev, rank, world)
+    elif args.workload == "dynamic_mixed":
+        line = run_dynamic_mixed(args, dev, rank, world)
     elif args.workload in ("hits", "rwr"):
         line = run_hits_rwr(args, dev, rank, world)
     else:

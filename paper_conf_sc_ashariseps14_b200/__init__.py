@@ -281,4 +281,4 @@ def version() -> int:
     return int(_lib.acsr_version())
 
 
-from .matrix import ACSRMatrix, hits, hits_matrix, pagerank, rwr, spmv_from_host  # noqa: E402
+from .matrix import ACSRMatrix, degree_relabel, hits, hits_matrix, pagerank, rwr, spmv_from_host  # noqa: E402

@@ -154,6 +154,7 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
         hdr->work_ctr = 0;
         hdr->exit_ticket = 0;
         hdr->d2_hi = 0;
+        hdr->d2_mid = 0;
         hdr->d2_lo = 0;
         hdr->scan_ticket = 0;
         (void)n_rows;

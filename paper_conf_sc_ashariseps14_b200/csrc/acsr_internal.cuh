@@ -71,7 +71,7 @@ struct PlanHeader {
     int32_t xc_valid;       // 1 if the x-cache table was built (col_idx given)
     int32_t xc_stride;      // sampling stride used for the counts
     int64_t n_cols;
-    uint64_t d2_hi, d2_lo;  // exact fixed-point Delta^2 accumulator (PageRank)
+    uint64_t d2_hi, d2_mid, d2_lo;  // exact 192-bit fixed-point Delta^2 accumulator (PageRank/RWR)
     int64_t off_units, off_partial, off_ticket, off_xc_vote, off_xc_tag, off_xc_val;
     int32_t totals[NBINS + 2 + 2];  // per scan row totals (bins, light units, heavy units)
 };

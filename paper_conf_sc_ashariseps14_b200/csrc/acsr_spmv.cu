@@ -104,31 +104,36 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t phase)
     }
 }
 
-// 128-bit fixed point, LSB = 2^-120, for exact order-independent sums of
-// non-negative doubles < 2^8 (PageRank Delta^2 <= 2).
-struct Fix128 {
-    uint64_t hi, lo;  // value = hi * 2^-56 + lo * 2^-120
+// 192-bit fixed point (value = hi + mid * 2^-64 + lo * 2^-128) for exact,
+// order-independent sums of non-negative doubles below 2^64: Delta^2 of any step is
+// deterministic under dynamic scheduling.  Each term is split exactly (53-bit mantissa)
+// and truncated below 2^-128.
+struct Fix192 {
+    uint64_t hi, mid, lo;
 };
 
-__device__ __forceinline__ void fix_add(Fix128 &a, double d)
-{
-    if (!(d > 0.0)) return;
-    if (d >= 256.0) d = 255.99999999999997;  // saturate (never reached for PageRank)
-    const double hs = d * 72057594037927936.0;  // 2^56 (exact scaling)
-    const double hf = floor(hs);
-    const uint64_t h = (uint64_t)hf;
-    const double rem = hs - hf;                                     // exact
-    const uint64_t l = (uint64_t)(rem * 18446744073709551616.0);   // * 2^64, truncated
-    const uint64_t lo = a.lo + l;
-    a.hi += h + (lo < a.lo ? 1u : 0u);
-    a.lo = lo;
-}
-
-__device__ __forceinline__ void fix_merge(Fix128 &a, uint64_t hi, uint64_t lo)
+__device__ __forceinline__ void fix_merge(Fix192 &a, uint64_t hi, uint64_t mid, uint64_t lo)
 {
     const uint64_t nlo = a.lo + lo;
-    a.hi += hi + (nlo < a.lo ? 1u : 0u);
+    const uint64_t c1 = nlo < a.lo ? 1u : 0u;
+    const uint64_t m1 = a.mid + mid;
+    const uint64_t c2a = m1 < a.mid ? 1u : 0u;
+    const uint64_t m2 = m1 + c1;
+    const uint64_t c2b = m2 < m1 ? 1u : 0u;
     a.lo = nlo;
+    a.mid = m2;
+    a.hi += hi + c2a + c2b;
+}
+
+__device__ __forceinline__ void fix_add(Fix192 &a, double d)
+{
+    if (!(d > 0.0)) return;
+    if (d >= 18446744073709549568.0) d = 18446744073709549568.0;  // < 2^64 (saturate)
+    const double hf = floor(d);
+    const double r1 = (d - hf) * 18446744073709551616.0;  // exact: * 2^64
+    const double mf = floor(r1);
+    const double r2 = (r1 - mf) * 18446744073709551616.0;
+    fix_merge(a, (uint64_t)hf, (uint64_t)mf, (uint64_t)floor(r2));
 }
 
 // ----------------------------------------------------------------- load flavours
@@ -314,7 +319,7 @@ struct Kern {
     }
 
     // write the row result (or the PageRank epilogue for local row r)
-    static __device__ __forceinline__ void finish(const A &a, int r, double s, Fix128 &d2)
+    static __device__ __forceinline__ void finish(const A &a, int r, double s, Fix192 &d2)
     {
         if (PR) {
             const double xn = a.teleport + a.damping * s + (r == a.restart ? a.restart_weight : 0.0);
@@ -330,7 +335,7 @@ struct Kern {
 
     // bins 1..6: W = 2^{b-1} lanes per row, each lane <= 2 elements (Alg. 2)
     template <int W>
-    static __device__ __forceinline__ void light_sub(const A &a, int start, int cnt, int lane, Fix128 &d2)
+    static __device__ __forceinline__ void light_sub(const A &a, int start, int cnt, int lane, Fix192 &d2)
     {
         constexpr int RPP = 32 / W;           // rows per pass
         constexpr int U = (W >= 16) ? 2 : 4;  // passes in flight
@@ -456,7 +461,7 @@ struct Kern {
     }
 
     // bins 7..10: a warp per row
-    static __device__ __forceinline__ void light_warp(const A &a, int start, int cnt, int lane, Fix128 &d2)
+    static __device__ __forceinline__ void light_warp(const A &a, int start, int cnt, int lane, Fix192 &d2)
     {
         const int myr = lane < cnt ? __ldg(a.bin_rows + start + lane) : 0;
         int mb = 0, me = 0;
@@ -470,13 +475,13 @@ struct Kern {
         }
     }
 
-    static __device__ __forceinline__ void empty_rows(const A &a, int start, int cnt, int lane, Fix128 &d2)
+    static __device__ __forceinline__ void empty_rows(const A &a, int start, int cnt, int lane, Fix192 &d2)
     {
         for (int i = lane; i < cnt; i += 32) finish(a, __ldg(a.bin_rows + start + i), 0.0, d2);
     }
 
     // one HEAVY_CHUNK chunk of a long row; last arriver combines in chunk order
-    static __device__ __forceinline__ void heavy(const A &a, int u, int r, int c, int lane, Fix128 &d2)
+    static __device__ __forceinline__ void heavy(const A &a, int u, int r, int c, int lane, Fix192 &d2)
     {
         int beg, end;
         row_bounds(a, r, beg, end);
@@ -507,7 +512,7 @@ struct Kern {
         }
     }
 
-    static __device__ __forceinline__ void unit(const A &a, int u, int lane, Fix128 &d2)
+    static __device__ __forceinline__ void unit(const A &a, int u, int lane, Fix192 &d2)
     {
         const int2 d = __ldg(a.units + u);
         const uint32_t y = (uint32_t)d.y;
@@ -571,7 +576,7 @@ spmv_kernel(SpmvArgs<V> a)
         a.xval = sval;
         a.xtag = stag;
     }
-    Fix128 d2{0, 0};
+    Fix192 d2{0, 0, 0};
 #if ACSR_SCHED_STATIC
     for (int u = gw; u < n_units; u += nw) K::unit(a, u, lane, d2);
 #else
@@ -585,18 +590,22 @@ spmv_kernel(SpmvArgs<V> a)
     }
 #endif
     if (PR) {
-        // exact fixed-point warp sum, then two 64-bit atomics per warp
+        // exact fixed-point warp sum, then three 64-bit atomics per warp with carries
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
             const uint64_t h = __shfl_xor_sync(0xffffffffu, d2.hi, o);
+            const uint64_t m = __shfl_xor_sync(0xffffffffu, d2.mid, o);
             const uint64_t l = __shfl_xor_sync(0xffffffffu, d2.lo, o);
-            fix_merge(d2, h, l);
+            fix_merge(d2, h, m, l);
         }
-        if (lane == 0 && (d2.hi | d2.lo)) {
-            const unsigned long long old =
-                atomicAdd((unsigned long long *)&hdr->d2_lo, (unsigned long long)d2.lo);
-            const uint64_t carry = (old + d2.lo < old) ? 1u : 0u;
-            atomicAdd((unsigned long long *)&hdr->d2_hi, (unsigned long long)(d2.hi + carry));
+        if (lane == 0 && (d2.hi | d2.mid | d2.lo)) {
+            const unsigned long long ol = atomicAdd((unsigned long long *)&hdr->d2_lo, (unsigned long long)d2.lo);
+            const uint64_t c1 = (ol + d2.lo < ol) ? 1u : 0u;
+            const uint64_t madd = d2.mid + c1;
+            const uint64_t cm = (madd < d2.mid) ? 1u : 0u;  // d2.mid == 2^64-1 and c1
+            const unsigned long long om = atomicAdd((unsigned long long *)&hdr->d2_mid, (unsigned long long)madd);
+            const uint64_t c2 = (om + madd < om) ? 1u : 0u;
+            atomicAdd((unsigned long long *)&hdr->d2_hi, (unsigned long long)(d2.hi + c2 + cm));
         }
     }
     // last warp out publishes Delta^2 and resets the counters for the next call
@@ -606,9 +615,11 @@ spmv_kernel(SpmvArgs<V> a)
             __threadfence();
             if (PR) {
                 const uint64_t hi = *(volatile uint64_t *)&hdr->d2_hi;
+                const uint64_t mid = *(volatile uint64_t *)&hdr->d2_mid;
                 const uint64_t lo = *(volatile uint64_t *)&hdr->d2_lo;
-                *a.delta2 = (double)hi * 1.3877787807814457e-17 + (double)lo * 7.52316384526264e-37;
+                *a.delta2 = (double)hi + ((double)mid + (double)lo * 5.421010862427522e-20) * 5.421010862427522e-20;
                 hdr->d2_hi = 0;
+                hdr->d2_mid = 0;
                 hdr->d2_lo = 0;
             }
             hdr->work_ctr = 0;

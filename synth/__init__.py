@@ -339,3 +339,43 @@ def mixed_batches(row_ptr: np.ndarray, col: np.ndarray, n_cols: int, frac_rows: 
             keep = np.setdiff1d(cur, dels, assume_unique=False)
             cols[r] = np.concatenate([cur[np.isin(cur, keep)], adds])
         yield encode_changes(n, np.asarray(ir), np.asarray(ic), np.asarray(dr), np.asarray(dc))
+
+
+def mixed_epoch(row_begin: torch.Tensor, row_end: torch.Tensor, col: torch.Tensor, n_cols: int,
+                frac_rows: float, seed: int):
+    """Paper-shaped change list (reading R3) generated on the graph's device from the
+    CURRENT live entries of a slack CSR: rows are picked with probability frac_rows; scanning
+    a picked row's columns, each column is deleted or "another column" (uniform, not already
+    in the row, not a duplicate) is added, each with probability 1/2.  Returns the change
+    dict (host int32 numpy arrays, "in CSR format")."""
+    dev = row_begin.device
+    n = row_begin.numel()
+    rid = torch.arange(n, device=dev, dtype=torch.int64)
+    pick = uniform53(hash64(seed, 41, rid)) < frac_rows
+    ln = (row_end - row_begin).long()
+    lnp = torch.where(pick, ln, torch.zeros_like(ln))
+    rows = torch.repeat_interleave(rid, lnp)
+    start = torch.repeat_interleave(row_begin.long(), lnp)
+    first = torch.zeros(n + 1, dtype=torch.int64, device=dev)
+    first[1:] = torch.cumsum(lnp, 0)
+    pos = torch.arange(rows.numel(), device=dev, dtype=torch.int64) - first[rows]
+    cols = col[(start + pos)].long()
+    key_e = rows * (1 << 32) + pos
+    coin = uniform53(hash64(seed, 43, key_e)) < 0.5
+    del_r, del_c = rows[coin], cols[coin]
+    add_r = rows[~coin]
+    add_c = _srl(hash64(seed, 45, key_e[~coin]), 1) % n_cols
+    # drop adds already in the row (live entries) and duplicate adds
+    live_r = torch.repeat_interleave(rid, ln)
+    lfirst = torch.zeros(n + 1, dtype=torch.int64, device=dev)
+    lfirst[1:] = torch.cumsum(ln, 0)
+    lpos = torch.arange(live_r.numel(), device=dev, dtype=torch.int64) - lfirst[live_r]
+    live_c = col[(torch.repeat_interleave(row_begin.long(), ln) + lpos)].long()
+    live_keys = torch.sort(live_r * n_cols + live_c).values
+    ak = torch.unique(add_r * n_cols + add_c)
+    p = torch.searchsorted(live_keys, ak)
+    present = (p < live_keys.numel()) & (live_keys[torch.clamp(p, max=max(live_keys.numel() - 1, 0))] == ak)
+    ak = ak[~present]
+    dk = torch.unique(del_r * n_cols + del_c)
+    akh, dkh = ak.cpu().numpy(), dk.cpu().numpy()
+    return encode_changes(n, akh // n_cols, akh % n_cols, dkh // n_cols, dkh % n_cols)

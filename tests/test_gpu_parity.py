@@ -522,3 +522,40 @@ def test_hits_parity(acsr, cuda, scale):
         a_ref, h_ref, _ = oracle.hits(rp.numpy(), ci.numpy(), rpT.numpy(), ciT.numpy(), eps=0.0, max_iter=it)
     assert np.allclose(a.cpu().numpy(), a_ref, rtol=1e-9, atol=1e-15)
     assert np.allclose(h.cpu().numpy(), h_ref, rtol=1e-9, atol=1e-15)
+
+
+def test_degree_relabel_pagerank_equivalent(acsr, cuda):
+    # P A P^T relabelling (degree order) is a pure renumbering: PR'[perm[v]] == PR[v]
+    rp, ci, od, n = _inlink(14, cuda)
+    rp2, ci2, od2, perm = acsr.degree_relabel(rp.to(cuda), ci.to(cuda), od.to(cuda))
+    assert torch.all(od2[:-1] >= od2[1:])
+    m = acsr.ACSRMatrix(rp2, ci2)
+    x2, it2, _ = acsr.pagerank(m, od2, eps=1e-6)
+    x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)
+    assert abs(it2 - it_ref) <= 1
+    if it2 != it_ref:
+        x_ref, _, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=0.0, max_iter=it2)
+    back = x2[perm].cpu().numpy()
+    assert np.all(np.abs(back - x_ref) <= 1e-11 * x_ref + 1e-18)
+
+
+def test_paper_epoch_update_bitwise(acsr, cuda):
+    # P:337 paper-shaped epoch generated on the device from the live graph (synth.mixed_epoch)
+    n, rb, re, cap, col, val, od, rp, ci = _slack_graph(14, frac=1)
+    m = acsr.ACSRMatrix(rb.to(cuda), col.to(cuda), None, row_end=re.to(cuda), row_cap=cap.to(cuda),
+                        nnz_max=col.numel())
+    odd = od.to(cuda)
+    re_h, col_h, od_h = re.numpy().copy(), col.numpy().copy(), od.numpy().copy()
+    for ep in range(3):
+        ch = synth.mixed_epoch(m.row_begin, m.row_end, m.col_idx, n, 0.1, 77 + ep)
+        code, _ = oracle.update(n, rb.numpy(), re_h, cap.numpy(), col_h, None, ch["upd_rows"], ch["del_ptr"],
+                                ch["del_cols"], ch["ins_ptr"], ch["ins_cols"], None, od_h)
+        st = m.update(_dev_changes(ch, cuda), outdeg=odd)
+        torch.cuda.synchronize()
+        assert st.cpu().tolist() == [code, -1 if code == 0 else st.cpu().tolist()[1]]
+        if code != 0:
+            break
+        assert np.array_equal(m.row_end.cpu().numpy(), re_h)
+        live = np.concatenate([np.arange(b, e) for b, e in zip(rb.numpy(), re_h)])
+        assert np.array_equal(m.col_idx.cpu().numpy()[live], col_h[live])
+        assert np.array_equal(odd.cpu().numpy(), od_h)

@@ -32,6 +32,14 @@
 
 #include "acsr_internal.cuh"
 
+#ifndef ACSR_BRANCHY_SUB
+#define ACSR_BRANCHY_SUB 0  // 1: branchy element loads in the Alg. 2 sub-warp path (A/B builds)
+#endif
+#ifndef ACSR_NO_VEC
+#define ACSR_NO_VEC 0  // 1: never use the 128-bit vector path (A/B builds)
+#endif
+
+
 namespace acsr {
 
 template <typename V>
@@ -356,8 +364,15 @@ struct Kern {
 #pragma unroll
             for (int u = 0; u < U; u++) {
                 const int k0 = beg[u] + li, k1 = k0 + W;
+#if ACSR_BRANCHY_SUB
+                double sacc = 0.0;
+                if (k0 < end[u]) sacc = prod(a, k0);
+                if (k1 < end[u]) sacc += prod(a, k1);
+                acc[u] = sacc;
+#else
                 acc[u] = fmacp(a, k0 < end[u], k0, 0.0);
                 acc[u] = fmacp(a, k1 < end[u], k1, acc[u]);
+#endif
             }
 #pragma unroll
             for (int u = 0; u < U; u++) {
@@ -749,7 +764,7 @@ static int xcache_bits()
 template <typename V, bool PR>
 static int dispatch(SpmvArgs<V> a, cudaStream_t s)
 {
-    a.vph = vec_phase<V>(a.col, a.val);
+    a.vph = ACSR_NO_VEC ? -1 : vec_phase<V>(a.col, a.val);
     a.xc_bits = xcache_bits();
     if (xcache_enabled() && a.x != nullptr) {
         xc_fill_kernel<V><<<((1 << a.xc_bits) + 255) / 256, 256, 0, s>>>(a.hdr, a.x, a.xc_bits,

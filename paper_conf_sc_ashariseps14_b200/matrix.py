@@ -50,11 +50,14 @@ class ACSRMatrix:
                                  changes.get("del_cols"), outdeg, status, ws, stream=stream)
 
     def grow(self, min_slack=8, frac=2, stream=None):
-        """Re-lay the slack CSR out with cap_r = len_r + max(min_slack, ceil(len_r / frac))
-        (reading R4: after a CAPACITY rejection), then re-bin."""
+        """Re-lay the slack CSR out with more room (reading R4: after a CAPACITY rejection):
+        cap_r <- max(cap_r + max(min_slack, ceil(cap_r / frac)), len_r + max(min_slack,
+        ceil(len_r / frac))) -- every row grows, so repeated rejections always progress.
+        Then re-bin."""
         assert self.row_end is not None
         ln = (self.row_end - self.row_begin).to(torch.int64)
-        cap = torch.maximum(self.row_cap.to(torch.int64),
+        old = self.row_cap.to(torch.int64)
+        cap = torch.maximum(old + torch.clamp((old + frac - 1) // frac, min=min_slack),
                             ln + torch.clamp((ln + frac - 1) // frac, min=min_slack))
         nb = torch.zeros_like(cap)
         nb[1:] = torch.cumsum(cap, 0)[:-1]

@@ -16,6 +16,9 @@ for v in "$@"; do
     t256) build t256 -DACSR_SPMV_THREADS=256 ;;
     t512) build t512 -DACSR_SPMV_THREADS=512 ;;
     t256st) build t256st -DACSR_SPMV_THREADS=256 -DACSR_SCHED_STATIC=1 ;;
+    nv) build nv -DACSR_NO_VEC=1 ;;
+    br) build br -DACSR_BRANCHY_SUB=1 ;;
+    nvbr) build nvbr -DACSR_NO_VEC=1 -DACSR_BRANCHY_SUB=1 ;;
   esac
 done
 wait

@@ -11,12 +11,16 @@
 //   3. bin_scatter one CTA per tile: stable ranks (warp __match_any_sync + per-warp
 //                  counts scanned across warps, 16 rounds of 256 rows in row
 //                  order) -> bin_rows; then writes the tile's work units.
+#include <cooperative_groups.h>
 #include <cuda_runtime.h>
+#include <stddef.h>
 #include <stdlib.h>
 
 #include "acsr_internal.cuh"
 
 namespace acsr {
+
+namespace cg = cooperative_groups;
 
 template <bool HAS_END>
 __device__ __forceinline__ int row_length(const int32_t *__restrict__ rb,
@@ -27,19 +31,37 @@ __device__ __forceinline__ int row_length(const int32_t *__restrict__ rb,
     return e - b;
 }
 
+// Shared scratch of the binning phases (one union per CTA; the fused kernel runs the
+// phases back to back in the same CTA).
+struct BinSmem {
+    // count
+    int hist[NBINS];
+    int heavy;
+    // scan
+    int warp_sums[32];
+    int carry;
+    int is_last;
+    // scatter
+    int run[NBINS];
+    int wcnt[BIN_THREADS / 32][NBINS];
+    int wbase[BIN_THREADS / 32][NBINS];
+    int seg[NBINS];
+    int hw[BIN_THREADS / 32];
+    int heavy_run;
+    int upre[LIGHT_MAX_BIN + 2];
+};
+
+// ---- phase 1: per-tile histogram of bin ids (+ light-unit / heavy-chunk counts)
 template <bool HAS_END>
-__global__ void __launch_bounds__(BIN_THREADS)
-bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
-                 int32_t *__restrict__ cnt, int n_tiles, PlanHeader *hdr)
+__device__ __forceinline__ void count_tile(BinSmem &sm, int64_t n, const int32_t *__restrict__ rb,
+                                           const int32_t *__restrict__ re, int32_t *__restrict__ cnt,
+                                           int n_tiles, int tile)
 {
-    __shared__ int hist[NBINS];
-    __shared__ int heavy;
     const int tid = threadIdx.x;
-    if (blockIdx.x == 0 && tid == 0) hdr->scan_ticket = 0;  // bin_scan runs after us
-    if (tid < NBINS) hist[tid] = 0;
-    if (tid == 0) heavy = 0;
+    if (tid < NBINS) sm.hist[tid] = 0;
+    if (tid == 0) sm.heavy = 0;
     __syncthreads();
-    const int64_t base = (int64_t)blockIdx.x * TILE_ROWS;
+    const int64_t base = (int64_t)tile * TILE_ROWS;
     int my_heavy = 0;
     int lens[TILE_ROUNDS];
 #pragma unroll
@@ -54,75 +76,89 @@ bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__res
         const int b = valid ? bin_of_len(len) : NBINS;
         // warp-aggregated histogram update: one shared atomic per distinct bin
         const unsigned m = __match_any_sync(0xffffffffu, b);
-        if (valid && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&hist[b], __popc(m));
+        if (valid && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&sm.hist[b], __popc(m));
         if (b >= HEAVY_BIN && valid) my_heavy += heavy_chunks(len);
     }
-    // warp-reduce the heavy chunk count
     for (int o = 16; o > 0; o >>= 1) my_heavy += __shfl_xor_sync(0xffffffffu, my_heavy, o);
-    if ((tid & 31) == 0 && my_heavy) atomicAdd(&heavy, my_heavy);
+    if ((tid & 31) == 0 && my_heavy) atomicAdd(&sm.heavy, my_heavy);
     __syncthreads();
-    if (tid < NBINS) cnt[(int64_t)tid * n_tiles + blockIdx.x] = hist[tid];
+    if (tid < NBINS) cnt[(int64_t)tid * n_tiles + tile] = sm.hist[tid];
     if (tid == NBINS) {
         int lu = 0;
 #pragma unroll
-        for (int b = 0; b <= LIGHT_MAX_BIN; b++) lu += (hist[b] + unit_rows(b) - 1) / unit_rows(b);
-        cnt[(int64_t)NBINS * n_tiles + blockIdx.x] = lu;
-        cnt[(int64_t)(NBINS + 1) * n_tiles + blockIdx.x] = heavy;
+        for (int b = 0; b <= LIGHT_MAX_BIN; b++) lu += (sm.hist[b] + unit_rows(b) - 1) / unit_rows(b);
+        cnt[(int64_t)NBINS * n_tiles + tile] = lu;
+        cnt[(int64_t)(NBINS + 1) * n_tiles + tile] = sm.heavy;
     }
+    __syncthreads();
 }
 
-constexpr int SCAN_THREADS = 1024;
+struct ScanArgs {
+    int32_t *bin_offsets;
+    int64_t n_cols, light_cap, heavy_cap;
+    PlanLayout L;
+    int xc_valid, xc_stride;
+};
 
-__global__ void __launch_bounds__(SCAN_THREADS)
-bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int n_tiles,
-                PlanHeader *hdr, int32_t *__restrict__ bin_offsets, int64_t n_rows, int64_t n_cols,
-                int64_t light_cap, int64_t heavy_cap, PlanLayout L, int xc_valid, int xc_stride)
+// ---- phase 2: exclusive scan of one scan row over the tiles (coalesced chunks of T
+// with a running carry); the last of the SCAN_ROWS rows to finish turns the totals
+// into bin_offsets and the plan header.
+template <int T, int IPT>
+__device__ __forceinline__ void scan_row(BinSmem &sm, const int32_t *__restrict__ cnt,
+                                         int32_t *__restrict__ toff, int n_tiles, PlanHeader *hdr,
+                                         const ScanArgs &sa, int row)
 {
-    __shared__ int warp_sums[SCAN_THREADS / 32];
-    __shared__ int is_last;
-    const int row = blockIdx.x;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int32_t *a = cnt + (int64_t)row * n_tiles;
     int32_t *o = toff + (int64_t)row * n_tiles;
-    // coalesced block scan over chunks of SCAN_THREADS elements with a running carry
-    __shared__ int carry;
-    if (tid == 0) carry = 0;
+    if (tid == 0) sm.carry = 0;
     __syncthreads();
-    for (int c0 = 0; c0 < n_tiles; c0 += SCAN_THREADS) {
-        const int i = c0 + tid;
-        const int s = i < n_tiles ? a[i] : 0;
+    // chunks of T * IPT elements; thread t owns IPT consecutive elements of a chunk
+    for (int c0 = 0; c0 < n_tiles; c0 += T * IPT) {
+        const int i0 = c0 + tid * IPT;
+        int v[IPT];
+        int s = 0;
+#pragma unroll
+        for (int j = 0; j < IPT; j++) {
+            v[j] = i0 + j < n_tiles ? a[i0 + j] : 0;
+            s += v[j];
+        }
         int incl = s;
         for (int d = 1; d < 32; d <<= 1) {
             const int t = __shfl_up_sync(0xffffffffu, incl, d);
             if (lane >= d) incl += t;
         }
-        if (lane == 31) warp_sums[warp] = incl;
+        if (lane == 31) sm.warp_sums[warp] = incl;
         __syncthreads();
         if (warp == 0) {
-            const int w = warp_sums[lane];
+            const int w = lane < T / 32 ? sm.warp_sums[lane] : 0;
             int wi = w;
             for (int d = 1; d < 32; d <<= 1) {
                 const int t = __shfl_up_sync(0xffffffffu, wi, d);
                 if (lane >= d) wi += t;
             }
-            warp_sums[lane] = wi - w;  // exclusive
+            if (lane < T / 32) sm.warp_sums[lane] = wi - w;  // exclusive
         }
         __syncthreads();
-        const int base_c = carry;
-        if (i < n_tiles) o[i] = base_c + warp_sums[warp] + incl - s;
+        const int base_c = sm.carry;
+        int run = base_c + sm.warp_sums[warp] + incl - s;
+#pragma unroll
+        for (int j = 0; j < IPT; j++) {
+            if (i0 + j < n_tiles) o[i0 + j] = run;
+            run += v[j];
+        }
         __syncthreads();
-        if (tid == SCAN_THREADS - 1) carry = base_c + warp_sums[warp] + incl;
+        if (tid == T - 1) sm.carry = run;
         __syncthreads();
     }
-    if (tid == 0) hdr->totals[row] = carry;
-    // last CTA: bin offsets + unit totals
+    if (tid == 0) hdr->totals[row] = sm.carry;
     __syncthreads();
     if (tid == 0) {
         __threadfence();
-        is_last = (atomicAdd(&hdr->scan_ticket, 1) == SCAN_ROWS - 1);
+        sm.is_last = (atomicAdd(&hdr->scan_ticket, 1) == SCAN_ROWS - 1);
     }
     __syncthreads();
-    if (is_last && warp == 0) {
+    if (sm.is_last && warp == 0) {
         // one parallel load per lane (not a serial chain of L2 round trips)
         __threadfence();
         const int t = __ldcg(hdr->totals + lane);
@@ -131,34 +167,197 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
             const int v = __shfl_up_sync(0xffffffffu, incl, d);
             if (lane >= d) incl += v;
         }
-        bin_offsets[lane] = incl - t;
-        if (lane == 31) bin_offsets[NBINS] = incl;  // == n_rows
+        sa.bin_offsets[lane] = incl - t;
+        if (lane == 31) sa.bin_offsets[NBINS] = incl;  // == n_rows
     }
-    if (is_last && tid == 0) {
+    if (sm.is_last && tid == 0) {
         const int nl = __ldcg(hdr->totals + NBINS), nh = __ldcg(hdr->totals + NBINS + 1);
-        int ovf = (nl > light_cap) || (nh > heavy_cap);
+        const int ovf = (nl > sa.light_cap) || (nh > sa.heavy_cap);
         hdr->overflow = ovf;
         hdr->n_light_units = ovf ? 0 : nl;
         hdr->n_heavy_units = ovf ? 0 : nh;
         hdr->n_units = ovf ? 0 : nl + nh;
         hdr->n_tiles = n_tiles;
-        hdr->off_units = (int64_t)L.off_units;
-        hdr->off_partial = (int64_t)L.off_partial;
-        hdr->off_ticket = (int64_t)L.off_ticket;
-        hdr->off_xc_vote = (int64_t)L.off_xc_vote;
-        hdr->off_xc_tag = (int64_t)L.off_xc_tag;
-        hdr->off_xc_val = (int64_t)L.off_xc_val;
-        hdr->xc_valid = xc_valid;
-        hdr->xc_stride = xc_stride;
-        hdr->n_cols = n_cols;
+        hdr->off_units = (int64_t)sa.L.off_units;
+        hdr->off_partial = (int64_t)sa.L.off_partial;
+        hdr->off_ticket = (int64_t)sa.L.off_ticket;
+        hdr->off_xc_vote = (int64_t)sa.L.off_xc_vote;
+        hdr->off_xc_tag = (int64_t)sa.L.off_xc_tag;
+        hdr->off_xc_val = (int64_t)sa.L.off_xc_val;
+        hdr->xc_valid = sa.xc_valid;
+        hdr->xc_stride = sa.xc_stride;
+        hdr->n_cols = sa.n_cols;
         hdr->work_ctr = 0;
         hdr->exit_ticket = 0;
         hdr->d2_hi = 0;
         hdr->d2_mid = 0;
         hdr->d2_lo = 0;
         hdr->scan_ticket = 0;
-        (void)n_rows;
     }
+    __syncthreads();
+}
+
+// ---- phase 3: stable scatter of one tile + its work units
+template <bool HAS_END>
+__device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32_t *__restrict__ rb,
+                                             const int32_t *__restrict__ re, int32_t *__restrict__ bin_rows,
+                                             const int32_t *bin_offsets, const int32_t *toff, int n_tiles,
+                                             const PlanHeader *hdr, int2 *__restrict__ units,
+                                             int32_t *__restrict__ tickets, int64_t heavy_cap, int tile)
+{
+    constexpr int NW = BIN_THREADS / 32;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int overflow = hdr->overflow;
+    const int n_heavy = hdr->n_heavy_units;
+    if (tid < NBINS) {
+        sm.run[tid] = 0;
+        sm.seg[tid] = bin_offsets[tid] + toff[(int64_t)tid * n_tiles + tile];
+    }
+    for (int i = tid; i < NW * NBINS; i += BIN_THREADS) (&sm.wcnt[0][0])[i] = 0;
+    if (tid == 0) sm.heavy_run = toff[(int64_t)(NBINS + 1) * n_tiles + tile];
+    __syncthreads();
+    const int64_t base = (int64_t)tile * TILE_ROWS;
+    const unsigned lt = (1u << lane) - 1u;
+    int lens[TILE_ROUNDS];
+#pragma unroll
+    for (int k = 0; k < TILE_ROUNDS; k++) {  // all row-length loads in flight at once
+        const int64_t r = base + k * BIN_THREADS + tid;
+        lens[k] = r < n ? row_length<HAS_END>(rb, re, r) : 0;
+    }
+#pragma unroll
+    for (int k = 0; k < TILE_ROUNDS; k++) {
+        const int64_t r = base + k * BIN_THREADS + tid;
+        const bool valid = r < n;
+        const int len = lens[k];
+        const int b = valid ? bin_of_len(len) : NBINS;  // NBINS = sentinel for past-the-end rows
+        const unsigned mask = __match_any_sync(0xffffffffu, b);
+        const int rank = __popc(mask & lt);
+        if (valid && rank == 0) sm.wcnt[warp][b] = __popc(mask);
+        const int hc = (valid && b >= HEAVY_BIN) ? heavy_chunks(len) : 0;
+        int hincl = hc;
+        for (int d = 1; d < 32; d <<= 1) {
+            const int t = __shfl_up_sync(0xffffffffu, hincl, d);
+            if (lane >= d) hincl += t;
+        }
+        if (lane == 31) sm.hw[warp] = hincl;
+        __syncthreads();
+        if (tid < NBINS) {
+            int acc = sm.run[tid];
+#pragma unroll
+            for (int w = 0; w < NW; w++) {
+                sm.wbase[w][tid] = acc;
+                acc += sm.wcnt[w][tid];
+                sm.wcnt[w][tid] = 0;
+            }
+            sm.run[tid] = acc;
+        } else if (tid == NBINS) {
+            int acc = sm.heavy_run;
+#pragma unroll
+            for (int w = 0; w < NW; w++) {
+                const int t = sm.hw[w];
+                sm.hw[w] = acc;
+                acc += t;
+            }
+            sm.heavy_run = acc;
+        }
+        __syncthreads();
+        if (valid) {
+            bin_rows[sm.seg[b] + sm.wbase[warp][b] + rank] = (int32_t)r;
+            if (hc > 0 && !overflow) {
+                const int u0 = sm.hw[warp] + hincl - hc;
+                for (int c = 0; c < hc; c++)
+                    if (u0 + c < heavy_cap) units[u0 + c] = make_int2((int)r, (int)(HEAVY_FLAG | (uint32_t)c));
+                if (u0 < heavy_cap) tickets[u0] = 0;
+            }
+        }
+        __syncthreads();
+    }
+    if (!overflow) {
+        // light work units of this tile: bins 0..10, in bin order, row-contiguous
+        if (tid == 0) {
+            int acc = 0;
+            for (int b = 0; b <= LIGHT_MAX_BIN; b++) {
+                sm.upre[b] = acc;
+                acc += (sm.run[b] + unit_rows(b) - 1) / unit_rows(b);
+            }
+            sm.upre[LIGHT_MAX_BIN + 1] = acc;
+        }
+        __syncthreads();
+        const int ubase = n_heavy + toff[(int64_t)NBINS * n_tiles + tile];
+        const int total = sm.upre[LIGHT_MAX_BIN + 1];
+        for (int j = tid; j < total; j += BIN_THREADS) {
+            int b = 0;
+            while (sm.upre[b + 1] <= j) b++;
+            const int q = j - sm.upre[b];
+            const int K = unit_rows(b);
+            const int c = min(K, sm.run[b] - q * K);
+            units[ubase + j] = make_int2(sm.seg[b] + q * K, (b << 24) | c);
+        }
+    }
+    __syncthreads();
+}
+
+// ---- three-launch path (used when a cooperative launch is not possible)
+template <bool HAS_END>
+__global__ void __launch_bounds__(BIN_THREADS)
+bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
+                 int32_t *__restrict__ cnt, int n_tiles, PlanHeader *hdr)
+{
+    __shared__ BinSmem sm;
+    if (blockIdx.x == 0 && threadIdx.x == 0) hdr->scan_ticket = 0;  // bin_scan runs after us
+    count_tile<HAS_END>(sm, n, rb, re, cnt, n_tiles, blockIdx.x);
+}
+
+constexpr int SCAN_THREADS = 1024;
+
+__global__ void __launch_bounds__(SCAN_THREADS)
+bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int n_tiles,
+                PlanHeader *hdr, ScanArgs sa)
+{
+    __shared__ BinSmem sm;
+    scan_row<SCAN_THREADS, 1>(sm, cnt, toff, n_tiles, hdr, sa, blockIdx.x);
+}
+
+template <bool HAS_END>
+__global__ void __launch_bounds__(BIN_THREADS)
+bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
+                   int32_t *__restrict__ bin_rows, const int32_t *__restrict__ bin_offsets,
+                   const int32_t *__restrict__ toff, int n_tiles, const PlanHeader *__restrict__ hdr,
+                   int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap)
+{
+    __shared__ BinSmem sm;
+    scatter_tile<HAS_END>(sm, n, rb, re, bin_rows, bin_offsets, toff, n_tiles, hdr, units, tickets, heavy_cap,
+                          blockIdx.x);
+}
+
+// ---- one cooperative launch: count -> grid barrier -> scan -> grid barrier -> scatter
+// (two grid-wide barriers instead of two kernel boundaries; tiles are grid-strided)
+struct FusedArgs {
+    int64_t n;
+    const int32_t *rb, *re;
+    int32_t *cnt, *toff, *bin_rows, *tickets;
+    int2 *units;
+    PlanHeader *hdr;
+    int n_tiles;
+    ScanArgs sa;
+};
+
+template <bool HAS_END>
+__global__ void __launch_bounds__(BIN_THREADS)
+bin_fused_kernel(FusedArgs f)
+{
+    __shared__ BinSmem sm;
+    cg::grid_group grid = cg::this_grid();
+    if (blockIdx.x == 0 && threadIdx.x == 0) f.hdr->scan_ticket = 0;
+    for (int t = blockIdx.x; t < f.n_tiles; t += gridDim.x)
+        count_tile<HAS_END>(sm, f.n, f.rb, f.re, f.cnt, f.n_tiles, t);
+    grid.sync();
+    for (int row = blockIdx.x; row < SCAN_ROWS; row += gridDim.x)
+        scan_row<BIN_THREADS, 8>(sm, f.cnt, f.toff, f.n_tiles, f.hdr, f.sa, row);
+    grid.sync();
+    for (int t = blockIdx.x; t < f.n_tiles; t += gridDim.x)
+        scatter_tile<HAS_END>(sm, f.n, f.rb, f.re, f.bin_rows, f.sa.bin_offsets, f.toff, f.n_tiles, f.hdr, f.units,
+                              f.tickets, f.sa.heavy_cap, t);
 }
 
 // x-cache table: sampled occurrence counts, per-slot winner (count, column).
@@ -175,115 +374,36 @@ __global__ void xc_count_kernel(const int32_t *__restrict__ col, int64_t nnz_max
     atomicMax(best + (c & (XC_SLOTS - 1)), ((unsigned long long)cnt << 32) | (unsigned)c);
 }
 
-template <bool HAS_END>
-__global__ void __launch_bounds__(BIN_THREADS)
-bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
-                   int32_t *__restrict__ bin_rows, const int32_t *__restrict__ bin_offsets,
-                   const int32_t *__restrict__ toff, int n_tiles, const PlanHeader *__restrict__ hdr,
-                   int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap)
-{
-    constexpr int NW = BIN_THREADS / 32;
-    __shared__ int run[NBINS];
-    __shared__ int wcnt[NW][NBINS];
-    __shared__ int wbase[NW][NBINS];
-    __shared__ int seg[NBINS];       // global start of this tile's segment of bin b
-    __shared__ int hw[NW];           // per-warp heavy chunk totals -> exclusive bases
-    __shared__ int heavy_run;
-    __shared__ int upre[LIGHT_MAX_BIN + 2];
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int tile = blockIdx.x;
-    const int overflow = hdr->overflow;
-    const int n_heavy = hdr->n_heavy_units;
-    if (tid < NBINS) {
-        run[tid] = 0;
-        seg[tid] = bin_offsets[tid] + toff[(int64_t)tid * n_tiles + tile];
-    }
-    for (int i = tid; i < NW * NBINS; i += BIN_THREADS) (&wcnt[0][0])[i] = 0;
-    if (tid == 0) heavy_run = toff[(int64_t)(NBINS + 1) * n_tiles + tile];
-    __syncthreads();
-    const int64_t base = (int64_t)tile * TILE_ROWS;
-    const unsigned lt = (1u << lane) - 1u;
-    int lens[TILE_ROUNDS];
-#pragma unroll
-    for (int k = 0; k < TILE_ROUNDS; k++) {  // all row-length loads in flight at once
-        const int64_t r = base + k * BIN_THREADS + tid;
-        lens[k] = r < n ? row_length<HAS_END>(rb, re, r) : 0;
-    }
-#pragma unroll
-    for (int k = 0; k < TILE_ROUNDS; k++) {
-        int64_t r = base + k * BIN_THREADS + tid;
-        bool valid = r < n;
-        int len = lens[k];
-        int b = valid ? bin_of_len(len) : NBINS;  // NBINS = sentinel for past-the-end rows
-        unsigned mask = __match_any_sync(0xffffffffu, b);
-        int rank = __popc(mask & lt);
-        if (valid && rank == 0) wcnt[warp][b] = __popc(mask);
-        int hc = (valid && b >= HEAVY_BIN) ? heavy_chunks(len) : 0;
-        int hincl = hc;
-        for (int d = 1; d < 32; d <<= 1) {
-            int t = __shfl_up_sync(0xffffffffu, hincl, d);
-            if (lane >= d) hincl += t;
-        }
-        if (lane == 31) hw[warp] = hincl;
-        __syncthreads();
-        if (tid < NBINS) {
-            int acc = run[tid];
-#pragma unroll
-            for (int w = 0; w < NW; w++) {
-                wbase[w][tid] = acc;
-                acc += wcnt[w][tid];
-                wcnt[w][tid] = 0;
-            }
-            run[tid] = acc;
-        } else if (tid == NBINS) {
-            int acc = heavy_run;
-#pragma unroll
-            for (int w = 0; w < NW; w++) {
-                int t = hw[w];
-                hw[w] = acc;
-                acc += t;
-            }
-            heavy_run = acc;
-        }
-        __syncthreads();
-        if (valid) {
-            bin_rows[seg[b] + wbase[warp][b] + rank] = (int32_t)r;
-            if (hc > 0 && !overflow) {
-                int u0 = hw[warp] + hincl - hc;
-                for (int c = 0; c < hc; c++) {
-                    if (u0 + c < heavy_cap) units[u0 + c] = make_int2((int)r, (int)(HEAVY_FLAG | (uint32_t)c));
-                }
-                if (u0 < heavy_cap) tickets[u0] = 0;
-            }
-        }
-        __syncthreads();
-    }
-    if (overflow) return;
-    // light work units of this tile: bins 0..10, in bin order, row-contiguous
-    if (tid == 0) {
-        int acc = 0;
-        for (int b = 0; b <= LIGHT_MAX_BIN; b++) {
-            upre[b] = acc;
-            acc += (run[b] + unit_rows(b) - 1) / unit_rows(b);
-        }
-        upre[LIGHT_MAX_BIN + 1] = acc;
-    }
-    __syncthreads();
-    const int ubase = n_heavy + toff[(int64_t)NBINS * n_tiles + tile];
-    const int total = upre[LIGHT_MAX_BIN + 1];
-    for (int j = tid; j < total; j += BIN_THREADS) {
-        int b = 0;
-        while (upre[b + 1] <= j) b++;
-        int q = j - upre[b];
-        int K = unit_rows(b);
-        int c = min(K, run[b] - q * K);
-        units[ubase + j] = make_int2(seg[b] + q * K, (b << 24) | c);
-    }
-}
-
 }  // namespace acsr
 
 using namespace acsr;
+
+// ACSR_BIN_FUSED=0 selects the three-launch path (A/B measurements, or no cooperative launch)
+static bool fused_enabled()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("ACSR_BIN_FUSED");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
+static int fused_grid(bool has_end)
+{
+    static int g[2] = {0, 0};
+    int &gg = g[has_end ? 1 : 0];
+    if (!gg) {
+        int per_sm = 0;
+        if (has_end)
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bin_fused_kernel<true>, BIN_THREADS, 0);
+        else
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bin_fused_kernel<false>, BIN_THREADS, 0);
+        if (per_sm < 1) per_sm = 1;
+        gg = per_sm * acsr_num_sms();
+    }
+    return gg;
+}
 
 extern "C" size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t n_cols, int64_t nnz_max)
 {
@@ -318,18 +438,28 @@ extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
     int2 *units = (int2 *)(ws + L.off_units);
     int32_t *tickets = (int32_t *)(ws + L.off_ticket);
     const int nt = (int)L.n_tiles;
-    if (row_end)
-        bin_count_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
-    else
-        bin_count_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
     // the x-cache table is built only when the (experimental, default-off) cache is enabled
     const char *xe = getenv("ACSR_XCACHE");
     const int xc_valid = xe && xe[0] == '1' && col_idx != nullptr && n_cols > 0 &&
                          n_cols < ((int64_t)XC_NOTAG << XC_BITS);
     int64_t stride64 = nnz_max >> XC_SAMPLE_LOG2;
     const int xc_stride = (int)(stride64 < 1 ? 1 : (stride64 > (1 << 30) ? (1 << 30) : stride64));
-    bin_scan_kernel<<<SCAN_ROWS, SCAN_THREADS, 0, stream>>>(
-        cnt, toff, nt, hdr, bin_offsets, n_rows, n_cols, L.light_cap, L.heavy_cap, L, xc_valid, xc_stride);
+    ScanArgs sa{bin_offsets, n_cols, L.light_cap, L.heavy_cap, L, xc_valid, xc_stride};
+    if (fused_enabled()) {
+        FusedArgs f{n_rows, row_begin, row_end, cnt, toff, bin_rows, tickets, units, hdr, nt, sa};
+        const int grid = fused_grid(row_end != nullptr);
+        void *args[] = {&f};
+        const cudaError_t e = row_end
+            ? cudaLaunchCooperativeKernel((void *)bin_fused_kernel<true>, grid, BIN_THREADS, args, 0, stream)
+            : cudaLaunchCooperativeKernel((void *)bin_fused_kernel<false>, grid, BIN_THREADS, args, 0, stream);
+        if (e == cudaSuccess) goto xc;
+        cudaGetLastError();  // not supported here (e.g. MPS limits): fall back to three launches
+    }
+    if (row_end)
+        bin_count_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
+    else
+        bin_count_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
+    bin_scan_kernel<<<SCAN_ROWS, SCAN_THREADS, 0, stream>>>(cnt, toff, nt, hdr, sa);
     if (row_end)
         bin_scatter_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, bin_rows,
                                                                    bin_offsets, toff, nt, hdr, units,
@@ -338,6 +468,7 @@ extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
         bin_scatter_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, bin_rows,
                                                                     bin_offsets, toff, nt, hdr, units,
                                                                     tickets, L.heavy_cap);
+xc:
     if (xc_valid) {
         cudaMemsetAsync(ws + L.off_xc_vote, 0, sizeof(uint64_t) * XC_SLOTS, stream);
         cudaMemsetAsync(ws + L.off_xc_count, 0, sizeof(int32_t) * (size_t)n_cols, stream);

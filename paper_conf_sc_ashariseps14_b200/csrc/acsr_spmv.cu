@@ -38,6 +38,9 @@
 #ifndef ACSR_NO_VEC
 #define ACSR_NO_VEC 0  // 1: never use the 128-bit vector path (A/B builds)
 #endif
+#ifndef ACSR_VEC_MIN
+#define ACSR_VEC_MIN 512  // rows (chunks) shorter than this use the lane-strided scalar path
+#endif
 
 
 namespace acsr {
@@ -428,7 +431,7 @@ struct Kern {
     {
         double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
         int k;
-        if (a.vph >= 0 && ke - kb >= 64) {
+        if (a.vph >= 0 && ke - kb >= ACSR_VEC_MIN) {
             const int ja = ((kb + a.vph + 3) & ~3) - a.vph;  // first aligned index >= kb
             s0 = fmacp(a, lane < ja - kb, kb + lane, s0);
             int j = ja;

@@ -19,6 +19,10 @@ for v in "$@"; do
     nv) build nv -DACSR_NO_VEC=1 ;;
     br) build br -DACSR_BRANCHY_SUB=1 ;;
     nvbr) build nvbr -DACSR_NO_VEC=1 -DACSR_BRANCHY_SUB=1 ;;
+    v256) build v256 -DACSR_VEC_MIN=256 ;;
+    v512) build v512 -DACSR_VEC_MIN=512 ;;
+    v1024) build v1024 -DACSR_VEC_MIN=1024 ;;
+    v512br) build v512br -DACSR_VEC_MIN=512 -DACSR_BRANCHY_SUB=1 ;;
   esac
 done
 wait

@@ -378,13 +378,16 @@ __global__ void xc_count_kernel(const int32_t *__restrict__ col, int64_t nnz_max
 
 using namespace acsr;
 
-// ACSR_BIN_FUSED=0 selects the three-launch path (A/B measurements, or no cooperative launch)
+// ACSR_BIN_FUSED=1 selects the single cooperative launch.  Measured slower on B200
+// (C2: 28.7 vs 25.6 us; LiveJournal-like: 65.5 vs 48.1 us; s26: 0.87 vs 0.61 ms -- the
+// grid-wide syncs and the cooperative launch cost more than the two kernel boundaries
+// they replace), so the three-launch path is the default.
 static bool fused_enabled()
 {
     static int v = -1;
     if (v < 0) {
         const char *e = getenv("ACSR_BIN_FUSED");
-        v = (e && e[0] == '0') ? 0 : 1;
+        v = (e && e[0] == '1') ? 1 : 0;
     }
     return v == 1;
 }

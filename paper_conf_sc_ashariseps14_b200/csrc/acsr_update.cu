@@ -9,6 +9,7 @@
 // appends the inserts lane-parallel.  Out-degrees change by integer atomics, so
 // the result is exact and independent of scheduling.
 #include <cuda_runtime.h>
+#include <stddef.h>
 #include <string.h>
 
 #include "acsr_internal.cuh"
@@ -17,6 +18,16 @@ namespace acsr {
 
 constexpr int UPD_THREADS = 256;
 constexpr unsigned long long NO_FAIL = ~0ull;
+// rows longer than this with a non-empty delete list are validated and compacted by a
+// whole CTA (block-scan compaction) instead of one warp: hub rows of power-law graphs
+constexpr int LONG_ROW = 2048;
+
+struct UpdWs {
+    unsigned long long key;  // (first failing index << 3) | code, or NO_FAIL
+    unsigned int n_long;     // number of long-row updates appended to long_list
+    unsigned int pad;
+    int32_t long_list[1];    // [n_upd]
+};
 
 __device__ __forceinline__ bool member(const int32_t *__restrict__ d, int lo, int hi, int c)
 {
@@ -35,8 +46,9 @@ update_validate_kernel(int64_t n_rows, int64_t n_cols, const int32_t *__restrict
                        const int32_t *__restrict__ col, int64_t n_upd,
                        const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
                        const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
-                       const int32_t *__restrict__ icol, unsigned long long *key)
+                       const int32_t *__restrict__ icol, UpdWs *ws)
 {
+    unsigned long long *key = &ws->key;
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
     if (i >= n_upd) return;
@@ -64,6 +76,10 @@ update_validate_kernel(int64_t n_rows, int64_t n_cols, const int32_t *__restrict
     }
     if (code == ACSR_OK) {
         const int b = __ldg(rb + r), e = __ldg(re + r);
+        if (d1 > d0 && e - b > LONG_ROW) {  // deferred to the CTA-per-row kernel
+            if (lane == 0) ws->long_list[atomicAdd(&ws->n_long, 1u)] = (int32_t)i;
+            return;
+        }
         int dels = 0;
         if (d1 > d0)
             for (int k = b + lane; k < e; k += 32) dels += member(dcol, d0, d1, __ldg(col + k)) ? 1 : 0;
@@ -74,6 +90,119 @@ update_validate_kernel(int64_t n_rows, int64_t n_cols, const int32_t *__restrict
     if (code != ACSR_OK && lane == 0) atomicMin(key, ((unsigned long long)i << 3) | (unsigned)code);
 }
 
+__device__ __forceinline__ int block_exclusive_scan(int v, int &total, int *sh)
+{
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int incl = v;
+    for (int d = 1; d < 32; d <<= 1) {
+        const int t = __shfl_up_sync(0xffffffffu, incl, d);
+        if (lane >= d) incl += t;
+    }
+    if (lane == 31) sh[w] = incl;
+    __syncthreads();
+    if (w == 0) {
+        const int x = lane < UPD_THREADS / 32 ? sh[lane] : 0;
+        int xi = x;
+        for (int d = 1; d < 32; d <<= 1) {
+            const int t = __shfl_up_sync(0xffffffffu, xi, d);
+            if (lane >= d) xi += t;
+        }
+        if (lane < UPD_THREADS / 32) sh[lane] = xi - x;
+        if (lane == UPD_THREADS / 32 - 1) sh[32] = xi;
+    }
+    __syncthreads();
+    const int r = sh[w] + incl - v;
+    total = sh[32];
+    __syncthreads();
+    return r;
+}
+
+// capacity check of the long rows (one CTA per long update, grid-strided over the list)
+__global__ void __launch_bounds__(UPD_THREADS)
+update_validate_long_kernel(const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
+                            const int32_t *__restrict__ cap, const int32_t *__restrict__ col,
+                            const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
+                            const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr, UpdWs *ws)
+{
+    __shared__ int sh[33];
+    const unsigned n_long = *(volatile unsigned *)&ws->n_long;
+    for (unsigned j = blockIdx.x; j < n_long; j += gridDim.x) {
+        const int i = ws->long_list[j];
+        const int r = __ldg(upd + i);
+        const int b = __ldg(rb + r), e = __ldg(re + r);
+        const int d0 = __ldg(dptr + i), d1 = __ldg(dptr + i + 1);
+        int dels = 0;
+        for (int k = b + threadIdx.x; k < e; k += UPD_THREADS) dels += member(dcol, d0, d1, __ldg(col + k)) ? 1 : 0;
+        int total;
+        block_exclusive_scan(dels, total, sh);
+        const long long new_len = (long long)(e - b) - total + (__ldg(iptr + i + 1) - __ldg(iptr + i));
+        if (threadIdx.x == 0 && new_len > __ldg(cap + r))
+            atomicMin(&ws->key, ((unsigned long long)i << 3) | (unsigned)ACSR_ERR_CAPACITY);
+    }
+}
+
+// stable in-place compaction + append of the long rows: chunks of 4 * UPD_THREADS entries,
+// thread t owns 4 consecutive entries; every entry of a chunk is read before any write
+// (a destination never passes its source), kept entries move to w + block prefix.
+template <typename T>
+__global__ void __launch_bounds__(UPD_THREADS)
+update_apply_long_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re, int32_t *__restrict__ col,
+                         T *__restrict__ val, const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
+                         const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
+                         const int32_t *__restrict__ icol, const T *__restrict__ ival, T one,
+                         int32_t *__restrict__ outdeg, UpdWs *ws)
+{
+    __shared__ int sh[33];
+    if (*(volatile unsigned long long *)&ws->key != NO_FAIL) return;
+    const unsigned n_long = *(volatile unsigned *)&ws->n_long;
+    constexpr int E = 4;
+    for (unsigned j = blockIdx.x; j < n_long; j += gridDim.x) {
+        const int i = ws->long_list[j];
+        const int r = __ldg(upd + i);
+        const int b = __ldg(rb + r), e = re[r];
+        const int d0 = __ldg(dptr + i), d1 = __ldg(dptr + i + 1);
+        int w = b;
+        for (int k0 = b; k0 < e; k0 += E * UPD_THREADS) {
+            int c[E];
+            T v[E];
+            bool keep[E], del[E];
+            int cnt = 0;
+#pragma unroll
+            for (int q = 0; q < E; q++) {
+                const int kk = k0 + threadIdx.x * E + q;
+                const bool valid = kk < e;
+                c[q] = valid ? col[kk] : 0;
+                v[q] = (val && valid) ? val[kk] : T();
+                del[q] = valid && member(dcol, d0, d1, c[q]);
+                keep[q] = valid && !del[q];
+                cnt += keep[q] ? 1 : 0;
+            }
+            int total;
+            int dst = w + block_exclusive_scan(cnt, total, sh);  // includes a __syncthreads: reads done
+#pragma unroll
+            for (int q = 0; q < E; q++) {
+                if (keep[q]) {
+                    col[dst] = c[q];
+                    if (val) val[dst] = v[q];
+                    dst++;
+                }
+                if (del[q] && outdeg) atomicSub(outdeg + c[q], 1);
+            }
+            w += total;
+            __syncthreads();
+        }
+        const int i0 = __ldg(iptr + i), i1 = __ldg(iptr + i + 1);
+        for (int q = i0 + threadIdx.x; q < i1; q += UPD_THREADS) {
+            const int cc = __ldg(icol + q);
+            col[w + (q - i0)] = cc;
+            if (val) val[w + (q - i0)] = ival ? ival[q] : one;
+            if (outdeg) atomicAdd(outdeg + cc, 1);
+        }
+        if (threadIdx.x == 0) re[r] = w + (i1 - i0);
+        __syncthreads();
+    }
+}
+
 template <typename T>
 __global__ void __launch_bounds__(UPD_THREADS)
 update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
@@ -81,10 +210,9 @@ update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
                     const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
                     const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
                     const int32_t *__restrict__ icol, const T *__restrict__ ival, T one,
-                    int32_t *__restrict__ outdeg, const unsigned long long *key,
-                    int32_t *__restrict__ status)
+                    int32_t *__restrict__ outdeg, const UpdWs *ws, int32_t *__restrict__ status)
 {
-    const unsigned long long k = *(volatile const unsigned long long *)key;
+    const unsigned long long k = *(volatile const unsigned long long *)&ws->key;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         status[0] = k == NO_FAIL ? ACSR_OK : (int32_t)(k & 7);
         status[1] = k == NO_FAIL ? -1 : (int32_t)(k >> 3);
@@ -98,6 +226,7 @@ update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
     const int b = __ldg(rb + r), e = re[r];
     int w = e;
     const int d0 = dptr ? __ldg(dptr + i) : 0, d1 = dptr ? __ldg(dptr + i + 1) : 0;
+    if (d1 > d0 && e - b > LONG_ROW) return;  // update_apply_long_kernel
     if (d1 > d0) {
         w = b;
         for (int k0 = b; k0 < e; k0 += 32) {
@@ -180,8 +309,7 @@ extern "C" acsr_status acsr_relayout(acsr_dtype dt, int64_t n_rows, const int32_
 
 extern "C" size_t acsr_update_workspace_bytes(int64_t n_upd)
 {
-    (void)n_upd;
-    return 256;
+    return align_up(offsetof(UpdWs, long_list) + sizeof(int32_t) * (size_t)(n_upd > 0 ? n_upd : 1), 256);
 }
 
 extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
@@ -203,8 +331,10 @@ extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t 
         acsr_set_error("acsr_update_edges: workspace too small");
         return ACSR_ERR_WORKSPACE;
     }
-    unsigned long long *key = (unsigned long long *)ws;
-    cudaMemsetAsync(key, 0xff, sizeof(unsigned long long), stream);
+    UpdWs *uw = (UpdWs *)ws;
+    cudaMemsetAsync(&uw->key, 0xff, sizeof(unsigned long long), stream);
+    cudaMemsetAsync(&uw->n_long, 0, sizeof(unsigned int), stream);
+    const int long_grid = 4 * acsr_num_sms();
     const int wpb = UPD_THREADS / 32;
     const int64_t blocks64 = n_upd > 0 ? (n_upd + wpb - 1) / wpb : 1;
     if (blocks64 > 0x7fffffff) return ACSR_ERR_INVALID_VALUE;
@@ -213,21 +343,33 @@ extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t 
         update_validate_kernel<<<blocks, UPD_THREADS, 0, stream>>>(n_rows, n_cols, row_begin, row_end,
                                                                    row_cap, col_idx, n_upd, upd_rows,
                                                                    del_ptr, del_cols, ins_ptr, ins_cols,
-                                                                   key);
+                                                                   uw);
+    if (n_upd > 0 && del_ptr)
+        update_validate_long_kernel<<<long_grid, UPD_THREADS, 0, stream>>>(row_begin, row_end, row_cap, col_idx,
+                                                                          upd_rows, del_ptr, del_cols, ins_ptr,
+                                                                          uw);
     if (dt == ACSR_F64) {
         uint64_t one;
         double d1 = 1.0;
         memcpy(&one, &d1, 8);
         update_apply_kernel<uint64_t><<<blocks, UPD_THREADS, 0, stream>>>(
             row_begin, row_end, col_idx, (uint64_t *)values, n_upd, upd_rows, del_ptr, del_cols, ins_ptr,
-            ins_cols, (const uint64_t *)ins_vals, one, outdeg, key, status);
+            ins_cols, (const uint64_t *)ins_vals, one, outdeg, uw, status);
+        if (n_upd > 0 && del_ptr)
+            update_apply_long_kernel<uint64_t><<<long_grid, UPD_THREADS, 0, stream>>>(
+                row_begin, row_end, col_idx, (uint64_t *)values, upd_rows, del_ptr, del_cols, ins_ptr, ins_cols,
+                (const uint64_t *)ins_vals, one, outdeg, uw);
     } else {
         uint32_t one;
         float f1 = 1.0f;
         memcpy(&one, &f1, 4);
         update_apply_kernel<uint32_t><<<blocks, UPD_THREADS, 0, stream>>>(
             row_begin, row_end, col_idx, (uint32_t *)values, n_upd, upd_rows, del_ptr, del_cols, ins_ptr,
-            ins_cols, (const uint32_t *)ins_vals, one, outdeg, key, status);
+            ins_cols, (const uint32_t *)ins_vals, one, outdeg, uw, status);
+        if (n_upd > 0 && del_ptr)
+            update_apply_long_kernel<uint32_t><<<long_grid, UPD_THREADS, 0, stream>>>(
+                row_begin, row_end, col_idx, (uint32_t *)values, upd_rows, del_ptr, del_cols, ins_ptr, ins_cols,
+                (const uint32_t *)ins_vals, one, outdeg, uw);
     }
     return acsr_check_launch("acsr_update_edges");
 }

@@ -559,3 +559,53 @@ def test_paper_epoch_update_bitwise(acsr, cuda):
         live = np.concatenate([np.arange(b, e) for b, e in zip(rb.numpy(), re_h)])
         assert np.array_equal(m.col_idx.cpu().numpy()[live], col_h[live])
         assert np.array_equal(odd.cpu().numpy(), od_h)
+
+
+def test_update_long_row_cta_path(acsr, cuda):
+    # hub rows (> 2048 entries) with deletes take the CTA-per-row validate/compact path
+    lens = [3, 10000, 5, 40000, 0, 2049]
+    rp, ci = synth.boundary_csr(lens, 1 << 17, 11)
+    val = synth.values(ci.numel(), 12)
+    rb, re, cap, col, v2 = synth.with_slack(rp, ci, val)
+    n = len(lens)
+    od = torch.bincount(ci.long(), minlength=1 << 17).to(torch.int32)
+    rng = np.random.default_rng(3)
+    upd = np.array([1, 2, 3, 5], np.int32)
+    dels, inss = [], []
+    for r in upd:
+        cur = ci.numpy()[rp[r]:rp[r + 1]]
+        dels.append(np.unique(rng.choice(cur, size=len(cur) // 2)))
+        inss.append(rng.integers(0, 1 << 17, size=min(len(cur) // 5, 40)).astype(np.int32))
+    ch = {"upd_rows": upd,
+          "del_ptr": np.concatenate([[0], np.cumsum([d.size for d in dels])]).astype(np.int32),
+          "del_cols": np.concatenate(dels).astype(np.int32),
+          "ins_ptr": np.concatenate([[0], np.cumsum([a.size for a in inss])]).astype(np.int32),
+          "ins_cols": np.concatenate(inss).astype(np.int32)}
+    re_h, col_h, v_h, od_h = re.numpy().copy(), col.numpy().copy(), v2.numpy().copy(), od.numpy().copy()
+    code, _ = oracle.update(1 << 17, rb.numpy(), re_h, cap.numpy(), col_h, v_h, ch["upd_rows"], ch["del_ptr"],
+                            ch["del_cols"], ch["ins_ptr"], ch["ins_cols"], None, od_h)
+    assert code == 0
+    m = acsr.ACSRMatrix(rb.to(cuda), col.to(cuda), v2.to(cuda), n_cols=1 << 17, row_end=re.to(cuda),
+                        row_cap=cap.to(cuda), nnz_max=col.numel())
+    odd = od.to(cuda)
+    st = m.update(_dev_changes(ch, cuda), outdeg=odd)
+    torch.cuda.synchronize()
+    assert st.cpu().tolist() == [0, -1]
+    assert np.array_equal(m.row_end.cpu().numpy(), re_h)
+    live = np.concatenate([np.arange(b, e) for b, e in zip(rb.numpy(), re_h)])
+    assert np.array_equal(m.col_idx.cpu().numpy()[live], col_h[live])
+    assert np.array_equal(m.values.cpu().numpy()[live].view(np.uint8), v_h[live].view(np.uint8))
+    assert np.array_equal(odd.cpu().numpy(), od_h)
+    # a long-row capacity failure is reported at its index, nothing applied
+    snap = [t.clone() for t in (m.row_end, m.col_idx, odd)]
+    r = 3
+    free = int(m.row_cap[r] - (m.row_end[r] - m.row_begin[r]))
+    bad = {"upd_rows": np.array([0, r], np.int32), "del_ptr": np.array([0, 0, 1], np.int32),
+           "del_cols": np.array([int(m.col_idx[m.row_begin[r]])], np.int32),
+           "ins_ptr": np.array([0, 1, 1 + free + 2], np.int32),
+           "ins_cols": np.arange(free + 3, dtype=np.int32)}
+    st = m.update(_dev_changes(bad, cuda), outdeg=odd)
+    torch.cuda.synchronize()
+    assert st.cpu().tolist() == [3, 1]
+    for a, b in zip((m.row_end, m.col_idx, odd), snap):
+        assert torch.equal(a, b)

@@ -609,3 +609,27 @@ def test_update_long_row_cta_path(acsr, cuda):
     assert st.cpu().tolist() == [3, 1]
     for a, b in zip((m.row_end, m.col_idx, odd), snap):
         assert torch.equal(a, b)
+
+
+def test_c_abi_from_plain_c(cuda):
+    # the boundary is usable without Python: compile tests/c/capi_smoke.c against
+    # include/acsr.h and libacsr.so and run it
+    import os
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    lib = os.path.join(root, "paper_conf_sc_ashariseps14_b200", "lib")
+    exe = os.path.join(lib, "capi_smoke")
+    subprocess.check_call(["nvcc", "-Wno-deprecated-gpu-targets", "-o", exe, os.path.join(root, "tests", "c", "capi_smoke.c"),
+                           "-L" + lib, "-lacsr", "-Xlinker", "-rpath=" + lib])
+    out = subprocess.run([exe], capture_output=True, text=True, timeout=120)
+    assert out.returncode == 0, out.stdout + out.stderr
+    assert "capi_smoke OK" in out.stdout
+
+
+def test_spmv_from_host_e2e(acsr, cuda):
+    rp, ci = synth.rmat_csr(13)
+    val = synth.values(ci.numel(), 3)
+    x = synth.vector(rp.numel() - 1, 4)
+    y = acsr.spmv_from_host(rp.pin_memory(), ci.pin_memory(), val.pin_memory(), x.pin_memory(), device=cuda)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y.numpy(), y_ref, den, torch.float64)

@@ -235,7 +235,7 @@ def run_acsr(args, dev, rank, world):
         "e2e": {"value": round(2.0 * nnz / (t_e2e * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
                 "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
                 "ms_per_step": round(t_e2e, 4)},
-        "gpu_launches": 5 * K,
+        "gpu_launches": 4 * K,  # per step: bin_count, bin_scan, bin_scatter, spmv_kernel
         "clocks": clk.summary(),
     }
     if not args.no_cpu_baseline:
@@ -654,10 +654,16 @@ def main():
         dev = torch.device("cuda", local) if torch.cuda.is_available() else torch.device("cpu")
         print(json.dumps(run_reference(args, dev)), flush=True)
         return
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    ndev = torch.cuda.device_count()
+    local_dev = local % max(ndev, 1)  # (ranks > GPUs only in the single-GPU test of this path)
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
     if world > 1:
-        torch.distributed.init_process_group("nccl", device_id=dev)
+        backend = os.environ.get("ACSR_DIST_BACKEND", "nccl")  # gloo: test the path on one GPU
+        if backend == "nccl":
+            torch.distributed.init_process_group("nccl", device_id=dev)
+        else:
+            torch.distributed.init_process_group(backend)
     if args.workload == "pagerank":
         line = run_pagerank(args, dev, rank, world)
     elif args.workload == "pagerank_dist":

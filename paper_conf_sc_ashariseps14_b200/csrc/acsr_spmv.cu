@@ -556,8 +556,12 @@ struct Kern {
 #define ACSR_SCHED_STATIC 0  // 1: static round-robin units (A/B builds)
 #endif
 
+#ifndef ACSR_MIN_BLOCKS
+#define ACSR_MIN_BLOCKS (1024 / SPMV_THREADS)  // 64 registers per thread
+#endif
+
 template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
-__global__ void __launch_bounds__(SPMV_THREADS, 1024 / SPMV_THREADS)
+__global__ void __launch_bounds__(SPMV_THREADS, ACSR_MIN_BLOCKS)
 spmv_kernel(SpmvArgs<V> a)
 {
     using K = Kern<V, HAS_VAL, HAS_END, PR, XC>;

@@ -20,6 +20,10 @@ for v in "$@"; do
     br) build br -DACSR_BRANCHY_SUB=1 ;;
     nvbr) build nvbr -DACSR_NO_VEC=1 -DACSR_BRANCHY_SUB=1 ;;
     v256) build v256 -DACSR_VEC_MIN=256 ;;
+    mb2) build mb2 -DACSR_MIN_BLOCKS=2 ;;
+    t512mb3) build t512mb3 -DACSR_SPMV_THREADS=512 -DACSR_MIN_BLOCKS=3 ;;
+    t256mb6) build t256mb6 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=6 ;;
+    t256mb8) build t256mb8 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=8 ;;
     v512) build v512 -DACSR_VEC_MIN=512 ;;
     v1024) build v1024 -DACSR_VEC_MIN=1024 ;;
     v512br) build v512br -DACSR_VEC_MIN=512 -DACSR_BRANCHY_SUB=1 ;;

@@ -140,6 +140,13 @@ typedef struct {
     double *delta2;               /* [1] local sum of squared differences */
     int64_t restart;              /* RWR restart row (local index) or -1 */
     double restart_weight;        /* added to x_new[restart]: (1-c) for RWR */
+    int32_t *ctrl;                /* NULL, or [2] device: device-side convergence control.
+                                   * If ctrl[0] != 0 the call is a no-op (nothing written);
+                                   * otherwise the step runs, ctrl[1] += 1 and ctrl[0] = 1 when
+                                   * *delta2 <= eps2.  Lets the host enqueue several steps
+                                   * between synchronisations with results identical to a
+                                   * test after every step (single GPU). */
+    double eps2;                  /* convergence threshold on delta2 (eps^2) */
 } acsr_pr_args;
 
 acsr_status acsr_pagerank_step(const acsr_pr_args *args, cudaStream_t stream);

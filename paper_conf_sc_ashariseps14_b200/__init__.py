@@ -73,7 +73,7 @@ class PrArgs(ctypes.Structure):
                 ("col_idx", _vp), ("bin_rows", _vp), ("bin_offsets", _vp), ("plan_ws", _vp),
                 ("plan_ws_bytes", _sz), ("xs", _vp), ("x", _vp), ("outdeg", _vp), ("x_new", _vp),
                 ("xs_next", _vp), ("damping", _dbl), ("teleport", _dbl), ("delta2", _vp),
-                ("restart", _i64), ("restart_weight", _dbl)]
+                ("restart", _i64), ("restart_weight", _dbl), ("ctrl", _vp), ("eps2", _dbl)]
 
 
 _lib.acsr_pagerank_step.argtypes = [ctypes.POINTER(PrArgs), _vp]
@@ -192,7 +192,7 @@ def acsr_pagerank_scale(x, outdeg, xs=None, stream=None):
 
 def acsr_pagerank_step(row_begin, col_idx, bin_rows, bin_offsets, plan_ws, xs, x, outdeg, x_new,
                        xs_next, delta2, damping=0.85, teleport=None, n_global=None, row_end=None,
-                       stream=None, restart=-1, restart_weight=0.0):
+                       stream=None, restart=-1, restart_weight=0.0, ctrl=None, eps2=-1.0):
     """One fused PageRank step on the local rows (Alg. 5).  delta2: 1-element float64.
     With teleport=0, damping=c, restart=i, restart_weight=1-c it is an RWR step (Eq. 8)."""
     n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
@@ -208,7 +208,8 @@ def acsr_pagerank_step(row_begin, col_idx, bin_rows, bin_offsets, plan_ws, xs, x
                _dev(outdeg, torch.int32, "outdeg") if n else None,
                _dev(x_new, torch.float64, "x_new") if n else None,
                _dev(xs_next, torch.float64, "xs_next") if n else None, float(damping), float(tel),
-               _dev(delta2, torch.float64, "delta2"), int(restart), float(restart_weight))
+               _dev(delta2, torch.float64, "delta2"), int(restart), float(restart_weight),
+               _dev(ctrl, torch.int32, "ctrl", True), float(eps2))
     _check(_lib.acsr_pagerank_step(ctypes.byref(a), _stream(stream)), "acsr_pagerank_step")
     return x_new, xs_next, delta2
 

@@ -74,6 +74,8 @@ struct SpmvArgs {
     double *delta2;
     int64_t restart;
     double restart_weight;
+    int32_t *ctrl;  // device-side convergence: [0] stop flag, [1] executed steps (nullable)
+    double eps2;
 };
 
 // ----------------------------------------------------------------- PTX helpers
@@ -571,6 +573,7 @@ spmv_kernel(SpmvArgs<V> a)
     const int gw = blockIdx.x * SPMV_WARPS + (threadIdx.x >> 5);
     const int nw = gridDim.x * SPMV_WARPS;
     PlanHeader *hdr = a.hdr;
+    if (PR && a.ctrl && *(volatile int32_t *)a.ctrl) return;  // converged earlier: no-op step
     const int n_units = hdr->n_units;
     {
         char *ws = (char *)hdr;
@@ -639,7 +642,12 @@ spmv_kernel(SpmvArgs<V> a)
                 const uint64_t hi = *(volatile uint64_t *)&hdr->d2_hi;
                 const uint64_t mid = *(volatile uint64_t *)&hdr->d2_mid;
                 const uint64_t lo = *(volatile uint64_t *)&hdr->d2_lo;
-                *a.delta2 = (double)hi + ((double)mid + (double)lo * 5.421010862427522e-20) * 5.421010862427522e-20;
+                const double d2v = (double)hi + ((double)mid + (double)lo * 5.421010862427522e-20) * 5.421010862427522e-20;
+                *a.delta2 = d2v;
+                if (a.ctrl) {
+                    a.ctrl[1] += 1;
+                    if (d2v <= a.eps2) a.ctrl[0] = 1;
+                }
                 hdr->d2_hi = 0;
                 hdr->d2_mid = 0;
                 hdr->d2_lo = 0;
@@ -861,6 +869,7 @@ extern "C" acsr_status acsr_pagerank_step(const acsr_pr_args *p, cudaStream_t st
     a.x_old = p->x; a.outdeg = p->outdeg; a.x_new = p->x_new; a.xs_next = p->xs_next;
     a.damping = p->damping; a.teleport = p->teleport; a.delta2 = p->delta2;
     a.restart = p->restart; a.restart_weight = p->restart_weight;
+    a.ctrl = p->ctrl; a.eps2 = p->eps2;
     dispatch<double, true>(a, stream);
     return acsr_check_launch("acsr_pagerank_step");
 }

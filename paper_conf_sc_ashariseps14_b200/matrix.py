@@ -94,32 +94,45 @@ def spmv_from_host(row_ptr_h, col_h, val_h, x_h, y_h=None, device="cuda", stream
     return y_h
 
 
-def pagerank(m: ACSRMatrix, outdeg, x0=None, damping=0.85, eps=1e-6, max_iter=1000, stream=None):
-    """Alg. 5 on one GPU over the in-link pattern matrix m.  Returns (x, iterations, delta2).
-    The convergence test reads one double per iteration (the paper's host loop)."""
+def _power_loop(m: ACSRMatrix, outdeg, x, damping, teleport, eps, max_iter, check_every, stream,
+                restart=-1, restart_weight=0.0):
+    """Alg. 5-style loop with device-side convergence: up to check_every fused steps are
+    enqueued between host synchronisations; a step after convergence is a no-op (ctrl[0]),
+    so results equal a host test after every step.  Returns (x, iterations, delta2)."""
+    n = m.n_rows
+    dev = m.row_begin.device
+    bufs = [x, torch.empty_like(x)]
+    sbufs = [acsr_pagerank_scale(x, outdeg, stream=stream), torch.empty_like(x)]
+    d2 = torch.zeros(1, dtype=torch.float64, device=dev)
+    ctrl = torch.zeros(2, dtype=torch.int32, device=dev)
+    eps2 = eps * eps if eps >= 0 else -1.0
+    k = 0
+    while k < max_iter:
+        for _ in range(min(check_every, max_iter - k)):
+            acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, sbufs[k % 2],
+                               bufs[k % 2], outdeg, bufs[(k + 1) % 2], sbufs[(k + 1) % 2], d2, damping,
+                               teleport, n, m.row_end, stream, restart=restart, restart_weight=restart_weight,
+                               ctrl=ctrl, eps2=eps2)
+            k += 1
+        c = ctrl.cpu()
+        if int(c[0]):
+            break
+    it = int(c[1])
+    return bufs[it % 2], it, float(d2.item())
+
+
+def pagerank(m: ACSRMatrix, outdeg, x0=None, damping=0.85, eps=1e-6, max_iter=1000, stream=None,
+             check_every=8):
+    """Alg. 5 on one GPU over the in-link pattern matrix m (stop when
+    ||x' - x||_2 <= eps, reading Q9).  Returns (x, iterations, delta2)."""
     n = m.n_rows
     dev = m.row_begin.device
     x = torch.full((n,), 1.0 / n, dtype=torch.float64, device=dev) if x0 is None else x0.clone()
-    xs = acsr_pagerank_scale(x, outdeg, stream=stream)
-    x_new = torch.empty_like(x)
-    xs_next = torch.empty_like(x)
-    d2 = torch.zeros(1, dtype=torch.float64, device=dev)
-    teleport = (1.0 - damping) / n
-    it = 0
-    delta2 = float("inf")
-    while it < max_iter:
-        acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xs, x,
-                           outdeg, x_new, xs_next, d2, damping, teleport, n, m.row_end, stream)
-        x, x_new = x_new, x
-        xs, xs_next = xs_next, xs
-        it += 1
-        delta2 = float(d2.item())
-        if delta2 ** 0.5 <= eps:
-            break
-    return x, it, delta2
+    return _power_loop(m, outdeg, x, damping, (1.0 - damping) / n, eps, max_iter, check_every, stream)
 
 
-def rwr(m: ACSRMatrix, outdeg, restart: int, c=0.85, eps=1e-6, max_iter=1000, r0=None, stream=None):
+def rwr(m: ACSRMatrix, outdeg, restart: int, c=0.85, eps=1e-6, max_iter=1000, r0=None, stream=None,
+        check_every=8):
     """Random Walk with Restart (Eq. 8; reading R5) on the in-link pattern m:
     r' = c (W r) + (1-c) e_restart, r^0 = e_restart.  One fused acsr_pagerank_step per
     iteration (teleport 0, restart weight 1-c).  Returns (r, iterations, delta2)."""
@@ -130,21 +143,8 @@ def rwr(m: ACSRMatrix, outdeg, restart: int, c=0.85, eps=1e-6, max_iter=1000, r0
         r[restart] = 1.0
     else:
         r = r0.clone()
-    rs = acsr_pagerank_scale(r, outdeg, stream=stream)
-    r_new, rs_next = torch.empty_like(r), torch.empty_like(r)
-    d2 = torch.zeros(1, dtype=torch.float64, device=dev)
-    it, delta2 = 0, float("inf")
-    while it < max_iter:
-        acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, rs, r, outdeg,
-                           r_new, rs_next, d2, c, 0.0, n, m.row_end, stream, restart=restart,
-                           restart_weight=1.0 - c)
-        r, r_new = r_new, r
-        rs, rs_next = rs_next, rs
-        it += 1
-        delta2 = float(d2.item())
-        if delta2 ** 0.5 <= eps:
-            break
-    return r, it, delta2
+    return _power_loop(m, outdeg, r, c, 0.0, eps, max_iter, check_every, stream, restart=restart,
+                       restart_weight=1.0 - c)
 
 
 def hits_matrix(out_ptr, out_col, n=None):

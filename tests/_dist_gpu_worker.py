@@ -1,0 +1,31 @@
+"""Worker for tests/test_gpu_parity.py::test_dist_pagerank_two_ranks_one_gpu (spawned)."""
+import os
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+
+def worker(rank, world, port, scale, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import synth
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+    dev = torch.device("cuda:0")
+    rp, ci = synth.rmat_csr(scale, transpose=True)
+    n = rp.numel() - 1
+    od = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    splits = pdist.partition_rows(np.diff(rp.numpy()), world)
+    lo, hi = int(splits[rank]), int(splits[rank + 1])
+    rpl = (rp[lo:hi + 1] - rp[lo]).to(dev)
+    cil = ci[int(rp[lo]):int(rp[hi])].to(dev)
+    pr = pdist.DistPageRank(rpl, cil, od[lo:hi].to(dev), splits, n)
+    x, it, d2 = pr.run(eps=1e-6)
+    parts = [torch.zeros(pr.L, dtype=torch.float64) for _ in range(world)]
+    xp = torch.zeros(pr.L, dtype=torch.float64)
+    xp[: x.numel()] = x.cpu()
+    dist.all_gather(parts, xp)
+    if rank == 0:
+        full = torch.cat([parts[k][: int(splits[k + 1] - splits[k])] for k in range(world)])
+        q.put((full.numpy(), it))
+    dist.destroy_process_group()

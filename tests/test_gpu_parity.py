@@ -6,6 +6,8 @@ order is exact).  SpMV on U(-1,1) data: |y - y_ref| <= 1e-12 * (|A||x|)_r in fp6
 (+0.0 for empty rows).  PageRank: step-wise at the fp64 bar, loop iteration count within
 +-1 of the oracle (reading Q18).
 """
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -633,3 +635,45 @@ def test_spmv_from_host_e2e(acsr, cuda):
     y = acsr.spmv_from_host(rp.pin_memory(), ci.pin_memory(), val.pin_memory(), x.pin_memory(), device=cuda)
     y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
     check_spmv(y.numpy(), y_ref, den, torch.float64)
+
+
+def test_dist_pagerank_two_ranks_one_gpu(cuda):
+    # the partitioned driver with two ranks sharing the GPU (gloo for the exchange): CUDA
+    # step + column renumbering + padded all-gather + Delta^2 all-reduce vs the oracle
+    import socket
+    import sys
+    import torch.multiprocessing as mp
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    import _dist_gpu_worker
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_dist_gpu_worker.worker, args=(r, 2, port, 14, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    full, it = q.get(timeout=300)
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    rp, ci, od, n = _inlink(14, cuda)
+    x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)
+    assert abs(it - it_ref) <= 1
+    if it != it_ref:
+        x_ref, _, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=0.0, max_iter=it)
+    assert np.all(np.abs(full - x_ref) <= 1e-11 * x_ref + 1e-18)
+
+
+def test_device_side_convergence_identical(acsr, cuda):
+    # enqueueing 8 steps between host checks (ctrl no-op steps after convergence) gives the
+    # same iterate, iteration count and Delta^2 as a host test after every step
+    rp, ci, od, n = _inlink(15, cuda)
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda))
+    x1, it1, d1 = acsr.pagerank(m, od.to(cuda), eps=1e-6, check_every=1)
+    x8, it8, d8 = acsr.pagerank(m, od.to(cuda), eps=1e-6, check_every=8)
+    assert it1 == it8 and d1 == d8 and torch.equal(x1, x8)
+    r1, j1, _ = acsr.rwr(m, od.to(cuda), 3, check_every=1)
+    r8, j8, _ = acsr.rwr(m, od.to(cuda), 3, check_every=8)
+    assert j1 == j8 and torch.equal(r1, r8)

@@ -14,7 +14,10 @@ namespace acsr {
 // of 256 rows in row order).  The per-(bin, tile) counts double as the row-space
 // locality unit of the SpMV work map.
 constexpr int BIN_THREADS = 256;
-constexpr int TILE_ROWS = 1024;
+#ifndef ACSR_TILE_ROWS
+#define ACSR_TILE_ROWS 1024
+#endif
+constexpr int TILE_ROWS = ACSR_TILE_ROWS;
 constexpr int TILE_ROUNDS = TILE_ROWS / BIN_THREADS;
 constexpr int NBINS = ACSR_NBINS;
 
@@ -27,11 +30,25 @@ constexpr int LIGHT_MAX_BIN = 10;
 constexpr int HEAVY_BIN = LIGHT_MAX_BIN + 1;
 constexpr int HEAVY_CHUNK = 1024;  // power of two
 
-// rows per light work unit, by bin (~6-12 KB of CSR traffic per unit)
-__host__ __device__ constexpr int unit_rows(int b)
+// rows per light work unit, by bin (~6-12 KB of CSR traffic per unit); ACSR_UNIT_SHIFT
+// scales them by 2^shift for A/B builds
+#ifndef ACSR_UNIT_SHIFT
+#define ACSR_UNIT_SHIFT 0
+#endif
+#ifndef ACSR_UNIT_WARP_SHIFT
+#define ACSR_UNIT_WARP_SHIFT 0  // extra right shift for the warp-per-row bins 7..10 (A/B)
+#endif
+__host__ __device__ constexpr int unit_rows_base(int b)
 {
     return b == 0 ? 1024 : b == 1 ? 256 : b == 2 ? 128 : b == 3 ? 128 : b == 4 ? 64
-         : b == 5 ? 32 : b == 6 ? 16 : b == 7 ? 8 : b == 8 ? 4 : b == 9 ? 2 : 1;
+         : b == 5 ? 32 : b == 6 ? 16
+         : ((b == 7 ? 8 : b == 8 ? 4 : b == 9 ? 2 : 1) >> ACSR_UNIT_WARP_SHIFT) > 0
+             ? ((b == 7 ? 8 : b == 8 ? 4 : b == 9 ? 2 : 1) >> ACSR_UNIT_WARP_SHIFT) : 1;
+}
+__host__ __device__ constexpr int unit_rows(int b)
+{
+    return ACSR_UNIT_SHIFT >= 0 ? unit_rows_base(b) << ACSR_UNIT_SHIFT
+                                : (unit_rows_base(b) >> -ACSR_UNIT_SHIFT) > 0 ? unit_rows_base(b) >> -ACSR_UNIT_SHIFT : 1;
 }
 
 // Persistent CTAs (grid = resident CTAs per SM x SMs).  1024 threads: the whole SM

@@ -38,6 +38,9 @@
 #ifndef ACSR_NO_VEC
 #define ACSR_NO_VEC 0  // 1: never use the 128-bit vector path (A/B builds)
 #endif
+#ifndef ACSR_PAIR_ROWS
+#define ACSR_PAIR_ROWS 0  // 1: warp-per-row bins process two rows at a time (A/B builds)
+#endif
 #ifndef ACSR_VEC_MIN
 #define ACSR_VEC_MIN 512  // rows (chunks) shorter than this use the lane-strided scalar path
 #endif
@@ -486,6 +489,34 @@ struct Kern {
         const int myr = lane < cnt ? __ldg(a.bin_rows + start + lane) : 0;
         int mb = 0, me = 0;
         if (lane < cnt) row_bounds(a, myr, mb, me);
+#if ACSR_PAIR_ROWS
+        // two rows in flight: element k of a row feeds accumulator (k mod 64) < 32 ? p : q,
+        // whether or not the row has a partner -> per-row order independent of pairing
+        for (int i = 0; i < cnt; i += 2) {
+            const bool has1 = i + 1 < cnt;
+            const int r0 = __shfl_sync(0xffffffffu, myr, i);
+            const int b0 = __shfl_sync(0xffffffffu, mb, i);
+            const int l0 = __shfl_sync(0xffffffffu, me, i) - b0;
+            const int r1 = __shfl_sync(0xffffffffu, myr, has1 ? i + 1 : i);
+            const int b1 = __shfl_sync(0xffffffffu, mb, has1 ? i + 1 : i);
+            const int l1 = has1 ? __shfl_sync(0xffffffffu, me, i + 1) - b1 : 0;
+            double p0 = 0.0, q0 = 0.0, p1 = 0.0, q1 = 0.0;
+            const int L = max(l0, l1);
+            for (int k = lane; k < L; k += 64) {
+                p0 = fmacp(a, k < l0, b0 + k, p0);
+                q0 = fmacp(a, k + 32 < l0, b0 + k + 32, q0);
+                p1 = fmacp(a, k < l1, b1 + k, p1);
+                q1 = fmacp(a, k + 32 < l1, b1 + k + 32, q1);
+            }
+            const double s0 = warp_sum(p0 + q0);
+            const double s1 = warp_sum(p1 + q1);
+            if (lane == 0) {
+                finish(a, r0, s0, d2);
+                if (has1) finish(a, r1, s1, d2);
+            }
+        }
+        return;
+#endif
         for (int i = 0; i < cnt; i++) {
             const int r = __shfl_sync(0xffffffffu, myr, i);
             const int beg = __shfl_sync(0xffffffffu, mb, i);

@@ -21,6 +21,15 @@ for v in "$@"; do
     nvbr) build nvbr -DACSR_NO_VEC=1 -DACSR_BRANCHY_SUB=1 ;;
     v256) build v256 -DACSR_VEC_MIN=256 ;;
     mb2) build mb2 -DACSR_MIN_BLOCKS=2 ;;
+    u1) build u1 -DACSR_UNIT_SHIFT=1 ;;
+    uw1) build uw1 -DACSR_UNIT_WARP_SHIFT=1 ;;
+    pr) build pr -DACSR_PAIR_ROWS=1 ;;
+    pruw1) build pruw1 -DACSR_PAIR_ROWS=1 -DACSR_UNIT_WARP_SHIFT=1 ;;
+    uw2) build uw2 -DACSR_UNIT_WARP_SHIFT=2 ;;
+    um1uw0) build um1uw0 -DACSR_UNIT_SHIFT=-1 ;;
+    um1) build um1 -DACSR_UNIT_SHIFT=-1 ;;
+    tile2k) build tile2k -DACSR_TILE_ROWS=2048 ;;
+    tile512) build tile512 -DACSR_TILE_ROWS=512 ;;
     t512mb3) build t512mb3 -DACSR_SPMV_THREADS=512 -DACSR_MIN_BLOCKS=3 ;;
     t256mb6) build t256mb6 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=6 ;;
     t256mb8) build t256mb8 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=8 ;;

@@ -20,13 +20,24 @@ def main():
         rp, ci = synth.powerlaw_csr(seed=4, device=dev, **synth.LIVEJOURNAL)
     n, nnz = rp.numel() - 1, ci.numel()
     val = synth.values(nnz, 1014, dtype, dev); x = synth.vector(n, 2014, dtype, dev)
+    colperm = os.environ.get("COLPERM") == "1"
+    t_relabel = None
+    if colperm:  # experiment: columns renumbered by decreasing frequency (x gathered through q)
+        torch.cuda.synchronize(); t0 = time.perf_counter()
+        cnt = torch.bincount(ci.long(), minlength=n)
+        q = torch.sort(cnt, descending=True, stable=True).indices
+        p = torch.empty_like(q); p[q] = torch.arange(n, device=dev)
+        ci = p[ci.long()].to(torch.int32)
+        torch.cuda.synchronize(); t_relabel = time.perf_counter() - t0
     m = acsr.ACSRMatrix(rp, ci, val)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     tb, ts = [], []
     for i in range(reps + 3):
         flush.zero_()
         e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
-        e[0].record(); m.rebin(); e[1].record(); y = m.spmv(x); e[2].record()
+        e[0].record(); m.rebin(); e[1].record()
+        y = m.spmv(x[q] if colperm else x)
+        e[2].record()
         torch.cuda.synchronize()
         if i >= 3:
             tb.append(e[0].elapsed_time(e[1])); ts.append(e[1].elapsed_time(e[2]))
@@ -36,6 +47,7 @@ def main():
     print(json.dumps({"wl": wl, "env": {k: v for k, v in os.environ.items() if k.startswith("ACSR_")},
                       "t_bin_us": round(1e3 * float(np.median(tb)), 2), "t_spmv_us": round(1e3 * float(np.median(ts)), 2),
                       "t_spmv_min_us": round(1e3 * float(np.min(ts)), 2),
-                      "spmv_GBs": round(alg / (np.median(ts) * 1e-3) / 1e9, 1), "nnz": nnz, "n": n}))
+                      "spmv_GBs": round(alg / (np.median(ts) * 1e-3) / 1e9, 1), "nnz": nnz, "n": n,
+                      "colperm": colperm, "t_relabel_s": t_relabel}))
 
 main()

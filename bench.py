@@ -46,8 +46,16 @@ def peaks():
 
 
 class Clocks:
-    """Sample nvidia-smi clocks + throttle reasons during the timed region."""
+    """Sample SM clocks + throttle reasons DURING the timed region.
 
+    NVML (pynvml) is polled from a thread every ~2 ms, so even a few-ms timed region
+    gets samples; `nvidia-smi -lms 100` is the fallback when NVML is unavailable.  The
+    sampler is started (and its first sample awaited) before the timed region."""
+
+    REASONS = (("hw_slowdown", "nvmlClocksEventReasonHwSlowdown"),
+               ("hw_thermal_slowdown", "nvmlClocksEventReasonHwThermalSlowdown"),
+               ("sw_thermal_slowdown", "nvmlClocksEventReasonSwThermalSlowdown"),
+               ("sw_power_cap", "nvmlClocksEventReasonSwPowerCap"))
     Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
@@ -56,8 +64,48 @@ class Clocks:
         self.index = index
         self.proc = None
         self.lines = []
+        self.samples = []  # (sm_mhz, max_mhz, reasons bitmask)
+        self.stop = threading.Event()
+        self.nv = None
+
+    def _nvml_handle(self):
+        import pynvml
+        pynvml.nvmlInit()
+        idx = self.index
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES", "")
+        ids = [v.strip() for v in vis.split(",") if v.strip()]
+        if ids and idx < len(ids):
+            if ids[idx].isdigit():
+                idx = int(ids[idx])
+            else:
+                return pynvml, pynvml.nvmlDeviceGetHandleByUUID(ids[idx])
+        return pynvml, pynvml.nvmlDeviceGetHandleByIndex(idx)
+
+    def _poll(self):
+        nv, h = self.nv
+        mx = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+        while True:
+            try:
+                sm = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
+                rs = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+                self.samples.append((float(sm), float(mx), int(rs)))
+            except Exception:
+                pass
+            if self.stop.wait(0.002):
+                break
 
     def __enter__(self):
+        try:
+            self.nv = self._nvml_handle()
+            self.t = threading.Thread(target=self._poll, daemon=True)
+            self.t.start()
+            t0 = time.perf_counter()
+            while not self.samples and time.perf_counter() - t0 < 2.0:
+                time.sleep(0.001)
+            self.n0 = len(self.samples)
+            return self
+        except Exception:
+            self.nv = None
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
                                           "--format=csv,noheader,nounits", "-lms", "100"],
@@ -73,6 +121,11 @@ class Clocks:
             self.lines.append(line.strip())
 
     def __exit__(self, *a):
+        if self.nv is not None:
+            self.n1 = len(self.samples)
+            self.stop.set()
+            self.t.join(1.0)
+            return
         if self.proc:
             time.sleep(0.25)
             self.proc.terminate()
@@ -82,8 +135,17 @@ class Clocks:
                 self.proc.kill()
 
     def summary(self):
+        if self.nv is not None:
+            nv = self.nv[0]
+            # samples taken while the timed region ran (plus the one awaited before it)
+            s = self.samples[max(0, self.n0 - 1):self.n1] or self.samples[-1:]
+            reasons = sorted({name for name, attr in self.REASONS
+                              for (_, _, rs) in s if rs & getattr(nv, attr, 0)})
+            return {"sm_mhz": float(np.median([v[0] for v in s])) if s else None,
+                    "sm_max_mhz": max(v[1] for v in s) if s else None,
+                    "reasons": reasons, "samples": len(s), "source": "nvml, 2 ms poll"}
         sm, mx, reasons = [], 0.0, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        names = [r[0] for r in self.REASONS]
         for l in self.lines:
             f = [x.strip() for x in l.split(",")]
             if len(f) < 6:
@@ -97,7 +159,7 @@ class Clocks:
                 if v.lower().startswith("active"):
                     reasons.add(n)
         return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx or None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+                "reasons": sorted(reasons), "samples": len(sm), "source": "nvidia-smi -lms 100"}
 
 
 # ------------------------------------------------------------------------------ workloads
@@ -640,7 +702,7 @@ def run_reference(args, dev):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="acsr", choices=["acsr", "reference"])
     ap.add_argument("--workload", default="rmat20")

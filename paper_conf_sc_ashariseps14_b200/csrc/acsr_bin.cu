@@ -86,7 +86,8 @@ __device__ __forceinline__ void count_tile(BinSmem &sm, int64_t n, const int32_t
     if (tid == NBINS) {
         int lu = 0;
 #pragma unroll
-        for (int b = 0; b <= LIGHT_MAX_BIN; b++) lu += (sm.hist[b] + unit_rows(b) - 1) / unit_rows(b);
+        for (int b = WIN_MAX_BIN + 1; b <= LIGHT_MAX_BIN; b++) lu += (sm.hist[b] + unit_rows(b) - 1) / unit_rows(b);
+        if (WIN_MAX_BIN >= 0) lu += win_units((int)min((int64_t)TILE_ROWS, n - base));
         cnt[(int64_t)NBINS * n_tiles + tile] = lu;
         cnt[(int64_t)(NBINS + 1) * n_tiles + tile] = sm.heavy;
     }
@@ -273,12 +274,15 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
         __syncthreads();
     }
     if (!overflow) {
-        // light work units of this tile: bins 0..10, in bin order, row-contiguous
+        // light work units of this tile: the short-row windows (row order), then the
+        // bins above WIN_MAX_BIN up to 10, in bin order, row-contiguous
+        const int tile_rows = (int)min((int64_t)TILE_ROWS, n - base);
+        const int nwin = WIN_MAX_BIN >= 0 ? win_units(tile_rows) : 0;
         if (tid == 0) {
-            int acc = 0;
+            int acc = nwin;
             for (int b = 0; b <= LIGHT_MAX_BIN; b++) {
                 sm.upre[b] = acc;
-                acc += (sm.run[b] + unit_rows(b) - 1) / unit_rows(b);
+                if (b > WIN_MAX_BIN) acc += (sm.run[b] + unit_rows(b) - 1) / unit_rows(b);
             }
             sm.upre[LIGHT_MAX_BIN + 1] = acc;
         }
@@ -286,6 +290,11 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
         const int ubase = n_heavy + toff[(int64_t)NBINS * n_tiles + tile];
         const int total = sm.upre[LIGHT_MAX_BIN + 1];
         for (int j = tid; j < total; j += BIN_THREADS) {
+            if (j < nwin) {
+                const int r0 = j * WIN_UNIT_ROWS;
+                units[ubase + j] = make_int2((int)(base + r0), (int)(WIN_FLAG | (uint32_t)min(WIN_UNIT_ROWS, tile_rows - r0)));
+                continue;
+            }
             int b = 0;
             while (sm.upre[b + 1] <= j) b++;
             const int q = j - sm.upre[b];
@@ -304,6 +313,7 @@ bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__res
                  int32_t *__restrict__ cnt, int n_tiles, PlanHeader *hdr)
 {
     __shared__ BinSmem sm;
+    pdl_enter();
     if (blockIdx.x == 0 && threadIdx.x == 0) hdr->scan_ticket = 0;  // bin_scan runs after us
     count_tile<HAS_END>(sm, n, rb, re, cnt, n_tiles, blockIdx.x);
 }
@@ -315,6 +325,7 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
                 PlanHeader *hdr, ScanArgs sa)
 {
     __shared__ BinSmem sm;
+    pdl_enter();
     scan_row<SCAN_THREADS, 1>(sm, cnt, toff, n_tiles, hdr, sa, blockIdx.x);
 }
 
@@ -326,6 +337,7 @@ bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__r
                    int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap)
 {
     __shared__ BinSmem sm;
+    pdl_enter();
     scatter_tile<HAS_END>(sm, n, rb, re, bin_rows, bin_offsets, toff, n_tiles, hdr, units, tickets, heavy_cap,
                           blockIdx.x);
 }
@@ -458,19 +470,24 @@ extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
         if (e == cudaSuccess) goto xc;
         cudaGetLastError();  // not supported here (e.g. MPS limits): fall back to three launches
     }
-    if (row_end)
-        bin_count_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
-    else
-        bin_count_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, cnt, nt, hdr);
-    bin_scan_kernel<<<SCAN_ROWS, SCAN_THREADS, 0, stream>>>(cnt, toff, nt, hdr, sa);
-    if (row_end)
-        bin_scatter_kernel<true><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, bin_rows,
-                                                                   bin_offsets, toff, nt, hdr, units,
-                                                                   tickets, L.heavy_cap);
-    else
-        bin_scatter_kernel<false><<<nt, BIN_THREADS, 0, stream>>>(n_rows, row_begin, row_end, bin_rows,
-                                                                    bin_offsets, toff, nt, hdr, units,
-                                                                    tickets, L.heavy_cap);
+    {
+        const int64_t nr = n_rows;
+        const int32_t *rb = row_begin, *re = row_end;
+        const int32_t *cbo = bin_offsets, *ctoff = toff;
+        const PlanHeader *chdr = hdr;
+        if (row_end)
+            launch_pdl(bin_count_kernel<true>, nt, BIN_THREADS, 0, stream, nr, rb, re, cnt, nt, hdr);
+        else
+            launch_pdl(bin_count_kernel<false>, nt, BIN_THREADS, 0, stream, nr, rb, re, cnt, nt, hdr);
+        const int32_t *ccnt = cnt;
+        launch_pdl(bin_scan_kernel, SCAN_ROWS, SCAN_THREADS, 0, stream, ccnt, toff, nt, hdr, sa);
+        if (row_end)
+            launch_pdl(bin_scatter_kernel<true>, nt, BIN_THREADS, 0, stream, nr, rb, re, bin_rows, cbo, ctoff, nt, chdr,
+                       units, tickets, L.heavy_cap);
+        else
+            launch_pdl(bin_scatter_kernel<false>, nt, BIN_THREADS, 0, stream, nr, rb, re, bin_rows, cbo, ctoff, nt,
+                       chdr, units, tickets, L.heavy_cap);
+    }
 xc:
     if (xc_valid) {
         cudaMemsetAsync(ws + L.off_xc_vote, 0, sizeof(uint64_t) * XC_SLOTS, stream);

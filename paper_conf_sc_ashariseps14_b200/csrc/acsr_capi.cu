@@ -2,6 +2,7 @@
 #include <cuda_runtime.h>
 #include <stdarg.h>
 #include <stdio.h>
+#include <stdlib.h>
 
 #include "acsr_internal.cuh"
 
@@ -23,6 +24,16 @@ acsr_status acsr_check_launch(const char *what)
         return ACSR_ERR_CUDA;
     }
     return ACSR_OK;
+}
+
+bool acsr::acsr_pdl_enabled()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("ACSR_PDL");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
 }
 
 int acsr_num_sms()

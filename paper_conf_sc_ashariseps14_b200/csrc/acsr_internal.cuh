@@ -71,9 +71,43 @@ constexpr int XC_SLOTS = 1 << XC_BITS;
 constexpr uint16_t XC_NOTAG = 0xFFFF;
 constexpr int XC_SAMPLE_LOG2 = 20;  // ~2^20 sampled entries per acsr_bin
 
+// ---------------------------------------------------------------- short-row windows
+// Rows of the shortest bins (0..WIN_MAX_BIN, i.e. len <= WIN_MAX_LEN) are not read
+// through bin_rows one sub-warp per row: a warp takes WIN_ROWS = 32 CONSECUTIVE rows
+// (one per lane), concatenates the nnz of its short rows (coalesced col/val loads of
+// what are contiguous CSR runs), gathers x, and each lane sums its own row's products
+// in element order from a per-warp shared-memory buffer.  Longer rows of the window
+// are left to their bin units.  Measured reason: in bin order every
+// short row costs a random row_ptr sector, partial col/val sectors and a random y
+// sector, 22-29 % extra L2 sectors on the power-law matrices.  ACSR_WINDOW=0 restores
+// the per-bin Alg. 2 mapping for bins 1..6 (A/B builds).
+#ifndef ACSR_WINDOW
+#define ACSR_WINDOW 1
+#endif
+#ifndef ACSR_WIN_MAX_BIN
+#define ACSR_WIN_MAX_BIN 5
+#endif
+#ifndef ACSR_WIN_UNIT_ROWS
+#define ACSR_WIN_UNIT_ROWS 128
+#endif
+#ifndef ACSR_WIN_G
+#define ACSR_WIN_G 4
+#endif
+constexpr int WIN_MAX_BIN = ACSR_WINDOW ? ACSR_WIN_MAX_BIN : -1;  // -1: no windows
+constexpr int WIN_MAX_LEN = 1 << (ACSR_WIN_MAX_BIN > 0 ? ACSR_WIN_MAX_BIN : 0);  // bin b holds len <= 2^b (b >= 1)
+constexpr int WIN_ROWS = 32;
+constexpr int WIN_UNIT_ROWS = ACSR_WIN_UNIT_ROWS;  // multiple of WIN_ROWS
+constexpr int WIN_G = ACSR_WIN_G;                  // 32-element groups in flight per chunk
+static_assert(WIN_UNIT_ROWS % WIN_ROWS == 0, "window unit = whole windows");
+static_assert(TILE_ROWS % WIN_UNIT_ROWS == 0, "tiles hold whole window units");
+
+__host__ __device__ constexpr int win_units(int tile_rows) { return (tile_rows + WIN_UNIT_ROWS - 1) / WIN_UNIT_ROWS; }
+
 // unit descriptor: light  x = first index into bin_rows, y = (bin << 24) | rows
 //                  heavy  x = row id,                     y = 0x80000000 | chunk
+//                  window x = first row,                  y = 0x40000000 | rows
 constexpr uint32_t HEAVY_FLAG = 0x80000000u;
+constexpr uint32_t WIN_FLAG = 0x40000000u;
 
 // ---------------------------------------------------------------- plan header
 struct PlanHeader {
@@ -152,6 +186,39 @@ __device__ __forceinline__ uint32_t mix32(uint32_t v)
     v *= 0x846ca68bU;
     v ^= v >> 16;
     return v;
+}
+
+// ---------------------------------------------------------------- programmatic dependent launch
+// The hot-path kernels of one step (bin_count -> bin_scan -> bin_scatter -> spmv, and
+// back-to-back PageRank steps) are launched with programmatic stream serialization:
+// the next grid is launched while the previous one runs and parks in
+// griddepcontrol.wait until the previous grid has completed and its writes are
+// visible, which hides the launch latency between the short kernels.  Every kernel
+// launched this way calls pdl_enter() before its first global-memory access.
+// ACSR_PDL=0 (environment) launches them plainly (A/B).
+__device__ __forceinline__ void pdl_enter()
+{
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
+bool acsr_pdl_enabled();
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t stream,
+                              Args... args)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = stream;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = acsr_pdl_enabled() ? 1 : 0;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
 }
 
 }  // namespace acsr

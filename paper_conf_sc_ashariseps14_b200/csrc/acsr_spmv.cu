@@ -526,6 +526,79 @@ struct Kern {
         }
     }
 
+    // masked product: val[k] * x[col[k]] when p, else 0 (no memory touched)
+    static __device__ __forceinline__ double prodp(const A &a, bool p, int k)
+    {
+        const int c = p ? lds_i(a.col + k) : 0;
+        const double xv = gxp(a, p, c);
+        if (HAS_VAL) return (p ? lds_v(a.val + k) : 0.0) * xv;
+        return xv;
+    }
+
+    // Short-row windows (acsr_internal.cuh): rows r0 .. r0+nrows-1, 32 per pass, lane i
+    // owns row r0 + w + i.  The nnz of the window's short rows (len <= WIN_MAX_LEN) are
+    // concatenated in row order; element t of the concatenation is loaded by lane
+    // t mod 32 (coalesced over the CSR runs), its row found from the head bitmask of the
+    // 32-element group and a per-warp (beg, pre) table of the non-empty short rows.
+    // Products go to a per-warp shared buffer; each lane then adds ITS row's products in
+    // element order, so a row's sum depends only on the row (as in every other mapping).
+    static __device__ __forceinline__ void window(const A &a, int r0, int nrows, int lane, Fix192 &d2,
+                                                  double *buf, int2 *tab)
+    {
+        constexpr unsigned FULL = 0xffffffffu;
+        const unsigned lt = (1u << lane) - 1u;
+        const unsigned le = 0xffffffffu >> (31 - lane);
+        for (int w = 0; w < nrows; w += WIN_ROWS) {
+            const int r = r0 + w + lane;
+            const bool in = w + lane < nrows;
+            int beg = 0, end = 0;
+            if (in) row_bounds(a, r, beg, end);
+            const int len = end - beg;
+            const bool mine = in && len <= WIN_MAX_LEN;
+            const int l = mine ? len : 0;
+            int incl = l;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const int t = __shfl_up_sync(FULL, incl, d);
+                if (lane >= d) incl += t;
+            }
+            const int pre = incl - l;
+            const int T = __shfl_sync(FULL, incl, 31);
+            const unsigned ne = __ballot_sync(FULL, l > 0);
+            if (l > 0) tab[__popc(ne & lt)] = make_int2(beg, pre);
+            __syncwarp();
+            double acc = 0.0;
+            for (int t0 = 0; t0 < T; t0 += 32 * WIN_G) {
+                double p[WIN_G];
+#pragma unroll
+                for (int g = 0; g < WIN_G; g++) {
+                    const int cb = t0 + 32 * g;
+                    const bool hd = l > 0 && pre >= cb && pre < cb + 32;
+                    const unsigned H = __reduce_or_sync(FULL, hd ? 1u << (pre - cb) : 0u);
+                    const int q0 = __popc(__ballot_sync(FULL, l > 0 && pre < cb));
+                    const int t = cb + lane;
+                    const bool v = t < T;
+                    int k = 0;
+                    if (v) {
+                        const int2 bp = tab[q0 + __popc(H & le) - 1];
+                        k = bp.x + (t - bp.y);
+                    }
+                    p[g] = prodp(a, v, k);
+                }
+#pragma unroll
+                for (int g = 0; g < WIN_G; g++) buf[32 * g + lane] = p[g];
+                __syncwarp();
+                if (l > 0) {
+                    const int i1 = min(pre + l, t0 + 32 * WIN_G) - t0;
+                    for (int i = max(pre, t0) - t0; i < i1; i++) acc += buf[i];
+                }
+                __syncwarp();
+            }
+            if (mine) finish(a, r, acc, d2);
+            __syncwarp();  // tab / buf reused by the next window
+        }
+    }
+
     static __device__ __forceinline__ void empty_rows(const A &a, int start, int cnt, int lane, Fix192 &d2)
     {
         for (int i = lane; i < cnt; i += 32) finish(a, __ldg(a.bin_rows + start + i), 0.0, d2);
@@ -563,12 +636,16 @@ struct Kern {
         }
     }
 
-    static __device__ __forceinline__ void unit(const A &a, int u, int lane, Fix192 &d2)
+    static __device__ __forceinline__ void unit(const A &a, int u, int lane, Fix192 &d2, double *wbuf, int2 *wtab)
     {
         const int2 d = __ldg(a.units + u);
         const uint32_t y = (uint32_t)d.y;
         if (y & HEAVY_FLAG) {
             heavy(a, u, d.x, (int)(y & ~HEAVY_FLAG), lane, d2);
+            return;
+        }
+        if (WIN_MAX_BIN >= 0 && (y & WIN_FLAG)) {
+            window(a, d.x, (int)(y & 0xFFFFFF), lane, d2, wbuf, wtab);
             return;
         }
         const int b = (int)(y >> 24), cnt = (int)(y & 0xFFFFFF);
@@ -604,6 +681,7 @@ spmv_kernel(SpmvArgs<V> a)
     const int gw = blockIdx.x * SPMV_WARPS + (threadIdx.x >> 5);
     const int nw = gridDim.x * SPMV_WARPS;
     PlanHeader *hdr = a.hdr;
+    pdl_enter();
     if (PR && a.ctrl && *(volatile int32_t *)a.ctrl) return;  // converged earlier: no-op step
     const int n_units = hdr->n_units;
     {
@@ -632,15 +710,20 @@ spmv_kernel(SpmvArgs<V> a)
         a.xval = sval;
         a.xtag = stag;
     }
+    // per-warp short-row window scratch (products + (beg, pre) table)
+    __shared__ double win_buf[WIN_MAX_BIN >= 0 ? SPMV_WARPS * 32 * WIN_G : 1];
+    __shared__ int2 win_tab[WIN_MAX_BIN >= 0 ? SPMV_WARPS * 32 : 1];
+    double *wbuf = win_buf + (WIN_MAX_BIN >= 0 ? (threadIdx.x >> 5) * 32 * WIN_G : 0);
+    int2 *wtab = win_tab + (WIN_MAX_BIN >= 0 ? (threadIdx.x >> 5) * 32 : 0);
     Fix192 d2{0, 0, 0};
 #if ACSR_SCHED_STATIC
-    for (int u = gw; u < n_units; u += nw) K::unit(a, u, lane, d2);
+    for (int u = gw; u < n_units; u += nw) K::unit(a, u, lane, d2, wbuf, wtab);
 #else
     int u = gw;
     int nxt = 0;
     if (lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
     while (u < n_units) {
-        K::unit(a, u, lane, d2);
+        K::unit(a, u, lane, d2, wbuf, wtab);
         u = __shfl_sync(0xffffffffu, nxt, 0) + nw;
         if (u < n_units && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
     }
@@ -743,7 +826,7 @@ static void launch(const SpmvArgs<V> &a, cudaStream_t s)
                                                       SPMV_THREADS, smem);
         if (per_sm < 1) per_sm = 1;
     }
-    spmv_kernel<V, HAS_VAL, HAS_END, PR, XC><<<per_sm * acsr_num_sms(), SPMV_THREADS, smem, s>>>(a);
+    launch_pdl(spmv_kernel<V, HAS_VAL, HAS_END, PR, XC>, per_sm * acsr_num_sms(), SPMV_THREADS, smem, s, a);
 }
 
 template <typename V, bool PR, bool XC>

@@ -36,6 +36,17 @@ for v in "$@"; do
     v512) build v512 -DACSR_VEC_MIN=512 ;;
     v1024) build v1024 -DACSR_VEC_MIN=1024 ;;
     v512br) build v512br -DACSR_VEC_MIN=512 -DACSR_BRANCHY_SUB=1 ;;
+    w0) build w0 -DACSR_WINDOW=0 ;;
+    wu128) build wu128 -DACSR_WIN_UNIT_ROWS=128 ;;
+    wu32) build wu32 -DACSR_WIN_UNIT_ROWS=32 ;;
+    wu64) build wu64 -DACSR_WIN_UNIT_ROWS=64 ;;
+    wg2) build wg2 -DACSR_WIN_G=2 ;;
+    wg8) build wg8 -DACSR_WIN_G=8 ;;
+    wb4) build wb4 -DACSR_WIN_MAX_BIN=4 ;;
+    wb6) build wb6 -DACSR_WIN_MAX_BIN=6 ;;
+    wb6u128) build wb6u128 -DACSR_WIN_MAX_BIN=6 -DACSR_WIN_UNIT_ROWS=128 ;;
+    wb6u256) build wb6u256 -DACSR_WIN_MAX_BIN=6 -DACSR_WIN_UNIT_ROWS=256 ;;
+    wu256) build wu256 -DACSR_WIN_UNIT_ROWS=256 ;;
   esac
 done
 wait

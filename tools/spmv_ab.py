@@ -47,6 +47,7 @@ def main():
     print(json.dumps({"wl": wl, "env": {k: v for k, v in os.environ.items() if k.startswith("ACSR_")},
                       "t_bin_us": round(1e3 * float(np.median(tb)), 2), "t_spmv_us": round(1e3 * float(np.median(ts)), 2),
                       "t_spmv_min_us": round(1e3 * float(np.min(ts)), 2),
+                      "t_spmv_mean_us": round(1e3 * float(np.mean(ts)), 2),
                       "spmv_GBs": round(alg / (np.median(ts) * 1e-3) / 1e9, 1), "nnz": nnz, "n": n,
                       "colperm": colperm, "t_relabel_s": t_relabel}))
 

@@ -84,10 +84,30 @@ acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
                      int32_t *bin_offsets /* [ACSR_NBINS + 1] out */,
                      void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream);
 
+/* acsr_bin_ex: acsr_bin with plan flags (acsr_bin == acsr_bin_ex(..., 0, stream)).
+ *   ACSR_BIN_SHORT_ALG2   rows of bins 0..5 (<= 32 non-zeros) get per-bin work units
+ *                         and the SpMV maps them exactly as Alg. 2: a
+ *                         sub-warp of 2^{b-1} lanes per row, width-2^{b-1} shuffle
+ *                         reduction, lane 0 writes.  Without the flag (default) they
+ *                         are processed in short-row windows: a warp takes 32
+ *                         consecutive rows (one per lane), loads the concatenated
+ *                         non-zeros of its short rows coalesced, and each lane sums
+ *                         its own row's products in element order (DESIGN.md §6:
+ *                         fewer L2 sectors per short row on B200).  Both are exact
+ *                         y = A x mappings (reading Q4); bin_rows/bin_offsets are
+ *                         identical either way.  Unknown flag bits ->
+ *                         ACSR_ERR_INVALID_VALUE. */
+enum { ACSR_BIN_SHORT_ALG2 = 1u };
+acsr_status acsr_bin_ex(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
+                        const int32_t *row_begin, const int32_t *row_end,
+                        const int32_t *col_idx, int32_t *bin_rows, int32_t *bin_offsets,
+                        void *plan_ws, size_t plan_ws_bytes, unsigned flags, cudaStream_t stream);
+
 /* ------------------------------------------------------------------------ */
 /* SpMV y = A x, computed directly on CSR with bin-specific mappings
- * (Alg. 2): bins 1..6 use a sub-warp of 2^{b-1} lanes per row with
- * shuffle reduction (exactly Alg. 2); bins 7..10 a warp per row; rows longer
+ * (Alg. 2): bins 0..5 in short-row windows (default plan) or, with an
+ * ACSR_BIN_SHORT_ALG2 plan, a sub-warp of 2^{b-1} lanes per row with shuffle
+ * reduction (exactly Alg. 2); bin 6 always Alg. 2 (32 lanes); bins 7..10 a warp per row; rows longer
  * than 1024 non-zeros are cut into fixed chunks processed by different warps and
  * combined in chunk order by the last-arriving warp (replaces the dynamic-
  * parallelism parent/child kernels of Alg. 3/4; reading Q4/Q7/Q8).

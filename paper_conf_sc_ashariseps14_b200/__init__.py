@@ -49,6 +49,8 @@ _lib.acsr_bin_workspace_bytes.argtypes = [_i64, _i64, _i64]
 _lib.acsr_bin_workspace_bytes.restype = _sz
 _lib.acsr_bin.argtypes = [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
 _lib.acsr_bin.restype = ctypes.c_int
+_lib.acsr_bin_ex.argtypes = [_i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _sz, ctypes.c_uint, _vp]
+_lib.acsr_bin_ex.restype = ctypes.c_int
 _lib.acsr_spmv.argtypes = [ctypes.c_int, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _sz,
                            _vp]
 _lib.acsr_spmv.restype = ctypes.c_int
@@ -83,7 +85,9 @@ _lib.acsr_hits_workspace_bytes.restype = _sz
 _lib.acsr_hits_normalize.argtypes = [_i64, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
 _lib.acsr_hits_normalize.restype = ctypes.c_int
 
-EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_spmv", "acsr_pagerank_step",
+ACSR_BIN_SHORT_ALG2 = 1  # include/acsr.h: per-bin Alg. 2 units for bins 0..5
+
+EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_bin_ex", "acsr_spmv", "acsr_pagerank_step",
             "acsr_pagerank_scale", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_relayout",
             "acsr_hits_workspace_bytes", "acsr_hits_normalize",
             "acsr_status_string", "acsr_last_error", "acsr_version")
@@ -135,9 +139,13 @@ def acsr_bin_workspace_bytes(n_rows: int, n_cols: int, nnz_max: int) -> int:
 
 
 def acsr_bin(row_begin, row_end=None, nnz_max=None, bin_rows=None, bin_offsets=None, plan_ws=None,
-             stream=None, col_idx=None, n_cols=0):
+             stream=None, col_idx=None, n_cols=0, short_rows="window"):
     """Bin the rows.  Returns (bin_rows, bin_offsets, plan_ws).  col_idx (with
-    n_cols) additionally builds the hot-column table of the SpMV x cache."""
+    n_cols) additionally builds the hot-column table of the SpMV x cache.  short_rows selects
+    the SpMV mapping of bins 0..5 recorded in the plan: "window" (default, acsr_bin) or
+    "alg2" (the paper's sub-warp per row, acsr_bin_ex(..., ACSR_BIN_SHORT_ALG2))."""
+    if short_rows not in ("window", "alg2"):
+        raise ValueError(f"short_rows must be 'window' or 'alg2', not {short_rows!r}")
     n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
     dev = row_begin.device
     if nnz_max is None:
@@ -149,12 +157,13 @@ def acsr_bin(row_begin, row_end=None, nnz_max=None, bin_rows=None, bin_offsets=N
     need = acsr_bin_workspace_bytes(n, n_cols, nnz_max)
     if plan_ws is None:
         plan_ws = torch.empty(need, dtype=torch.uint8, device=dev)
-    _check(_lib.acsr_bin(n, int(n_cols), int(nnz_max), _dev(row_begin, torch.int32, "row_begin"),
-                         _dev(row_end, torch.int32, "row_end", True),
-                         _dev(col_idx, torch.int32, "col_idx") if col_idx is not None and col_idx.numel() else None,
-                         _dev(bin_rows, torch.int32, "bin_rows") if n > 0 else None,
-                         _dev(bin_offsets, torch.int32, "bin_offsets"),
-                         _dev(plan_ws, torch.uint8, "plan_ws"), plan_ws.numel(), _stream(stream)),
+    _check(_lib.acsr_bin_ex(n, int(n_cols), int(nnz_max), _dev(row_begin, torch.int32, "row_begin"),
+                            _dev(row_end, torch.int32, "row_end", True),
+                            _dev(col_idx, torch.int32, "col_idx") if col_idx is not None and col_idx.numel() else None,
+                            _dev(bin_rows, torch.int32, "bin_rows") if n > 0 else None,
+                            _dev(bin_offsets, torch.int32, "bin_offsets"),
+                            _dev(plan_ws, torch.uint8, "plan_ws"), plan_ws.numel(),
+                            ACSR_BIN_SHORT_ALG2 if short_rows == "alg2" else 0, _stream(stream)),
            "acsr_bin")
     return bin_rows, bin_offsets, plan_ws
 

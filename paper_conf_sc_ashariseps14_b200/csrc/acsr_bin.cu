@@ -55,7 +55,7 @@ struct BinSmem {
 template <bool HAS_END>
 __device__ __forceinline__ void count_tile(BinSmem &sm, int64_t n, const int32_t *__restrict__ rb,
                                            const int32_t *__restrict__ re, int32_t *__restrict__ cnt,
-                                           int n_tiles, int tile)
+                                           int n_tiles, int tile, int wmb)
 {
     const int tid = threadIdx.x;
     if (tid < NBINS) sm.hist[tid] = 0;
@@ -86,8 +86,8 @@ __device__ __forceinline__ void count_tile(BinSmem &sm, int64_t n, const int32_t
     if (tid == NBINS) {
         int lu = 0;
 #pragma unroll
-        for (int b = WIN_MAX_BIN + 1; b <= LIGHT_MAX_BIN; b++) lu += (sm.hist[b] + unit_rows(b) - 1) / unit_rows(b);
-        if (WIN_MAX_BIN >= 0) lu += win_units((int)min((int64_t)TILE_ROWS, n - base));
+        for (int b = wmb + 1; b <= LIGHT_MAX_BIN; b++) lu += (sm.hist[b] + unit_rows(b) - 1) / unit_rows(b);
+        if (wmb >= 0) lu += win_units((int)min((int64_t)TILE_ROWS, n - base));
         cnt[(int64_t)NBINS * n_tiles + tile] = lu;
         cnt[(int64_t)(NBINS + 1) * n_tiles + tile] = sm.heavy;
     }
@@ -204,7 +204,7 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
                                              const int32_t *__restrict__ re, int32_t *__restrict__ bin_rows,
                                              const int32_t *bin_offsets, const int32_t *toff, int n_tiles,
                                              const PlanHeader *hdr, int2 *__restrict__ units,
-                                             int32_t *__restrict__ tickets, int64_t heavy_cap, int tile)
+                                             int32_t *__restrict__ tickets, int64_t heavy_cap, int tile, int wmb)
 {
     constexpr int NW = BIN_THREADS / 32;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -275,14 +275,15 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
     }
     if (!overflow) {
         // light work units of this tile: the short-row windows (row order), then the
-        // bins above WIN_MAX_BIN up to 10, in bin order, row-contiguous
+        // bins above wmb up to 10, in bin order, row-contiguous (wmb = -1: no windows,
+        // bins 0..10 as per-bin units -- Alg. 2 for the short bins)
         const int tile_rows = (int)min((int64_t)TILE_ROWS, n - base);
-        const int nwin = WIN_MAX_BIN >= 0 ? win_units(tile_rows) : 0;
+        const int nwin = wmb >= 0 ? win_units(tile_rows) : 0;
         if (tid == 0) {
             int acc = nwin;
             for (int b = 0; b <= LIGHT_MAX_BIN; b++) {
                 sm.upre[b] = acc;
-                if (b > WIN_MAX_BIN) acc += (sm.run[b] + unit_rows(b) - 1) / unit_rows(b);
+                if (b > wmb) acc += (sm.run[b] + unit_rows(b) - 1) / unit_rows(b);
             }
             sm.upre[LIGHT_MAX_BIN + 1] = acc;
         }
@@ -310,12 +311,12 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
 template <bool HAS_END>
 __global__ void __launch_bounds__(BIN_THREADS)
 bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
-                 int32_t *__restrict__ cnt, int n_tiles, PlanHeader *hdr)
+                 int32_t *__restrict__ cnt, int n_tiles, PlanHeader *hdr, int wmb)
 {
     __shared__ BinSmem sm;
     pdl_enter();
     if (blockIdx.x == 0 && threadIdx.x == 0) hdr->scan_ticket = 0;  // bin_scan runs after us
-    count_tile<HAS_END>(sm, n, rb, re, cnt, n_tiles, blockIdx.x);
+    count_tile<HAS_END>(sm, n, rb, re, cnt, n_tiles, blockIdx.x, wmb);
 }
 
 constexpr int SCAN_THREADS = 1024;
@@ -334,12 +335,12 @@ __global__ void __launch_bounds__(BIN_THREADS)
 bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
                    int32_t *__restrict__ bin_rows, const int32_t *__restrict__ bin_offsets,
                    const int32_t *__restrict__ toff, int n_tiles, const PlanHeader *__restrict__ hdr,
-                   int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap)
+                   int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap, int wmb)
 {
     __shared__ BinSmem sm;
     pdl_enter();
     scatter_tile<HAS_END>(sm, n, rb, re, bin_rows, bin_offsets, toff, n_tiles, hdr, units, tickets, heavy_cap,
-                          blockIdx.x);
+                          blockIdx.x, wmb);
 }
 
 // ---- one cooperative launch: count -> grid barrier -> scan -> grid barrier -> scatter
@@ -352,6 +353,7 @@ struct FusedArgs {
     PlanHeader *hdr;
     int n_tiles;
     ScanArgs sa;
+    int wmb;
 };
 
 template <bool HAS_END>
@@ -362,14 +364,14 @@ bin_fused_kernel(FusedArgs f)
     cg::grid_group grid = cg::this_grid();
     if (blockIdx.x == 0 && threadIdx.x == 0) f.hdr->scan_ticket = 0;
     for (int t = blockIdx.x; t < f.n_tiles; t += gridDim.x)
-        count_tile<HAS_END>(sm, f.n, f.rb, f.re, f.cnt, f.n_tiles, t);
+        count_tile<HAS_END>(sm, f.n, f.rb, f.re, f.cnt, f.n_tiles, t, f.wmb);
     grid.sync();
     for (int row = blockIdx.x; row < SCAN_ROWS; row += gridDim.x)
         scan_row<BIN_THREADS, 8>(sm, f.cnt, f.toff, f.n_tiles, f.hdr, f.sa, row);
     grid.sync();
     for (int t = blockIdx.x; t < f.n_tiles; t += gridDim.x)
         scatter_tile<HAS_END>(sm, f.n, f.rb, f.re, f.bin_rows, f.sa.bin_offsets, f.toff, f.n_tiles, f.hdr, f.units,
-                              f.tickets, f.sa.heavy_cap, t);
+                              f.tickets, f.sa.heavy_cap, t, f.wmb);
 }
 
 // x-cache table: sampled occurrence counts, per-slot winner (count, column).
@@ -426,11 +428,16 @@ extern "C" size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t n_cols, int64
     return plan_layout(n_rows, n_cols, nnz_max).total;
 }
 
-extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
-                                const int32_t *row_begin, const int32_t *row_end,
-                                const int32_t *col_idx, int32_t *bin_rows, int32_t *bin_offsets,
-                                void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream)
+extern "C" acsr_status acsr_bin_ex(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
+                                   const int32_t *row_begin, const int32_t *row_end,
+                                   const int32_t *col_idx, int32_t *bin_rows, int32_t *bin_offsets,
+                                   void *plan_ws, size_t plan_ws_bytes, unsigned flags, cudaStream_t stream)
 {
+    if ((flags & ~(unsigned)ACSR_BIN_SHORT_ALG2) != 0) {
+        acsr_set_error("acsr_bin_ex: unknown flags 0x%x", flags);
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    const int wmb = (flags & ACSR_BIN_SHORT_ALG2) ? -1 : WIN_MAX_BIN;
     if (n_rows < 0 || n_cols < 0 || nnz_max < 0 || n_rows >= (int64_t)1 << 31 || !bin_offsets ||
         (n_rows > 0 && (!row_begin || !bin_rows))) {
         acsr_set_error("acsr_bin: invalid argument");
@@ -461,7 +468,7 @@ extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
     const int xc_stride = (int)(stride64 < 1 ? 1 : (stride64 > (1 << 30) ? (1 << 30) : stride64));
     ScanArgs sa{bin_offsets, n_cols, L.light_cap, L.heavy_cap, L, xc_valid, xc_stride};
     if (fused_enabled()) {
-        FusedArgs f{n_rows, row_begin, row_end, cnt, toff, bin_rows, tickets, units, hdr, nt, sa};
+        FusedArgs f{n_rows, row_begin, row_end, cnt, toff, bin_rows, tickets, units, hdr, nt, sa, wmb};
         const int grid = fused_grid(row_end != nullptr);
         void *args[] = {&f};
         const cudaError_t e = row_end
@@ -476,17 +483,17 @@ extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
         const int32_t *cbo = bin_offsets, *ctoff = toff;
         const PlanHeader *chdr = hdr;
         if (row_end)
-            launch_pdl(bin_count_kernel<true>, nt, BIN_THREADS, 0, stream, nr, rb, re, cnt, nt, hdr);
+            launch_pdl(bin_count_kernel<true>, nt, BIN_THREADS, 0, stream, nr, rb, re, cnt, nt, hdr, wmb);
         else
-            launch_pdl(bin_count_kernel<false>, nt, BIN_THREADS, 0, stream, nr, rb, re, cnt, nt, hdr);
+            launch_pdl(bin_count_kernel<false>, nt, BIN_THREADS, 0, stream, nr, rb, re, cnt, nt, hdr, wmb);
         const int32_t *ccnt = cnt;
         launch_pdl(bin_scan_kernel, SCAN_ROWS, SCAN_THREADS, 0, stream, ccnt, toff, nt, hdr, sa);
         if (row_end)
             launch_pdl(bin_scatter_kernel<true>, nt, BIN_THREADS, 0, stream, nr, rb, re, bin_rows, cbo, ctoff, nt, chdr,
-                       units, tickets, L.heavy_cap);
+                       units, tickets, L.heavy_cap, wmb);
         else
             launch_pdl(bin_scatter_kernel<false>, nt, BIN_THREADS, 0, stream, nr, rb, re, bin_rows, cbo, ctoff, nt,
-                       chdr, units, tickets, L.heavy_cap);
+                       chdr, units, tickets, L.heavy_cap, wmb);
     }
 xc:
     if (xc_valid) {
@@ -498,4 +505,13 @@ xc:
             (unsigned long long *)(ws + L.off_xc_vote));
     }
     return acsr_check_launch("acsr_bin");
+}
+
+extern "C" acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
+                                const int32_t *row_begin, const int32_t *row_end,
+                                const int32_t *col_idx, int32_t *bin_rows, int32_t *bin_offsets,
+                                void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream)
+{
+    return acsr_bin_ex(n_rows, n_cols, nnz_max, row_begin, row_end, col_idx, bin_rows, bin_offsets, plan_ws,
+                       plan_ws_bytes, 0u, stream);
 }

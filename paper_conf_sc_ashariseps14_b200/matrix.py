@@ -17,7 +17,8 @@ class ACSRMatrix:
     """Device CSR + ACSR bins.  row_end None => standard CSR (row_begin has n+1 entries)."""
 
     def __init__(self, row_begin, col_idx, values=None, n_cols=None, row_end=None, row_cap=None,
-                 nnz_max=None):
+                 nnz_max=None, short_rows="window"):
+        self.short_rows = short_rows  # SpMV mapping of bins 0..5: "window" or "alg2" (acsr_bin_ex)
         self.row_begin = row_begin
         self.row_end = row_end
         self.row_cap = row_cap
@@ -35,7 +36,7 @@ class ACSRMatrix:
 
     def rebin(self, stream=None):
         acsr_bin(self.row_begin, self.row_end, self.nnz_max, self.bin_rows, self.bin_offsets,
-                 self.plan_ws, stream, col_idx=self.col_idx, n_cols=self.n_cols)
+                 self.plan_ws, stream, col_idx=self.col_idx, n_cols=self.n_cols, short_rows=self.short_rows)
 
     def spmv(self, x, y=None, stream=None):
         return acsr_spmv(self.row_begin, self.col_idx, self.values, x, self.bin_rows,

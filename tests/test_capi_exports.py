@@ -36,5 +36,8 @@ def test_host_side_queries_without_gpu():
     assert acsr._lib.acsr_status_string(3) == b"ACSR_ERR_CAPACITY"
     # host-detected argument errors return synchronously without touching a device
     assert acsr._lib.acsr_bin(-1, 0, 0, None, None, None, None, None, None, 0, None) == acsr.ACSR_ERR_INVALID_VALUE
+    # acsr_bin_ex: unknown plan flags are rejected before anything is enqueued
+    assert acsr._lib.acsr_bin_ex(10, 10, 10, None, None, None, None, None, None, 0, 0x80,
+                                 None) == acsr.ACSR_ERR_INVALID_VALUE
     assert acsr._lib.acsr_spmv(7, 0, 0, None, None, None, None, None, None, None, None, None, 0,
                                None) == acsr.ACSR_ERR_INVALID_VALUE

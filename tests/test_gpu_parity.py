@@ -34,11 +34,14 @@ def check_spmv(y_gpu, y_ref, den, dtype, exact=False):
     assert not bad.any(), (np.flatnonzero(bad)[:10], err[bad][:5], den[bad][:5])
 
 
-def run_csr(acsr, rp, ci, val, x, dev, row_end=None):
+MAPPINGS = ["window", "alg2"]  # SpMV mapping of bins 0..5 (acsr_bin / acsr_bin_ex ACSR_BIN_SHORT_ALG2)
+
+
+def run_csr(acsr, rp, ci, val, x, dev, row_end=None, short_rows="window"):
     rbd = rp.to(dev)
     red = None if row_end is None else row_end.to(dev)
     m = acsr.ACSRMatrix(rbd, ci.to(dev), None if val is None else val.to(dev),
-                        n_cols=x.numel(), row_end=red, nnz_max=max(ci.numel(), 1))
+                        n_cols=x.numel(), row_end=red, nnz_max=max(ci.numel(), 1), short_rows=short_rows)
     y = m.spmv(x.to(dev))
     torch.cuda.synchronize()
     return m, y.cpu()
@@ -82,26 +85,28 @@ def test_bins_edge_sizes(acsr, cuda, n):
 
 
 # ------------------------------------------------------------------------------ SpMV exact
+@pytest.mark.parametrize("mapping", MAPPINGS)
 @pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
-def test_spmv_integer_bitwise_rmat14(acsr, cuda, dtype):
+def test_spmv_integer_bitwise_rmat14(acsr, cuda, dtype, mapping):
     rp, ci = synth.rmat_csr(14)
     n = rp.numel() - 1
     val = synth.values(ci.numel(), 1014, dtype, integer=True)
     x = synth.vector(n, 2014, dtype, integer=True)
-    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda, short_rows=mapping)
     y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
     check_spmv(y.numpy(), y_ref, den, dtype, exact=True)
 
 
+@pytest.mark.parametrize("mapping", MAPPINGS)
 @pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
-def test_spmv_integer_bitwise_boundary(acsr, cuda, dtype):
+def test_spmv_integer_bitwise_boundary(acsr, cuda, dtype, mapping):
     # one row per bin edge up to 2^17+1 nnz: every mapping (sub-warp widths 1..32, warp,
     # split rows with many chunks) is exercised; integer data makes every order exact.
     lens = synth.boundary_lengths(17)
     rp, ci = synth.boundary_csr(lens, 1 << 18, 3)
     val = synth.values(ci.numel(), 7, dtype, integer=True)
     x = synth.vector(1 << 18, 8, dtype, integer=True)
-    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda, short_rows=mapping)
     y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
     check_spmv(y.numpy(), y_ref, den, dtype, exact=True)
 
@@ -118,25 +123,27 @@ def test_identity_permutation_pattern(acsr, cuda):
 
 
 # ------------------------------------------------------------------------------ SpMV float
+@pytest.mark.parametrize("mapping", MAPPINGS)
 @pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
 @pytest.mark.parametrize("scale", [14, 16])
-def test_spmv_float_rmat(acsr, cuda, dtype, scale):
+def test_spmv_float_rmat(acsr, cuda, dtype, scale, mapping):
     rp, ci = synth.rmat_csr(scale)
     n = rp.numel() - 1
     val = synth.values(ci.numel(), 1014, dtype)
     x = synth.vector(n, 2014, dtype)
-    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda, short_rows=mapping)
     y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
     check_spmv(y.numpy(), y_ref, den, dtype)
 
 
+@pytest.mark.parametrize("mapping", MAPPINGS)
 @pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
-def test_spmv_float_boundary(acsr, cuda, dtype):
+def test_spmv_float_boundary(acsr, cuda, dtype, mapping):
     lens = synth.boundary_lengths(17)
     rp, ci = synth.boundary_csr(lens, 1 << 18, 9)
     val = synth.values(ci.numel(), 10, dtype)
     x = synth.vector(1 << 18, 11, dtype)
-    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda, short_rows=mapping)
     y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
     check_spmv(y.numpy(), y_ref, den, dtype)
 
@@ -154,26 +161,54 @@ def test_adversarial_long_equal_row(acsr, cuda, dtype, L):
     check_spmv(y.numpy(), y_ref, den, dtype)
 
 
-def test_powerlaw_webgoogle_like(acsr, cuda):
+@pytest.mark.parametrize("mapping", MAPPINGS)
+def test_powerlaw_webgoogle_like(acsr, cuda, mapping):
     rp, ci = synth.powerlaw_csr(seed=3, **dict(synth.WEB_GOOGLE, n=200_000))
     n = rp.numel() - 1
     val = synth.values(ci.numel(), 4)
     x = synth.vector(n, 5)
-    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda, short_rows=mapping)
     y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
     check_spmv(y.numpy(), y_ref, den, torch.float64)
 
 
-def test_slack_csr_equals_standard_and_determinism(acsr, cuda):
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+def test_window_rows_are_in_order_sums(acsr, cuda, dtype):
+    """Short-row windows: a row with <= 32 non-zeros is summed by one lane in element
+    order from rounded products, i.e. exactly the oracle's plain sequential loop (O4',
+    compiled without FMA contraction; fp32 accumulated in double, rounded once) -- so
+    those rows must match oracle.spmv_plain BIT FOR BIT, and a row's result must not
+    depend on its neighbours (lengths of other rows changed -> same bits)."""
+    rp, ci = synth.rmat_csr(16)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 31, dtype)
+    x = synth.vector(n, 32, dtype)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda)
+    y_plain = oracle.spmv_plain(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    ln = (rp[1:] - rp[:-1]).numpy()
+    short = ln <= 32
+    assert short.sum() > n // 2
+    assert np.array_equal(y.numpy()[short].view(np.uint8), y_plain[short].view(np.uint8))
+    # drop the last non-zero of every third row: the other rows keep their bits
+    rb, re = rp[:-1].clone(), rp[1:].clone()
+    cut = (torch.arange(n) % 3 == 0) & (re > rb)
+    re[cut] -= 1
+    _, y2 = run_csr(acsr, rb, ci, val, x, cuda, row_end=re)
+    keep = ~cut.numpy()
+    assert np.array_equal(y2.numpy()[keep].view(np.uint8), y.numpy()[keep].view(np.uint8))
+
+
+@pytest.mark.parametrize("mapping", MAPPINGS)
+def test_slack_csr_equals_standard_and_determinism(acsr, cuda, mapping):
     rp, ci = synth.rmat_csr(15)
     n = rp.numel() - 1
     val = synth.values(ci.numel(), 1)
     x = synth.vector(n, 2)
-    m, y1 = run_csr(acsr, rp, ci, val, x, cuda)
+    m, y1 = run_csr(acsr, rp, ci, val, x, cuda, short_rows=mapping)
     y2 = m.spmv(x.to(cuda)).cpu()
     assert torch.equal(y1, y2)  # run-to-run bitwise
     rb, re, cap, c2, v2 = synth.with_slack(rp, ci, val)
-    _, y3 = run_csr(acsr, rb, c2, v2, x, cuda, row_end=re)
+    _, y3 = run_csr(acsr, rb, c2, v2, x, cuda, row_end=re, short_rows=mapping)
     y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
     check_spmv(y3.numpy(), y_ref, den, torch.float64)
 

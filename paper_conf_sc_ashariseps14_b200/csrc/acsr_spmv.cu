@@ -719,17 +719,40 @@ spmv_kernel(SpmvArgs<V> a)
 #if ACSR_SCHED_STATIC
     for (int u = gw; u < n_units; u += nw) K::unit(a, u, lane, d2, wbuf, wtab);
 #else
+    // first prefetched claims: one atomic per CTA (a same-address atomic per warp at
+    // launch costs microseconds of serialisation at the L2 slice)
+    __shared__ int s_claim;
+    if (threadIdx.x == 0) s_claim = atomicAdd(&hdr->work_ctr, SPMV_WARPS);
+    __syncthreads();
     int u = gw;
-    int nxt = 0;
-    if (lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
+    int nxt = s_claim + (threadIdx.x >> 5);
     while (u < n_units) {
         K::unit(a, u, lane, d2, wbuf, wtab);
         u = __shfl_sync(0xffffffffu, nxt, 0) + nw;
         if (u < n_units && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
     }
 #endif
+    // CTA-level exit: Delta^2 (exact fixed point) reduced warp -> CTA in shared memory,
+    // then ONE set of atomics and ONE exit ticket per CTA
+    __shared__ uint64_t s_d2[SPMV_WARPS][3];
     if (PR) {
-        // exact fixed-point warp sum, then three 64-bit atomics per warp with carries
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            const uint64_t h = __shfl_xor_sync(0xffffffffu, d2.hi, o);
+            const uint64_t m = __shfl_xor_sync(0xffffffffu, d2.mid, o);
+            const uint64_t l = __shfl_xor_sync(0xffffffffu, d2.lo, o);
+            fix_merge(d2, h, m, l);
+        }
+        if (lane == 0) {
+            s_d2[threadIdx.x >> 5][0] = d2.hi;
+            s_d2[threadIdx.x >> 5][1] = d2.mid;
+            s_d2[threadIdx.x >> 5][2] = d2.lo;
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x >= 32) return;
+    if (PR) {
+        d2 = lane < SPMV_WARPS ? Fix192{s_d2[lane][0], s_d2[lane][1], s_d2[lane][2]} : Fix192{0, 0, 0};
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
             const uint64_t h = __shfl_xor_sync(0xffffffffu, d2.hi, o);
@@ -747,10 +770,10 @@ spmv_kernel(SpmvArgs<V> a)
             atomicAdd((unsigned long long *)&hdr->d2_hi, (unsigned long long)(d2.hi + c2 + cm));
         }
     }
-    // last warp out publishes Delta^2 and resets the counters for the next call
+    // last CTA out publishes Delta^2 and resets the counters for the next call
     if (lane == 0) {
         __threadfence();
-        if (atomicAdd(&hdr->exit_ticket, 1) == nw - 1) {
+        if (atomicAdd(&hdr->exit_ticket, 1) == (int)gridDim.x - 1) {
             __threadfence();
             if (PR) {
                 const uint64_t hi = *(volatile uint64_t *)&hdr->d2_hi;

@@ -485,7 +485,9 @@ def run_pagerank_dist(args, dev, rank, world):
             "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"pagerank_rmat{S}_inlink_partitioned", "n_rows": n, "nnz": nnz,
-                       "parallelism": f"row-partitioned x{world}", "padded_slice": pr.L},
+                       "parallelism": f"row-partitioned x{world}", "padded_slice": pr.L,
+                       "exchange_slice": pr.Lx, "exchange_bytes_in_per_rank_per_iter": pr.exchange_bytes_per_rank(),
+                       "exchange_layout": "non-dangling only (lossless)" if pr.compact else "all vertices"},
             "gpu_launches": K, "clocks": clk.summary()}
 
 

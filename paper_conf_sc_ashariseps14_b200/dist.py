@@ -55,16 +55,41 @@ def renumber_columns(col: torch.Tensor, splits: np.ndarray, L: int) -> torch.Ten
     return (owner * L + (c - start)).to(torch.int32)
 
 
+def permute_rows(row_ptr: torch.Tensor, col: torch.Tensor, perm: torch.Tensor):
+    """CSR with its rows reordered: new row i = old row perm[i] (columns untouched)."""
+    rp = row_ptr.to(torch.int64)
+    lens = (rp[1:] - rp[:-1])[perm]
+    new_rp = torch.zeros_like(rp)
+    torch.cumsum(lens, 0, out=new_rp[1:])
+    nnz = int(new_rp[-1])
+    row_of = torch.repeat_interleave(torch.arange(perm.numel(), device=rp.device), lens, output_size=nnz)
+    old = rp[perm][row_of] + torch.arange(nnz, device=rp.device) - new_rp[:-1][row_of]
+    return new_rp.to(torch.int32), col[old].contiguous()
+
+
 class DistPageRank:
     """PageRank over P ranks.  Each rank passes its local in-link CSR rows
     [splits[rank], splits[rank+1]) with GLOBAL column ids; the object renumbers the
     columns once and owns the replicated padded xs buffers.
 
-    step_fn(local, xs, x, x_new, xs_next_slice, delta2) computes one local step; the
-    default runs the CUDA kernel (acsr_pagerank_step)."""
+    Exchange layouts (world > 1):
+      compact=False  every vertex has a slot: slice length L = max rows per rank.
+      compact=True   (default) only vertices with outdeg > 0 have a slot.  xs_u = 0
+                     exactly when outdeg_u = 0 (Alg. 5 with reading Q11) and such a
+                     vertex is never a column of the in-link pattern, so the all-gather
+                     carries only the non-dangling entries (R-MAT: about half of the
+                     vertices are dangling) -- lossless.  Each rank
+                     orders its local rows non-dangling first (a local relabelling, undone
+                     on output), so its exchanged slice is a prefix of its local xs.
+                     A column whose vertex is dangling (inconsistent outdeg input) reads a
+                     trailing slot that is always 0, as Alg. 5 prescribes.
+
+    step_fn(xs, x, x_new, xs_next_local, delta2) computes one local step on
+    (self.row_ptr, self.col, self.outdeg); the default runs the CUDA kernel
+    (acsr_pagerank_step)."""
 
     def __init__(self, row_ptr_local, col_local, outdeg_local, splits, n_global, damping=0.85,
-                 group=None, step_fn=None, scale_fn=None, device=None):
+                 group=None, step_fn=None, scale_fn=None, device=None, compact=True):
         self.group = group
         self.rank = dist.get_rank(group) if dist.is_initialized() else 0
         self.world = dist.get_world_size(group) if dist.is_initialized() else 1
@@ -76,23 +101,65 @@ class DistPageRank:
         self.damping = float(damping)
         self.teleport = (1.0 - self.damping) / self.n_global  # computed once, same bits on all ranks
         self.device = row_ptr_local.device if device is None else device
-        self.row_ptr = row_ptr_local
-        self.col = renumber_columns(col_local, self.splits, self.L) if self.world > 1 else col_local
-        self.outdeg = outdeg_local
+        self.compact = bool(compact) and self.world > 1
+        self.perm = None
+        if self.compact:
+            self._setup_compact(row_ptr_local, col_local, outdeg_local)
+        else:
+            self.row_ptr = row_ptr_local
+            self.col = renumber_columns(col_local, self.splits, self.L) if self.world > 1 else col_local
+            self.outdeg = outdeg_local
+            self.Lx = self.L
         use_cuda = step_fn is None
         self.step_fn = step_fn or self._cuda_step
         self.scale_fn = scale_fn or self._cuda_scale
         dev = self.device
-        self.xs = torch.zeros(self.world * self.L, dtype=torch.float64, device=dev)
+        # replicated gathered xs (+1 trailing always-zero slot in the compact layout)
+        nx = self.world * self.Lx + (1 if self.compact else 0)
+        self.xs = torch.zeros(nx, dtype=torch.float64, device=dev)
         self.xs_next = torch.zeros_like(self.xs)
+        # compact: the kernel writes the local xs here; its first Lx entries are exchanged
+        self.xs_loc = (torch.zeros(max(self.n_local, self.Lx), dtype=torch.float64, device=dev)
+                       if self.compact else None)
         self.delta2 = torch.zeros(1, dtype=torch.float64, device=dev)
         self._m = None
         if use_cuda:
             from .matrix import ACSRMatrix
             self._m = ACSRMatrix(self.row_ptr, self.col, None, n_cols=self.xs.numel())
 
-    def _slice(self, buf):
-        return buf[self.rank * self.L: self.rank * self.L + self.n_local]
+    def _setup_compact(self, row_ptr_local, col_local, outdeg_local):
+        dev = row_ptr_local.device
+        world, L = self.world, self.L
+        nd_local = (outdeg_local > 0)
+        # global non-dangling mask: all-gather the padded local masks (setup, once)
+        pad = torch.zeros(L, dtype=torch.uint8, device=dev)
+        pad[: self.n_local] = nd_local.to(torch.uint8)
+        allm = torch.zeros(world * L, dtype=torch.uint8, device=dev)
+        dist.all_gather_into_tensor(allm, pad.clone() if dev.type == "cpu" else pad, group=self.group)
+        sizes = np.diff(self.splits)
+        nd = torch.cat([allm[k * L: k * L + int(sizes[k])] for k in range(world)]).to(torch.bool)
+        nnd = [int(allm[k * L: k * L + int(sizes[k])].sum()) for k in range(world)]
+        self.n_nd = nnd
+        self.Lx = max(1, max(nnd))
+        # compact position of every vertex: owner * Lx + rank among the owner's non-dangling
+        sp = torch.as_tensor(self.splits, dtype=torch.int64, device=dev)
+        csum = torch.cumsum(nd.to(torch.int64), 0)
+        ex = csum - nd.to(torch.int64)  # exclusive prefix over all vertices
+        owner = torch.searchsorted(sp[1:-1], torch.arange(self.n_global, device=dev), right=True)
+        base = torch.cat([torch.zeros(1, dtype=torch.int64, device=dev), csum])[sp[:-1]][owner]
+        pos = torch.where(nd, owner * self.Lx + (ex - base), torch.full_like(ex, world * self.Lx))
+        col = pos[col_local.to(torch.int64)].to(torch.int32)
+        # local rows: non-dangling first (stable), so the exchanged slice is a prefix
+        perm = torch.cat([torch.nonzero(nd_local).flatten(), torch.nonzero(~nd_local).flatten()])
+        self.perm = perm
+        self.row_ptr, self.col = permute_rows(row_ptr_local, col, perm)
+        self.outdeg = outdeg_local[perm].contiguous()
+
+    def _local_out(self):
+        """Where the local step writes its xs slice."""
+        if self.compact:
+            return self.xs_loc[: self.n_local]
+        return self.xs_next[self.rank * self.L: self.rank * self.L + self.n_local]
 
     def _cuda_step(self, xs, x, x_new, xs_next_slice, delta2):
         from . import acsr_pagerank_step
@@ -106,25 +173,37 @@ class DistPageRank:
         acsr_pagerank_scale(x, outdeg, out)
 
     def exchange(self, buf):
-        if self.world > 1:
+        """Gather every rank's slice into buf (the replicated xs of the next step)."""
+        if self.compact:
+            dist.all_gather_into_tensor(buf[: self.world * self.Lx], self.xs_loc[: self.Lx], group=self.group)
+        elif self.world > 1:
             chunk = buf[self.rank * self.L:(self.rank + 1) * self.L]  # padded: tail stays 0
             dist.all_gather_into_tensor(buf, chunk.clone() if buf.device.type == "cpu" else chunk,
                                         group=self.group)
 
+    def exchange_bytes_per_rank(self):
+        """Bytes each rank receives per iteration from the all-gather."""
+        return (self.world - 1) * self.Lx * 8
+
     def run(self, x0_local=None, eps=1e-6, max_iter=1000):
-        """Alg. 5 loop; returns (x_local, iterations, delta2_global)."""
+        """Alg. 5 loop; returns (x_local, iterations, delta2_global) with x_local in the
+        caller's local row order."""
         dev = self.device
         if x0_local is None:
             x = torch.full((self.n_local,), 1.0 / self.n_global, dtype=torch.float64, device=dev)
         else:
-            x = x0_local.clone()
+            x = x0_local.clone() if self.perm is None else x0_local[self.perm].contiguous()
         # xs^0 slice = x^0 / outdeg (IEEE division), then gather
-        self.scale_fn(x, self.outdeg, self._slice(self.xs))
-        self.exchange(self.xs)
+        if self.compact:
+            self.scale_fn(x, self.outdeg, self._local_out())
+            self.exchange(self.xs)
+        else:
+            self.scale_fn(x, self.outdeg, self.xs[self.rank * self.L: self.rank * self.L + self.n_local])
+            self.exchange(self.xs)
         x_new = torch.empty_like(x)
         it, d2 = 0, float("inf")
         while it < max_iter:
-            self.step_fn(self.xs, x, x_new, self._slice(self.xs_next), self.delta2)
+            self.step_fn(self.xs, x, x_new, self._local_out(), self.delta2)
             self.exchange(self.xs_next)
             if self.world > 1:
                 dist.all_reduce(self.delta2, group=self.group)
@@ -134,4 +213,8 @@ class DistPageRank:
             d2 = float(self.delta2.item())
             if d2 ** 0.5 <= eps:
                 break
+        if self.perm is not None:
+            out = torch.empty_like(x)
+            out[self.perm] = x
+            x = out
         return x, it, d2

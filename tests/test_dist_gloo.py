@@ -24,7 +24,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, scale, out):
+def _worker(rank, world, port, scale, out, compact=True):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     rp, ci = synth.rmat_csr(scale, transpose=True)
@@ -37,39 +37,45 @@ def _worker(rank, world, port, scale, out):
     odl = od[lo:hi].contiguous()
 
     def step(xs, x, x_new, xs_next_slice, delta2):
-        xn, d2 = oracle.pagerank_step(rpl.numpy(), pr.col.numpy(), np.ones(xs.numel(), np.int32),
+        # the local CSR / outdeg as the object holds them (rows possibly reordered,
+        # columns renumbered into the exchange layout)
+        xn, d2 = oracle.pagerank_step(pr.row_ptr.numpy(), pr.col.numpy(), np.ones(xs.numel(), np.int32),
                                       xs.numpy(), pr.teleport, pr.damping)
         # oracle with outdeg = 1 gathers xs itself: y_v = sum xs_u  (xs already scaled)
+        od_l = pr.outdeg
         x_new.copy_(torch.from_numpy(xn))
-        xs_next_slice.copy_(torch.where(odl > 0, x_new / odl.clamp(min=1).double(), torch.zeros_like(x_new)))
+        xs_next_slice.copy_(torch.where(od_l > 0, x_new / od_l.clamp(min=1).double(), torch.zeros_like(x_new)))
         delta2.fill_(float(((x_new - x) ** 2).sum()))
 
     def scale(x, outdeg, outv):
         outv.copy_(torch.where(outdeg > 0, x / outdeg.clamp(min=1).double(), torch.zeros_like(x)))
 
     pr = acsr_dist.DistPageRank(rpl, cil, odl, splits, n, step_fn=step, scale_fn=scale,
-                                device=torch.device("cpu"))
+                                device=torch.device("cpu"), compact=compact)
     x, it, d2 = pr.run(eps=1e-8)
+    # exchange volume: the compact layout carries only the non-dangling vertices
+    nb = torch.tensor([pr.exchange_bytes_per_rank(), pr.Lx, pr.L], dtype=torch.int64)
     xs_all = [torch.zeros(pr.L, dtype=torch.float64) for _ in range(world)]
     xp = torch.zeros(pr.L, dtype=torch.float64)
     xp[: x.numel()] = x
     dist.all_gather(xs_all, xp)
     if rank == 0:
         full = torch.cat([xs_all[k][: int(splits[k + 1] - splits[k])] for k in range(world)])
-        out.put((full.numpy(), it, d2, splits))
+        out.put((full.numpy(), it, d2, splits, nb.tolist()))
     dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("compact", [True, False])
 @pytest.mark.parametrize("world", [2])
-def test_partitioned_pagerank_matches_single(world):
+def test_partitioned_pagerank_matches_single(world, compact):
     scale = 11
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, scale, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, scale, q, compact)) for r in range(world)]
     for p in procs:
         p.start()
-    full, it, d2, splits = q.get(timeout=240)
+    full, it, d2, splits, (xbytes, Lx, L) = q.get(timeout=240)
     for p in procs:
         p.join(60)
         assert p.exitcode == 0
@@ -80,6 +86,13 @@ def test_partitioned_pagerank_matches_single(world):
     assert abs(it - it_ref) <= 1
     assert np.allclose(full, x_ref, rtol=1e-11, atol=1e-18)
     assert splits[0] == 0 and splits[-1] == n and np.all(np.diff(splits) > 0)
+    if compact:
+        # slot per non-dangling vertex only: the largest per-rank count of outdeg > 0
+        nnd = max(int((od[splits[k]:splits[k + 1]] > 0).sum()) for k in range(world))
+        assert Lx == nnd < L
+        assert xbytes == (world - 1) * nnd * 8
+    else:
+        assert Lx == L
 
 
 def test_partition_matches_oracle_rule():
@@ -98,3 +111,14 @@ def test_renumber_roundtrip():
     assert torch.equal(owner, torch.tensor([0] * 5 + [1] * 7 + [2] * 8))
     back = torch.tensor(splits[:-1])[owner.long()] + c2 % L
     assert torch.equal(back.to(torch.int32), col)
+
+
+def test_permute_rows_roundtrip():
+    rp, ci = synth.rmat_csr(9)
+    n = rp.numel() - 1
+    perm = torch.randperm(n, generator=torch.Generator().manual_seed(3))
+    rp2, ci2 = acsr_dist.permute_rows(rp, ci, perm)
+    for i in range(0, n, 7):
+        r = int(perm[i])
+        assert torch.equal(ci2[int(rp2[i]):int(rp2[i + 1])], ci[int(rp[r]):int(rp[r + 1])])
+    assert int(rp2[-1]) == ci.numel()

@@ -225,6 +225,34 @@ def test_empty_and_all_empty(acsr, cuda):
     assert not torch.signbit(y).any()
 
 
+@pytest.mark.parametrize("mapping", MAPPINGS)
+@pytest.mark.parametrize("n", [1, 31, 33, 4097, 70001])
+def test_spmv_ragged_sizes(acsr, cuda, n, mapping):
+    """Row counts that end inside a 32-row window / a 1024-row tile, with a mix of
+    empty, short (1..32), bin-6 (33..64), warp (65..1024) and split (> 1024) rows;
+    integer data, so every mapping must match the oracle bit for bit."""
+    g = torch.Generator().manual_seed(n)
+    kind = torch.randint(0, 10, (n,), generator=g)
+    ln = torch.where(kind < 3, torch.zeros(n, dtype=torch.int64),
+                     torch.where(kind < 8, torch.randint(1, 33, (n,), generator=g),
+                                 torch.where(kind < 9, torch.randint(33, 65, (n,), generator=g),
+                                             torch.randint(65, 1025, (n,), generator=g))))
+    if n > 100:
+        ln[n // 3] = 5000
+        ln[-1] = 17  # a short row in the ragged last window
+    rp = torch.zeros(n + 1, dtype=torch.int64)
+    rp[1:] = torch.cumsum(ln, 0)
+    nnz = int(rp[-1])
+    n_cols = 50_000
+    ci = torch.randint(0, n_cols, (nnz,), generator=g).to(torch.int32)
+    rp = rp.to(torch.int32)
+    val = synth.values(nnz, n, torch.float64, integer=True)
+    x = synth.vector(n_cols, n + 1, torch.float64, integer=True)
+    _, y = run_csr(acsr, rp, ci, val, x, cuda, short_rows=mapping)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y.numpy(), y_ref, den, torch.float64, exact=True)
+
+
 def sampled_parity(rp, ci, val, x, y, bins_check=None, n_random=4000, seed=0):
     """Check y (host numpy) on a sample of rows -- random rows, the longest rows and the
     first rows of every bin -- against the oracle computed row by row on the sample."""

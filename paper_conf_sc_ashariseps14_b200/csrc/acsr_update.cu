@@ -48,6 +48,7 @@ update_validate_kernel(int64_t n_rows, int64_t n_cols, const int32_t *__restrict
                        const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
                        const int32_t *__restrict__ icol, UpdWs *ws)
 {
+    pdl_enter();
     unsigned long long *key = &ws->key;
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
@@ -124,6 +125,7 @@ update_validate_long_kernel(const int32_t *__restrict__ rb, const int32_t *__res
                             const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
                             const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr, UpdWs *ws)
 {
+    pdl_enter();
     __shared__ int sh[33];
     const unsigned n_long = *(volatile unsigned *)&ws->n_long;
     for (unsigned j = blockIdx.x; j < n_long; j += gridDim.x) {
@@ -152,6 +154,7 @@ update_apply_long_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ r
                          const int32_t *__restrict__ icol, const T *__restrict__ ival, T one,
                          int32_t *__restrict__ outdeg, UpdWs *ws)
 {
+    pdl_enter();
     __shared__ int sh[33];
     if (*(volatile unsigned long long *)&ws->key != NO_FAIL) return;
     const unsigned n_long = *(volatile unsigned *)&ws->n_long;
@@ -212,6 +215,7 @@ update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
                     const int32_t *__restrict__ icol, const T *__restrict__ ival, T one,
                     int32_t *__restrict__ outdeg, const UpdWs *ws, int32_t *__restrict__ status)
 {
+    pdl_enter();
     const unsigned long long k = *(volatile const unsigned long long *)&ws->key;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         status[0] = k == NO_FAIL ? ACSR_OK : (int32_t)(k & 7);
@@ -312,6 +316,13 @@ extern "C" size_t acsr_update_workspace_bytes(int64_t n_upd)
     return align_up(offsetof(UpdWs, long_list) + sizeof(int32_t) * (size_t)(n_upd > 0 ? n_upd : 1), 256);
 }
 
+__global__ void update_init_kernel(UpdWs *ws)
+{
+    pdl_enter();
+    ws->key = NO_FAIL;
+    ws->n_long = 0;
+}
+
 extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
                                          const int32_t *row_begin, int32_t *row_end,
                                          const int32_t *row_cap, int32_t *col_idx, void *values,
@@ -332,42 +343,41 @@ extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t 
         return ACSR_ERR_WORKSPACE;
     }
     UpdWs *uw = (UpdWs *)ws;
-    cudaMemsetAsync(&uw->key, 0xff, sizeof(unsigned long long), stream);
-    cudaMemsetAsync(&uw->n_long, 0, sizeof(unsigned int), stream);
+    launch_pdl(update_init_kernel, 1, 1, 0, stream, uw);
     const int long_grid = 4 * acsr_num_sms();
     const int wpb = UPD_THREADS / 32;
     const int64_t blocks64 = n_upd > 0 ? (n_upd + wpb - 1) / wpb : 1;
     if (blocks64 > 0x7fffffff) return ACSR_ERR_INVALID_VALUE;
     const int blocks = (int)blocks64;
     if (n_upd > 0)
-        update_validate_kernel<<<blocks, UPD_THREADS, 0, stream>>>(n_rows, n_cols, row_begin, row_end,
+        launch_pdl(update_validate_kernel, blocks, UPD_THREADS, 0, stream, n_rows, n_cols, row_begin, row_end,
                                                                    row_cap, col_idx, n_upd, upd_rows,
                                                                    del_ptr, del_cols, ins_ptr, ins_cols,
                                                                    uw);
     if (n_upd > 0 && del_ptr)
-        update_validate_long_kernel<<<long_grid, UPD_THREADS, 0, stream>>>(row_begin, row_end, row_cap, col_idx,
+        launch_pdl(update_validate_long_kernel, long_grid, UPD_THREADS, 0, stream, row_begin, row_end, row_cap, col_idx,
                                                                           upd_rows, del_ptr, del_cols, ins_ptr,
                                                                           uw);
     if (dt == ACSR_F64) {
         uint64_t one;
         double d1 = 1.0;
         memcpy(&one, &d1, 8);
-        update_apply_kernel<uint64_t><<<blocks, UPD_THREADS, 0, stream>>>(
+        launch_pdl(update_apply_kernel<uint64_t>, blocks, UPD_THREADS, 0, stream, 
             row_begin, row_end, col_idx, (uint64_t *)values, n_upd, upd_rows, del_ptr, del_cols, ins_ptr,
             ins_cols, (const uint64_t *)ins_vals, one, outdeg, uw, status);
         if (n_upd > 0 && del_ptr)
-            update_apply_long_kernel<uint64_t><<<long_grid, UPD_THREADS, 0, stream>>>(
+            launch_pdl(update_apply_long_kernel<uint64_t>, long_grid, UPD_THREADS, 0, stream, 
                 row_begin, row_end, col_idx, (uint64_t *)values, upd_rows, del_ptr, del_cols, ins_ptr, ins_cols,
                 (const uint64_t *)ins_vals, one, outdeg, uw);
     } else {
         uint32_t one;
         float f1 = 1.0f;
         memcpy(&one, &f1, 4);
-        update_apply_kernel<uint32_t><<<blocks, UPD_THREADS, 0, stream>>>(
+        launch_pdl(update_apply_kernel<uint32_t>, blocks, UPD_THREADS, 0, stream, 
             row_begin, row_end, col_idx, (uint32_t *)values, n_upd, upd_rows, del_ptr, del_cols, ins_ptr,
             ins_cols, (const uint32_t *)ins_vals, one, outdeg, uw, status);
         if (n_upd > 0 && del_ptr)
-            update_apply_long_kernel<uint32_t><<<long_grid, UPD_THREADS, 0, stream>>>(
+            launch_pdl(update_apply_long_kernel<uint32_t>, long_grid, UPD_THREADS, 0, stream, 
                 row_begin, row_end, col_idx, (uint32_t *)values, upd_rows, del_ptr, del_cols, ins_ptr, ins_cols,
                 (const uint32_t *)ins_vals, one, outdeg, uw);
     }

@@ -576,14 +576,19 @@ struct Kern {
                     const bool hd = l > 0 && pre >= cb && pre < cb + 32;
                     const unsigned H = __reduce_or_sync(FULL, hd ? 1u << (pre - cb) : 0u);
                     const int q0 = __popc(__ballot_sync(FULL, l > 0 && pre < cb));
-                    const int t = cb + lane;
-                    const bool v = t < T;
-                    int k = 0;
-                    if (v) {
-                        const int2 bp = tab[q0 + __popc(H & le) - 1];
-                        k = bp.x + (t - bp.y);
-                    }
-                    p[g] = prodp(a, v, k);
+                    // element t, clamped to the last one (T-1) past the end so that every
+                    // lane loads from a valid address: no branches, all WIN_G groups'
+                    // loads are issued back to back (the f32 build serialised them when
+                    // the loads sat behind a branch).  No row starts at or past T, so the
+                    // row found for a clamped lane is the last non-empty row, which holds T-1.
+                    const bool v = cb + lane < T;
+                    const int t = v ? cb + lane : T - 1;
+                    const int2 bp = tab[q0 + __popc(H & le) - 1];
+                    const int k = bp.x + (t - bp.y);
+                    const int c = lds_i(a.col + k);
+                    const double xv = gx(a, c);
+                    const double pv = HAS_VAL ? lds_v(a.val + k) * xv : xv;
+                    p[g] = v ? pv : 0.0;
                 }
 #pragma unroll
                 for (int g = 0; g < WIN_G; g++) buf[32 * g + lane] = p[g];

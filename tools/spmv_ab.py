@@ -29,7 +29,7 @@ def main():
         p = torch.empty_like(q); p[q] = torch.arange(n, device=dev)
         ci = p[ci.long()].to(torch.int32)
         torch.cuda.synchronize(); t_relabel = time.perf_counter() - t0
-    m = acsr.ACSRMatrix(rp, ci, val)
+    m = acsr.ACSRMatrix(rp, ci, val, short_rows=os.environ.get("SHORT_ROWS", "window"))
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     tb, ts = [], []
     for i in range(reps + 3):
@@ -44,7 +44,7 @@ def main():
     sv = 8 if dtype == torch.float64 else 4
     n_c = int((torch.bincount(ci.long(), minlength=n) > 0).sum())
     alg = (sv + 4) * nnz + 8 * n + 4 + sv * n_c + sv * n
-    print(json.dumps({"wl": wl, "env": {k: v for k, v in os.environ.items() if k.startswith("ACSR_")},
+    print(json.dumps({"wl": wl, "env": {k: v for k, v in os.environ.items() if k.startswith("ACSR_") or k == "SHORT_ROWS"},
                       "t_bin_us": round(1e3 * float(np.median(tb)), 2), "t_spmv_us": round(1e3 * float(np.median(ts)), 2),
                       "t_spmv_min_us": round(1e3 * float(np.min(ts)), 2),
                       "t_spmv_mean_us": round(1e3 * float(np.mean(ts)), 2),

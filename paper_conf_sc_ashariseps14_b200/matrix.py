@@ -96,10 +96,16 @@ def spmv_from_host(row_ptr_h, col_h, val_h, x_h, y_h=None, device="cuda", stream
 
 
 def _power_loop(m: ACSRMatrix, outdeg, x, damping, teleport, eps, max_iter, check_every, stream,
-                restart=-1, restart_weight=0.0):
+                restart=-1, restart_weight=0.0, graph=False):
     """Alg. 5-style loop with device-side convergence: up to check_every fused steps are
     enqueued between host synchronisations; a step after convergence is a no-op (ctrl[0]),
-    so results equal a host test after every step.  Returns (x, iterations, delta2)."""
+    so results equal a host test after every step.  With graph=True (and the default
+    stream) the block of check_every steps is captured once into a CUDA graph and
+    replayed, so the host issues one launch per block instead of one per step (the
+    buffers alternate with the step parity and check_every is even, so every block sees
+    the same pointers).  Capturing costs milliseconds (torch.cuda.graph synchronises and
+    collects), so it pays only for long solves on small matrices, where a step is shorter
+    than its host launch; off by default.  Returns (x, iterations, delta2)."""
     n = m.n_rows
     dev = m.row_begin.device
     bufs = [x, torch.empty_like(x)]
@@ -107,14 +113,30 @@ def _power_loop(m: ACSRMatrix, outdeg, x, damping, teleport, eps, max_iter, chec
     d2 = torch.zeros(1, dtype=torch.float64, device=dev)
     ctrl = torch.zeros(2, dtype=torch.int32, device=dev)
     eps2 = eps * eps if eps >= 0 else -1.0
+
+    def step(k):
+        acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, sbufs[k % 2],
+                           bufs[k % 2], outdeg, bufs[(k + 1) % 2], sbufs[(k + 1) % 2], d2, damping,
+                           teleport, n, m.row_end, stream, restart=restart, restart_weight=restart_weight,
+                           ctrl=ctrl, eps2=eps2)
+
+    use_graph = graph and stream is None and check_every % 2 == 0 and check_every > 0
+    g = None
     k = 0
     while k < max_iter:
-        for _ in range(min(check_every, max_iter - k)):
-            acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, sbufs[k % 2],
-                               bufs[k % 2], outdeg, bufs[(k + 1) % 2], sbufs[(k + 1) % 2], d2, damping,
-                               teleport, n, m.row_end, stream, restart=restart, restart_weight=restart_weight,
-                               ctrl=ctrl, eps2=eps2)
-            k += 1
+        nblk = min(check_every, max_iter - k)
+        if use_graph and k > 0 and nblk == check_every:
+            if g is None:  # the first block ran eagerly (lazy kernel attributes are set)
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g):
+                    for j in range(check_every):
+                        step(j)
+            g.replay()
+            k += check_every
+        else:
+            for _ in range(nblk):
+                step(k)
+                k += 1
         c = ctrl.cpu()
         if int(c[0]):
             break
@@ -123,17 +145,18 @@ def _power_loop(m: ACSRMatrix, outdeg, x, damping, teleport, eps, max_iter, chec
 
 
 def pagerank(m: ACSRMatrix, outdeg, x0=None, damping=0.85, eps=1e-6, max_iter=1000, stream=None,
-             check_every=8):
+             check_every=8, graph=False):
     """Alg. 5 on one GPU over the in-link pattern matrix m (stop when
     ||x' - x||_2 <= eps, reading Q9).  Returns (x, iterations, delta2)."""
     n = m.n_rows
     dev = m.row_begin.device
     x = torch.full((n,), 1.0 / n, dtype=torch.float64, device=dev) if x0 is None else x0.clone()
-    return _power_loop(m, outdeg, x, damping, (1.0 - damping) / n, eps, max_iter, check_every, stream)
+    return _power_loop(m, outdeg, x, damping, (1.0 - damping) / n, eps, max_iter, check_every, stream,
+                       graph=graph)
 
 
 def rwr(m: ACSRMatrix, outdeg, restart: int, c=0.85, eps=1e-6, max_iter=1000, r0=None, stream=None,
-        check_every=8):
+        check_every=8, graph=False):
     """Random Walk with Restart (Eq. 8; reading R5) on the in-link pattern m:
     r' = c (W r) + (1-c) e_restart, r^0 = e_restart.  One fused acsr_pagerank_step per
     iteration (teleport 0, restart weight 1-c).  Returns (r, iterations, delta2)."""
@@ -145,7 +168,7 @@ def rwr(m: ACSRMatrix, outdeg, restart: int, c=0.85, eps=1e-6, max_iter=1000, r0
     else:
         r = r0.clone()
     return _power_loop(m, outdeg, r, c, 0.0, eps, max_iter, check_every, stream, restart=restart,
-                       restart_weight=1.0 - c)
+                       restart_weight=1.0 - c, graph=graph)
 
 
 def hits_matrix(out_ptr, out_col, n=None):

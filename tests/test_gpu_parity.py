@@ -740,3 +740,35 @@ def test_device_side_convergence_identical(acsr, cuda):
     r1, j1, _ = acsr.rwr(m, od.to(cuda), 3, check_every=1)
     r8, j8, _ = acsr.rwr(m, od.to(cuda), 3, check_every=8)
     assert j1 == j8 and torch.equal(r1, r8)
+    # blocks of 8 steps replayed from one CUDA graph (PDL edges inside) -- same bits
+    xg, itg, dg = acsr.pagerank(m, od.to(cuda), eps=1e-6, check_every=8, graph=True)
+    xe, ite, de = acsr.pagerank(m, od.to(cuda), eps=1e-6, check_every=8, graph=False)
+    assert itg == ite == it1 and dg == de and torch.equal(xg, xe) and torch.equal(xg, x1)
+    # a tight eps forces several graph replays (and a ragged eager tail via max_iter)
+    xg, itg, _ = acsr.pagerank(m, od.to(cuda), eps=1e-13, max_iter=43, graph=True)
+    xe, ite, _ = acsr.pagerank(m, od.to(cuda), eps=1e-13, max_iter=43, graph=False)
+    assert itg == ite and torch.equal(xg, xe)
+
+
+def test_graph_captured_bin_spmv(acsr, cuda):
+    """acsr_bin + acsr_spmv captured into a CUDA graph (the calls are stream-ordered and
+    allocation-free, PDL edges included) and replayed: same bits as eager calls."""
+    rp, ci = synth.rmat_csr(15)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 5).to(cuda)
+    x = synth.vector(n, 6).to(cuda)
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda), val)
+    y_e = m.spmv(x).clone()
+    y = torch.empty_like(y_e)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        m.rebin()
+        m.spmv(x, y)
+    y.zero_()
+    g.replay()
+    torch.cuda.synchronize()
+    assert torch.equal(y, y_e)
+    x.mul_(-2.0)  # inputs updated in place -> the replay sees them
+    g.replay()
+    torch.cuda.synchronize()
+    assert torch.equal(y, m.spmv(x))

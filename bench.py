@@ -477,7 +477,7 @@ def run_pagerank_dist(args, dev, rank, world):
     nnz_local = cil.numel()
     del rp, ci
     torch.cuda.empty_cache()
-    pr = pdist.DistPageRank(rpl, cil, odl, splits, n)
+    pr = pdist.DistPageRank(rpl, cil, odl, splits, n, exchange=args.exchange)
     for _ in range(args.warmup):
         pr.run(max_iter=1)
     torch.cuda.synchronize()
@@ -487,7 +487,10 @@ def run_pagerank_dist(args, dev, rank, world):
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with Clocks(torch.cuda.current_device()) as clk:
         e0.record()
-        x, it, d2 = pr.run(eps=0.0, max_iter=K)
+        if args.exchange == "peer":  # device-side stop flag: 8 (step, Delta^2) pairs per host sync
+            x, it, d2 = pr.run(eps=0.0, max_iter=K, check_every=8)
+        else:
+            x, it, d2 = pr.run(eps=0.0, max_iter=K)
         e1.record()
         torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / K
@@ -502,15 +505,18 @@ def run_pagerank_dist(args, dev, rank, world):
         nnz = nnz_local
     if rank != 0:
         return None
-    return {"metric": "PageRank iteration GTEPS, row-partitioned (NCCL all-gather of xs)",
+    how = ("exchange fused into the step: P2P stores of xs over peer memory" if args.exchange == "peer"
+           else "NCCL all-gather of xs")
+    return {"metric": f"PageRank iteration GTEPS, row-partitioned ({how})",
             "value": round(nnz / (ms * 1e-3) / 1e9, 3), "unit": "GTEPS", "n_gpus": world, "steps": K,
             "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"pagerank_rmat{S}_inlink_partitioned", "n_rows": n, "nnz": nnz,
                        "parallelism": f"row-partitioned x{world}", "padded_slice": pr.L,
                        "exchange_slice": pr.Lx, "exchange_bytes_in_per_rank_per_iter": pr.exchange_bytes_per_rank(),
-                       "exchange_layout": "non-dangling only (lossless)" if pr.compact else "all vertices"},
-            "gpu_launches": K, "clocks": clk.summary()}
+                       "exchange_layout": "non-dangling only (lossless)" if pr.compact else "all vertices",
+                       "exchange": args.exchange},
+            "gpu_launches": K * (2 if args.exchange == "peer" else 1), "clocks": clk.summary()}
 
 
 def run_hits_rwr(args, dev, rank, world):
@@ -736,6 +742,9 @@ def main():
     ap.add_argument("--scale", type=int, default=None, help="R-MAT scale for pagerank/dynamic")
     ap.add_argument("--batches", type=int, default=None, help="dynamic: number of insertion batches")
     ap.add_argument("--relabel", action="store_true", help="pagerank: degree-ordered vertex relabelling")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "peer"],
+                    help="pagerank_dist: NCCL all-gather after the step, or the exchange fused into the "
+                         "step over peer memory (acsr_pagerank_step_peer)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     world = int(os.environ.get("WORLD_SIZE", "1"))

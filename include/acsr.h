@@ -182,6 +182,70 @@ acsr_status acsr_pagerank_scale(int64_t n, const double *x, const int32_t *outde
                                 cudaStream_t stream);
 
 /* ------------------------------------------------------------------------ */
+/* Multi-GPU PageRank with the exchange FUSED into the step over peer memory
+ * (§VIII row split, reading Q19; SURVEY §8(e) lever 1 / §8(f) N1).
+ * Row-partitioned PageRank needs every rank's slice of xs' = PR'/outdeg in every
+ * rank's replicated xs after each step.  Here the fused step kernel stores each
+ * finished slice entry directly into all ranks' xs buffers (NVLink/NVSwitch P2P
+ * stores, overlapped with the rest of the step), and its last CTA publishes the
+ * push -- the Delta^2 partial and a release flag -- to every rank.  The next step
+ * waits on those flags at entry; no host-side collective is involved.
+ *
+ * One acsr_peer per rank (single node, one process per GPU; several processes may
+ * share a GPU).  The library owns one device region per rank: a state block and two
+ * replicated xs buffers of xs_len doubles (alternating by push parity; zeroed at
+ * create, so slots nobody writes -- e.g. the trailing always-zero slot of the
+ * dangling-free layout -- read +0.0).  Protocol:
+ *   1. acsr_peer_create on every rank -> ACSR_IPC_HANDLE_BYTES of HOST bytes;
+ *   2. the caller all-gathers the handles (any host transport, rank order);
+ *   3. acsr_peer_open maps every other rank's region (cudaIpcOpenMemHandle);
+ *   4. acsr_peer_push: xs = x / outdeg of the local rows (first iterate, or a
+ *      warm start), rows [0, slice_len) stored at slots slice_off + r of every
+ *      rank's next buffer;
+ *   5. per iteration: acsr_pagerank_step_peer (acsr_pagerank_step semantics; args->xs
+ *      is ignored -- the step reads the buffer of the previous push; args->n_cols must
+ *      equal xs_len; args->xs_next may be NULL, else it also receives the local xs';
+ *      args->delta2 receives this rank's partial).  With args->ctrl, a step first
+ *      waits for the previous push of every rank, adds their exact Delta^2 partials and,
+ *      when the sum is <= eps2, sets ctrl[0] and does nothing (every rank decides
+ *      alike): consecutive steps need no host round trip or extra launch.
+ *   6. acsr_peer_delta2 whenever the host wants the GLOBAL Delta^2 of the last push.
+ * Every rank must issue the same sequence of push / step calls.  Waits are bounded
+ * (20 s): a timed-out wait sets the error word read by acsr_peer_query and the call
+ * proceeds with invalid results rather than hanging the GPU.  Results are bitwise
+ * identical to the same partition with a plain all-gather (the per-row sums do not
+ * depend on where xs came from).  Not thread-safe; one stream per acsr_peer. */
+enum { ACSR_PEER_MAX = 8, ACSR_IPC_HANDLE_BYTES = 64 };
+typedef struct acsr_peer acsr_peer;
+
+/* slice_off/slice_len: this rank's exchanged slots [slice_off, slice_off+slice_len)
+ * of xs (local rows 0..slice_len-1 in order).  handle: HOST out, 64 bytes. */
+acsr_status acsr_peer_create(acsr_peer **out, int nranks, int rank, int64_t xs_len,
+                             int64_t slice_off, int64_t slice_len, void *handle);
+/* handles: HOST, nranks * ACSR_IPC_HANDLE_BYTES in rank order (own entry ignored). */
+acsr_status acsr_peer_open(acsr_peer *p, const void *handles);
+/* synchronises the device, unmaps the peers, frees the region. */
+acsr_status acsr_peer_destroy(acsr_peer *p);
+/* x, outdeg: [n] local rows (n >= slice_len); xs_local: NULL or [n] (also gets xs). */
+acsr_status acsr_peer_push(acsr_peer *p, int64_t n, const double *x, const int32_t *outdeg,
+                           double *xs_local, cudaStream_t stream);
+acsr_status acsr_pagerank_step_peer(const acsr_pr_args *args, acsr_peer *p, cudaStream_t stream);
+/* delta2: [1] device out, the global sum of every rank's partial of the last push
+ * (exact fixed-point partials: the same bits on every rank).  ctrl: NULL or [2] as in
+ * acsr_pr_args -- ctrl[0] is set here when delta2 <= eps2 (every rank decides alike),
+ * and a call with ctrl[0] set does nothing, so blocks of (step, delta2) pairs can be
+ * enqueued between host synchronisations. */
+acsr_status acsr_peer_delta2(acsr_peer *p, double *delta2, int32_t *ctrl, double eps2,
+                             cudaStream_t stream);
+/* HOST query (synchronous copy): pushes completed by this rank, the error word, and
+ * the local buffer holding the last push (NULL before the first push). */
+acsr_status acsr_peer_query(const acsr_peer *p, int64_t *pushes, int32_t *error,
+                            const double **xs_current);
+/* dst: [xs_len] device; receives (stream-ordered) this rank's replicated xs as left by
+ * the last push (zeros before the first push). */
+acsr_status acsr_peer_read_xs(const acsr_peer *p, double *dst, cudaStream_t stream);
+
+/* ------------------------------------------------------------------------ */
 /* HITS normalisation (Eq. 5-7).  The HITS step is one acsr_spmv on the
  * 2n x 2n pattern matrix [[0, A^T], [A, 0]] applied to v = [a; h] (Eq. 7); this call
  * then scales each half of y = [A^T h; A a] to unit Euclidean norm (reading R6; a zero

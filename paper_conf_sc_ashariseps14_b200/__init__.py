@@ -80,15 +80,34 @@ class PrArgs(ctypes.Structure):
 
 _lib.acsr_pagerank_step.argtypes = [ctypes.POINTER(PrArgs), _vp]
 _lib.acsr_pagerank_step.restype = ctypes.c_int
+_lib.acsr_pagerank_step_peer.argtypes = [ctypes.POINTER(PrArgs), _vp, _vp]
+_lib.acsr_pagerank_step_peer.restype = ctypes.c_int
+_lib.acsr_peer_create.argtypes = [ctypes.POINTER(_vp), ctypes.c_int, ctypes.c_int, _i64, _i64, _i64, _vp]
+_lib.acsr_peer_create.restype = ctypes.c_int
+_lib.acsr_peer_open.argtypes = [_vp, _vp]
+_lib.acsr_peer_open.restype = ctypes.c_int
+_lib.acsr_peer_destroy.argtypes = [_vp]
+_lib.acsr_peer_destroy.restype = ctypes.c_int
+_lib.acsr_peer_push.argtypes = [_vp, _i64, _vp, _vp, _vp, _vp]
+_lib.acsr_peer_push.restype = ctypes.c_int
+_lib.acsr_peer_delta2.argtypes = [_vp, _vp, _vp, _dbl, _vp]
+_lib.acsr_peer_delta2.restype = ctypes.c_int
+_lib.acsr_peer_query.argtypes = [_vp, ctypes.POINTER(_i64), ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(_vp)]
+_lib.acsr_peer_query.restype = ctypes.c_int
+_lib.acsr_peer_read_xs.argtypes = [_vp, _vp, _vp]
+_lib.acsr_peer_read_xs.restype = ctypes.c_int
 _lib.acsr_hits_workspace_bytes.argtypes = [_i64]
 _lib.acsr_hits_workspace_bytes.restype = _sz
 _lib.acsr_hits_normalize.argtypes = [_i64, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
 _lib.acsr_hits_normalize.restype = ctypes.c_int
 
 ACSR_BIN_SHORT_ALG2 = 1  # include/acsr.h: per-bin Alg. 2 units for bins 0..5
+ACSR_PEER_MAX = 8
+ACSR_IPC_HANDLE_BYTES = 64
 
 EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_bin_ex", "acsr_spmv", "acsr_pagerank_step",
-            "acsr_pagerank_scale", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_relayout",
+            "acsr_pagerank_scale", "acsr_pagerank_step_peer", "acsr_peer_create", "acsr_peer_open",
+            "acsr_peer_destroy", "acsr_peer_push", "acsr_peer_delta2", "acsr_peer_query", "acsr_peer_read_xs", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_relayout",
             "acsr_hits_workspace_bytes", "acsr_hits_normalize",
             "acsr_status_string", "acsr_last_error", "acsr_version")
 
@@ -221,6 +240,95 @@ def acsr_pagerank_step(row_begin, col_idx, bin_rows, bin_offsets, plan_ws, xs, x
                _dev(ctrl, torch.int32, "ctrl", True), float(eps2))
     _check(_lib.acsr_pagerank_step(ctypes.byref(a), _stream(stream)), "acsr_pagerank_step")
     return x_new, xs_next, delta2
+
+
+# --------------------------------------------------------------------------- peer exchange
+class AcsrPeer:
+    """Owner of one ``acsr_peer`` (include/acsr.h): the library-owned region holding this
+    rank's replicated xs double buffer and exchange flags, mapped into every other rank.
+    Protocol: ``handle`` (64 host bytes) -> caller all-gathers -> ``open(handles)``."""
+
+    def __init__(self, nranks, rank, xs_len, slice_off, slice_len):
+        self._p = _vp()
+        self.handle = ctypes.create_string_buffer(ACSR_IPC_HANDLE_BYTES)
+        _check(_lib.acsr_peer_create(ctypes.byref(self._p), int(nranks), int(rank), int(xs_len),
+                                     int(slice_off), int(slice_len), self.handle), "acsr_peer_create")
+        self.nranks, self.rank, self.xs_len = int(nranks), int(rank), int(xs_len)
+        self.slice_off, self.slice_len = int(slice_off), int(slice_len)
+
+    def handle_bytes(self) -> bytes:
+        return bytes(self.handle.raw)
+
+    def open(self, handles):
+        """handles: list of every rank's handle_bytes() in rank order."""
+        if len(handles) != self.nranks:
+            raise ValueError("one handle per rank")
+        buf = ctypes.create_string_buffer(b"".join(bytes(h) for h in handles), ACSR_IPC_HANDLE_BYTES * self.nranks)
+        _check(_lib.acsr_peer_open(self._p, buf), "acsr_peer_open")
+
+    def push(self, x, outdeg, xs_local=None, stream=None):
+        n = x.numel()
+        _check(_lib.acsr_peer_push(self._p, n, _dev(x, torch.float64, "x") if n else None,
+                                   _dev(outdeg, torch.int32, "outdeg") if n else None,
+                                   _dev(xs_local, torch.float64, "xs_local", True), _stream(stream)),
+               "acsr_peer_push")
+
+    def delta2(self, out, ctrl=None, eps2=-1.0, stream=None):
+        _check(_lib.acsr_peer_delta2(self._p, _dev(out, torch.float64, "delta2"),
+                                     _dev(ctrl, torch.int32, "ctrl", True), float(eps2), _stream(stream)),
+               "acsr_peer_delta2")
+        return out
+
+    def query(self):
+        """(pushes, error word, device address of the buffer holding the last push)."""
+        pushes, err, ptr = _i64(), ctypes.c_int32(), _vp()
+        _check(_lib.acsr_peer_query(self._p, ctypes.byref(pushes), ctypes.byref(err), ctypes.byref(ptr)),
+               "acsr_peer_query")
+        return int(pushes.value), int(err.value), ptr.value
+
+    def read_xs(self, out=None, stream=None):
+        """This rank's replicated xs as left by the last push (enqueued copy)."""
+        if out is None:
+            out = torch.empty(self.xs_len, dtype=torch.float64, device="cuda")
+        _check(_lib.acsr_peer_read_xs(self._p, _dev(out, torch.float64, "out"), _stream(stream)),
+               "acsr_peer_read_xs")
+        return out
+
+    def close(self):
+        if self._p:
+            _check(_lib.acsr_peer_destroy(self._p), "acsr_peer_destroy")
+            self._p = _vp()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def acsr_pagerank_step_peer(peer: AcsrPeer, row_begin, col_idx, bin_rows, bin_offsets, plan_ws, x, outdeg,
+                            x_new, xs_next, delta2, damping=0.85, teleport=None, n_global=None, row_end=None,
+                            stream=None, ctrl=None, eps2=-1.0):
+    """One fused PageRank step whose xs' slice is stored straight into every rank's
+    replicated xs (peer memory); reads the xs of the previous push.  xs_next may be None
+    (no local copy).  delta2 receives this rank's partial; the global one comes from
+    peer.delta2().  With ctrl, the step is a no-op once the global Delta^2 of the previous
+    step is <= eps2 (ctrl[0] set, identically on every rank)."""
+    n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
+    ng = peer.xs_len if n_global is None else n_global
+    tel = (1.0 - damping) / ng if teleport is None else teleport
+    a = PrArgs(n, peer.xs_len, _dev(row_begin, torch.int32, "row_begin"),
+               _dev(row_end, torch.int32, "row_end", True),
+               _dev(col_idx, torch.int32, "col_idx") if col_idx.numel() else None,
+               _dev(bin_rows, torch.int32, "bin_rows") if n else None,
+               _dev(bin_offsets, torch.int32, "bin_offsets"), _dev(plan_ws, torch.uint8, "plan_ws"),
+               plan_ws.numel(), None, _dev(x, torch.float64, "x") if n else None,
+               _dev(outdeg, torch.int32, "outdeg") if n else None,
+               _dev(x_new, torch.float64, "x_new") if n else None,
+               _dev(xs_next, torch.float64, "xs_next", True) if n else None, float(damping), float(tel),
+               _dev(delta2, torch.float64, "delta2"), -1, 0.0, _dev(ctrl, torch.int32, "ctrl", True), float(eps2))
+    _check(_lib.acsr_pagerank_step_peer(ctypes.byref(a), peer._p, _stream(stream)), "acsr_pagerank_step_peer")
+    return x_new, delta2
 
 
 # --------------------------------------------------------------------------- update

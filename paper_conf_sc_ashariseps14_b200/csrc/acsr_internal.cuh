@@ -169,6 +169,132 @@ inline PlanLayout plan_layout(int64_t n_rows, int64_t n_cols, int64_t nnz_max)
     return L;
 }
 
+// ---------------------------------------------------------------- peer-memory exchange
+// (acsr_peer.cu; NEXT N1 of SURVEY §8(f)).  Every rank owns one device region with the
+// same layout, mapped into every other rank's address space (CUDA IPC over NVLink /
+// NVSwitch P2P, or two processes on one GPU):
+//   PeerState at offset 0, then the two replicated xs buffers (push parity 0 / 1).
+// Rank q writes flag[q] and d2[.][q] in EVERY region (its own included) and xs slices
+// into every region's buffer; the owner alone writes `pushes`, `err`, `ticket`.
+//   pushes  number of completed pushes of this rank (init scale-push or fused step);
+//           push c+1 writes buffer c & 1 and reads buffer (c-1) & 1 (fused step)
+//   flag[q] = pushes of rank q once its stores of that push are visible (release.sys)
+//   d2[p][q] the 192-bit fixed-point Delta^2 partial of rank q's push with parity p
+constexpr int PEER_MAX = ACSR_PEER_MAX;
+struct PeerState;
+
+// kernel-side view of one acsr_peer.  The SpMV/PageRank kernel reads it through a
+// pointer (a copy lives in the owner's region): dynamic indexing of base[] in a
+// by-value kernel argument forced the whole argument block to local memory (spills).
+struct PeerArgs {
+    char *base[PEER_MAX];  // region base of rank q as mapped in this process
+    PeerState *st;         // == (PeerState *)base[rank]
+    int64_t off_buf[2];    // byte offset of xs buffer 0 / 1 inside a region
+    int64_t slice_off;     // first xs slot of this rank's slice
+    int64_t slice_len;     // local rows [0, slice_len) are exchanged
+    int64_t xs_len;        // doubles per xs buffer
+    int nranks, rank;
+};
+
+struct PeerState {
+    unsigned long long flag[PEER_MAX];
+    unsigned long long d2[2][PEER_MAX][3];
+    unsigned long long pushes;
+    unsigned int err;     // 1: a barrier wait timed out (results of that call are invalid)
+    unsigned int ticket;  // last-CTA detection of the push kernel
+    unsigned int last_step;  // 1 if this rank's last push was a fused step (has Delta^2 partials)
+    PeerArgs view;        // this process's view (owner-written at acsr_peer_open)
+};
+constexpr size_t PEER_BUF_ALIGN = 4096;
+
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p)
+{
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v)
+{
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long globaltimer_ns()
+{
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+// One thread: wait until every rank has completed `target` pushes.  Bounded (20 s):
+// on timeout st->err is set and the caller proceeds (the host checks err), so a lost
+// peer never hangs the GPU.
+__device__ __forceinline__ void peer_wait(const PeerArgs &p, unsigned long long target)
+{
+    const unsigned long long t0 = globaltimer_ns();
+    for (int q = 0; q < p.nranks; q++) {
+        while (ld_acquire_sys(&p.st->flag[q]) < target) {
+            if (globaltimer_ns() - t0 > 20000000000ull) {
+                atomicExch(&p.st->err, 1u);
+                return;
+            }
+            __nanosleep(256);
+        }
+    }
+}
+
+// One thread, after a system-scope fence that orders this push's data stores:
+// publish the Delta^2 partial (PR) and the new push count to every rank.
+__device__ __forceinline__ void peer_signal(const PeerArgs &p, unsigned long long newc, bool with_d2,
+                                            unsigned long long hi, unsigned long long mid, unsigned long long lo)
+{
+    if (with_d2) {
+        for (int q = 0; q < p.nranks; q++) {
+            PeerState *s = (PeerState *)p.base[q];
+            s->d2[newc & 1][p.rank][0] = hi;
+            s->d2[newc & 1][p.rank][1] = mid;
+            s->d2[newc & 1][p.rank][2] = lo;
+        }
+        __threadfence_system();
+    }
+    for (int q = 0; q < p.nranks; q++) st_release_sys(&((PeerState *)p.base[q])->flag[p.rank], newc);
+    p.st->pushes = newc;
+    p.st->last_step = with_d2 ? 1u : 0u;
+}
+
+// Global Delta^2 of push c: the exact sum of every rank's 192-bit partial (the same bits
+// on every rank, whatever the order), after peer_wait(p, c).
+__device__ __forceinline__ double peer_sum_d2(const PeerArgs &p, unsigned long long c)
+{
+    unsigned long long hi = 0, mid = 0, lo = 0;
+    for (int q = 0; q < p.nranks; q++) {
+        const volatile unsigned long long *s = p.st->d2[c & 1][q];
+        const unsigned long long h = s[0], m = s[1], l = s[2];
+        const unsigned long long nlo = lo + l;
+        const unsigned long long c1 = nlo < lo;
+        const unsigned long long m1 = mid + m;
+        const unsigned long long c2a = m1 < mid;
+        const unsigned long long m2 = m1 + c1;
+        const unsigned long long c2b = m2 < m1;
+        lo = nlo;
+        mid = m2;
+        hi += h + c2a + c2b;
+    }
+    return (double)hi + ((double)mid + (double)lo * 5.421010862427522e-20) * 5.421010862427522e-20;
+}
+
+}  // namespace acsr
+
+// host-side object behind the opaque acsr_peer handle (acsr_peer.cu)
+struct acsr_peer {
+    int nranks = 0, rank = 0, device = 0;
+    int64_t xs_len = 0, slice_off = 0, slice_len = 0;
+    size_t bytes = 0;
+    char *region = nullptr;  // this rank's region (cudaMalloc, library-owned)
+    bool opened = false;     // peers' regions mapped
+    acsr::PeerArgs args{};   // kernel view (valid once opened)
+};
+
+namespace acsr {
+
 // ---------------------------------------------------------------- device helpers
 __device__ __forceinline__ int bin_of_len(int len)
 {

@@ -79,6 +79,9 @@ struct SpmvArgs {
     double restart_weight;
     int32_t *ctrl;  // device-side convergence: [0] stop flag, [1] executed steps (nullable)
     double eps2;
+    // fused peer-memory exchange of xs_next (acsr_pagerank_step_peer; peer.nranks == 0: off)
+    const PeerArgs *peer;  // device copy (PeerState::view) or NULL
+    int64_t peer_next;  // byte offset of the buffer this step pushes into (set in-kernel)
 };
 
 // ----------------------------------------------------------------- PTX helpers
@@ -341,7 +344,18 @@ struct Kern {
             const double xn = a.teleport + a.damping * s + (r == a.restart ? a.restart_weight : 0.0);
             a.x_new[r] = xn;
             const int od = __ldg(a.outdeg + r);
-            a.xs_next[r] = od > 0 ? xn / (double)od : 0.0;
+            const double xs = od > 0 ? xn / (double)od : 0.0;
+            if (a.xs_next) a.xs_next[r] = xs;  // NULL: peer exchange only
+            if (a.peer) {
+                // the exchange, fused: store the slice entry straight into every rank's
+                // replicated xs (NVLink P2P stores; window rows give coalesced 256-B runs)
+                const PeerArgs *P = a.peer;
+                if (r < P->slice_len) {
+                    const int64_t o = a.peer_next + 8 * (P->slice_off + r);
+                    const int nr = P->nranks;
+                    for (int q = 0; q < nr; q++) *(double *)(P->base[q] + o) = xs;
+                }
+            }
             const double diff = xn - __ldg(a.x_old + r);
             fix_add(d2, diff * diff);
         } else {
@@ -688,6 +702,27 @@ spmv_kernel(SpmvArgs<V> a)
     PlanHeader *hdr = a.hdr;
     pdl_enter();
     if (PR && a.ctrl && *(volatile int32_t *)a.ctrl) return;  // converged earlier: no-op step
+    unsigned long long pc = 0;  // peer exchange: pushes completed before this step
+    if (PR && a.peer) {
+        const PeerArgs *P = a.peer;
+        pc = *(volatile unsigned long long *)&P->st->pushes;
+        a.x = (const V *)(P->base[P->rank] + P->off_buf[(pc + 1) & 1]);  // filled by push pc
+        a.peer_next = P->off_buf[pc & 1];
+        // every rank has completed push pc: buffer (pc-1)&1 is complete everywhere, and
+        // nobody still reads buffer pc&1 (the previous step of every rank read it)
+        // device-side convergence across ranks: the global Delta^2 of the previous step
+        // is complete now -- every CTA takes the same decision from the same partials
+        __shared__ int s_stop;
+        if (threadIdx.x == 0) {
+            peer_wait(*P, pc);
+            s_stop = (a.ctrl && P->st->last_step && peer_sum_d2(*P, pc) <= a.eps2) ? 1 : 0;
+        }
+        __syncthreads();
+        if (s_stop) {
+            if (blockIdx.x == 0 && threadIdx.x == 0) a.ctrl[0] = 1;
+            return;
+        }
+    }
     const int n_units = hdr->n_units;
     {
         char *ws = (char *)hdr;
@@ -777,7 +812,10 @@ spmv_kernel(SpmvArgs<V> a)
     }
     // last CTA out publishes Delta^2 and resets the counters for the next call
     if (lane == 0) {
-        __threadfence();
+        // peer exchange: the CTA's remote xs stores must be visible system-wide before
+        // the push is signalled (barrier above + system-scope fence, then the ticket chain)
+        if (PR && a.peer) __threadfence_system();
+        else __threadfence();
         if (atomicAdd(&hdr->exit_ticket, 1) == (int)gridDim.x - 1) {
             __threadfence();
             if (PR) {
@@ -785,10 +823,16 @@ spmv_kernel(SpmvArgs<V> a)
                 const uint64_t mid = *(volatile uint64_t *)&hdr->d2_mid;
                 const uint64_t lo = *(volatile uint64_t *)&hdr->d2_lo;
                 const double d2v = (double)hi + ((double)mid + (double)lo * 5.421010862427522e-20) * 5.421010862427522e-20;
-                *a.delta2 = d2v;
+                *a.delta2 = d2v;  // with the peer exchange: this rank's partial
+                if (a.peer) {
+                    __threadfence_system();
+                    peer_signal(*a.peer, pc + 1, true, hi, mid, lo);
+                }
                 if (a.ctrl) {
                     a.ctrl[1] += 1;
-                    if (d2v <= a.eps2) a.ctrl[0] = 1;
+                    // peer exchange: the global test runs at the next step's entry (or in
+                    // acsr_peer_delta2), once every rank's partial has arrived
+                    if (!a.peer && d2v <= a.eps2) a.ctrl[0] = 1;
                 }
                 hdr->d2_hi = 0;
                 hdr->d2_mid = 0;
@@ -1014,6 +1058,40 @@ extern "C" acsr_status acsr_pagerank_step(const acsr_pr_args *p, cudaStream_t st
     a.ctrl = p->ctrl; a.eps2 = p->eps2;
     dispatch<double, true>(a, stream);
     return acsr_check_launch("acsr_pagerank_step");
+}
+
+extern "C" acsr_status acsr_pagerank_step_peer(const acsr_pr_args *p, acsr_peer *peer, cudaStream_t stream)
+{
+    if (!peer || !peer->opened) {
+        acsr_set_error("acsr_pagerank_step_peer: peer object missing or not opened (acsr_peer_open)");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    if (!p || p->n_rows < 0 || p->n_rows >= ((int64_t)1 << 31) || !p->delta2 || p->n_cols != peer->xs_len ||
+        p->n_rows < peer->slice_len ||
+        (p->n_rows > 0 && (!p->row_begin || !p->x || !p->outdeg || !p->x_new))) {
+        acsr_set_error("acsr_pagerank_step_peer: invalid argument (n_cols must equal the peer xs_len, "
+                       "n_rows >= slice_len)");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    if (!plan_ok(p->n_rows, p->bin_rows, p->bin_offsets, p->plan_ws, p->plan_ws_bytes)) {
+        acsr_set_error("acsr_pagerank_step_peer: plan workspace missing or too small");
+        return ACSR_ERR_WORKSPACE;
+    }
+    if (p->n_rows == 0) {  // nothing local: still take part in the barrier / signal
+        acsr_set_error("acsr_pagerank_step_peer: a rank needs at least one row");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    SpmvArgs<double> a{};
+    a.rb = p->row_begin; a.re = p->row_end; a.col = p->col_idx;
+    a.val = nullptr; a.x = nullptr; a.y = nullptr;  // x: the peer buffer, chosen in-kernel
+    a.bin_rows = p->bin_rows; a.hdr = (PlanHeader *)p->plan_ws;
+    a.x_old = p->x; a.outdeg = p->outdeg; a.x_new = p->x_new; a.xs_next = p->xs_next;
+    a.damping = p->damping; a.teleport = p->teleport; a.delta2 = p->delta2;
+    a.restart = p->restart; a.restart_weight = p->restart_weight;
+    a.ctrl = p->ctrl; a.eps2 = p->eps2;
+    a.peer = &((const PeerState *)peer->region)->view;
+    dispatch<double, true>(a, stream);
+    return acsr_check_launch("acsr_pagerank_step_peer");
 }
 
 extern "C" acsr_status acsr_pagerank_scale(int64_t n, const double *x, const int32_t *outdeg,

@@ -10,6 +10,13 @@ Delta^2 partial), then
     all-gather; the only data-path exchange, A9 in SURVEY §8(a)),
   * all-reduces the 8-byte Delta^2 (the convergence test of Alg. 5, reading Q9).
 
+With ``exchange="peer"`` the all-gather disappears: the fused step kernel itself stores
+every finished xs' slice entry into all ranks' replicated xs over peer memory (NVLink /
+NVSwitch P2P stores through CUDA IPC mappings, overlapped with the rest of the step) and
+signals the push with a release flag; the next step waits on the flags at entry, and
+the global Delta^2 is the exact sum of the ranks' fixed-point partials
+(``acsr_pagerank_step_peer`` / ``acsr_peer_delta2``, include/acsr.h).
+
 Host logic here (partition, column renumbering into the padded layout, the loop) is
 device-agnostic so it is unit-tested with the gloo backend on CPU (tests/test_dist_gloo.py)
 by injecting a CPU step function; on GPUs the step is the CUDA kernel.
@@ -89,7 +96,12 @@ class DistPageRank:
     (acsr_pagerank_step)."""
 
     def __init__(self, row_ptr_local, col_local, outdeg_local, splits, n_global, damping=0.85,
-                 group=None, step_fn=None, scale_fn=None, device=None, compact=True):
+                 group=None, step_fn=None, scale_fn=None, device=None, compact=True, exchange="nccl"):
+        if exchange not in ("nccl", "peer"):
+            raise ValueError(f"exchange must be 'nccl' (collective all-gather) or 'peer', not {exchange!r}")
+        if exchange == "peer" and (step_fn is not None or scale_fn is not None):
+            raise ValueError("exchange='peer' fuses the exchange into the CUDA step (no step_fn)")
+        self.exchange_mode = exchange
         self.group = group
         self.rank = dist.get_rank(group) if dist.is_initialized() else 0
         self.world = dist.get_world_size(group) if dist.is_initialized() else 1
@@ -116,8 +128,14 @@ class DistPageRank:
         dev = self.device
         # replicated gathered xs (+1 trailing always-zero slot in the compact layout)
         nx = self.world * self.Lx + (1 if self.compact else 0)
-        self.xs = torch.zeros(nx, dtype=torch.float64, device=dev)
-        self.xs_next = torch.zeros_like(self.xs)
+        self.nx = nx
+        self.peer = None
+        if exchange == "peer":
+            self._setup_peer(nx)
+            self.xs = self.xs_next = torch.zeros(0, dtype=torch.float64, device=dev)  # in the peer regions
+        else:
+            self.xs = torch.zeros(nx, dtype=torch.float64, device=dev)
+            self.xs_next = torch.zeros_like(self.xs)
         # compact: the kernel writes the local xs here; its first Lx entries are exchanged
         self.xs_loc = (torch.zeros(max(self.n_local, self.Lx), dtype=torch.float64, device=dev)
                        if self.compact else None)
@@ -125,7 +143,22 @@ class DistPageRank:
         self._m = None
         if use_cuda:
             from .matrix import ACSRMatrix
-            self._m = ACSRMatrix(self.row_ptr, self.col, None, n_cols=self.xs.numel())
+            self._m = ACSRMatrix(self.row_ptr, self.col, None, n_cols=nx)
+
+    def _setup_peer(self, nx):
+        """acsr_peer regions: xs double buffer + flags per rank, handles all-gathered once."""
+        from . import AcsrPeer
+        if self.compact:
+            off, ln = self.rank * self.Lx, self.n_nd[self.rank]
+        else:
+            off, ln = self.rank * self.L, self.n_local
+        self.peer = AcsrPeer(self.world, self.rank, nx, off, ln)
+        if self.world > 1:
+            hs = [None] * self.world
+            dist.all_gather_object(hs, self.peer.handle_bytes(), group=self.group)
+        else:
+            hs = [self.peer.handle_bytes()]
+        self.peer.open(hs)
 
     def _setup_compact(self, row_ptr_local, col_local, outdeg_local):
         dev = row_ptr_local.device
@@ -181,18 +214,55 @@ class DistPageRank:
             dist.all_gather_into_tensor(buf, chunk.clone() if buf.device.type == "cpu" else chunk,
                                         group=self.group)
 
+    def _run_peer(self, x, eps, max_iter, check_every):
+        """Steps are enqueued back to back (no per-step collective or extra launch); each
+        step tests the global Delta^2 of the previous one at entry (device-side stop
+        flag), and the host reads the global Delta^2 every check_every steps."""
+        from . import acsr_pagerank_step_peer
+        m, peer = self._m, self.peer
+        peer.push(x, self.outdeg)
+        bufs = [x, torch.empty_like(x)]
+        part = torch.zeros(1, dtype=torch.float64, device=self.device)
+        ctrl = torch.zeros(2, dtype=torch.int32, device=self.device)
+        eps2 = eps * eps if eps >= 0 else -1.0
+        k = 0
+        while k < max_iter:
+            for _ in range(min(check_every, max_iter - k)):
+                acsr_pagerank_step_peer(peer, m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws,
+                                        bufs[k % 2], self.outdeg, bufs[(k + 1) % 2], None, part,
+                                        self.damping, self.teleport, self.n_global, ctrl=ctrl, eps2=eps2)
+                k += 1
+            peer.delta2(self.delta2)  # global Delta^2 of the last executed step
+            c = ctrl.cpu()
+            if int(c[0]) or float(self.delta2.item()) <= eps2:
+                break
+        it = int(ctrl[1].item())
+        _, err, _ = peer.query()
+        if err:
+            raise RuntimeError("acsr_peer: a peer barrier timed out (a rank stopped issuing steps?)")
+        return bufs[it % 2], it, float(self.delta2.item())
+
     def exchange_bytes_per_rank(self):
         """Bytes each rank receives per iteration from the all-gather."""
         return (self.world - 1) * self.Lx * 8
 
-    def run(self, x0_local=None, eps=1e-6, max_iter=1000):
+    def run(self, x0_local=None, eps=1e-6, max_iter=1000, check_every=1):
         """Alg. 5 loop; returns (x_local, iterations, delta2_global) with x_local in the
-        caller's local row order."""
+        caller's local row order.  check_every (peer exchange only): (step, Delta^2) pairs
+        enqueued between host synchronisations, steps after convergence are no-ops on
+        every rank (device-side stop flag) -- same results as checking every step."""
         dev = self.device
         if x0_local is None:
             x = torch.full((self.n_local,), 1.0 / self.n_global, dtype=torch.float64, device=dev)
         else:
             x = x0_local.clone() if self.perm is None else x0_local[self.perm].contiguous()
+        if self.peer is not None:
+            x, it, d2 = self._run_peer(x, eps, max_iter, max(1, int(check_every)))
+            if self.perm is not None:
+                out = torch.empty_like(x)
+                out[self.perm] = x
+                x = out
+            return x, it, d2
         # xs^0 slice = x^0 / outdeg (IEEE division), then gather
         if self.compact:
             self.scale_fn(x, self.outdeg, self._local_out())

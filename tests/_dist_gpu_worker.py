@@ -6,7 +6,7 @@ import torch
 import torch.distributed as dist
 
 
-def worker(rank, world, port, scale, q):
+def worker(rank, world, port, scale, q, exchange="nccl", compact=True, check_every=1):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     import synth
@@ -19,13 +19,22 @@ def worker(rank, world, port, scale, q):
     lo, hi = int(splits[rank]), int(splits[rank + 1])
     rpl = (rp[lo:hi + 1] - rp[lo]).to(dev)
     cil = ci[int(rp[lo]):int(rp[hi])].to(dev)
-    pr = pdist.DistPageRank(rpl, cil, od[lo:hi].to(dev), splits, n)
-    x, it, d2 = pr.run(eps=1e-6)
+    pr = pdist.DistPageRank(rpl, cil, od[lo:hi].to(dev), splits, n, exchange=exchange, compact=compact)
+    if exchange == "peer":
+        x, it, d2 = pr.run(eps=1e-6, check_every=check_every)
+        # every rank's replicated xs after the last push is the same vector
+        xs = pr.peer.read_xs()
+        allx = [torch.zeros_like(xs.cpu()) for _ in range(world)]
+        dist.all_gather(allx, xs.cpu())
+        assert all(torch.equal(allx[0], a) for a in allx), "replicated xs differ across ranks"
+        pr.peer.close()
+    else:
+        x, it, d2 = pr.run(eps=1e-6)
     parts = [torch.zeros(pr.L, dtype=torch.float64) for _ in range(world)]
     xp = torch.zeros(pr.L, dtype=torch.float64)
     xp[: x.numel()] = x.cpu()
     dist.all_gather(parts, xp)
     if rank == 0:
         full = torch.cat([parts[k][: int(splits[k + 1] - splits[k])] for k in range(world)])
-        q.put((full.numpy(), it))
+        q.put((full.numpy(), it, d2))
     dist.destroy_process_group()

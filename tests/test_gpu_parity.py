@@ -700,9 +700,7 @@ def test_spmv_from_host_e2e(acsr, cuda):
     check_spmv(y.numpy(), y_ref, den, torch.float64)
 
 
-def test_dist_pagerank_two_ranks_one_gpu(cuda):
-    # the partitioned driver with two ranks sharing the GPU (gloo for the exchange): CUDA
-    # step + column renumbering + padded all-gather + Delta^2 all-reduce vs the oracle
+def _two_ranks(scale, **kw):
     import socket
     import sys
     import torch.multiprocessing as mp
@@ -714,19 +712,91 @@ def test_dist_pagerank_two_ranks_one_gpu(cuda):
     s.close()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_dist_gpu_worker.worker, args=(r, 2, port, 14, q)) for r in range(2)]
+    procs = [ctx.Process(target=_dist_gpu_worker.worker, args=(r, 2, port, scale, q), kwargs=kw)
+             for r in range(2)]
     for p in procs:
         p.start()
-    full, it = q.get(timeout=300)
+    full, it, d2 = q.get(timeout=300)
     for p in procs:
         p.join(60)
         assert p.exitcode == 0
+    return full, it, d2
+
+
+def test_dist_pagerank_two_ranks_one_gpu(cuda):
+    # the partitioned driver with two ranks sharing the GPU (gloo for the exchange): CUDA
+    # step + column renumbering + padded all-gather + Delta^2 all-reduce vs the oracle
+    full, it, _ = _two_ranks(14)
     rp, ci, od, n = _inlink(14, cuda)
     x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)
     assert abs(it - it_ref) <= 1
     if it != it_ref:
         x_ref, _, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=0.0, max_iter=it)
     assert np.all(np.abs(full - x_ref) <= 1e-11 * x_ref + 1e-18)
+
+
+@pytest.mark.parametrize("compact", [True, False])
+def test_peer_exchange_two_ranks_one_gpu(cuda, compact):
+    # N1: the exchange fused into the step over peer memory (two processes sharing the GPU,
+    # CUDA IPC mappings, in-kernel P2P stores + release/acquire flags, exact Delta^2
+    # partials).  Same partition and layout as the collective all-gather path -> the same
+    # bits (iterate, iteration count, Delta^2); every rank's replicated xs identical
+    # (checked in the worker); and the oracle bar.
+    full_p, it_p, d2_p = _two_ranks(14, exchange="peer", compact=compact)
+    full_c, it_c, d2_c = _two_ranks(14, exchange="nccl", compact=compact)
+    assert it_p == it_c and np.array_equal(full_p, full_c)
+    # Delta^2: the collective path all-reduces two rounded doubles, the peer path adds the
+    # exact fixed-point partials and rounds once -> equal up to that one rounding
+    assert abs(d2_p - d2_c) <= 4e-16 * d2_c
+    full_8, it_8, d2_8 = _two_ranks(14, exchange="peer", compact=compact, check_every=8)
+    assert it_8 == it_p and d2_8 == d2_p and np.array_equal(full_8, full_p)
+    rp, ci, od, n = _inlink(14, cuda)
+    x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)
+    assert abs(it_p - it_ref) <= 1
+    if it_p != it_ref:
+        x_ref, _, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=0.0, max_iter=it_p)
+    assert np.all(np.abs(full_p - x_ref) <= 1e-11 * x_ref + 1e-18)
+
+
+def test_peer_exchange_single_rank_equals_pagerank(acsr, cuda):
+    # one rank: the peer path (push to itself, flags, Delta^2 via the partial) gives the
+    # single-GPU pagerank() bits, and a second run on the same acsr_peer (push count
+    # continues, buffer parity flips) gives them again
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+    rp, ci, od, n = _inlink(15, cuda)
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda))
+    x1, it1, d1 = acsr.pagerank(m, od.to(cuda), eps=1e-6, check_every=1)
+    pr = pdist.DistPageRank(rp.to(cuda), ci.to(cuda), od.to(cuda), np.array([0, n]), n, exchange="peer")
+    for _ in range(2):
+        xp, itp, dp = pr.run(eps=1e-6)
+        assert itp == it1 and dp == d1 and torch.equal(xp, x1)
+    x3, it3, d3 = pr.run(eps=1e-6, check_every=8)
+    assert it3 == it1 and d3 == d1 and torch.equal(x3, x1)
+    pushes, err, _ = pr.peer.query()
+    assert err == 0 and pushes == 3 * (it1 + 1)
+    # the replicated xs is the scaled final iterate
+    xs = pr.peer.read_xs()
+    ref = acsr.acsr_pagerank_scale(x1, od.to(cuda))
+    assert torch.equal(xs, ref)
+    pr.peer.close()
+
+
+def test_peer_argument_errors(acsr, cuda):
+    with pytest.raises(acsr.ACSRError):
+        acsr.AcsrPeer(9, 0, 10, 0, 5)  # more ranks than ACSR_PEER_MAX
+    with pytest.raises(acsr.ACSRError):
+        acsr.AcsrPeer(2, 0, 10, 8, 5)  # slice outside xs
+    p = acsr.AcsrPeer(1, 0, 10, 0, 10)
+    x = torch.ones(10, dtype=torch.float64, device=cuda)
+    od = torch.ones(10, dtype=torch.int32, device=cuda)
+    with pytest.raises(acsr.ACSRError):
+        p.push(x, od)  # not opened
+    p.open([p.handle_bytes()])
+    with pytest.raises(acsr.ACSRError):
+        p.push(x[:5], od[:5])  # fewer local rows than the slice
+    p.push(x, od)
+    assert torch.equal(p.read_xs(), x)
+    p.close()
 
 
 def test_device_side_convergence_identical(acsr, cuda):

@@ -557,6 +557,23 @@ def run_hits_rwr(args, dev, rank, world):
 
 
 # ------------------------------------------------------------------------------ dynamic graph (C5)
+def host_inclusive_batch(m, chd, outdeg, st, uws, x, xs_tmp, y):
+    """Wall time (ms) of update + re-bin + scale + SpMV issued from an idle GPU through
+    the Python API, on a scratch copy of the slack CSR (the live matrix is not touched)."""
+    import paper_conf_sc_ashariseps14_b200 as acsr
+    mm = acsr.ACSRMatrix(m.row_begin, m.col_idx.clone(), None, row_end=m.row_end.clone(),
+                         row_cap=m.row_cap, nnz_max=m.nnz_max)
+    od = outdeg.clone()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    mm.update(chd, outdeg=od, status=st, ws=uws)
+    mm.rebin()
+    acsr.acsr_pagerank_scale(x, od, xs_tmp)
+    mm.spmv(xs_tmp, y)
+    torch.cuda.synchronize()
+    return (time.perf_counter() - t0) * 1e3
+
+
 def run_dynamic(args, dev, rank, world):
     """C5: R-MAT s20 in-link pattern with slack (cap = len + max(4, len/4)); per batch of
     16,384 inserted edges: H2D of the change lists, acsr_update_edges, acsr_bin, one SpMV
@@ -586,6 +603,10 @@ def run_dynamic(args, dev, rank, world):
         pinned = {kk: torch.from_numpy(v).pin_memory() for kk, v in ch.items()}
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(5)]
         torch.cuda.synchronize()
+        # device time of each phase: the batch is enqueued behind a ~0.5 ms GPU sleep, so
+        # the host's launch/marshalling time does not show up as gaps between the events;
+        # the host-inclusive time (sync -> enqueue -> sync, no sleep) is reported beside it
+        torch.cuda._sleep(1_000_000)
         ev[0].record()
         chd = {kk: v.to(dev, non_blocking=True) for kk, v in pinned.items()}
         ev[1].record()
@@ -606,12 +627,15 @@ def run_dynamic(args, dev, rank, world):
             torch.cuda.synchronize()
             regrow += 1
         relayouts += regrow
+        # host-inclusive: the same update + re-bin + SpMV issued from an idle GPU (a
+        # re-applied insert batch only appends duplicates, so time it on a scratch copy)
+        t_host = host_inclusive_batch(m, chd, outdeg, st, uws, x, xs_tmp, y) if b >= args.warmup else 0.0
         t0 = time.perf_counter()
         x, it, _ = acsr.pagerank(m, outdeg, x0=x, eps=1e-6)
         torch.cuda.synchronize()
         t_pr = time.perf_counter() - t0
         if b >= args.warmup:
-            rec.append([ev[i].elapsed_time(ev[i + 1]) for i in range(4)] + [t_pr * 1e3, it, k])
+            rec.append([ev[i].elapsed_time(ev[i + 1]) for i in range(4)] + [t_pr * 1e3, it, k, t_host])
     r = np.array(rec)
     if rank != 0:
         return None
@@ -626,6 +650,9 @@ def run_dynamic(args, dev, rank, world):
                           "t_spmv_ms": round(t_spmv, 5), "bin_lt_spmv": bool(t_bin < t_spmv),
                           "pt_st": round(t_bin / t_spmv, 3),
                           "rebuild_plus_spmv_ms": round(t_upd + t_bin + t_spmv, 5),
+                          "rebuild_plus_spmv_host_inclusive_ms": round(float(r[:, 7].mean()), 5),
+                          "timing": "phases: CUDA events, batch enqueued behind a GPU sleep (device time); "
+                                    "host_inclusive: wall clock from an idle GPU through the Python API",
                           "pagerank_warm_ms": round(float(r[:, 4].mean()), 4),
                           "warm_iterations_mean": round(float(r[:, 5].mean()), 2),
                           "inserted_edges_mean": round(float(r[:, 6].mean()), 1),
@@ -662,6 +689,7 @@ def run_dynamic_mixed(args, dev, rank, world):
         pinned = {k: torch.from_numpy(v).pin_memory() for k, v in ch.items()}
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
         torch.cuda.synchronize()
+        torch.cuda._sleep(1_000_000)  # device time: enqueue behind a GPU sleep (as run_dynamic)
         ev[0].record()
         chd = {k: v.to(dev, non_blocking=True) for k, v in pinned.items()}
         ev[1].record()

@@ -81,7 +81,14 @@ struct SpmvArgs {
     double eps2;
     // fused peer-memory exchange of xs_next (acsr_pagerank_step_peer; peer.nranks == 0: off)
     const PeerArgs *peer;  // device copy (PeerState::view) or NULL
-    int64_t peer_next;  // byte offset of the buffer this step pushes into (set in-kernel)
+    // set in-kernel from *peer (registers + a shared copy of the region bases), so the
+    // per-row epilogue does not re-load the peer view
+    char *const *pbase;    // shared: region base of every rank
+    char *pself;           // region base of this rank
+    int64_t peer_next;     // byte offset of the buffer this step pushes into
+    int64_t peer_off;      // slice_off
+    int peer_len, peer_n;  // slice_len (< 2^31, local rows), nranks
+    int peer_rank;
 };
 
 // ----------------------------------------------------------------- PTX helpers
@@ -302,7 +309,14 @@ __device__ __forceinline__ double ldx(const float *p)
 #endif
 }
 
-template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
+// xs' slice entry -> every OTHER rank's replicated buffer (byte offset o in each region)
+__device__ __noinline__ void peer_store(char *const *pbase, int nranks, int self, int64_t o, double v)
+{
+    for (int q = 0; q < nranks; q++)
+        if (q != self) *(double *)(pbase[q] + o) = v;
+}
+
+template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC, bool PEER = false>
 struct Kern {
     using A = SpmvArgs<V>;
 
@@ -346,15 +360,14 @@ struct Kern {
             const int od = __ldg(a.outdeg + r);
             const double xs = od > 0 ? xn / (double)od : 0.0;
             if (a.xs_next) a.xs_next[r] = xs;  // NULL: peer exchange only
-            if (a.peer) {
-                // the exchange, fused: store the slice entry straight into every rank's
-                // replicated xs (NVLink P2P stores; window rows give coalesced 256-B runs)
-                const PeerArgs *P = a.peer;
-                if (r < P->slice_len) {
-                    const int64_t o = a.peer_next + 8 * (P->slice_off + r);
-                    const int nr = P->nranks;
-                    for (int q = 0; q < nr; q++) *(double *)(P->base[q] + o) = xs;
-                }
+            // the exchange, fused: store the slice entry straight into every rank's
+            // replicated xs (NVLink P2P stores; window rows give coalesced 256-B runs).
+            // The remote loop is out of line: inlined at every finish() site it cost
+            // I-cache misses (ncu no_instruction stalls 0.9 -> 3.3 per issue, +13 %).
+            if (PEER && r < a.peer_len) {
+                const int64_t o = a.peer_next + 8 * (a.peer_off + r);
+                *(double *)(a.pself + o) = xs;  // own replicated buffer: inline
+                if (a.peer_n > 1) peer_store(a.pbase, a.peer_n, a.peer_rank, o, xs);
             }
             const double diff = xn - __ldg(a.x_old + r);
             fix_add(d2, diff * diff);
@@ -689,11 +702,12 @@ struct Kern {
 #define ACSR_MIN_BLOCKS (1024 / SPMV_THREADS)  // 64 registers per thread
 #endif
 
-template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
+template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC, bool PEER = false>
 __global__ void __launch_bounds__(SPMV_THREADS, ACSR_MIN_BLOCKS)
 spmv_kernel(SpmvArgs<V> a)
 {
-    using K = Kern<V, HAS_VAL, HAS_END, PR, XC>;
+    static_assert(!PEER || (PR && !XC), "the peer exchange is a PageRank-step epilogue");
+    using K = Kern<V, HAS_VAL, HAS_END, PR, XC, PEER>;
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t bar;
     const int lane = threadIdx.x & 31;
@@ -703,11 +717,19 @@ spmv_kernel(SpmvArgs<V> a)
     pdl_enter();
     if (PR && a.ctrl && *(volatile int32_t *)a.ctrl) return;  // converged earlier: no-op step
     unsigned long long pc = 0;  // peer exchange: pushes completed before this step
-    if (PR && a.peer) {
+    __shared__ char *s_pbase[PEER_MAX];
+    if (PEER) {
         const PeerArgs *P = a.peer;
         pc = *(volatile unsigned long long *)&P->st->pushes;
         a.x = (const V *)(P->base[P->rank] + P->off_buf[(pc + 1) & 1]);  // filled by push pc
         a.peer_next = P->off_buf[pc & 1];
+        a.peer_off = P->slice_off;
+        a.peer_len = (int)P->slice_len;
+        a.peer_n = P->nranks;
+        a.peer_rank = P->rank;
+        a.pself = P->base[P->rank];
+        if (threadIdx.x < PEER_MAX) s_pbase[threadIdx.x] = threadIdx.x < P->nranks ? P->base[threadIdx.x] : nullptr;
+        a.pbase = s_pbase;
         // every rank has completed push pc: buffer (pc-1)&1 is complete everywhere, and
         // nobody still reads buffer pc&1 (the previous step of every rank read it)
         // device-side convergence across ranks: the global Delta^2 of the previous step
@@ -814,7 +836,7 @@ spmv_kernel(SpmvArgs<V> a)
     if (lane == 0) {
         // peer exchange: the CTA's remote xs stores must be visible system-wide before
         // the push is signalled (barrier above + system-scope fence, then the ticket chain)
-        if (PR && a.peer) __threadfence_system();
+        if (PEER) __threadfence_system();
         else __threadfence();
         if (atomicAdd(&hdr->exit_ticket, 1) == (int)gridDim.x - 1) {
             __threadfence();
@@ -824,7 +846,7 @@ spmv_kernel(SpmvArgs<V> a)
                 const uint64_t lo = *(volatile uint64_t *)&hdr->d2_lo;
                 const double d2v = (double)hi + ((double)mid + (double)lo * 5.421010862427522e-20) * 5.421010862427522e-20;
                 *a.delta2 = d2v;  // with the peer exchange: this rank's partial
-                if (a.peer) {
+                if (PEER) {
                     __threadfence_system();
                     peer_signal(*a.peer, pc + 1, true, hi, mid, lo);
                 }
@@ -832,7 +854,7 @@ spmv_kernel(SpmvArgs<V> a)
                     a.ctrl[1] += 1;
                     // peer exchange: the global test runs at the next step's entry (or in
                     // acsr_peer_delta2), once every rank's partial has arrived
-                    if (!a.peer && d2v <= a.eps2) a.ctrl[0] = 1;
+                    if (!PEER && d2v <= a.eps2) a.ctrl[0] = 1;
                 }
                 hdr->d2_hi = 0;
                 hdr->d2_mid = 0;
@@ -882,23 +904,23 @@ static size_t spmv_smem(int bits)
     return (XC ? (sizeof(V) + sizeof(uint16_t)) * ((size_t)1 << bits) : 0) + (size_t)reserve;
 }
 
-template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC>
+template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC, bool PEER = false>
 static void launch(const SpmvArgs<V> &a, cudaStream_t s)
 {
     static size_t configured = 0;
     const size_t smem = spmv_smem<V, XC>(a.xc_bits);
     if (smem > configured) {
-        cudaFuncSetAttribute(spmv_kernel<V, HAS_VAL, HAS_END, PR, XC>,
+        cudaFuncSetAttribute(spmv_kernel<V, HAS_VAL, HAS_END, PR, XC, PEER>,
                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         configured = smem;
     }
     static int per_sm = 0;
     if (!per_sm) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmv_kernel<V, HAS_VAL, HAS_END, PR, XC>,
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmv_kernel<V, HAS_VAL, HAS_END, PR, XC, PEER>,
                                                       SPMV_THREADS, smem);
         if (per_sm < 1) per_sm = 1;
     }
-    launch_pdl(spmv_kernel<V, HAS_VAL, HAS_END, PR, XC>, per_sm * acsr_num_sms(), SPMV_THREADS, smem, s, a);
+    launch_pdl(spmv_kernel<V, HAS_VAL, HAS_END, PR, XC, PEER>, per_sm * acsr_num_sms(), SPMV_THREADS, smem, s, a);
 }
 
 template <typename V, bool PR, bool XC>
@@ -967,6 +989,11 @@ static int dispatch(SpmvArgs<V> a, cudaStream_t s)
 {
     a.vph = ACSR_NO_VEC ? -1 : vec_phase<V>(a.col, a.val);
     a.xc_bits = xcache_bits();
+    if (PR && a.peer) {  // fused peer exchange: pattern matrix, no x cache
+        if (a.re) launch<V, false, true, true, false, true>(a, s);
+        else launch<V, false, false, true, false, true>(a, s);
+        return 1;
+    }
     if (xcache_enabled() && a.x != nullptr) {
         xc_fill_kernel<V><<<((1 << a.xc_bits) + 255) / 256, 256, 0, s>>>(a.hdr, a.x, a.xc_bits,
                                                                           xcache_force_miss());

@@ -366,6 +366,51 @@ def test_pagerank_converged_parity(acsr, cuda, scale):
     assert np.all(np.abs(x.cpu().numpy() - xr) <= 1e-11 * xr + 1e-18)
 
 
+def test_pagerank_s26_first_steps_sampled(acsr, cuda):
+    """C4 at BASELINE size (R-MAT s26 in-link pattern: 67 M rows, ~1.06 B nnz), in the
+    launch configuration bench.py times (one fused acsr_pagerank_step per iteration from
+    the cold start): bins bitwise, and for each of the first three steps the sampled rows
+    (random, the longest, the first rows of every bin) against the oracle step taken from
+    the same iterate ("at s26, check parity on the first 3 PageRank steps")."""
+    rp, ci = synth.rmat_csr(26, device=cuda, transpose=True)
+    n = rp.numel() - 1
+    od = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    m = acsr.ACSRMatrix(rp, ci)
+    rph = rp.cpu().numpy()
+    br, off = oracle.bins(rph)
+    assert np.array_equal(m.bin_offsets.cpu().numpy(), off)
+    assert np.array_equal(m.bin_rows.cpu().numpy(), br)
+    ln = np.diff(rph)
+    rng = np.random.default_rng(26)
+    sample = set(rng.choice(n, 3000, replace=False).tolist()) | set(np.argsort(ln)[-20:].tolist())
+    for b in range(32):
+        sample |= set(br[off[b]:off[b + 1]][:10].tolist())
+    rows = np.array(sorted(sample))
+    sub_rp = np.zeros(rows.size + 1, np.int64)
+    sub_rp[1:] = np.cumsum(ln[rows])
+    idx = torch.cat([torch.arange(int(rph[r]), int(rph[r + 1]), device=cuda) for r in rows])
+    sub_ci = ci[idx].cpu().numpy()
+    odh = od.cpu().numpy()
+    teleport = (1.0 - 0.85) / n
+    x = torch.full((n,), 1.0 / n, dtype=torch.float64, device=cuda)
+    xs = acsr.acsr_pagerank_scale(x, od)
+    xn, xsn = torch.empty_like(x), torch.empty_like(x)
+    d2 = torch.zeros(1, dtype=torch.float64, device=cuda)
+    for step in range(3):
+        acsr.acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xs, x, od,
+                                xn, xsn, d2, 0.85, teleport, n)
+        xh = x.cpu().numpy()
+        ref, _ = oracle.pagerank_step(sub_rp.astype(np.int32), sub_ci, odh, xh, teleport, 0.85)
+        got = xn.cpu().numpy()[rows]
+        # step bar (fp64 O5): |err| <= 1e-12 * (teleport + d * sum |xs|), all terms >= 0
+        assert np.all(np.abs(got - ref) <= 1e-12 * ref), (step, np.max(np.abs(got - ref) / ref))
+        # the scaled vector the next step gathers is x'/outdeg (IEEE division)
+        xs_ref = np.where(odh[rows] > 0, got / np.maximum(odh[rows], 1), 0.0)
+        assert np.array_equal(xsn.cpu().numpy()[rows], xs_ref)
+        x, xn = xn, x
+        xs, xsn = xsn, xs
+
+
 def test_pagerank_closed_forms(acsr, cuda):
     # directed cycle -> uniform 1/n after one step
     n = 10007

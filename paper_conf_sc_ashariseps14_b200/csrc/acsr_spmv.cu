@@ -41,6 +41,12 @@
 #ifndef ACSR_PAIR_ROWS
 #define ACSR_PAIR_ROWS 0  // 1: warp-per-row bins process two rows at a time (A/B builds)
 #endif
+#ifndef ACSR_WIN_LDS4
+#define ACSR_WIN_LDS4 0  // 1: four shared loads in flight per add group (A/B: C3a +6 %, C2 +2 %, slower)
+#endif
+#ifndef ACSR_WIN_PREFETCH
+#define ACSR_WIN_PREFETCH 0  // 1: prefetch the next window's row bounds (A/B: no gain on C3a, LiveJournal-like +5 %)
+#endif
 #ifndef ACSR_VEC_MIN
 #define ACSR_VEC_MIN 512  // rows (chunks) shorter than this use the lane-strided scalar path
 #endif
@@ -575,11 +581,24 @@ struct Kern {
         constexpr unsigned FULL = 0xffffffffu;
         const unsigned lt = (1u << lane) - 1u;
         const unsigned le = 0xffffffffu >> (31 - lane);
+#if ACSR_WIN_PREFETCH
+        // the next window's row bounds are loaded while this window runs (one dependent
+        // DRAM round trip less per window on short-row matrices)
+        int nbeg = 0, nend = 0;
+        if (lane < nrows) row_bounds(a, r0 + lane, nbeg, nend);
+#endif
         for (int w = 0; w < nrows; w += WIN_ROWS) {
             const int r = r0 + w + lane;
             const bool in = w + lane < nrows;
             int beg = 0, end = 0;
+#if ACSR_WIN_PREFETCH
+            beg = nbeg;
+            end = nend;
+            nbeg = nend = 0;
+            if (w + WIN_ROWS + lane < nrows) row_bounds(a, r + WIN_ROWS, nbeg, nend);
+#else
             if (in) row_bounds(a, r, beg, end);
+#endif
             const int len = end - beg;
             const bool mine = in && len <= WIN_MAX_LEN;
             const int l = mine ? len : 0;
@@ -622,7 +641,19 @@ struct Kern {
                 __syncwarp();
                 if (l > 0) {
                     const int i1 = min(pre + l, t0 + 32 * WIN_G) - t0;
-                    for (int i = max(pre, t0) - t0; i < i1; i++) acc += buf[i];
+                    int i = max(pre, t0) - t0;
+#if ACSR_WIN_LDS4
+                    // four shared loads in flight, then the adds in element order (the sum
+                    // is the same bits as the one-at-a-time loop; only the loads overlap)
+                    for (; i + 4 <= i1; i += 4) {
+                        const double b0 = buf[i], b1 = buf[i + 1], b2 = buf[i + 2], b3 = buf[i + 3];
+                        acc += b0;
+                        acc += b1;
+                        acc += b2;
+                        acc += b3;
+                    }
+#endif
+                    for (; i < i1; i++) acc += buf[i];
                 }
                 __syncwarp();
             }

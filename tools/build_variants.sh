@@ -47,6 +47,13 @@ for v in "$@"; do
     wb6u128) build wb6u128 -DACSR_WIN_MAX_BIN=6 -DACSR_WIN_UNIT_ROWS=128 ;;
     wb6u256) build wb6u256 -DACSR_WIN_MAX_BIN=6 -DACSR_WIN_UNIT_ROWS=256 ;;
     wu256) build wu256 -DACSR_WIN_UNIT_ROWS=256 ;;
+    wp1) build wp1 -DACSR_WIN_PREFETCH=1 ;;
+    l41) build l41 -DACSR_WIN_LDS4=1 ;;
+    wu64) build wu64 -DACSR_WIN_UNIT_ROWS=64 ;;
+    wu32) build wu32 -DACSR_WIN_UNIT_ROWS=32 ;;
+
+    wg8) build wg8 -DACSR_WIN_G=8 ;;
+    wb6) build wb6 -DACSR_WIN_MAX_BIN=6 ;;
   esac
 done
 wait

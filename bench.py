@@ -9,7 +9,8 @@ factor 16, fp64 (C2).  `value` = GFLOP/s = 2*nnz per step / device time of the s
 L2 is flushed (256 MiB write) between timed steps, outside the step's events.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl acsr|reference]
-                  [--workload rmat20|rmat20_f32|webgoogle|livejournal|pagerank|dynamic]
+                  [--workload rmat20|rmat20_f32|webgoogle|livejournal|rmat20_split|pagerank|
+                              pagerank_dist|dynamic|dynamic_mixed|hits|rwr]
 
 With N > 1 (torchrun) every rank runs its own independent matrix (seed + rank): the
 units are independent problems, no data-path collective, scaling "weak"; the time is
@@ -458,6 +459,63 @@ def run_pagerank(args, dev, rank, world):
             "gpu_launches": K, "clocks": clk.summary()}
 
 
+def run_spmv_split(args, dev, rank, world):
+    """N4: ONE C2 matrix (R-MAT s20 fp64, the same seed on every rank) row-split across
+    the ranks (nnz-balanced contiguous ranges, cost 12 len + 16), every rank bins
+    its rows and runs acsr_spmv on them each step; y stays distributed (no exchange in the
+    step).  Strong scaling: value = 2 nnz per step / max-over-ranks step time."""
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+
+    rp, ci = synth.rmat_csr(20, seed=20, device=dev)
+    n, nnz = rp.numel() - 1, ci.numel()
+    val = synth.values(nnz, 1014, torch.float64, dev)
+    x = synth.vector(n, 2014, torch.float64, dev)
+    splits = pdist.partition_rows((rp[1:] - rp[:-1]).cpu().numpy(), world, b_nnz=12, b_row=16)
+    sp = pdist.DistSpMV(rp, ci, val, splits)
+    nnz_local = sp.col.numel()
+    del rp, ci, val
+    y = torch.empty(sp.n_local, dtype=torch.float64, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+    for _ in range(args.warmup):
+        flush.zero_()
+        sp.rebin()
+        sp.spmv(x, y)
+    torch.cuda.synchronize()
+    K = args.steps
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(K)]
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    with Clocks(torch.cuda.current_device()) as clk:
+        for k in range(K):
+            flush.zero_()
+            ev[k][0].record(stream)
+            sp.rebin()
+            ev[k][1].record(stream)
+            sp.spmv(x, y)
+            ev[k][2].record(stream)
+        torch.cuda.synchronize()
+    t_bin = float(np.mean([ev[k][0].elapsed_time(ev[k][1]) for k in range(K)]))
+    t_spmv = float(np.mean([ev[k][1].elapsed_time(ev[k][2]) for k in range(K)]))
+    tot = t_bin + t_spmv
+    if world > 1:
+        tt = torch.tensor([tot, t_bin, t_spmv], dtype=torch.float64, device=dev)
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        tot, t_bin, t_spmv = (float(v) for v in tt.tolist())
+    if rank != 0:
+        return None
+    return {"metric": "SpMV GFLOP/s (bin+SpMV per step), one matrix row-split across GPUs",
+            "value": round(2.0 * nnz / (tot * 1e-3) / 1e9, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K,
+            "warmup": args.warmup, "ms_per_step": round(tot, 5), "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": "rmat20_ef16_f64_row_split", "n_rows": n, "nnz": nnz,
+                       "nnz_rank0": nnz_local, "parallelism": f"row-split x{world} (P:345)",
+                       "l2": "flushed: 256 MiB write between timed steps (outside the step events)"},
+            "breakdown": {"t_bin_ms_max_rank": round(t_bin, 5), "t_spmv_ms_max_rank": round(t_spmv, 5)},
+            "gpu_launches": 4 * K * world, "clocks": clk.summary()}
+
+
 def run_pagerank_dist(args, dev, rank, world):
     """C4 row-partitioned across the ranks (reading Q19): every rank builds the
     in-link graph, keeps its nnz-balanced contiguous row range, and per iteration runs
@@ -796,6 +854,8 @@ def main():
             torch.distributed.init_process_group(backend)
     if args.workload == "pagerank":
         line = run_pagerank(args, dev, rank, world)
+    elif args.workload == "rmat20_split":
+        line = run_spmv_split(args, dev, rank, world)
     elif args.workload == "pagerank_dist":
         line = run_pagerank_dist(args, dev, rank, world)
     elif args.workload == "dynamic":

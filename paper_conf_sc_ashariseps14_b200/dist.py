@@ -288,3 +288,76 @@ class DistPageRank:
             out[self.perm] = x
             x = out
         return x, it, d2
+
+
+def aligned_slice(t: torch.Tensor, start: int, stop: int, elems_per_16b: int) -> torch.Tensor:
+    """Copy t[start:stop] into a fresh buffer whose first element sits at the same
+    16-byte phase as t[start] does in t (elements of width 16/elems_per_16b).  The SpMV
+    groups 128-bit vector loads by that phase, so a row's summation order -- and its
+    result bits -- are the same in the slice as in the whole array (SURVEY §8(c),
+    "P-invariance")."""
+    ph = start % elems_per_16b
+    buf = torch.empty(stop - start + ph, dtype=t.dtype, device=t.device)
+    out = buf[ph:]
+    out.copy_(t[start:stop])
+    return out
+
+
+class DistSpMV:
+    """One SpMV y = A x row-split across P ranks (§VIII: "map half of the rows in
+    each bin to each device, each GPU is thus responsible for computing half the
+    results", generalised to P ranks as contiguous nnz-balanced row ranges, reading Q19;
+    SURVEY §8(f) N4).  Rank k holds rows [splits[k], splits[k+1]) with GLOBAL column ids
+    and the whole x; it bins its rows once (acsr_bin) and every call runs acsr_spmv on
+    them -- no exchange in the SpMV itself.  gather() all-gathers the y slices (padded,
+    in place) when every rank needs the whole y.
+
+    The local col/val keep their global 16-byte phase (aligned_slice), so every row is
+    summed exactly as on one GPU: the P-rank y equals the 1-GPU y bit for bit.
+
+    spmv_fn(row_ptr, col, val, x) -> y_local overrides the CUDA call (CPU tests)."""
+
+    def __init__(self, row_ptr, col, val, splits, group=None, spmv_fn=None, b_nnz=None, b_row=16):
+        self.group = group
+        self.rank = dist.get_rank(group) if dist.is_initialized() else 0
+        self.world = dist.get_world_size(group) if dist.is_initialized() else 1
+        self.splits = np.asarray(splits, dtype=np.int64)
+        assert self.splits.size == self.world + 1
+        lo, hi = int(self.splits[self.rank]), int(self.splits[self.rank + 1])
+        rp = row_ptr.to(torch.int64)
+        k0, k1 = int(rp[lo]), int(rp[hi])
+        self.row_ptr = (rp[lo:hi + 1] - k0).to(torch.int32)
+        self.col = aligned_slice(col, k0, k1, 4)
+        self.val = None if val is None else aligned_slice(val, k0, k1, 16 // val.element_size())
+        self.n_local = hi - lo
+        self.L = padded_layout(self.splits)
+        self._m = None
+        self.spmv_fn = spmv_fn
+        self.n_cols = None
+
+    def _matrix(self, n_cols):
+        if self._m is None:
+            from .matrix import ACSRMatrix
+            self._m = ACSRMatrix(self.row_ptr, self.col, self.val, n_cols=n_cols)
+        return self._m
+
+    def spmv(self, x, y_local=None):
+        """This rank's rows of A x."""
+        if self.spmv_fn is not None:
+            return self.spmv_fn(self.row_ptr, self.col, self.val, x)
+        return self._matrix(x.numel()).spmv(x, y_local)
+
+    def rebin(self):
+        if self._m is not None:
+            self._m.rebin()
+
+    def gather(self, y_local):
+        """Whole y on every rank (padded equal-size all-gather of the slices)."""
+        if self.world == 1:
+            return y_local
+        pad = torch.zeros(self.L, dtype=y_local.dtype, device=y_local.device)
+        pad[: self.n_local] = y_local
+        allp = torch.empty(self.world * self.L, dtype=y_local.dtype, device=y_local.device)
+        dist.all_gather_into_tensor(allp, pad, group=self.group)
+        sizes = np.diff(self.splits)
+        return torch.cat([allp[k * self.L: k * self.L + int(sizes[k])] for k in range(self.world)])

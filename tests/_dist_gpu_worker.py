@@ -38,3 +38,27 @@ def worker(rank, world, port, scale, q, exchange="nccl", compact=True, check_eve
         full = torch.cat([parts[k][: int(splits[k + 1] - splits[k])] for k in range(world)])
         q.put((full.numpy(), it, d2))
     dist.destroy_process_group()
+
+
+def spmv_worker(rank, world, port, scale, dtype_name, q):
+    """N4: C2-shaped matrix row-split over `world` ranks sharing the GPU (gloo for the
+    y gather); rank 0 returns the gathered y."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import synth
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+    dev = torch.device("cuda:0")
+    dtype = getattr(torch, dtype_name)
+    rp, ci = synth.rmat_csr(scale, device=dev)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 1014, dtype, dev)
+    x = synth.vector(n, 2014, dtype, dev)
+    splits = pdist.partition_rows((rp[1:] - rp[:-1]).cpu().numpy(), world, b_nnz=4 + val.element_size(), b_row=16)
+    sp = pdist.DistSpMV(rp, ci, val, splits)
+    y = sp.spmv(x)
+    y2 = sp.spmv(x)  # a second call on the same plan: identical
+    assert torch.equal(y, y2)
+    yall = sp.gather(y.cpu())
+    if rank == 0:
+        q.put(yall.numpy())
+    dist.destroy_process_group()

@@ -122,3 +122,49 @@ def test_permute_rows_roundtrip():
         r = int(perm[i])
         assert torch.equal(ci2[int(rp2[i]):int(rp2[i + 1])], ci[int(rp[r]):int(rp[r + 1])])
     assert int(rp2[-1]) == ci.numel()
+
+
+def _spmv_worker(rank, world, port, out):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    rp, ci = synth.rmat_csr(12)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 7)
+    x = synth.vector(n, 8)
+    splits = acsr_dist.partition_rows(np.diff(rp.numpy()), world, b_nnz=12, b_row=16)
+
+    def local(row_ptr, col, v, xx):
+        y, _ = oracle.spmv(row_ptr.numpy(), col.numpy(), v.numpy(), xx.numpy())
+        return torch.from_numpy(y)
+
+    sp = acsr_dist.DistSpMV(rp, ci, val, splits, spmv_fn=local)
+    # the local arrays keep the global 16-byte phase of their first element
+    k0 = int(rp[int(splits[rank])])
+    assert sp.col.data_ptr() % 16 == (ci.data_ptr() + 4 * k0) % 16
+    assert sp.val.data_ptr() % 16 == (val.data_ptr() + 8 * k0) % 16
+    y = sp.gather(sp.spmv(x))
+    if rank == 0:
+        out.put((y.numpy(), splits))
+    dist.destroy_process_group()
+
+
+def test_dist_spmv_row_split_gloo_ws2():
+    """N4: one SpMV split by rows over two ranks (gloo, CPU; the oracle as the local SpMV):
+    nnz-balanced split points equal the oracle's O8 partition, the gathered y equals the
+    oracle on the whole matrix bit for bit."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_spmv_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    y, splits = q.get(timeout=120)
+    for p in ps:
+        p.join(60)
+        assert p.exitcode == 0
+    rp, ci = synth.rmat_csr(12)
+    val = synth.values(ci.numel(), 7)
+    x = synth.vector(rp.numel() - 1, 8)
+    y_ref, _ = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    assert np.array_equal(y, y_ref)
+    assert np.array_equal(splits, oracle.partition(rp.numpy(), 2, 12, 16))

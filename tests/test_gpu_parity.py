@@ -780,6 +780,39 @@ def test_dist_pagerank_two_ranks_one_gpu(cuda):
     assert np.all(np.abs(full - x_ref) <= 1e-11 * x_ref + 1e-18)
 
 
+@pytest.mark.parametrize("dtype", ["float64", "float32"])
+def test_dist_spmv_row_split_bitwise(acsr, cuda, dtype):
+    """N4 (P:345 row split): one SpMV row-split over three ranks sharing the GPU equals the
+    one-GPU acsr_spmv bit for bit (local col/val keep their global 16-byte phase), and the
+    oracle bar."""
+    import socket
+    import sys
+    import torch.multiprocessing as mp
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    import _dist_gpu_worker
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_dist_gpu_worker.spmv_worker, args=(r, 3, port, 16, dtype, q)) for r in range(3)]
+    for p in procs:
+        p.start()
+    y_split = q.get(timeout=300)
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    dt = getattr(torch, dtype)
+    rp, ci = synth.rmat_csr(16, device=cuda)
+    val = synth.values(ci.numel(), 1014, dt, cuda)
+    x = synth.vector(rp.numel() - 1, 2014, dt, cuda)
+    y1 = acsr.ACSRMatrix(rp, ci, val).spmv(x).cpu().numpy()
+    assert np.array_equal(y_split, y1)
+    y_ref, den = oracle.spmv(rp.cpu().numpy(), ci.cpu().numpy(), val.cpu().numpy(), x.cpu().numpy())
+    check_spmv(y_split, y_ref, den, dt)
+
+
 @pytest.mark.parametrize("compact", [True, False])
 def test_peer_exchange_two_ranks_one_gpu(cuda, compact):
     # N1: the exchange fused into the step over peer memory (two processes sharing the GPU,

@@ -211,8 +211,9 @@ acsr_status acsr_pagerank_scale(int64_t n, const double *x, const int32_t *outde
  *      alike): consecutive steps need no host round trip or extra launch.
  *   6. acsr_peer_delta2 whenever the host wants the GLOBAL Delta^2 of the last push.
  * Every rank must issue the same sequence of push / step calls.  Waits are bounded
- * (20 s): a timed-out wait sets the error word read by acsr_peer_query and the call
- * proceeds with invalid results rather than hanging the GPU.  Results are bitwise
+ * (20 s, or ACSR_PEER_TIMEOUT_MS read at acsr_peer_open): a timed-out wait sets the
+ * error word read by acsr_peer_query and the call proceeds with invalid results
+ * rather than hanging the GPU.  Results are bitwise
  * identical to the same partition with a plain all-gather (the per-row sums do not
  * depend on where xs came from).  Not thread-safe; one stream per acsr_peer. */
 enum { ACSR_PEER_MAX = 8, ACSR_IPC_HANDLE_BYTES = 64 };

@@ -193,6 +193,7 @@ struct PeerArgs {
     int64_t slice_off;     // first xs slot of this rank's slice
     int64_t slice_len;     // local rows [0, slice_len) are exchanged
     int64_t xs_len;        // doubles per xs buffer
+    unsigned long long timeout_ns;  // bound of every flag wait (ACSR_PEER_TIMEOUT_MS, default 20 s)
     int nranks, rank;
 };
 
@@ -224,15 +225,15 @@ __device__ __forceinline__ unsigned long long globaltimer_ns()
     return t;
 }
 
-// One thread: wait until every rank has completed `target` pushes.  Bounded (20 s):
-// on timeout st->err is set and the caller proceeds (the host checks err), so a lost
-// peer never hangs the GPU.
+// One thread: wait until every rank has completed `target` pushes.  Bounded
+// (p.timeout_ns, 20 s by default): on timeout st->err is set and the caller proceeds
+// (the host checks err), so a lost peer never hangs the GPU.
 __device__ __forceinline__ void peer_wait(const PeerArgs &p, unsigned long long target)
 {
     const unsigned long long t0 = globaltimer_ns();
     for (int q = 0; q < p.nranks; q++) {
         while (ld_acquire_sys(&p.st->flag[q]) < target) {
-            if (globaltimer_ns() - t0 > 20000000000ull) {
+            if (globaltimer_ns() - t0 > p.timeout_ns) {
                 atomicExch(&p.st->err, 1u);
                 return;
             }

@@ -16,6 +16,7 @@
 // e.g. torch.distributed.all_gather_object).
 #include <cuda_runtime.h>
 #include <stddef.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <new>
@@ -131,6 +132,11 @@ extern "C" acsr_status acsr_peer_open(acsr_peer *p, const void *handles)
     a.slice_off = p->slice_off;
     a.slice_len = p->slice_len;
     a.xs_len = p->xs_len;
+    {
+        const char *e = getenv("ACSR_PEER_TIMEOUT_MS");
+        const long long ms = (e && e[0]) ? atoll(e) : 20000;
+        a.timeout_ns = (unsigned long long)(ms > 0 ? ms : 20000) * 1000000ull;
+    }
     for (int q = 0; q < p->nranks; q++) {
         if (q == p->rank) {
             a.base[q] = p->region;

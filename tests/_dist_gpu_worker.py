@@ -62,3 +62,30 @@ def spmv_worker(rank, world, port, scale, dtype_name, q):
     if rank == 0:
         q.put(yall.numpy())
     dist.destroy_process_group()
+
+
+def peer_timeout_worker(rank, world, port, q):
+    """Rank 1 maps the regions and then stops issuing pushes; rank 0's push and steps must
+    time out (ACSR_PEER_TIMEOUT_MS), set the error word and return, not hang."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), ACSR_PEER_TIMEOUT_MS="300")
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import time
+    import paper_conf_sc_ashariseps14_b200 as acsr
+    dev = torch.device("cuda:0")
+    n = 1000
+    peer = acsr.AcsrPeer(world, rank, 2 * n, rank * n, n)
+    hs = [None] * world
+    dist.all_gather_object(hs, peer.handle_bytes())
+    peer.open(hs)
+    if rank == 0:
+        x = torch.full((n,), 1.0 / n, dtype=torch.float64, device=dev)
+        od = torch.ones(n, dtype=torch.int32, device=dev)
+        peer.push(x, od)          # waits only for pushes >= 0: passes
+        peer.push(x, od)          # needs rank 1's first push: times out
+        t0 = time.perf_counter()
+        torch.cuda.synchronize()
+        pushes, err, _ = peer.query()
+        q.put((pushes, err, time.perf_counter() - t0))
+    dist.barrier()
+    peer.close()
+    dist.destroy_process_group()

@@ -859,6 +859,30 @@ def test_peer_exchange_single_rank_equals_pagerank(acsr, cuda):
     pr.peer.close()
 
 
+def test_peer_wait_times_out_instead_of_hanging(cuda):
+    """A rank that stops issuing pushes: the other rank's flag wait gives up after the
+    bound (ACSR_PEER_TIMEOUT_MS = 300 here), sets the error word and the GPU stays usable."""
+    import socket
+    import sys
+    import torch.multiprocessing as mp
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    import _dist_gpu_worker
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_dist_gpu_worker.peer_timeout_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    pushes, err, waited = q.get(timeout=120)
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    assert err == 1 and pushes == 2 and waited < 30.0
+
+
 def test_peer_argument_errors(acsr, cuda):
     with pytest.raises(acsr.ACSRError):
         acsr.AcsrPeer(9, 0, 10, 0, 5)  # more ranks than ACSR_PEER_MAX

@@ -275,6 +275,10 @@ def run_acsr(args, dev, rank, world):
     e1.record(stream)
     torch.cuda.synchronize()
     t_e2e = e0.elapsed_time(e1) / ke
+    if world > 1:  # whole job: every rank ran its own e2e loop concurrently; max over ranks
+        te = torch.tensor([t_e2e], dtype=torch.float64, device=dev)
+        torch.distributed.all_reduce(te, op=torch.distributed.ReduceOp.MAX)
+        t_e2e = float(te.item())
     h2d = sum(t.numel() * t.element_size() for t in (rp_h, ci_h, val_h, x_h))
     d2h = y_h.numel() * y_h.element_size()
     ctx = cusparse_context(rp, ci, val, x, n)
@@ -307,13 +311,13 @@ def run_acsr(args, dev, rank, world):
                      "frac": round(achieved / peak, 4), "traffic": ncu_traffic(label),
                      "kernel": "acsr::spmv_kernel", "peak_kind": peak_kind,
                      "algorithmic_bytes_per_launch": int(alg_bytes)},
-        "e2e": {"value": round(2.0 * nnz / (t_e2e * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
-                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+        "e2e": {"value": round(2.0 * nnz * world / (t_e2e * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
+                "h2d_bytes_per_step": int(h2d) * world, "d2h_bytes_per_step": int(d2h) * world,
                 "ms_per_step": round(t_e2e, 4)},
-        "gpu_launches": 4 * K,  # per step: bin_count, bin_scan, bin_scatter, spmv_kernel
+        "gpu_launches": 4 * K * world,  # per step and rank: bin_count, bin_scan, bin_scatter, spmv_kernel
         "clocks": clk.summary(),
     }
-    if not args.no_cpu_baseline:
+    if not args.no_cpu_baseline and world == 1:  # the oracle baseline: rank 0 at N = 1 only
         line["cpu_baseline"] = cpu_baseline(rp, ci, val, x, dtype)
     return line
 

@@ -812,7 +812,7 @@ def run_reference(args, dev):
     dt = (time.perf_counter() - t0) / K
     v = 2.0 * cih.size / dt / 1e9
     return {"metric": "SpMV GFLOP/s (bin+SpMV per step) & HBM GB/s vs peak", "impl": "reference",
-            "value": round(v, 4), "unit": "GFLOP/s", "n_gpus": 1, "steps": K, "warmup": args.warmup,
+            "value": round(v, 4), "unit": "GFLOP/s", "n_gpus": int(os.environ.get("WORLD_SIZE", "1")), "steps": K, "warmup": args.warmup,
             "ms_per_step": round(dt * 1e3, 3), "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64" if dtype == torch.float64 else "f32", "data": "synthetic",
             "config": {"workload": label, "n_rows": int(rph.size - 1), "nnz": int(cih.size)},

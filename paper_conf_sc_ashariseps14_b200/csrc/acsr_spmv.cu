@@ -41,6 +41,9 @@
 #ifndef ACSR_PAIR_ROWS
 #define ACSR_PAIR_ROWS 0  // 1: warp-per-row bins process two rows at a time (A/B builds)
 #endif
+#ifndef ACSR_MERGED_WARP_PATH
+#define ACSR_MERGED_WARP_PATH 0  // 1: heavy + warp-per-row in one loop (A/B: PageRank s26 -0.8 %, SpMV C2/C3 +2-3 %)
+#endif
 #ifndef ACSR_WIN_LDS4
 #define ACSR_WIN_LDS4 0  // 1: four shared loads in flight per add group (A/B: C3a +6 %, C2 +2 %, slower)
 #endif
@@ -699,14 +702,72 @@ struct Kern {
         }
     }
 
+#if ACSR_MERGED_WARP_PATH
+    // Heavy chunks and the warp-per-row bins 7..10 in ONE loop, so the vectorised
+    // strided_dot and the epilogue are inlined once for both (I-cache: the PageRank
+    // kernel's executed code did not fit, ncu no_instruction stalls).
+    static __device__ __forceinline__ void warp_rows(const A &a, int u, int2 d, int lane, Fix192 &d2)
+    {
+        const uint32_t y = (uint32_t)d.y;
+        const bool hv = (y & HEAVY_FLAG) != 0;
+        int cnt, myr = 0, mb = 0, me = 0, c = 0, nch = 0;
+        if (hv) {
+            c = (int)(y & ~HEAVY_FLAG);
+            int beg, end;
+            row_bounds(a, d.x, beg, end);
+            cnt = 1;
+            myr = d.x;
+            mb = beg + c * HEAVY_CHUNK;
+            me = min(mb + HEAVY_CHUNK, end);
+            nch = heavy_chunks(end - beg);
+        } else {
+            cnt = (int)(y & 0xFFFFFF);
+            if (lane < cnt) {
+                myr = __ldg(a.bin_rows + d.x + lane);
+                row_bounds(a, myr, mb, me);
+            }
+        }
+        for (int i = 0; i < cnt; i++) {
+            const int r = __shfl_sync(0xffffffffu, myr, i);
+            const int kb = __shfl_sync(0xffffffffu, mb, i);
+            const int ke = __shfl_sync(0xffffffffu, me, i);
+            double s = warp_sum(strided_dot(a, kb, ke, lane));
+            if (hv && nch > 1) {  // one chunk of a long row: last arriver combines in chunk order
+                const int u0 = u - c;
+                int last = 0;
+                if (lane == 0) {
+                    a.partial[u] = s;
+                    __threadfence();
+                    last = (atomicAdd(a.ticket + u0, 1) == nch - 1);
+                }
+                last = __shfl_sync(0xffffffffu, last, 0);
+                if (!last) return;
+                __threadfence();
+                double t = 0.0;
+                for (int j = lane; j < nch; j += 32) t += __ldcg(a.partial + u0 + j);
+                s = warp_sum(t);
+                if (lane == 0) a.ticket[u0] = 0;  // ready for the next call on this plan
+            }
+            if (lane == 0) finish(a, r, s, d2);
+        }
+    }
+#endif
+
     static __device__ __forceinline__ void unit(const A &a, int u, int lane, Fix192 &d2, double *wbuf, int2 *wtab)
     {
         const int2 d = __ldg(a.units + u);
         const uint32_t y = (uint32_t)d.y;
+#if ACSR_MERGED_WARP_PATH
+        if ((y & HEAVY_FLAG) || (!(y & WIN_FLAG) && (int)(y >> 24) > 6)) {
+            warp_rows(a, u, d, lane, d2);
+            return;
+        }
+#else
         if (y & HEAVY_FLAG) {
             heavy(a, u, d.x, (int)(y & ~HEAVY_FLAG), lane, d2);
             return;
         }
+#endif
         if (WIN_MAX_BIN >= 0 && (y & WIN_FLAG)) {
             window(a, d.x, (int)(y & 0xFFFFFF), lane, d2, wbuf, wtab);
             return;
@@ -720,7 +781,9 @@ struct Kern {
             case 4: light_sub<8>(a, d.x, cnt, lane, d2); break;
             case 5: light_sub<16>(a, d.x, cnt, lane, d2); break;
             case 6: light_sub<32>(a, d.x, cnt, lane, d2); break;
+#if !ACSR_MERGED_WARP_PATH
             default: light_warp(a, d.x, cnt, lane, d2); break;
+#endif
         }
     }
 };

@@ -49,6 +49,7 @@ for v in "$@"; do
     wu256) build wu256 -DACSR_WIN_UNIT_ROWS=256 ;;
     wp1) build wp1 -DACSR_WIN_PREFETCH=1 ;;
     l41) build l41 -DACSR_WIN_LDS4=1 ;;
+    mw1) build mw1 -DACSR_MERGED_WARP_PATH=1 ;;
     wu64) build wu64 -DACSR_WIN_UNIT_ROWS=64 ;;
     wu32) build wu32 -DACSR_WIN_UNIT_ROWS=32 ;;
 

@@ -184,6 +184,29 @@ def make_workload(name, dev, rank):
     return label, dtype, rp, ci, val, x
 
 
+def read_stream_gbs(dev, gib=2, reps=5):
+    """Read-only streaming bandwidth measured in the same job (quote the
+    roofline against the spec, the measured copy and a read-only stream): a 2 GiB fp32
+    reduction (torch.sum, far larger than L2), best of `reps`."""
+    buf = torch.ones((gib << 30) // 4, dtype=torch.float32, device=dev)
+    buf.sum()
+    torch.cuda.synchronize()
+    best = 0.0
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        buf.sum()
+        e1.record()
+        torch.cuda.synchronize()
+        best = max(best, buf.numel() * 4 / (e0.elapsed_time(e1) * 1e-3) / 1e9)
+    del buf
+    torch.cuda.empty_cache()
+    return best
+
+
+HBM_SPEC_GBS = 8000.0  # B200 HBM3e nominal (the north star's denominator)
+
+
 def algorithmic_bytes(rp, ci, dtype):
     """(s_v+4) nnz + 4(n+1) row_ptr + 4n bin_rows + s_v n_c x + s_v n y."""
     n = rp.numel() - 1
@@ -282,6 +305,7 @@ def run_acsr(args, dev, rank, world):
     h2d = sum(t.numel() * t.element_size() for t in (rp_h, ci_h, val_h, x_h))
     d2h = y_h.numel() * y_h.element_size()
     ctx = cusparse_context(rp, ci, val, x, n)
+    rs = read_stream_gbs(dev)
     if rank != 0:
         return None
     peak, peak_kind = peaks()
@@ -310,7 +334,11 @@ def run_acsr(args, dev, rank, world):
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": ncu_traffic(label),
                      "kernel": "acsr::spmv_kernel", "peak_kind": peak_kind,
-                     "algorithmic_bytes_per_launch": int(alg_bytes)},
+                     "algorithmic_bytes_per_launch": int(alg_bytes),
+                     "vs_other_peaks": {"read_stream_measured_gbs": round(rs, 1),
+                                        "frac_vs_read_stream": round(achieved / rs, 4),
+                                        "spec_gbs": HBM_SPEC_GBS,
+                                        "frac_vs_spec": round(achieved / HBM_SPEC_GBS, 4)}},
         "e2e": {"value": round(2.0 * nnz * world / (t_e2e * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
                 "h2d_bytes_per_step": int(h2d) * world, "d2h_bytes_per_step": int(d2h) * world,
                 "ms_per_step": round(t_e2e, 4)},

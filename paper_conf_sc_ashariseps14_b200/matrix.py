@@ -189,13 +189,16 @@ def hits_matrix(out_ptr, out_col, n=None):
     return row_ptr, col
 
 
-def hits(out_ptr, out_col, eps=1e-6, max_iter=1000, stream=None):
+def hits(out_ptr, out_col, eps=1e-6, max_iter=1000, stream=None, B=None):
     """HITS (Eq. 5-7; reading R6): one acsr_spmv on [[0, A^T], [A, 0]] per
-    iteration plus acsr_hits_normalize.  a^0 = h^0 = 1/|V|.  Returns (a, h, iters)."""
+    iteration plus acsr_hits_normalize.  a^0 = h^0 = 1/|V|.  B: the binned block
+    matrix (ACSRMatrix of hits_matrix(out_ptr, out_col)), built here when None.  Returns
+    (a, h, iters)."""
     n = out_ptr.numel() - 1
     dev = out_ptr.device
-    rp, col = hits_matrix(out_ptr, out_col, n)
-    B = ACSRMatrix(rp, col, None, n_cols=2 * n)
+    if B is None:
+        rp, col = hits_matrix(out_ptr, out_col, n)
+        B = ACSRMatrix(rp, col, None, n_cols=2 * n)
     v = torch.full((2 * n,), 1.0 / n, dtype=torch.float64, device=dev)
     y, vn = torch.empty_like(v), torch.empty_like(v)
     d2 = torch.zeros(2, dtype=torch.float64, device=dev)

@@ -85,9 +85,10 @@ __device__ __forceinline__ void count_tile(BinSmem &sm, int64_t n, const int32_t
     if (tid < NBINS) cnt[(int64_t)tid * n_tiles + tile] = sm.hist[tid];
     if (tid == NBINS) {
         int lu = 0;
+        const bool tl = tail_tile(tile, n_tiles);
 #pragma unroll
-        for (int b = wmb + 1; b <= LIGHT_MAX_BIN; b++) lu += (sm.hist[b] + unit_rows(b) - 1) / unit_rows(b);
-        if (wmb >= 0) lu += win_units((int)min((int64_t)TILE_ROWS, n - base));
+        for (int b = wmb + 1; b <= LIGHT_MAX_BIN; b++) lu += (sm.hist[b] + unit_rows_t(b, tl) - 1) / unit_rows_t(b, tl);
+        if (wmb >= 0) lu += win_units_t((int)min((int64_t)TILE_ROWS, n - base), tl);
         cnt[(int64_t)NBINS * n_tiles + tile] = lu;
         cnt[(int64_t)(NBINS + 1) * n_tiles + tile] = sm.heavy;
     }
@@ -278,12 +279,14 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
         // bins above wmb up to 10, in bin order, row-contiguous (wmb = -1: no windows,
         // bins 0..10 as per-bin units -- Alg. 2 for the short bins)
         const int tile_rows = (int)min((int64_t)TILE_ROWS, n - base);
-        const int nwin = wmb >= 0 ? win_units(tile_rows) : 0;
+        const bool tl = tail_tile(tile, n_tiles);
+        const int wur = win_unit_rows_t(tl);
+        const int nwin = wmb >= 0 ? win_units_t(tile_rows, tl) : 0;
         if (tid == 0) {
             int acc = nwin;
             for (int b = 0; b <= LIGHT_MAX_BIN; b++) {
                 sm.upre[b] = acc;
-                if (b > wmb) acc += (sm.run[b] + unit_rows(b) - 1) / unit_rows(b);
+                if (b > wmb) acc += (sm.run[b] + unit_rows_t(b, tl) - 1) / unit_rows_t(b, tl);
             }
             sm.upre[LIGHT_MAX_BIN + 1] = acc;
         }
@@ -292,14 +295,14 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
         const int total = sm.upre[LIGHT_MAX_BIN + 1];
         for (int j = tid; j < total; j += BIN_THREADS) {
             if (j < nwin) {
-                const int r0 = j * WIN_UNIT_ROWS;
-                units[ubase + j] = make_int2((int)(base + r0), (int)(WIN_FLAG | (uint32_t)min(WIN_UNIT_ROWS, tile_rows - r0)));
+                const int r0 = j * wur;
+                units[ubase + j] = make_int2((int)(base + r0), (int)(WIN_FLAG | (uint32_t)min(wur, tile_rows - r0)));
                 continue;
             }
             int b = 0;
             while (sm.upre[b + 1] <= j) b++;
             const int q = j - sm.upre[b];
-            const int K = unit_rows(b);
+            const int K = unit_rows_t(b, tl);
             const int c = min(K, sm.run[b] - q * K);
             units[ubase + j] = make_int2(sm.seg[b] + q * K, (b << 24) | c);
         }

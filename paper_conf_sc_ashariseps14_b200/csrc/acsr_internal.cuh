@@ -103,6 +103,29 @@ static_assert(TILE_ROWS % WIN_UNIT_ROWS == 0, "tiles hold whole window units");
 
 __host__ __device__ constexpr int win_units(int tile_rows) { return (tile_rows + WIN_UNIT_ROWS - 1) / WIN_UNIT_ROWS; }
 
+// Tail tiles: the last max(1, n_tiles / ACSR_TAIL_DIV) tiles of the work list get 4x
+// smaller work units (32-row windows, a quarter of the rows per bin unit), so the last
+// claims of the dynamic schedule are short and warps run out of work together
+// (0: off; A/B builds).
+#ifndef ACSR_TAIL_DIV
+#define ACSR_TAIL_DIV 0
+#endif
+__host__ __device__ inline bool tail_tile(int tile, int n_tiles)
+{
+    if (ACSR_TAIL_DIV <= 0) return false;
+    const int k = n_tiles / (ACSR_TAIL_DIV > 0 ? ACSR_TAIL_DIV : 1);
+    return tile >= n_tiles - (k > 1 ? k : 1);
+}
+__host__ __device__ inline int unit_rows_t(int b, bool tail)
+{
+    return tail ? (unit_rows(b) / 4 > 1 ? unit_rows(b) / 4 : 1) : unit_rows(b);
+}
+__host__ __device__ inline int win_unit_rows_t(bool tail) { return tail ? WIN_ROWS : WIN_UNIT_ROWS; }
+__host__ __device__ inline int win_units_t(int tile_rows, bool tail)
+{
+    return (tile_rows + win_unit_rows_t(tail) - 1) / win_unit_rows_t(tail);
+}
+
 // unit descriptor: light  x = first index into bin_rows, y = (bin << 24) | rows
 //                  heavy  x = row id,                     y = 0x80000000 | chunk
 //                  window x = first row,                  y = 0x40000000 | rows

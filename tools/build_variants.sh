@@ -50,6 +50,9 @@ for v in "$@"; do
     wp1) build wp1 -DACSR_WIN_PREFETCH=1 ;;
     l41) build l41 -DACSR_WIN_LDS4=1 ;;
     mw1) build mw1 -DACSR_MERGED_WARP_PATH=1 ;;
+    td16) build td16 -DACSR_TAIL_DIV=16 ;;
+    td8) build td8 -DACSR_TAIL_DIV=8 ;;
+    td32) build td32 -DACSR_TAIL_DIV=32 ;;
     wu64) build wu64 -DACSR_WIN_UNIT_ROWS=64 ;;
     wu32) build wu32 -DACSR_WIN_UNIT_ROWS=32 ;;
 

@@ -88,6 +88,7 @@ struct SpmvArgs {
     double restart_weight;
     int32_t *ctrl;  // device-side convergence: [0] stop flag, [1] executed steps (nullable)
     double eps2;
+    int64_t x_prefetch;  // bytes of x to bulk-prefetch into L2 at entry (0: none)
     // fused peer-memory exchange of xs_next (acsr_pagerank_step_peer; peer.nranks == 0: off)
     const PeerArgs *peer;  // device copy (PeerState::view) or NULL
     // set in-kernel from *peer (registers + a shared copy of the region bases), so the
@@ -808,6 +809,24 @@ spmv_kernel(SpmvArgs<V> a)
     const int gw = blockIdx.x * SPMV_WARPS + (threadIdx.x >> 5);
     const int nw = gridDim.x * SPMV_WARPS;
     PlanHeader *hdr = a.hdr;
+    if (a.x_prefetch > 0 && threadIdx.x < 32) {
+        // x fits L2: every CTA bulk-prefetches its slice into L2 before waiting for the
+        // previous grid (PDL), so the first gather of each sector does not pay a DRAM
+        // round trip.  A prefetch is only a cache hint -- L2 is the point of coherence,
+        // so prefetching before the producer of x has finished can never return stale data.
+        const uintptr_t x0 = ((uintptr_t)a.x + 15) & ~(uintptr_t)15;
+        const uintptr_t x1 = ((uintptr_t)a.x + (uintptr_t)a.x_prefetch) & ~(uintptr_t)15;
+        if (x1 > x0) {
+            const uintptr_t per = (((x1 - x0) + gridDim.x - 1) / gridDim.x + 15) & ~(uintptr_t)15;
+            const uintptr_t b0 = x0 + per * blockIdx.x;
+            const uintptr_t b1 = b0 + per < x1 ? b0 + per : x1;
+            constexpr uintptr_t CH = 8192;
+            for (uintptr_t p = b0 + CH * (threadIdx.x & 31); p < b1; p += CH * 32) {
+                const uint32_t sz = (uint32_t)(b1 - p < CH ? b1 - p : CH);
+                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(sz) : "memory");
+            }
+        }
+    }
     pdl_enter();
     if (PR && a.ctrl && *(volatile int32_t *)a.ctrl) return;  // converged earlier: no-op step
     unsigned long long pc = 0;  // peer exchange: pushes completed before this step
@@ -1078,6 +1097,18 @@ static int xcache_bits()
     return v;
 }
 
+// x is bulk-prefetched into L2 at SpMV entry when it is at most this large (a quarter of
+// the ~126 MB L2); ACSR_XPREFETCH=0 switches it off (A/B)
+static int64_t x_prefetch_bytes(int64_t bytes)
+{
+    static int on = -1;
+    if (on < 0) {
+        const char *e = getenv("ACSR_XPREFETCH");
+        on = (e && e[0] == '0') ? 0 : 1;
+    }
+    return (on && bytes <= ((int64_t)32 << 20)) ? bytes : 0;
+}
+
 template <typename V, bool PR>
 static int dispatch(SpmvArgs<V> a, cudaStream_t s)
 {
@@ -1143,12 +1174,14 @@ extern "C" acsr_status acsr_spmv(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
         a.rb = row_begin; a.re = row_end; a.col = col_idx;
         a.val = (const double *)values; a.x = n_cols > 0 ? (const double *)x : nullptr; a.y = (double *)y;
         a.bin_rows = bin_rows; a.hdr = (PlanHeader *)plan_ws;
+        a.x_prefetch = a.x ? x_prefetch_bytes(n_cols * (int64_t)sizeof(double)) : 0;
         dispatch<double, false>(a, stream);
     } else {
         SpmvArgs<float> a{};
         a.rb = row_begin; a.re = row_end; a.col = col_idx;
         a.val = (const float *)values; a.x = n_cols > 0 ? (const float *)x : nullptr; a.y = (float *)y;
         a.bin_rows = bin_rows; a.hdr = (PlanHeader *)plan_ws;
+        a.x_prefetch = a.x ? x_prefetch_bytes(n_cols * (int64_t)sizeof(float)) : 0;
         dispatch<float, false>(a, stream);
     }
     return acsr_check_launch("acsr_spmv");
@@ -1177,6 +1210,7 @@ extern "C" acsr_status acsr_pagerank_step(const acsr_pr_args *p, cudaStream_t st
     a.damping = p->damping; a.teleport = p->teleport; a.delta2 = p->delta2;
     a.restart = p->restart; a.restart_weight = p->restart_weight;
     a.ctrl = p->ctrl; a.eps2 = p->eps2;
+    a.x_prefetch = a.x ? x_prefetch_bytes(p->n_cols * (int64_t)sizeof(double)) : 0;
     dispatch<double, true>(a, stream);
     return acsr_check_launch("acsr_pagerank_step");
 }

@@ -184,6 +184,21 @@ def make_workload(name, dev, rank):
     return label, dtype, rp, ci, val, x
 
 
+def bin_stats(rp, bin_offsets, heavy_chunk=1024):
+    """The B200 analogue of the paper's Table V: rows per bin
+    (from acsr_bin's bin_offsets), non-empty bins, rows split across warps (> 1024 nnz)
+    and their chunks."""
+    off = bin_offsets.cpu().numpy().astype(np.int64)
+    cnt = np.diff(off)
+    ln = (rp[1:] - rp[:-1]).to(torch.int64)
+    heavy = ln[ln > heavy_chunk]
+    return {"rows_per_bin": {int(b): int(c) for b, c in enumerate(cnt) if c},
+            "nonempty_bins": int((cnt[1:] > 0).sum()),
+            "split_rows": int(heavy.numel()),
+            "split_chunks": int(((heavy + heavy_chunk - 1) // heavy_chunk).sum()) if heavy.numel() else 0,
+            "split_nnz_share": round(float(heavy.sum()) / max(1, int(ln.sum())), 4)}
+
+
 def read_stream_gbs(dev, gib=2, reps=5):
     """Read-only streaming bandwidth measured in the same job (quote the
     roofline against the spec, the measured copy and a read-only stream): a 2 GiB fp32
@@ -329,6 +344,7 @@ def run_acsr(args, dev, rank, world):
     d2h = y_h.numel() * y_h.element_size()
     ctx = cusparse_context(rp, ci, val, x, n)
     rs = read_stream_gbs(dev)
+    bstats = bin_stats(rp, bo)
     if rank != 0:
         return None
     peak, peak_kind = peaks()
@@ -354,6 +370,7 @@ def run_acsr(args, dev, rank, world):
                       "gather_roofline_note": "pure random 8-byte gathers from an L2-resident x run at ~197 G/s "
                                               "on this B200 (profiles/r1_gather_bench.jsonl); one gather per nnz"},
         "context": ctx,
+        "bins": bstats,
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": ncu_traffic(label),
                      "kernel": "acsr::spmv_kernel", "peak_kind": peak_kind,

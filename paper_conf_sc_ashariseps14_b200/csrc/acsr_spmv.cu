@@ -1017,6 +1017,27 @@ static size_t spmv_smem(int bits)
     return (XC ? (sizeof(V) + sizeof(uint16_t)) * ((size_t)1 << bits) : 0) + (size_t)reserve;
 }
 
+// ACSR_X_PERSIST_MB=m (experiment, default off): an L2 access-policy window marks the
+// first m MB of x persisting for every SpMV / PageRank launch (the persisting L2 set-aside
+// is sized once, capped by the device maximum)
+static int64_t x_persist_bytes()
+{
+    static int64_t v = -1;
+    if (v < 0) {
+        const char *e = getenv("ACSR_X_PERSIST_MB");
+        v = (e && e[0]) ? (int64_t)atoll(e) << 20 : 0;
+        if (v > 0) {
+            int dev = 0, mx = 0, mw = 0;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, dev);
+            cudaDeviceGetAttribute(&mw, cudaDevAttrMaxAccessPolicyWindowSize, dev);
+            if (v > mw) v = mw;
+            cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)(v < mx ? v : mx));
+        }
+    }
+    return v;
+}
+
 template <typename V, bool HAS_VAL, bool HAS_END, bool PR, bool XC, bool PEER = false>
 static void launch(const SpmvArgs<V> &a, cudaStream_t s)
 {
@@ -1032,6 +1053,29 @@ static void launch(const SpmvArgs<V> &a, cudaStream_t s)
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmv_kernel<V, HAS_VAL, HAS_END, PR, XC, PEER>,
                                                       SPMV_THREADS, smem);
         if (per_sm < 1) per_sm = 1;
+    }
+    const int64_t persist = x_persist_bytes();
+    if (persist > 0 && a.x) {
+        // opt-in experiment: keep the first `persist` bytes of x persisting in L2 for this
+        // launch (with a hot-first vertex order these hold most gathers)
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = per_sm * acsr_num_sms();
+        cfg.blockDim = SPMV_THREADS;
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = s;
+        cudaLaunchAttribute at[2];
+        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[0].val.programmaticStreamSerializationAllowed = acsr_pdl_enabled() ? 1 : 0;
+        at[1].id = cudaLaunchAttributeAccessPolicyWindow;
+        at[1].val.accessPolicyWindow.base_ptr = (void *)a.x;
+        at[1].val.accessPolicyWindow.num_bytes = (size_t)persist;
+        at[1].val.accessPolicyWindow.hitRatio = 1.0f;
+        at[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        at[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.attrs = at;
+        cfg.numAttrs = 2;
+        cudaLaunchKernelEx(&cfg, spmv_kernel<V, HAS_VAL, HAS_END, PR, XC, PEER>, a);
+        return;
     }
     launch_pdl(spmv_kernel<V, HAS_VAL, HAS_END, PR, XC, PEER>, per_sm * acsr_num_sms(), SPMV_THREADS, smem, s, a);
 }

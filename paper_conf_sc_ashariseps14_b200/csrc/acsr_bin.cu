@@ -209,14 +209,16 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
 {
     constexpr int NW = BIN_THREADS / 32;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int overflow = hdr->overflow;
-    const int n_heavy = hdr->n_heavy_units;
+    // (L2 loads: in the fused scan+scatter launch these were written by other CTAs of the
+    // same grid)
+    const int overflow = __ldcg(&hdr->overflow);
+    const int n_heavy = __ldcg(&hdr->n_heavy_units);
     if (tid < NBINS) {
         sm.run[tid] = 0;
-        sm.seg[tid] = bin_offsets[tid] + toff[(int64_t)tid * n_tiles + tile];
+        sm.seg[tid] = __ldcg(bin_offsets + tid) + __ldcg(toff + (int64_t)tid * n_tiles + tile);
     }
     for (int i = tid; i < NW * NBINS; i += BIN_THREADS) (&sm.wcnt[0][0])[i] = 0;
-    if (tid == 0) sm.heavy_run = toff[(int64_t)(NBINS + 1) * n_tiles + tile];
+    if (tid == 0) sm.heavy_run = __ldcg(toff + (int64_t)(NBINS + 1) * n_tiles + tile);
     __syncthreads();
     const int64_t base = (int64_t)tile * TILE_ROWS;
     const unsigned lt = (1u << lane) - 1u;
@@ -291,7 +293,7 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
             sm.upre[LIGHT_MAX_BIN + 1] = acc;
         }
         __syncthreads();
-        const int ubase = n_heavy + toff[(int64_t)NBINS * n_tiles + tile];
+        const int ubase = n_heavy + __ldcg(toff + (int64_t)NBINS * n_tiles + tile);
         const int total = sm.upre[LIGHT_MAX_BIN + 1];
         for (int j = tid; j < total; j += BIN_THREADS) {
             if (j < nwin) {
@@ -318,7 +320,11 @@ bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__res
 {
     __shared__ BinSmem sm;
     pdl_enter();
-    if (blockIdx.x == 0 && threadIdx.x == 0) hdr->scan_ticket = 0;  // bin_scan runs after us
+    if (blockIdx.x == 0 && threadIdx.x == 0) {  // the scan (or fused scan+scatter) launch runs after us
+        hdr->scan_ticket = 0;
+        hdr->role_ticket = 0;
+        hdr->scan_done = 0;
+    }
     count_tile<HAS_END>(sm, n, rb, re, cnt, n_tiles, blockIdx.x, wmb);
 }
 
@@ -344,6 +350,50 @@ bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__r
     pdl_enter();
     scatter_tile<HAS_END>(sm, n, rb, re, bin_rows, bin_offsets, toff, n_tiles, hdr, units, tickets, heavy_cap,
                           blockIdx.x, wmb);
+}
+
+// ---- scan + scatter in ONE launch (opt-in, ACSR_BIN_SS=1): the first SCAN_ROWS CTAs to start (an
+// atomic role ticket, reset by bin_count) scan one row each -- the last of them writes
+// bin_offsets and the plan header -- and count themselves done; every other CTA takes a
+// tile, prefetches the tile's row offsets into L2, waits until all scan rows are done and
+// scatters.  The scanning CTAs are already running when anyone waits (they took the
+// first tickets), so the wait cannot deadlock.  Saves the scan kernel's launch boundary
+// but measured slower (see scan_scatter_fused).
+template <bool HAS_END>
+__global__ void __launch_bounds__(BIN_THREADS)
+bin_scan_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
+                        const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int32_t *__restrict__ bin_rows,
+                        int n_tiles, PlanHeader *hdr, ScanArgs sa, int2 *__restrict__ units,
+                        int32_t *__restrict__ tickets, int wmb)
+{
+    __shared__ BinSmem sm;
+    __shared__ int s_role;
+    pdl_enter();
+    if (threadIdx.x == 0) s_role = atomicAdd(&hdr->role_ticket, 1);
+    __syncthreads();
+    const int role = s_role;
+    if (role < SCAN_ROWS) {
+        scan_row<BIN_THREADS, 8>(sm, cnt, toff, n_tiles, hdr, sa, role);
+        if (threadIdx.x == 0) {
+            __threadfence();
+            atomicAdd(&hdr->scan_done, 1);
+        }
+        return;
+    }
+    const int tile = role - SCAN_ROWS;
+    {
+        const int64_t base = (int64_t)tile * TILE_ROWS;
+        const int64_t rows = min((int64_t)TILE_ROWS + 1, n + 1 - base);
+        const int64_t off = (int64_t)threadIdx.x * 32;  // 128-byte lines of the tile's offsets
+        if (off < rows) asm volatile("prefetch.global.L2 [%0];" ::"l"(rb + base + off));
+        if (HAS_END && off < rows - 1) asm volatile("prefetch.global.L2 [%0];" ::"l"(re + base + off));
+    }
+    if (threadIdx.x == 0)
+        while (*(volatile int32_t *)&hdr->scan_done < SCAN_ROWS) __nanosleep(64);
+    __syncthreads();
+    __threadfence();
+    scatter_tile<HAS_END>(sm, n, rb, re, bin_rows, sa.bin_offsets, toff, n_tiles, hdr, units, tickets, sa.heavy_cap,
+                          tile, wmb);
 }
 
 // ---- one cooperative launch: count -> grid barrier -> scan -> grid barrier -> scatter
@@ -404,6 +454,20 @@ static bool fused_enabled()
     static int v = -1;
     if (v < 0) {
         const char *e = getenv("ACSR_BIN_FUSED");
+        v = (e && e[0] == '1') ? 1 : 0;
+    }
+    return v == 1;
+}
+
+// ACSR_BIN_SS=1 selects the fused scan+scatter launch.  Measured slower on B200 (C2 bin
+// 27.6 vs 25.6 us, LiveJournal-like 93 vs 52 us, s26 1.30 vs 0.64 ms: the 34 scan rows on
+// 256-thread CTAs serialise in front of every waiting scatter CTA), so the separate scan
+// kernel is the default.
+static bool scan_scatter_fused()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("ACSR_BIN_SS");
         v = (e && e[0] == '1') ? 1 : 0;
     }
     return v == 1;
@@ -490,6 +554,15 @@ extern "C" acsr_status acsr_bin_ex(int64_t n_rows, int64_t n_cols, int64_t nnz_m
         else
             launch_pdl(bin_count_kernel<false>, nt, BIN_THREADS, 0, stream, nr, rb, re, cnt, nt, hdr, wmb);
         const int32_t *ccnt = cnt;
+        if (scan_scatter_fused()) {
+            if (row_end)
+                launch_pdl(bin_scan_scatter_kernel<true>, nt + SCAN_ROWS, BIN_THREADS, 0, stream, nr, rb, re, ccnt,
+                           toff, bin_rows, nt, hdr, sa, units, tickets, wmb);
+            else
+                launch_pdl(bin_scan_scatter_kernel<false>, nt + SCAN_ROWS, BIN_THREADS, 0, stream, nr, rb, re, ccnt,
+                           toff, bin_rows, nt, hdr, sa, units, tickets, wmb);
+            goto xc;
+        }
         launch_pdl(bin_scan_kernel, SCAN_ROWS, SCAN_THREADS, 0, stream, ccnt, toff, nt, hdr, sa);
         if (row_end)
             launch_pdl(bin_scatter_kernel<true>, nt, BIN_THREADS, 0, stream, nr, rb, re, bin_rows, cbo, ctoff, nt, chdr,

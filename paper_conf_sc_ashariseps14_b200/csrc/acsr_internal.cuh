@@ -138,6 +138,8 @@ struct PlanHeader {
     int32_t n_light_units;
     int32_t n_units;
     int32_t scan_ticket;    // last-CTA detection in the scan kernel
+    int32_t role_ticket;    // fused scan+scatter launch: CTA role order (reset by bin_count)
+    int32_t scan_done;      // fused scan+scatter launch: scan rows finished (reset by bin_count)
     int32_t work_ctr;       // dynamic unit counter (reset by the last warp)
     int32_t exit_ticket;    // last-warp detection at SpMV exit
     int32_t overflow;       // 1 if the unit list exceeded the workspace bounds

@@ -546,6 +546,32 @@ def test_spmv_unaligned_views(acsr, cuda, shift_c, shift_v):
     check_spmv(y, y_ref, den, torch.float64)
 
 
+@pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
+@pytest.mark.parametrize("shift_x", [0, 1, 3])
+def test_spmv_x_prefetch_views(acsr, cuda, dtype, shift_x):
+    # x given as an offset view (the L2 bulk prefetch of x is clipped inward to 16-byte
+    # bounds) and with the prefetch disabled by size (x of one column): results are the
+    # same bits as with an aligned x (bitwise on integer data)
+    rp, ci = synth.rmat_csr(13)
+    n = rp.numel() - 1
+    val = synth.values(ci.numel(), 31, dtype, integer=True)
+    x = synth.vector(n, 32, dtype, integer=True)
+    xbuf = torch.zeros(n + 4, dtype=dtype, device=cuda)
+    xv = xbuf[shift_x:shift_x + n]
+    xv.copy_(x.to(cuda))
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda), val.to(cuda))
+    y = m.spmv(xv).cpu().numpy()
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y, y_ref, den, dtype, exact=True)
+    # one column: every row sums val * x[0]
+    rp1 = torch.tensor([0, 3, 3, 5], dtype=torch.int32)
+    ci1 = torch.zeros(5, dtype=torch.int32)
+    v1 = torch.tensor([1, -2, 4, 3, 5], dtype=dtype)
+    x1 = torch.tensor([2], dtype=dtype)
+    m1 = acsr.ACSRMatrix(rp1.to(cuda), ci1.to(cuda), v1.to(cuda), n_cols=1)
+    assert m1.spmv(x1.to(cuda)).cpu().tolist() == [6.0, 0.0, 16.0]
+
+
 def test_dist_pagerank_single_rank_cuda(acsr, cuda):
     # the partitioned driver (dist.py) on one rank runs the same fused CUDA step: it must
     # reproduce the single-GPU loop bitwise and the oracle within the converged bar

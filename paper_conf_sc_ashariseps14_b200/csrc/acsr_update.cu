@@ -10,6 +10,7 @@
 // the result is exact and independent of scheduling.
 #include <cuda_runtime.h>
 #include <stddef.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include "acsr_internal.cuh"
@@ -28,6 +29,35 @@ struct UpdWs {
     unsigned int pad;
     int32_t long_list[1];    // [n_upd]
 };
+
+// hub rows: the delete list is staged in shared memory when it has at most del_cap entries
+// (dynamic shared memory, up to DEL_SMEM_MAX ints = 192 KB) and binary-searched there
+constexpr int DEL_SMEM_MAX = 48 * 1024;
+
+__device__ __forceinline__ bool member_s(const int32_t *d, int m, int c)
+{
+    int l = 0, h = m;
+    while (l < h) {
+        int mid = (l + h) >> 1;
+        if (d[mid] < c) l = mid + 1;
+        else h = mid;
+    }
+    return l < m && d[l] == c;
+}
+
+// short delete lists (<= 32 entries): lane t holds entry t in a register and membership is
+// tested with m warp shuffles instead of a dependent binary search in global memory
+// (called by all 32 lanes with the same m)
+__device__ __forceinline__ bool member_w(int dreg, int m, int c)
+{
+    bool hit = false;
+    for (int j = 0; j < m; j++) hit |= __shfl_sync(0xffffffffu, dreg, j) == c;
+    return hit;
+}
+
+#ifndef ACSR_UPD_WARPREG
+#define ACSR_UPD_WARPREG 0  // 1: register/shuffle membership for <= 32 deletes (A/B: neutral on N2)
+#endif
 
 __device__ __forceinline__ bool member(const int32_t *__restrict__ d, int lo, int hi, int c)
 {
@@ -82,8 +112,17 @@ update_validate_kernel(int64_t n_rows, int64_t n_cols, const int32_t *__restrict
             return;
         }
         int dels = 0;
-        if (d1 > d0)
+        const int m = d1 - d0;
+        if (ACSR_UPD_WARPREG && m > 0 && m <= 32) {
+            const int dreg = lane < m ? __ldg(dcol + d0 + lane) : 0;
+            for (int k0 = b; k0 < e; k0 += 32) {  // warp-uniform trip count (shuffles)
+                const bool valid = k0 + lane < e;
+                const int c = valid ? __ldg(col + k0 + lane) : 0;
+                dels += (member_w(dreg, m, c) && valid) ? 1 : 0;
+            }
+        } else if (m > 0) {
             for (int k = b + lane; k < e; k += 32) dels += member(dcol, d0, d1, __ldg(col + k)) ? 1 : 0;
+        }
         for (int o = 16; o > 0; o >>= 1) dels += __shfl_xor_sync(0xffffffffu, dels, o);
         long long new_len = (long long)(e - b) - dels + (i1 - i0);
         if (new_len > __ldg(cap + r)) code = ACSR_ERR_CAPACITY;
@@ -123,18 +162,29 @@ __global__ void __launch_bounds__(UPD_THREADS)
 update_validate_long_kernel(const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
                             const int32_t *__restrict__ cap, const int32_t *__restrict__ col,
                             const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
-                            const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr, UpdWs *ws)
+                            const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr, UpdWs *ws,
+                            int del_cap)
 {
     pdl_enter();
     __shared__ int sh[33];
+    extern __shared__ int32_t sdel[];
     const unsigned n_long = *(volatile unsigned *)&ws->n_long;
     for (unsigned j = blockIdx.x; j < n_long; j += gridDim.x) {
         const int i = ws->long_list[j];
         const int r = __ldg(upd + i);
         const int b = __ldg(rb + r), e = __ldg(re + r);
         const int d0 = __ldg(dptr + i), d1 = __ldg(dptr + i + 1);
+        const int m = d1 - d0;
+        const bool use_s = m <= del_cap;
+        if (use_s) {
+            for (int t = threadIdx.x; t < m; t += UPD_THREADS) sdel[t] = __ldg(dcol + d0 + t);
+            __syncthreads();
+        }
         int dels = 0;
-        for (int k = b + threadIdx.x; k < e; k += UPD_THREADS) dels += member(dcol, d0, d1, __ldg(col + k)) ? 1 : 0;
+        for (int k = b + threadIdx.x; k < e; k += UPD_THREADS) {
+            const int c = __ldg(col + k);
+            dels += (use_s ? member_s(sdel, m, c) : member(dcol, d0, d1, c)) ? 1 : 0;
+        }
         int total;
         block_exclusive_scan(dels, total, sh);
         const long long new_len = (long long)(e - b) - total + (__ldg(iptr + i + 1) - __ldg(iptr + i));
@@ -152,10 +202,11 @@ update_apply_long_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ r
                          T *__restrict__ val, const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
                          const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
                          const int32_t *__restrict__ icol, const T *__restrict__ ival, T one,
-                         int32_t *__restrict__ outdeg, UpdWs *ws)
+                         int32_t *__restrict__ outdeg, UpdWs *ws, int del_cap)
 {
     pdl_enter();
     __shared__ int sh[33];
+    extern __shared__ int32_t sdel[];
     if (*(volatile unsigned long long *)&ws->key != NO_FAIL) return;
     const unsigned n_long = *(volatile unsigned *)&ws->n_long;
     constexpr int E = 4;
@@ -164,6 +215,12 @@ update_apply_long_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ r
         const int r = __ldg(upd + i);
         const int b = __ldg(rb + r), e = re[r];
         const int d0 = __ldg(dptr + i), d1 = __ldg(dptr + i + 1);
+        const int m = d1 - d0;
+        const bool use_s = m <= del_cap;
+        if (use_s) {
+            for (int t = threadIdx.x; t < m; t += UPD_THREADS) sdel[t] = __ldg(dcol + d0 + t);
+            __syncthreads();
+        }
         int w = b;
         for (int k0 = b; k0 < e; k0 += E * UPD_THREADS) {
             int c[E];
@@ -176,7 +233,7 @@ update_apply_long_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ r
                 const bool valid = kk < e;
                 c[q] = valid ? col[kk] : 0;
                 v[q] = (val && valid) ? val[kk] : T();
-                del[q] = valid && member(dcol, d0, d1, c[q]);
+                del[q] = valid && (use_s ? member_s(sdel, m, c[q]) : member(dcol, d0, d1, c[q]));
                 keep[q] = valid && !del[q];
                 cnt += keep[q] ? 1 : 0;
             }
@@ -233,13 +290,17 @@ update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
     if (d1 > d0 && e - b > LONG_ROW) return;  // update_apply_long_kernel
     if (d1 > d0) {
         w = b;
+        const int m = d1 - d0;
+        const bool wr = ACSR_UPD_WARPREG && m <= 32;
+        const int dreg = (wr && lane < m) ? __ldg(dcol + d0 + lane) : 0;
         for (int k0 = b; k0 < e; k0 += 32) {
             int kk = k0 + lane;
             bool valid = kk < e;
             int c = valid ? col[kk] : 0;
             T v = T();
             if (val && valid) v = val[kk];
-            bool del = valid && member(dcol, d0, d1, c);
+            const bool hw = wr ? member_w(dreg, m, c) : false;  // every lane shuffles (wr is warp-uniform)
+            bool del = valid && (wr ? hw : member(dcol, d0, d1, c));
             bool keep = valid && !del;
             unsigned m = __ballot_sync(0xffffffffu, keep);
             __syncwarp();  // every lane has read its source before anyone writes
@@ -345,6 +406,23 @@ extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t 
     UpdWs *uw = (UpdWs *)ws;
     launch_pdl(update_init_kernel, 1, 1, 0, stream, uw);
     const int long_grid = 4 * acsr_num_sms();
+    // hub-row delete lists in shared memory (ACSR_UPD_SMEM=0: global binary search, A/B)
+    static int del_cap = -1;
+    if (del_cap < 0) {
+        const char *e = getenv("ACSR_UPD_SMEM");
+        del_cap = (e && e[0] == '0') ? 0 : DEL_SMEM_MAX;
+        if (del_cap) {
+            const int bytes = (int)(sizeof(int32_t) * DEL_SMEM_MAX);
+            if (cudaFuncSetAttribute(update_validate_long_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess ||
+                cudaFuncSetAttribute(update_apply_long_kernel<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess ||
+                cudaFuncSetAttribute(update_apply_long_kernel<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess) {
+                cudaGetLastError();
+                del_cap = 0;
+            }
+        }
+    }
+    const size_t long_smem = sizeof(int32_t) * (size_t)del_cap;
+    const int lgrid = del_cap ? acsr_num_sms() : long_grid;  // one 192 KB CTA per SM
     const int wpb = UPD_THREADS / 32;
     const int64_t blocks64 = n_upd > 0 ? (n_upd + wpb - 1) / wpb : 1;
     if (blocks64 > 0x7fffffff) return ACSR_ERR_INVALID_VALUE;
@@ -355,9 +433,8 @@ extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t 
                                                                    del_ptr, del_cols, ins_ptr, ins_cols,
                                                                    uw);
     if (n_upd > 0 && del_ptr)
-        launch_pdl(update_validate_long_kernel, long_grid, UPD_THREADS, 0, stream, row_begin, row_end, row_cap, col_idx,
-                                                                          upd_rows, del_ptr, del_cols, ins_ptr,
-                                                                          uw);
+        launch_pdl(update_validate_long_kernel, lgrid, UPD_THREADS, long_smem, stream, row_begin, row_end, row_cap,
+                   col_idx, upd_rows, del_ptr, del_cols, ins_ptr, uw, del_cap);
     if (dt == ACSR_F64) {
         uint64_t one;
         double d1 = 1.0;
@@ -366,9 +443,9 @@ extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t 
             row_begin, row_end, col_idx, (uint64_t *)values, n_upd, upd_rows, del_ptr, del_cols, ins_ptr,
             ins_cols, (const uint64_t *)ins_vals, one, outdeg, uw, status);
         if (n_upd > 0 && del_ptr)
-            launch_pdl(update_apply_long_kernel<uint64_t>, long_grid, UPD_THREADS, 0, stream, 
+            launch_pdl(update_apply_long_kernel<uint64_t>, lgrid, UPD_THREADS, long_smem, stream,
                 row_begin, row_end, col_idx, (uint64_t *)values, upd_rows, del_ptr, del_cols, ins_ptr, ins_cols,
-                (const uint64_t *)ins_vals, one, outdeg, uw);
+                (const uint64_t *)ins_vals, one, outdeg, uw, del_cap);
     } else {
         uint32_t one;
         float f1 = 1.0f;
@@ -377,9 +454,9 @@ extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t 
             row_begin, row_end, col_idx, (uint32_t *)values, n_upd, upd_rows, del_ptr, del_cols, ins_ptr,
             ins_cols, (const uint32_t *)ins_vals, one, outdeg, uw, status);
         if (n_upd > 0 && del_ptr)
-            launch_pdl(update_apply_long_kernel<uint32_t>, long_grid, UPD_THREADS, 0, stream, 
+            launch_pdl(update_apply_long_kernel<uint32_t>, lgrid, UPD_THREADS, long_smem, stream,
                 row_begin, row_end, col_idx, (uint32_t *)values, upd_rows, del_ptr, del_cols, ins_ptr, ins_cols,
-                (const uint32_t *)ins_vals, one, outdeg, uw);
+                (const uint32_t *)ins_vals, one, outdeg, uw, del_cap);
     }
     return acsr_check_launch("acsr_update_edges");
 }

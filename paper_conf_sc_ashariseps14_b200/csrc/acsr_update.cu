@@ -70,19 +70,15 @@ __device__ __forceinline__ bool member(const int32_t *__restrict__ d, int lo, in
     return l < hi && __ldg(d + l) == c;
 }
 
-__global__ void __launch_bounds__(UPD_THREADS)
-update_validate_kernel(int64_t n_rows, int64_t n_cols, const int32_t *__restrict__ rb,
-                       const int32_t *__restrict__ re, const int32_t *__restrict__ cap,
-                       const int32_t *__restrict__ col, int64_t n_upd,
-                       const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
-                       const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
-                       const int32_t *__restrict__ icol, UpdWs *ws)
+// validation of update i by one full warp (called warp-uniformly)
+__device__ __forceinline__ void validate_row(int64_t i, int lane, int64_t n_rows, int64_t n_cols,
+                                             const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
+                                             const int32_t *__restrict__ cap, const int32_t *__restrict__ col,
+                                             const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
+                                             const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
+                                             const int32_t *__restrict__ icol, UpdWs *ws)
 {
-    pdl_enter();
     unsigned long long *key = &ws->key;
-    const int lane = threadIdx.x & 31;
-    const int64_t i = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
-    if (i >= n_upd) return;
     int code = ACSR_OK;
     const int r = __ldg(upd + i);
     if (r < 0 || r >= n_rows || (i > 0 && r <= __ldg(upd + i - 1))) code = ACSR_ERR_INVALID_VALUE;
@@ -128,6 +124,70 @@ update_validate_kernel(int64_t n_rows, int64_t n_cols, const int32_t *__restrict
         if (new_len > __ldg(cap + r)) code = ACSR_ERR_CAPACITY;
     }
     if (code != ACSR_OK && lane == 0) atomicMin(key, ((unsigned long long)i << 3) | (unsigned)code);
+}
+
+// Short rows, four per warp: an 8-lane sub-warp per update (SUB_W lanes, SUB_R = 32/SUB_W
+// updates per warp) when every row of the warp has at most SUB_MAX entries -- the
+// per-row chain of dependent loads (update -> row bounds -> columns -> delete-list
+// search) is latency-bound, so more rows in flight per warp is what pays.  Otherwise
+// the warp validates its rows one after another with validate_row.
+constexpr int SUB_W = 8, SUB_R = 32 / SUB_W, SUB_MAX = 64;
+#ifndef ACSR_UPD_SUB
+#define ACSR_UPD_SUB 0  // 1: 8-lane sub-warps for short rows (A/B: N2 update 0.36 -> 0.45 ms, slower)
+#endif
+
+__global__ void __launch_bounds__(UPD_THREADS)
+update_validate_kernel(int64_t n_rows, int64_t n_cols, const int32_t *__restrict__ rb,
+                       const int32_t *__restrict__ re, const int32_t *__restrict__ cap,
+                       const int32_t *__restrict__ col, int64_t n_upd,
+                       const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
+                       const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
+                       const int32_t *__restrict__ icol, UpdWs *ws)
+{
+    pdl_enter();
+    const int lane = threadIdx.x & 31;
+    const int64_t wid = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
+    if (!ACSR_UPD_SUB) {
+        if (wid < n_upd) validate_row(wid, lane, n_rows, n_cols, rb, re, cap, col, upd, dptr, dcol, iptr, icol, ws);
+        return;
+    }
+    const int64_t ibase = wid * SUB_R;
+    if (ibase >= n_upd) return;
+    const int s = lane / SUB_W, li = lane % SUB_W;
+    const unsigned smask = 0xFFu << (s * SUB_W);
+    const int64_t i = ibase + s;
+    const bool has = i < n_upd;
+    int r = has ? __ldg(upd + i) : 0;
+    const bool rok = has && r >= 0 && r < n_rows;
+    const int b = rok ? __ldg(rb + r) : 0, e = rok ? __ldg(re + r) : 0;
+    const unsigned long_any = __ballot_sync(0xffffffffu, rok && e - b > SUB_MAX);
+    if (long_any) {  // a longer row in this warp: full-warp validation, row by row
+        for (int q = 0; q < SUB_R; q++)
+            if (ibase + q < n_upd)
+                validate_row(ibase + q, lane, n_rows, n_cols, rb, re, cap, col, upd, dptr, dcol, iptr, icol, ws);
+        return;
+    }
+    int code = ACSR_OK;
+    if (has && (!rok || (i > 0 && r <= __ldg(upd + i - 1)))) code = ACSR_ERR_INVALID_VALUE;
+    const int d0 = (has && dptr) ? __ldg(dptr + i) : 0, d1 = (has && dptr) ? __ldg(dptr + i + 1) : 0;
+    const int i0 = has ? __ldg(iptr + i) : 0, i1 = has ? __ldg(iptr + i + 1) : 0;
+    bool bad = false;
+    for (int j = d0 + 1 + li; j < d1; j += SUB_W) bad |= __ldg(dcol + j) < __ldg(dcol + j - 1);
+    for (int j = i0 + li; j < i1; j += SUB_W) {
+        const int c = __ldg(icol + j);
+        bad |= (c < 0 || c >= n_cols);
+    }
+    if (__ballot_sync(0xffffffffu, bad) & smask) code = code ? code : ACSR_ERR_INVALID_VALUE;
+    int dels = 0;
+    if (code == ACSR_OK && d1 > d0)
+        for (int k = b + li; k < e; k += SUB_W) dels += member(dcol, d0, d1, __ldg(col + k)) ? 1 : 0;
+#pragma unroll
+    for (int o = SUB_W / 2; o > 0; o >>= 1) dels += __shfl_xor_sync(0xffffffffu, dels, o, SUB_W);
+    if (code == ACSR_OK && has) {
+        const long long new_len = (long long)(e - b) - dels + (i1 - i0);
+        if (new_len > __ldg(cap + r)) code = ACSR_ERR_CAPACITY;
+    }
+    if (has && code != ACSR_OK && li == 0) atomicMin(&ws->key, ((unsigned long long)i << 3) | (unsigned)code);
 }
 
 __device__ __forceinline__ int block_exclusive_scan(int v, int &total, int *sh)
@@ -263,26 +323,16 @@ update_apply_long_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ r
     }
 }
 
+// compaction + append of update i by one full warp (called warp-uniformly)
 template <typename T>
-__global__ void __launch_bounds__(UPD_THREADS)
-update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
-                    int32_t *__restrict__ col, T *__restrict__ val, int64_t n_upd,
-                    const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
-                    const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
-                    const int32_t *__restrict__ icol, const T *__restrict__ ival, T one,
-                    int32_t *__restrict__ outdeg, const UpdWs *ws, int32_t *__restrict__ status)
+__device__ __forceinline__ void apply_row(int64_t i, int lane, const int32_t *__restrict__ rb,
+                                          int32_t *__restrict__ re, int32_t *__restrict__ col,
+                                          T *__restrict__ val, const int32_t *__restrict__ upd,
+                                          const int32_t *__restrict__ dptr, const int32_t *__restrict__ dcol,
+                                          const int32_t *__restrict__ iptr, const int32_t *__restrict__ icol,
+                                          const T *__restrict__ ival, T one, int32_t *__restrict__ outdeg)
 {
-    pdl_enter();
-    const unsigned long long k = *(volatile const unsigned long long *)&ws->key;
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        status[0] = k == NO_FAIL ? ACSR_OK : (int32_t)(k & 7);
-        status[1] = k == NO_FAIL ? -1 : (int32_t)(k >> 3);
-    }
-    if (k != NO_FAIL) return;  // all-or-nothing
-    const int lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
-    const int64_t i = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
-    if (i >= n_upd) return;
     const int r = __ldg(upd + i);
     const int b = __ldg(rb + r), e = re[r];
     int w = e;
@@ -322,6 +372,82 @@ update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
         if (outdeg) atomicAdd(outdeg + c, 1);
     }
     if (lane == 0) re[r] = w + (i1 - i0);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(UPD_THREADS)
+update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
+                    int32_t *__restrict__ col, T *__restrict__ val, int64_t n_upd,
+                    const int32_t *__restrict__ upd, const int32_t *__restrict__ dptr,
+                    const int32_t *__restrict__ dcol, const int32_t *__restrict__ iptr,
+                    const int32_t *__restrict__ icol, const T *__restrict__ ival, T one,
+                    int32_t *__restrict__ outdeg, const UpdWs *ws, int32_t *__restrict__ status)
+{
+    pdl_enter();
+    const unsigned long long k = *(volatile const unsigned long long *)&ws->key;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        status[0] = k == NO_FAIL ? ACSR_OK : (int32_t)(k & 7);
+        status[1] = k == NO_FAIL ? -1 : (int32_t)(k >> 3);
+    }
+    if (k != NO_FAIL) return;  // all-or-nothing
+    const int lane = threadIdx.x & 31;
+    const int64_t wid = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
+    if (!ACSR_UPD_SUB) {
+        if (wid < n_upd) apply_row<T>(wid, lane, rb, re, col, val, upd, dptr, dcol, iptr, icol, ival, one, outdeg);
+        return;
+    }
+    const int64_t ibase = wid * SUB_R;
+    if (ibase >= n_upd) return;
+    const int s = lane / SUB_W, li = lane % SUB_W;
+    const int64_t i = ibase + s;
+    const bool has = i < n_upd;
+    const int r = has ? __ldg(upd + i) : 0;
+    const int b = has ? __ldg(rb + r) : 0, e = has ? re[r] : 0;
+    if (__ballot_sync(0xffffffffu, has && e - b > SUB_MAX)) {  // the same decision as validation
+        for (int q = 0; q < SUB_R; q++)
+            if (ibase + q < n_upd)
+                apply_row<T>(ibase + q, lane, rb, re, col, val, upd, dptr, dcol, iptr, icol, ival, one, outdeg);
+        return;
+    }
+    const int d0 = (has && dptr) ? __ldg(dptr + i) : 0, d1 = (has && dptr) ? __ldg(dptr + i + 1) : 0;
+    int w = e;
+    if (__ballot_sync(0xffffffffu, d1 > d0)) {
+        // stable in-place compaction, SUB_W entries per round; the round count is the warp's
+        // maximum so the ballots are warp-uniform (rows <= SUB_MAX entries)
+        const int len = d1 > d0 ? e - b : 0;
+        const int lmax = __reduce_max_sync(0xffffffffu, (unsigned)len);
+        if (d1 > d0) w = b;
+        const unsigned lt = (1u << li) - 1u;
+        for (int t0 = 0; t0 < lmax; t0 += SUB_W) {
+            const bool valid = t0 + li < len;
+            const int kk = b + t0 + li;
+            const int c = valid ? col[kk] : 0;
+            T v = T();
+            if (val && valid) v = val[kk];
+            const bool del = valid && member(dcol, d0, d1, c);
+            const bool keep = valid && !del;
+            const unsigned m = (__ballot_sync(0xffffffffu, keep) >> (s * SUB_W)) & 0xFFu;
+            __syncwarp();  // every lane has read its source before anyone writes
+            if (keep) {
+                const int dst = w + __popc(m & lt);
+                col[dst] = c;
+                if (val) val[dst] = v;
+            }
+            if (del && outdeg) atomicSub(outdeg + c, 1);
+            w += __popc(m);
+            __syncwarp();
+        }
+    }
+    if (has) {
+        const int i0 = __ldg(iptr + i), i1 = __ldg(iptr + i + 1);
+        for (int j = i0 + li; j < i1; j += SUB_W) {
+            const int c = __ldg(icol + j);
+            col[w + (j - i0)] = c;
+            if (val) val[w + (j - i0)] = ival ? ival[j] : one;
+            if (outdeg) atomicAdd(outdeg + c, 1);
+        }
+        if (li == 0) re[r] = w + (i1 - i0);
+    }
 }
 
 // re-layout: copy row r from [ob[r], oe[r]) to [nb[r], nb[r] + len) (warp per row)
@@ -424,7 +550,8 @@ extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t 
     const size_t long_smem = sizeof(int32_t) * (size_t)del_cap;
     const int lgrid = del_cap ? acsr_num_sms() : long_grid;  // one 192 KB CTA per SM
     const int wpb = UPD_THREADS / 32;
-    const int64_t blocks64 = n_upd > 0 ? (n_upd + wpb - 1) / wpb : 1;
+    const int64_t upw = ACSR_UPD_SUB ? SUB_R : 1;  // updates per warp
+    const int64_t blocks64 = n_upd > 0 ? (n_upd + wpb * upw - 1) / (wpb * upw) : 1;
     if (blocks64 > 0x7fffffff) return ACSR_ERR_INVALID_VALUE;
     const int blocks = (int)blocks64;
     if (n_upd > 0)

@@ -230,9 +230,12 @@ acsr_status acsr_peer_destroy(acsr_peer *p);
 /* x, outdeg: [n] local rows (n >= slice_len); xs_local: NULL or [n] (also gets xs). */
 acsr_status acsr_peer_push(acsr_peer *p, int64_t n, const double *x, const int32_t *outdeg,
                            double *xs_local, cudaStream_t stream);
+/* args->n_rows >= 1 and >= slice_len (every rank owns at least one row); RWR fields
+ * (restart, restart_weight) work as in acsr_pagerank_step on the local rows. */
 acsr_status acsr_pagerank_step_peer(const acsr_pr_args *args, acsr_peer *p, cudaStream_t stream);
 /* delta2: [1] device out, the global sum of every rank's partial of the last push
- * (exact fixed-point partials: the same bits on every rank).  ctrl: NULL or [2] as in
+ * (exact fixed-point partials: the same bits on every rank; 0 if the last push was
+ * acsr_peer_push).  ctrl: NULL or [2] as in
  * acsr_pr_args -- ctrl[0] is set here when delta2 <= eps2 (every rank decides alike),
  * and a call with ctrl[0] set does nothing, so blocks of (step, delta2) pairs can be
  * enqueued between host synchronisations. */

@@ -345,6 +345,22 @@ def run_acsr(args, dev, rank, world):
     ctx = cusparse_context(rp, ci, val, x, n)
     rs = read_stream_gbs(dev)
     bstats = bin_stats(rp, bo)
+    # gather-only pass over the same column array, same L2 flush: x[col] with torch's
+    # index kernel (strictly less work than the SpMV: no values, no row sums) -- the
+    # in-job measure of the random-gather bound the SpMV sits against
+    g_out = torch.empty(nnz, dtype=dtype, device=dev)
+    tg = []
+    for k in range(max(5, min(K, 20))):
+        flush.zero_()
+        g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        g0.record(stream)
+        torch.index_select(x, 0, ci, out=g_out)  # int32 indices, as the SpMV reads them
+        g1.record(stream)
+        torch.cuda.synchronize()
+        if k >= 2:
+            tg.append(g0.elapsed_time(g1))
+    t_gather = float(np.median(tg))
+    del g_out
     if rank != 0:
         return None
     peak, peak_kind = peaks()
@@ -366,6 +382,10 @@ def run_acsr(args, dev, rank, world):
                       "t_spmv_median_ms": round(float(np.median(t_spmv)), 5),
                       "t_spmv_warm_back_to_back_ms": round(t_spmv_warm, 5),
                       "wall_s_timed_loop": round(wall, 4),
+                      "gather_pass_ms": round(t_gather, 5),
+                      "gather_pass_note": "torch.index_select(x, 0, col) over the same matrix, L2 flushed: "
+                                          "nnz random gathers + col read + nnz-value write, no row sums",
+                      "spmv_over_gather_pass": round(spmv_ms / t_gather, 3),
                       "gather_roofline_ms": round(nnz / 197e9 * 1e3, 5),
                       "gather_roofline_note": "pure random 8-byte gathers from an L2-resident x run at ~197 G/s "
                                               "on this B200 (profiles/r1_gather_bench.jsonl); one gather per nnz"},

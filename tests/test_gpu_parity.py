@@ -771,7 +771,7 @@ def test_spmv_from_host_e2e(acsr, cuda):
     check_spmv(y.numpy(), y_ref, den, torch.float64)
 
 
-def _two_ranks(scale, **kw):
+def _two_ranks(scale, world=2, **kw):
     import socket
     import sys
     import torch.multiprocessing as mp
@@ -783,8 +783,8 @@ def _two_ranks(scale, **kw):
     s.close()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_dist_gpu_worker.worker, args=(r, 2, port, scale, q), kwargs=kw)
-             for r in range(2)]
+    procs = [ctx.Process(target=_dist_gpu_worker.worker, args=(r, world, port, scale, q), kwargs=kw)
+             for r in range(world)]
     for p in procs:
         p.start()
     full, it, d2 = q.get(timeout=300)
@@ -855,6 +855,20 @@ def test_peer_exchange_two_ranks_one_gpu(cuda, compact):
     full_8, it_8, d2_8 = _two_ranks(14, exchange="peer", compact=compact, check_every=8)
     assert it_8 == it_p and d2_8 == d2_p and np.array_equal(full_8, full_p)
     rp, ci, od, n = _inlink(14, cuda)
+    x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)
+    assert abs(it_p - it_ref) <= 1
+    if it_p != it_ref:
+        x_ref, _, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=0.0, max_iter=it_p)
+    assert np.all(np.abs(full_p - x_ref) <= 1e-11 * x_ref + 1e-18)
+
+
+def test_peer_exchange_three_ranks_one_gpu(cuda):
+    # three ranks: every fused step stores its slice into two remote regions (the
+    # out-of-line remote loop with the self-skip); same bits as the collective path
+    full_p, it_p, _ = _two_ranks(13, world=3, exchange="peer", compact=True, check_every=4)
+    full_c, it_c, _ = _two_ranks(13, world=3, exchange="nccl", compact=True)
+    assert it_p == it_c and np.array_equal(full_p, full_c)
+    rp, ci, od, n = _inlink(13, cuda)
     x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)
     assert abs(it_p - it_ref) <= 1
     if it_p != it_ref:

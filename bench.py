@@ -716,15 +716,18 @@ def run_hits_rwr(args, dev, rank, world):
 
 
 # ------------------------------------------------------------------------------ dynamic graph (C5)
-def host_inclusive_batch(m, chd, outdeg, st, uws, x, xs_tmp, y):
-    """Wall time (ms) of update + re-bin + scale + SpMV issued from an idle GPU through
-    the Python API, on a scratch copy of the slack CSR (the live matrix is not touched)."""
+def host_inclusive_batch(m, pinned, outdeg, st, uws, x, xs_tmp, y):
+    """Wall time (ms) of the change-list H2D copies + update + re-bin + scale + SpMV issued
+    from an idle GPU through the Python API, on a scratch copy of the slack CSR (the live
+    matrix is not touched)."""
     import paper_conf_sc_ashariseps14_b200 as acsr
     mm = acsr.ACSRMatrix(m.row_begin, m.col_idx.clone(), None, row_end=m.row_end.clone(),
                          row_cap=m.row_cap, nnz_max=m.nnz_max)
     od = outdeg.clone()
+    dev = m.row_begin.device
     torch.cuda.synchronize()
     t0 = time.perf_counter()
+    chd = {kk: v.to(dev, non_blocking=True) for kk, v in pinned.items()}
     mm.update(chd, outdeg=od, status=st, ws=uws)
     mm.rebin()
     acsr.acsr_pagerank_scale(x, od, xs_tmp)
@@ -749,9 +752,11 @@ def run_dynamic(args, dev, rank, world):
     outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
     m = acsr.ACSRMatrix(rb, col, None, row_end=re, row_cap=cap, nnz_max=col.numel())
     x, it0, _ = acsr.pagerank(m, outdeg, eps=1e-6)
+    G = min(args.steps, 20)  # further batches replayed through one captured CUDA graph
     t_gen = time.perf_counter()
-    batches = [(ch, k) for ch, k in synth.insert_batches(S, B, 16384, keys, device=dev)]
+    all_batches = [(ch, k) for ch, k in synth.insert_batches(S, B + G, 16384, keys, device=dev)]
     t_gen = time.perf_counter() - t_gen
+    batches, gbatches = all_batches[:B], all_batches[B:]
     st = torch.empty(2, dtype=torch.int32, device=dev)
     uws = torch.empty(acsr.acsr_update_workspace_bytes(1 << 20), dtype=torch.uint8, device=dev)
     xs_tmp = torch.empty(n, dtype=torch.float64, device=dev)
@@ -788,13 +793,40 @@ def run_dynamic(args, dev, rank, world):
         relayouts += regrow
         # host-inclusive: the same update + re-bin + SpMV issued from an idle GPU (a
         # re-applied insert batch only appends duplicates, so time it on a scratch copy)
-        t_host = host_inclusive_batch(m, chd, outdeg, st, uws, x, xs_tmp, y) if b >= args.warmup else 0.0
+        t_host = host_inclusive_batch(m, pinned, outdeg, st, uws, x, xs_tmp, y) if b >= args.warmup else 0.0
         t0 = time.perf_counter()
         x, it, _ = acsr.pagerank(m, outdeg, x0=x, eps=1e-6)
         torch.cuda.synchronize()
         t_pr = time.perf_counter() - t0
         if b >= args.warmup:
             rec.append([ev[i].elapsed_time(ev[i + 1]) for i in range(4)] + [t_pr * 1e3, it, k, t_host])
+    # the same per-batch sequence (update -> re-bin -> scale -> SpMV) from ONE captured CUDA
+    # graph (acsr_update_edges_dev reads the batch size on the device), host-inclusive:
+    # sync -> pinned copies into the graph's capacity buffers + replay -> sync
+    x_g = x.clone()
+    cap_b = max(max(c["upd_rows"].size, c["ins_cols"].size) for c, _ in gbatches) if gbatches else 1
+    ug = acsr.UpdateGraph(m, outdeg, x_g, xs_tmp, y, max_upd=cap_b, max_ins=cap_b)
+    t_graph, g_regrow = [], 0
+    for ch, k in gbatches:
+        pinned = {kk: torch.from_numpy(v).pin_memory() for kk, v in ch.items()}
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        st = ug.replay(pinned)
+        torch.cuda.synchronize()
+        dt = time.perf_counter() - t0
+        if st.cpu().tolist() != [0, -1]:  # CAPACITY: grow (new buffers), apply eagerly, re-capture
+            assert int(st[0]) == acsr.ACSR_ERR_CAPACITY, st
+            m.grow()
+            chd = {kk: v.to(dev) for kk, v in pinned.items()}
+            while m.update(chd, outdeg=outdeg, status=st, ws=uws).cpu().tolist() != [0, -1]:
+                m.grow()
+            m.rebin()
+            ug = acsr.UpdateGraph(m, outdeg, x_g, xs_tmp, y, max_upd=cap_b, max_ins=cap_b)
+            g_regrow += 1
+        else:
+            t_graph.append(dt * 1e3)
+        x, it, _ = acsr.pagerank(m, outdeg, x0=x, eps=1e-6)
+        x_g.copy_(x)
     r = np.array(rec)
     if rank != 0:
         return None
@@ -810,8 +842,14 @@ def run_dynamic(args, dev, rank, world):
                           "pt_st": round(t_bin / t_spmv, 3),
                           "rebuild_plus_spmv_ms": round(t_upd + t_bin + t_spmv, 5),
                           "rebuild_plus_spmv_host_inclusive_ms": round(float(r[:, 7].mean()), 5),
+                          "rebuild_plus_spmv_graph_host_inclusive_ms": round(float(np.mean(t_graph)), 5)
+                          if t_graph else None,
+                          "graph_batches": len(t_graph), "graph_recaptures": g_regrow,
                           "timing": "phases: CUDA events, batch enqueued behind a GPU sleep (device time); "
-                                    "host_inclusive: wall clock from an idle GPU through the Python API",
+                                    "host_inclusive: wall clock from an idle GPU through the Python API, "
+                                    "change-list H2D copies included; "
+                                    "graph: further batches, copies + one CUDA-graph replay of "
+                                    "update_dev -> bin -> scale -> SpMV, wall clock",
                           "pagerank_warm_ms": round(float(r[:, 4].mean()), 4),
                           "warm_iterations_mean": round(float(r[:, 5].mean()), 2),
                           "inserted_edges_mean": round(float(r[:, 6].mean()), 1),

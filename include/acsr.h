@@ -290,6 +290,25 @@ acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
                               int32_t *status /* [2] out */,
                               void *ws, size_t ws_bytes, cudaStream_t stream);
 
+/* acsr_update_edges with the batch size read on the DEVICE: n_upd_dev[0] (int64) updates
+ * are applied, n_upd_max (>= it) sizes the launch and the workspace.  The launch
+ * configuration no longer depends on the batch, so the per-batch sequence (update ->
+ * acsr_bin -> ... -> acsr_spmv) can be captured into a CUDA graph once and replayed for
+ * every batch with the change lists copied into fixed buffers (CUDA graphs
+ * for the C5 update + re-bin + SpMV sequence).  A device count outside [0, n_upd_max]
+ * rejects the batch (status {ACSR_ERR_INVALID_VALUE, 0}, nothing modified). */
+acsr_status acsr_update_edges_dev(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
+                                  const int32_t *row_begin, int32_t *row_end, const int32_t *row_cap,
+                                  int32_t *col_idx, void *values /* NULL => pattern */,
+                                  int64_t n_upd_max, const int64_t *n_upd_dev /* [1] device */,
+                                  const int32_t *upd_rows,
+                                  const int32_t *del_ptr, const int32_t *del_cols,
+                                  const int32_t *ins_ptr, const int32_t *ins_cols,
+                                  const void *ins_vals /* NULL => ones */,
+                                  int32_t *outdeg /* NULL or [n_cols] */,
+                                  int32_t *status /* [2] out */,
+                                  void *ws, size_t ws_bytes, cudaStream_t stream);
+
 /* Re-layout of a slack CSR (§VII keeps "some additional memory ... at the end of
  * each CSR row"; what happens when a row outgrows it is unstated -- reading
  * R4 in DESIGN.md: after a CAPACITY rejection the caller re-lays the matrix out with

@@ -61,6 +61,9 @@ _lib.acsr_update_workspace_bytes.restype = _sz
 _lib.acsr_update_edges.argtypes = [ctypes.c_int, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _i64, _vp, _vp,
                                    _vp, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
 _lib.acsr_update_edges.restype = ctypes.c_int
+_lib.acsr_update_edges_dev.argtypes = [ctypes.c_int, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _i64, _vp, _vp, _vp,
+                                       _vp, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
+_lib.acsr_update_edges_dev.restype = ctypes.c_int
 _lib.acsr_relayout.argtypes = [ctypes.c_int, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp]
 _lib.acsr_relayout.restype = ctypes.c_int
 _lib.acsr_status_string.argtypes = [ctypes.c_int]
@@ -107,7 +110,7 @@ ACSR_IPC_HANDLE_BYTES = 64
 
 EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_bin_ex", "acsr_spmv", "acsr_pagerank_step",
             "acsr_pagerank_scale", "acsr_pagerank_step_peer", "acsr_peer_create", "acsr_peer_open",
-            "acsr_peer_destroy", "acsr_peer_push", "acsr_peer_delta2", "acsr_peer_query", "acsr_peer_read_xs", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_relayout",
+            "acsr_peer_destroy", "acsr_peer_push", "acsr_peer_delta2", "acsr_peer_query", "acsr_peer_read_xs", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_update_edges_dev", "acsr_relayout",
             "acsr_hits_workspace_bytes", "acsr_hits_normalize",
             "acsr_status_string", "acsr_last_error", "acsr_version")
 
@@ -338,8 +341,10 @@ def acsr_update_workspace_bytes(n_upd: int) -> int:
 
 def acsr_update_edges(n_cols, row_begin, row_end, row_cap, col_idx, values, upd_rows, ins_ptr,
                       ins_cols, ins_vals=None, del_ptr=None, del_cols=None, outdeg=None, status=None,
-                      ws=None, dtype=torch.float64, stream=None):
-    """Apply one change batch in place (§VII).  Returns the device status tensor [code, index]."""
+                      ws=None, dtype=torch.float64, stream=None, n_upd_dev=None):
+    """Apply one change batch in place (§VII).  Returns the device status tensor [code, index].
+    n_upd_dev (1-element int64 CUDA tensor): the batch size is read on the device and
+    upd_rows/ins_ptr/... are capacity buffers (acsr_update_edges_dev, graph-capturable)."""
     n = row_begin.numel()
     dev = row_begin.device
     n_upd = upd_rows.numel()
@@ -352,6 +357,20 @@ def acsr_update_edges(n_cols, row_begin, row_end, row_cap, col_idx, values, upd_
         del_ptr, del_cols = None, None  # insert-only batch
     dt = ACSR_F64 if vdt == torch.float64 else ACSR_F32
     opt = lambda t, d, nm: (_dev(t, d, nm) if t is not None and t.numel() else None)
+    if n_upd_dev is not None:
+        _check(_lib.acsr_update_edges_dev(dt, n, int(n_cols), _dev(row_begin, torch.int32, "row_begin"),
+                                          _dev(row_end, torch.int32, "row_end"),
+                                          _dev(row_cap, torch.int32, "row_cap"),
+                                          _dev(col_idx, torch.int32, "col_idx"), opt(values, vdt, "values"), n_upd,
+                                          _dev(n_upd_dev, torch.int64, "n_upd_dev"),
+                                          opt(upd_rows, torch.int32, "upd_rows"),
+                                          _dev(del_ptr, torch.int32, "del_ptr", True),
+                                          opt(del_cols, torch.int32, "del_cols") if del_ptr is not None else None,
+                                          opt(ins_ptr, torch.int32, "ins_ptr"), opt(ins_cols, torch.int32, "ins_cols"),
+                                          opt(ins_vals, vdt, "ins_vals"), _dev(outdeg, torch.int32, "outdeg", True),
+                                          _dev(status, torch.int32, "status"), _dev(ws, torch.uint8, "ws"),
+                                          ws.numel(), _stream(stream)), "acsr_update_edges_dev")
+        return status
     _check(_lib.acsr_update_edges(dt, n, int(n_cols), _dev(row_begin, torch.int32, "row_begin"),
                                   _dev(row_end, torch.int32, "row_end"), _dev(row_cap, torch.int32, "row_cap"),
                                   _dev(col_idx, torch.int32, "col_idx"), opt(values, vdt, "values"), n_upd,
@@ -399,4 +418,5 @@ def version() -> int:
     return int(_lib.acsr_version())
 
 
-from .matrix import ACSRMatrix, degree_relabel, hits, hits_matrix, pagerank, rwr, spmv_from_host  # noqa: E402
+from .matrix import (ACSRMatrix, UpdateGraph, degree_relabel, hits, hits_matrix, pagerank, rwr,  # noqa: E402
+                     spmv_from_host)

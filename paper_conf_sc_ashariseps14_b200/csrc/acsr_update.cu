@@ -27,6 +27,8 @@ struct UpdWs {
     unsigned long long key;  // (first failing index << 3) | code, or NO_FAIL
     unsigned int n_long;     // number of long-row updates appended to long_list
     unsigned int pad;
+    long long n_eff;         // updates of this batch (host count, or the device count of
+                             // acsr_update_edges_dev), written by update_init_kernel
     int32_t long_list[1];    // [n_upd]
 };
 
@@ -145,6 +147,7 @@ update_validate_kernel(int64_t n_rows, int64_t n_cols, const int32_t *__restrict
                        const int32_t *__restrict__ icol, UpdWs *ws)
 {
     pdl_enter();
+    n_upd = *(volatile long long *)&ws->n_eff;  // <= the launch's bound (init kernel)
     const int lane = threadIdx.x & 31;
     const int64_t wid = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
     if (!ACSR_UPD_SUB) {
@@ -390,6 +393,7 @@ update_apply_kernel(const int32_t *__restrict__ rb, int32_t *__restrict__ re,
         status[1] = k == NO_FAIL ? -1 : (int32_t)(k >> 3);
     }
     if (k != NO_FAIL) return;  // all-or-nothing
+    n_upd = *(volatile const long long *)&ws->n_eff;
     const int lane = threadIdx.x & 31;
     const int64_t wid = (int64_t)blockIdx.x * (UPD_THREADS / 32) + (threadIdx.x >> 5);
     if (!ACSR_UPD_SUB) {
@@ -503,21 +507,30 @@ extern "C" size_t acsr_update_workspace_bytes(int64_t n_upd)
     return align_up(offsetof(UpdWs, long_list) + sizeof(int32_t) * (size_t)(n_upd > 0 ? n_upd : 1), 256);
 }
 
-__global__ void update_init_kernel(UpdWs *ws)
+__global__ void update_init_kernel(UpdWs *ws, int64_t n_host, const int64_t *n_dev)
 {
     pdl_enter();
     ws->key = NO_FAIL;
     ws->n_long = 0;
+    long long n = n_host;
+    if (n_dev) {  // acsr_update_edges_dev: the batch size lives on the device
+        n = *n_dev;
+        if (n < 0 || n > n_host) {  // outside the launch's bound: the batch is rejected whole
+            ws->key = (unsigned long long)ACSR_ERR_INVALID_VALUE;  // index 0
+            n = 0;
+        }
+    }
+    ws->n_eff = n;
 }
 
-extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
+static acsr_status update_impl(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
                                          const int32_t *row_begin, int32_t *row_end,
                                          const int32_t *row_cap, int32_t *col_idx, void *values,
                                          int64_t n_upd, const int32_t *upd_rows,
                                          const int32_t *del_ptr, const int32_t *del_cols,
                                          const int32_t *ins_ptr, const int32_t *ins_cols,
                                          const void *ins_vals, int32_t *outdeg, int32_t *status,
-                                         void *ws, size_t ws_bytes, cudaStream_t stream)
+                                         void *ws, size_t ws_bytes, cudaStream_t stream, const int64_t *n_dev)
 {
     if (n_rows < 0 || n_cols < 0 || n_upd < 0 || !status || (dt != ACSR_F32 && dt != ACSR_F64) ||
         (n_upd > 0 && (!row_begin || !row_end || !row_cap || !col_idx || !upd_rows || !ins_ptr)) ||
@@ -530,7 +543,7 @@ extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t 
         return ACSR_ERR_WORKSPACE;
     }
     UpdWs *uw = (UpdWs *)ws;
-    launch_pdl(update_init_kernel, 1, 1, 0, stream, uw);
+    launch_pdl(update_init_kernel, 1, 1, 0, stream, uw, n_upd, n_dev);
     const int long_grid = 4 * acsr_num_sms();
     // hub-row delete lists in shared memory (ACSR_UPD_SMEM=0: global binary search, A/B)
     static int del_cap = -1;
@@ -586,4 +599,35 @@ extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t 
                 (const uint32_t *)ins_vals, one, outdeg, uw, del_cap);
     }
     return acsr_check_launch("acsr_update_edges");
+}
+
+extern "C" acsr_status acsr_update_edges(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
+                                         const int32_t *row_begin, int32_t *row_end,
+                                         const int32_t *row_cap, int32_t *col_idx, void *values,
+                                         int64_t n_upd, const int32_t *upd_rows,
+                                         const int32_t *del_ptr, const int32_t *del_cols,
+                                         const int32_t *ins_ptr, const int32_t *ins_cols,
+                                         const void *ins_vals, int32_t *outdeg, int32_t *status,
+                                         void *ws, size_t ws_bytes, cudaStream_t stream)
+{
+    return update_impl(dt, n_rows, n_cols, row_begin, row_end, row_cap, col_idx, values, n_upd, upd_rows, del_ptr,
+                       del_cols, ins_ptr, ins_cols, ins_vals, outdeg, status, ws, ws_bytes, stream, nullptr);
+}
+
+extern "C" acsr_status acsr_update_edges_dev(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
+                                             const int32_t *row_begin, int32_t *row_end,
+                                             const int32_t *row_cap, int32_t *col_idx, void *values,
+                                             int64_t n_upd_max, const int64_t *n_upd_dev,
+                                             const int32_t *upd_rows, const int32_t *del_ptr,
+                                             const int32_t *del_cols, const int32_t *ins_ptr,
+                                             const int32_t *ins_cols, const void *ins_vals, int32_t *outdeg,
+                                             int32_t *status, void *ws, size_t ws_bytes, cudaStream_t stream)
+{
+    if (!n_upd_dev) {
+        acsr_set_error("acsr_update_edges_dev: n_upd_dev is required");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    return update_impl(dt, n_rows, n_cols, row_begin, row_end, row_cap, col_idx, values, n_upd_max, upd_rows,
+                       del_ptr, del_cols, ins_ptr, ins_cols, ins_vals, outdeg, status, ws, ws_bytes, stream,
+                       n_upd_dev);
 }

@@ -10,7 +10,8 @@ from __future__ import annotations
 import torch
 
 from . import (acsr_bin, acsr_bin_workspace_bytes, acsr_hits_normalize, acsr_hits_workspace_bytes,
-               acsr_pagerank_scale, acsr_pagerank_step, acsr_relayout, acsr_spmv, acsr_update_edges)
+               acsr_pagerank_scale, acsr_pagerank_step, acsr_relayout, acsr_spmv, acsr_update_edges,
+               acsr_update_workspace_bytes)
 
 
 class ACSRMatrix:
@@ -42,13 +43,14 @@ class ACSRMatrix:
         return acsr_spmv(self.row_begin, self.col_idx, self.values, x, self.bin_rows,
                          self.bin_offsets, self.plan_ws, self.row_end, y, stream)
 
-    def update(self, changes, outdeg=None, ins_vals=None, status=None, ws=None, stream=None):
-        """changes: dict of CUDA int32 tensors upd_rows, ins_ptr, ins_cols[, del_ptr, del_cols]."""
+    def update(self, changes, outdeg=None, ins_vals=None, status=None, ws=None, stream=None, n_upd_dev=None):
+        """changes: dict of CUDA int32 tensors upd_rows, ins_ptr, ins_cols[, del_ptr, del_cols].
+        n_upd_dev: device batch size (the tensors are then capacity buffers; graph-capturable)."""
         assert self.row_end is not None and self.row_cap is not None, "update needs slack CSR"
         return acsr_update_edges(self.n_cols, self.row_begin, self.row_end, self.row_cap,
                                  self.col_idx, self.values, changes["upd_rows"], changes["ins_ptr"],
                                  changes["ins_cols"], ins_vals, changes.get("del_ptr"),
-                                 changes.get("del_cols"), outdeg, status, ws, stream=stream)
+                                 changes.get("del_cols"), outdeg, status, ws, stream=stream, n_upd_dev=n_upd_dev)
 
     def grow(self, min_slack=8, frac=2, stream=None):
         """Re-lay the slack CSR out with more room (reading R4: after a CAPACITY rejection):
@@ -79,6 +81,54 @@ class ACSRMatrix:
             self.plan_ws = torch.empty(acsr_bin_workspace_bytes(self.n_rows, self.n_cols, self.nnz_max),
                                        dtype=torch.uint8, device=dev)
         self.rebin(stream)
+
+
+class UpdateGraph:
+    """The C5 per-batch device sequence -- acsr_update_edges_dev -> acsr_bin ->
+    acsr_pagerank_scale -> acsr_spmv -- captured ONCE into a CUDA graph and
+    replayed for every insert-only batch: the change lists are copied into fixed capacity
+    buffers and the batch size into a device int64 (the update reads it there), so one
+    graph serves batches of any size up to the capacities.  Pointers are baked in: build a
+    new UpdateGraph after m.grow().  After replay(), self.status holds the update status and
+    y = A xs with xs = x / outdeg of the updated graph."""
+
+    def __init__(self, m: ACSRMatrix, outdeg, x, xs, y, max_upd: int, max_ins: int):
+        dev = m.row_begin.device
+        self.max_upd, self.max_ins = int(max_upd), int(max_ins)
+        self.n_dev = torch.zeros(1, dtype=torch.int64, device=dev)
+        self.n_host = torch.zeros(1, dtype=torch.int64).pin_memory()
+        self.bufs = {"upd_rows": torch.zeros(self.max_upd, dtype=torch.int32, device=dev),
+                     "ins_ptr": torch.zeros(self.max_upd + 1, dtype=torch.int32, device=dev),
+                     "ins_cols": torch.zeros(self.max_ins, dtype=torch.int32, device=dev)}
+        self.status = torch.zeros(2, dtype=torch.int32, device=dev)
+        self.ws = torch.empty(acsr_update_workspace_bytes(self.max_upd), dtype=torch.uint8, device=dev)
+
+        def seq():
+            m.update(self.bufs, outdeg=outdeg, status=self.status, ws=self.ws, n_upd_dev=self.n_dev)
+            m.rebin()
+            acsr_pagerank_scale(x, outdeg, xs)
+            m.spmv(xs, y)
+
+        self.n_dev.zero_()
+        seq()  # eager once with an empty batch: lazy kernel attributes are set outside the capture
+        torch.cuda.synchronize()
+        self.graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(self.graph):
+            seq()
+
+    def replay(self, changes_host):
+        """changes_host: dict of pinned host int32 tensors upd_rows, ins_ptr, ins_cols."""
+        n = changes_host["upd_rows"].numel()
+        k = changes_host["ins_cols"].numel()
+        if n > self.max_upd or k > self.max_ins:
+            raise ValueError("batch exceeds the UpdateGraph capacities")
+        self.bufs["upd_rows"][:n].copy_(changes_host["upd_rows"], non_blocking=True)
+        self.bufs["ins_ptr"][:n + 1].copy_(changes_host["ins_ptr"], non_blocking=True)
+        self.bufs["ins_cols"][:k].copy_(changes_host["ins_cols"], non_blocking=True)
+        self.n_host[0] = n
+        self.n_dev.copy_(self.n_host, non_blocking=True)
+        self.graph.replay()
+        return self.status
 
 
 def spmv_from_host(row_ptr_h, col_h, val_h, x_h, y_h=None, device="cuda", stream=None):

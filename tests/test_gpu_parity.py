@@ -476,6 +476,47 @@ def test_update_insert_bitwise(acsr, cuda, dtype):
     check_spmv(y, y_ref, den, dtype)
 
 
+def test_update_graph_replay_bitwise(acsr, cuda):
+    """C5 through one captured CUDA graph (acsr_update_edges_dev with the batch size on the
+    device -> acsr_bin -> acsr_pagerank_scale -> acsr_spmv), replayed for three insert
+    batches of different sizes: the pattern slack CSR, outdeg, bins and y equal the oracle
+    applied batch by batch; a device count above the capacity rejects the batch whole."""
+    n, rb, re, cap, col, _, od, rp, ci = _slack_graph(14, frac=1)
+    keys = np.sort(np.repeat(np.arange(n), np.diff(rp.numpy())).astype(np.int64) * n + ci.numpy())
+    batches = [ch for ch, _ in synth.insert_batches(14, 3, 4096, keys)]
+    m = acsr.ACSRMatrix(rb.to(cuda), col.to(cuda), None, row_end=re.to(cuda), row_cap=cap.to(cuda),
+                        nnz_max=col.numel())
+    odd = od.to(cuda)
+    x = (synth.vector(n, 7).abs() + 0.5).to(cuda)
+    xs, y = torch.empty_like(x), torch.empty_like(x)
+    g = acsr.UpdateGraph(m, odd, x, xs, y, max_upd=6000, max_ins=6000)
+    re_h, col_h, od_h = re.numpy().copy(), col.numpy().copy(), od.numpy().copy()
+    for ch in batches:
+        code, _ = oracle.update(n, rb.numpy(), re_h, cap.numpy(), col_h, None, ch["upd_rows"], None, None,
+                                ch["ins_ptr"], ch["ins_cols"], None, od_h)
+        assert code == 0
+        st = g.replay({k: torch.from_numpy(v).pin_memory() for k, v in ch.items()})
+        torch.cuda.synchronize()
+        assert st.cpu().tolist() == [0, -1]
+        assert np.array_equal(m.row_end.cpu().numpy(), re_h)
+        live = np.concatenate([np.arange(b, e) for b, e in zip(rb.numpy(), re_h)])
+        assert np.array_equal(m.col_idx.cpu().numpy()[live], col_h[live])
+        assert np.array_equal(odd.cpu().numpy(), od_h)
+        br, off = oracle.bins(rb.numpy(), re_h)
+        assert np.array_equal(m.bin_rows.cpu().numpy(), br)
+        xs_ref = np.where(od_h > 0, x.cpu().numpy() / np.maximum(od_h, 1), 0.0)
+        y_ref, den = oracle.spmv(rb.numpy(), col_h, None, xs_ref, row_end=re_h)
+        check_spmv(y.cpu().numpy(), y_ref, den, torch.float64)
+    # a device batch size beyond the capacity buffers: rejected, nothing modified
+    before = m.col_idx.clone(), m.row_end.clone()
+    g.n_host[0] = 7000
+    g.n_dev.copy_(g.n_host)
+    g.graph.replay()
+    torch.cuda.synchronize()
+    assert g.status.cpu().tolist() == [acsr.ACSR_ERR_INVALID_VALUE, 0]
+    assert torch.equal(m.col_idx, before[0]) and torch.equal(m.row_end, before[1])
+
+
 def test_update_mixed_bitwise(acsr, cuda):
     n, rb, re, cap, col, val, od, rp, ci = _slack_graph(12, frac=1)
     ch = next(synth.mixed_batches(rp.numpy(), ci.numpy(), n, 0.1, 5, 1))

@@ -81,30 +81,27 @@ __device__ __forceinline__ void validate_row(int64_t i, int lane, int64_t n_rows
                                              const int32_t *__restrict__ icol, UpdWs *ws)
 {
     unsigned long long *key = &ws->key;
-    int code = ACSR_OK;
+    // every load that does not depend on another is issued first (row id, previous row id,
+    // list bounds, then the row's bounds and capacity): the checks below overlap them
+    // instead of each waiting behind the previous check's warp vote
     const int r = __ldg(upd + i);
-    if (r < 0 || r >= n_rows || (i > 0 && r <= __ldg(upd + i - 1))) code = ACSR_ERR_INVALID_VALUE;
-    int d0 = 0, d1 = 0;
-    if (dptr) {
-        d0 = __ldg(dptr + i);
-        d1 = __ldg(dptr + i + 1);
-    }
-    if (code == ACSR_OK && dptr) {
-        bool bad = false;
-        for (int j = d0 + 1 + lane; j < d1; j += 32) bad |= __ldg(dcol + j) < __ldg(dcol + j - 1);
-        if (__any_sync(0xffffffffu, bad)) code = ACSR_ERR_INVALID_VALUE;
-    }
+    const int rprev = i > 0 ? __ldg(upd + i - 1) : -1;
+    const int d0 = dptr ? __ldg(dptr + i) : 0, d1 = dptr ? __ldg(dptr + i + 1) : 0;
     const int i0 = __ldg(iptr + i), i1 = __ldg(iptr + i + 1);
-    if (code == ACSR_OK) {
-        bool bad = false;
-        for (int j = i0 + lane; j < i1; j += 32) {
-            int c = __ldg(icol + j);
-            bad |= (c < 0 || c >= n_cols);
-        }
-        if (__any_sync(0xffffffffu, bad)) code = ACSR_ERR_INVALID_VALUE;
+    const bool rok = r >= 0 && r < n_rows;
+    const int b = rok ? __ldg(rb + r) : 0, e = rok ? __ldg(re + r) : 0;
+    const int cp = rok ? __ldg(cap + r) : 0;
+    // checks in reading R1's order: (a) row id, (b) delete list sorted, (c) insert columns
+    // in range -- (a)-(c) all give INVALID_VALUE, so one vote covers (b) and (c) -- then (d)
+    int code = (!rok || (i > 0 && r <= rprev)) ? ACSR_ERR_INVALID_VALUE : ACSR_OK;
+    bool bad = false;
+    for (int j = d0 + 1 + lane; j < d1; j += 32) bad |= __ldg(dcol + j) < __ldg(dcol + j - 1);
+    for (int j = i0 + lane; j < i1; j += 32) {
+        const int c = __ldg(icol + j);
+        bad |= (c < 0 || c >= n_cols);
     }
+    if (__any_sync(0xffffffffu, bad) && code == ACSR_OK) code = ACSR_ERR_INVALID_VALUE;
     if (code == ACSR_OK) {
-        const int b = __ldg(rb + r), e = __ldg(re + r);
         if (d1 > d0 && e - b > LONG_ROW) {  // deferred to the CTA-per-row kernel
             if (lane == 0) ws->long_list[atomicAdd(&ws->n_long, 1u)] = (int32_t)i;
             return;
@@ -123,7 +120,7 @@ __device__ __forceinline__ void validate_row(int64_t i, int lane, int64_t n_rows
         }
         for (int o = 16; o > 0; o >>= 1) dels += __shfl_xor_sync(0xffffffffu, dels, o);
         long long new_len = (long long)(e - b) - dels + (i1 - i0);
-        if (new_len > __ldg(cap + r)) code = ACSR_ERR_CAPACITY;
+        if (new_len > cp) code = ACSR_ERR_CAPACITY;
     }
     if (code != ACSR_OK && lane == 0) atomicMin(key, ((unsigned long long)i << 3) | (unsigned)code);
 }
@@ -337,9 +334,10 @@ __device__ __forceinline__ void apply_row(int64_t i, int lane, const int32_t *__
 {
     const unsigned lt = (1u << lane) - 1u;
     const int r = __ldg(upd + i);
+    const int d0 = dptr ? __ldg(dptr + i) : 0, d1 = dptr ? __ldg(dptr + i + 1) : 0;
+    const int i0 = __ldg(iptr + i), i1 = __ldg(iptr + i + 1);  // (independent loads first)
     const int b = __ldg(rb + r), e = re[r];
     int w = e;
-    const int d0 = dptr ? __ldg(dptr + i) : 0, d1 = dptr ? __ldg(dptr + i + 1) : 0;
     if (d1 > d0 && e - b > LONG_ROW) return;  // update_apply_long_kernel
     if (d1 > d0) {
         w = b;
@@ -367,7 +365,6 @@ __device__ __forceinline__ void apply_row(int64_t i, int lane, const int32_t *__
             __syncwarp();
         }
     }
-    const int i0 = __ldg(iptr + i), i1 = __ldg(iptr + i + 1);
     for (int j = i0 + lane; j < i1; j += 32) {
         int c = __ldg(icol + j);
         col[w + (j - i0)] = c;

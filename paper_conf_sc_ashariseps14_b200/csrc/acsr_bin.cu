@@ -49,6 +49,8 @@ struct BinSmem {
     int hw[BIN_THREADS / 32];
     int heavy_run;
     int upre[LIGHT_MAX_BIN + 2];
+    int boff[NBINS + 1];  // bin offsets as this CTA sees them (scatter)
+    int ovf, nheavy;
 };
 
 // ---- phase 1: per-tile histogram of bin ids (+ light-unit / heavy-chunk counts)
@@ -105,7 +107,7 @@ struct ScanArgs {
 // ---- phase 2: exclusive scan of one scan row over the tiles (coalesced chunks of T
 // with a running carry); the last of the SCAN_ROWS rows to finish turns the totals
 // into bin_offsets and the plan header.
-template <int T, int IPT>
+template <int T, int IPT, bool FINALIZE = true>
 __device__ __forceinline__ void scan_row(BinSmem &sm, const int32_t *__restrict__ cnt,
                                          int32_t *__restrict__ toff, int n_tiles, PlanHeader *hdr,
                                          const ScanArgs &sa, int row)
@@ -155,6 +157,7 @@ __device__ __forceinline__ void scan_row(BinSmem &sm, const int32_t *__restrict_
     }
     if (tid == 0) hdr->totals[row] = sm.carry;
     __syncthreads();
+    if (!FINALIZE) return;  // the scatter kernel turns the totals into offsets + header
     if (tid == 0) {
         __threadfence();
         sm.is_last = (atomicAdd(&hdr->scan_ticket, 1) == SCAN_ROWS - 1);
@@ -199,6 +202,67 @@ __device__ __forceinline__ void scan_row(BinSmem &sm, const int32_t *__restrict_
     __syncthreads();
 }
 
+// Scatter prologue, default path (warp 0): the 34 scan-row totals -> bin offsets (warp
+// scan), overflow and heavy-unit count, in shared memory; block 0 also publishes
+// bin_offsets and the plan header the SpMV reads.  Replaces the scan kernel's
+// last-CTA finalisation (ticket -> totals -> offsets: a chain of dependent L2 round trips).
+__device__ __forceinline__ void plan_from_totals(BinSmem &sm, PlanHeader *hdr, const ScanArgs &sa, int n_tiles,
+                                                 bool publish)
+{
+    const int lane = threadIdx.x & 31;
+    if (threadIdx.x >= 32) return;
+    const int t = __ldcg(hdr->totals + lane);  // NBINS == 32 == warp size
+    int incl = t;
+    for (int d = 1; d < 32; d <<= 1) {
+        const int v = __shfl_up_sync(0xffffffffu, incl, d);
+        if (lane >= d) incl += v;
+    }
+    sm.boff[lane] = incl - t;
+    if (lane == 31) sm.boff[NBINS] = incl;
+    const int nl = __ldcg(hdr->totals + NBINS), nh = __ldcg(hdr->totals + NBINS + 1);
+    const int ovf = (nl > sa.light_cap) || (nh > sa.heavy_cap);
+    if (lane == 0) {
+        sm.ovf = ovf;
+        sm.nheavy = ovf ? 0 : nh;
+    }
+    if (!publish) return;
+    sa.bin_offsets[lane] = incl - t;
+    if (lane == 31) sa.bin_offsets[NBINS] = incl;  // == n_rows
+    if (lane == 0) {
+        hdr->overflow = ovf;
+        hdr->n_light_units = ovf ? 0 : nl;
+        hdr->n_heavy_units = ovf ? 0 : nh;
+        hdr->n_units = ovf ? 0 : nl + nh;
+        hdr->n_tiles = n_tiles;
+        hdr->off_units = (int64_t)sa.L.off_units;
+        hdr->off_partial = (int64_t)sa.L.off_partial;
+        hdr->off_ticket = (int64_t)sa.L.off_ticket;
+        hdr->off_xc_vote = (int64_t)sa.L.off_xc_vote;
+        hdr->off_xc_tag = (int64_t)sa.L.off_xc_tag;
+        hdr->off_xc_val = (int64_t)sa.L.off_xc_val;
+        hdr->xc_valid = sa.xc_valid;
+        hdr->xc_stride = sa.xc_stride;
+        hdr->n_cols = sa.n_cols;
+        hdr->work_ctr = 0;
+        hdr->exit_ticket = 0;
+        hdr->d2_hi = 0;
+        hdr->d2_mid = 0;
+        hdr->d2_lo = 0;
+    }
+}
+
+// Scatter prologue of the fused paths: offsets and header were published by the
+// finalising scan CTA of the same grid (coherent L2 loads)
+__device__ __forceinline__ void plan_from_global(BinSmem &sm, const PlanHeader *hdr, const int32_t *bin_offsets)
+{
+    const int tid = threadIdx.x;
+    if (tid <= NBINS) sm.boff[tid] = __ldcg(bin_offsets + tid);
+    if (tid == 0) {
+        sm.ovf = __ldcg(&hdr->overflow);
+        sm.nheavy = __ldcg(&hdr->n_heavy_units);
+    }
+}
+
 // ---- phase 3: stable scatter of one tile + its work units
 template <bool HAS_END>
 __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32_t *__restrict__ rb,
@@ -209,13 +273,15 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
 {
     constexpr int NW = BIN_THREADS / 32;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    // (L2 loads: in the fused scan+scatter launch these were written by other CTAs of the
-    // same grid)
-    const int overflow = __ldcg(&hdr->overflow);
-    const int n_heavy = __ldcg(&hdr->n_heavy_units);
+    // sm.boff / sm.ovf / sm.nheavy were filled by the caller (plan_from_totals or
+    // plan_from_global) before a __syncthreads
+    (void)bin_offsets;
+    (void)hdr;
+    const int overflow = sm.ovf;
+    const int n_heavy = sm.nheavy;
     if (tid < NBINS) {
         sm.run[tid] = 0;
-        sm.seg[tid] = __ldcg(bin_offsets + tid) + __ldcg(toff + (int64_t)tid * n_tiles + tile);
+        sm.seg[tid] = sm.boff[tid] + __ldcg(toff + (int64_t)tid * n_tiles + tile);
     }
     for (int i = tid; i < NW * NBINS; i += BIN_THREADS) (&sm.wcnt[0][0])[i] = 0;
     if (tid == 0) sm.heavy_run = __ldcg(toff + (int64_t)(NBINS + 1) * n_tiles + tile);
@@ -336,20 +402,22 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
 {
     __shared__ BinSmem sm;
     pdl_enter();
-    scan_row<SCAN_THREADS, 1>(sm, cnt, toff, n_tiles, hdr, sa, blockIdx.x);
+    scan_row<SCAN_THREADS, 1, false>(sm, cnt, toff, n_tiles, hdr, sa, blockIdx.x);
 }
 
 template <bool HAS_END>
 __global__ void __launch_bounds__(BIN_THREADS)
 bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
-                   int32_t *__restrict__ bin_rows, const int32_t *__restrict__ bin_offsets,
-                   const int32_t *__restrict__ toff, int n_tiles, const PlanHeader *__restrict__ hdr,
-                   int2 *__restrict__ units, int32_t *__restrict__ tickets, int64_t heavy_cap, int wmb)
+                   int32_t *__restrict__ bin_rows, const int32_t *__restrict__ toff, int n_tiles,
+                   PlanHeader *hdr, int2 *__restrict__ units, int32_t *__restrict__ tickets, ScanArgs sa,
+                   int wmb)
 {
     __shared__ BinSmem sm;
     pdl_enter();
-    scatter_tile<HAS_END>(sm, n, rb, re, bin_rows, bin_offsets, toff, n_tiles, hdr, units, tickets, heavy_cap,
-                          blockIdx.x, wmb);
+    plan_from_totals(sm, hdr, sa, n_tiles, blockIdx.x == 0);
+    __syncthreads();
+    scatter_tile<HAS_END>(sm, n, rb, re, bin_rows, sa.bin_offsets, toff, n_tiles, hdr, units, tickets,
+                          sa.heavy_cap, blockIdx.x, wmb);
 }
 
 // ---- scan + scatter in ONE launch (opt-in, ACSR_BIN_SS=1): the first SCAN_ROWS CTAs to start (an
@@ -392,6 +460,8 @@ bin_scan_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t
         while (*(volatile int32_t *)&hdr->scan_done < SCAN_ROWS) __nanosleep(64);
     __syncthreads();
     __threadfence();
+    plan_from_global(sm, hdr, sa.bin_offsets);
+    __syncthreads();
     scatter_tile<HAS_END>(sm, n, rb, re, bin_rows, sa.bin_offsets, toff, n_tiles, hdr, units, tickets, sa.heavy_cap,
                           tile, wmb);
 }
@@ -422,6 +492,8 @@ bin_fused_kernel(FusedArgs f)
     for (int row = blockIdx.x; row < SCAN_ROWS; row += gridDim.x)
         scan_row<BIN_THREADS, 8>(sm, f.cnt, f.toff, f.n_tiles, f.hdr, f.sa, row);
     grid.sync();
+    plan_from_global(sm, f.hdr, f.sa.bin_offsets);
+    __syncthreads();
     for (int t = blockIdx.x; t < f.n_tiles; t += gridDim.x)
         scatter_tile<HAS_END>(sm, f.n, f.rb, f.re, f.bin_rows, f.sa.bin_offsets, f.toff, f.n_tiles, f.hdr, f.units,
                               f.tickets, f.sa.heavy_cap, t, f.wmb);
@@ -547,8 +619,7 @@ extern "C" acsr_status acsr_bin_ex(int64_t n_rows, int64_t n_cols, int64_t nnz_m
     {
         const int64_t nr = n_rows;
         const int32_t *rb = row_begin, *re = row_end;
-        const int32_t *cbo = bin_offsets, *ctoff = toff;
-        const PlanHeader *chdr = hdr;
+        const int32_t *ctoff = toff;
         if (row_end)
             launch_pdl(bin_count_kernel<true>, nt, BIN_THREADS, 0, stream, nr, rb, re, cnt, nt, hdr, wmb);
         else
@@ -565,11 +636,11 @@ extern "C" acsr_status acsr_bin_ex(int64_t n_rows, int64_t n_cols, int64_t nnz_m
         }
         launch_pdl(bin_scan_kernel, SCAN_ROWS, SCAN_THREADS, 0, stream, ccnt, toff, nt, hdr, sa);
         if (row_end)
-            launch_pdl(bin_scatter_kernel<true>, nt, BIN_THREADS, 0, stream, nr, rb, re, bin_rows, cbo, ctoff, nt, chdr,
-                       units, tickets, L.heavy_cap, wmb);
+            launch_pdl(bin_scatter_kernel<true>, nt, BIN_THREADS, 0, stream, nr, rb, re, bin_rows, ctoff, nt, hdr,
+                       units, tickets, sa, wmb);
         else
-            launch_pdl(bin_scatter_kernel<false>, nt, BIN_THREADS, 0, stream, nr, rb, re, bin_rows, cbo, ctoff, nt,
-                       chdr, units, tickets, L.heavy_cap, wmb);
+            launch_pdl(bin_scatter_kernel<false>, nt, BIN_THREADS, 0, stream, nr, rb, re, bin_rows, ctoff, nt, hdr,
+                       units, tickets, sa, wmb);
     }
 xc:
     if (xc_valid) {

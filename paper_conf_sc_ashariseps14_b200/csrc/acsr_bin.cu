@@ -264,36 +264,56 @@ __device__ __forceinline__ void plan_from_global(BinSmem &sm, const PlanHeader *
 }
 
 // ---- phase 3: stable scatter of one tile + its work units
+// The tile's inputs that do not depend on the plan (row lengths, the tile's row of the
+// per-tile prefixes) are loaded first, so their latency overlaps the plan prologue.
+struct ScatterPre {
+    int lens[TILE_ROUNDS];
+    int tof;   // toff[tid][tile] (tid < NBINS)
+    int hrun;  // toff[heavy row][tile] (tid == 0)
+    int lu;    // toff[light-unit row][tile] (every thread)
+};
+
 template <bool HAS_END>
-__device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32_t *__restrict__ rb,
-                                             const int32_t *__restrict__ re, int32_t *__restrict__ bin_rows,
-                                             const int32_t *bin_offsets, const int32_t *toff, int n_tiles,
-                                             const PlanHeader *hdr, int2 *__restrict__ units,
-                                             int32_t *__restrict__ tickets, int64_t heavy_cap, int tile, int wmb)
+__device__ __forceinline__ void scatter_preload(ScatterPre &pre, int64_t n, const int32_t *__restrict__ rb,
+                                                const int32_t *__restrict__ re, const int32_t *toff, int n_tiles,
+                                                int tile)
+{
+    const int tid = threadIdx.x;
+    const int64_t base = (int64_t)tile * TILE_ROWS;
+#pragma unroll
+    for (int k = 0; k < TILE_ROUNDS; k++) {  // all row-length loads in flight at once
+        const int64_t r = base + k * BIN_THREADS + tid;
+        pre.lens[k] = r < n ? row_length<HAS_END>(rb, re, r) : 0;
+    }
+    pre.tof = tid < NBINS ? __ldcg(toff + (int64_t)tid * n_tiles + tile) : 0;
+    pre.hrun = tid == 0 ? __ldcg(toff + (int64_t)(NBINS + 1) * n_tiles + tile) : 0;
+    pre.lu = __ldcg(toff + (int64_t)NBINS * n_tiles + tile);
+}
+
+template <bool HAS_END>
+__device__ __forceinline__ void scatter_tile(BinSmem &sm, const ScatterPre &pre, int64_t n,
+                                             int32_t *__restrict__ bin_rows, int n_tiles,
+                                             int2 *__restrict__ units, int32_t *__restrict__ tickets,
+                                             int64_t heavy_cap, int tile, int wmb)
 {
     constexpr int NW = BIN_THREADS / 32;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     // sm.boff / sm.ovf / sm.nheavy were filled by the caller (plan_from_totals or
     // plan_from_global) before a __syncthreads
-    (void)bin_offsets;
-    (void)hdr;
     const int overflow = sm.ovf;
     const int n_heavy = sm.nheavy;
     if (tid < NBINS) {
         sm.run[tid] = 0;
-        sm.seg[tid] = sm.boff[tid] + __ldcg(toff + (int64_t)tid * n_tiles + tile);
+        sm.seg[tid] = sm.boff[tid] + pre.tof;
     }
     for (int i = tid; i < NW * NBINS; i += BIN_THREADS) (&sm.wcnt[0][0])[i] = 0;
-    if (tid == 0) sm.heavy_run = __ldcg(toff + (int64_t)(NBINS + 1) * n_tiles + tile);
+    if (tid == 0) sm.heavy_run = pre.hrun;
     __syncthreads();
     const int64_t base = (int64_t)tile * TILE_ROWS;
     const unsigned lt = (1u << lane) - 1u;
     int lens[TILE_ROUNDS];
 #pragma unroll
-    for (int k = 0; k < TILE_ROUNDS; k++) {  // all row-length loads in flight at once
-        const int64_t r = base + k * BIN_THREADS + tid;
-        lens[k] = r < n ? row_length<HAS_END>(rb, re, r) : 0;
-    }
+    for (int k = 0; k < TILE_ROUNDS; k++) lens[k] = pre.lens[k];
 #pragma unroll
     for (int k = 0; k < TILE_ROUNDS; k++) {
         const int64_t r = base + k * BIN_THREADS + tid;
@@ -359,7 +379,7 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, int64_t n, const int32
             sm.upre[LIGHT_MAX_BIN + 1] = acc;
         }
         __syncthreads();
-        const int ubase = n_heavy + __ldcg(toff + (int64_t)NBINS * n_tiles + tile);
+        const int ubase = n_heavy + pre.lu;
         const int total = sm.upre[LIGHT_MAX_BIN + 1];
         for (int j = tid; j < total; j += BIN_THREADS) {
             if (j < nwin) {
@@ -414,10 +434,11 @@ bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__r
 {
     __shared__ BinSmem sm;
     pdl_enter();
+    ScatterPre pre;
+    scatter_preload<HAS_END>(pre, n, rb, re, toff, n_tiles, blockIdx.x);  // overlaps the prologue
     plan_from_totals(sm, hdr, sa, n_tiles, blockIdx.x == 0);
     __syncthreads();
-    scatter_tile<HAS_END>(sm, n, rb, re, bin_rows, sa.bin_offsets, toff, n_tiles, hdr, units, tickets,
-                          sa.heavy_cap, blockIdx.x, wmb);
+    scatter_tile<HAS_END>(sm, pre, n, bin_rows, n_tiles, units, tickets, sa.heavy_cap, blockIdx.x, wmb);
 }
 
 // ---- scan + scatter in ONE launch (opt-in, ACSR_BIN_SS=1): the first SCAN_ROWS CTAs to start (an
@@ -461,9 +482,10 @@ bin_scan_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t
     __syncthreads();
     __threadfence();
     plan_from_global(sm, hdr, sa.bin_offsets);
+    ScatterPre pre;
+    scatter_preload<HAS_END>(pre, n, rb, re, toff, n_tiles, tile);  // toff is complete after the wait
     __syncthreads();
-    scatter_tile<HAS_END>(sm, n, rb, re, bin_rows, sa.bin_offsets, toff, n_tiles, hdr, units, tickets, sa.heavy_cap,
-                          tile, wmb);
+    scatter_tile<HAS_END>(sm, pre, n, bin_rows, n_tiles, units, tickets, sa.heavy_cap, tile, wmb);
 }
 
 // ---- one cooperative launch: count -> grid barrier -> scan -> grid barrier -> scatter
@@ -494,9 +516,12 @@ bin_fused_kernel(FusedArgs f)
     grid.sync();
     plan_from_global(sm, f.hdr, f.sa.bin_offsets);
     __syncthreads();
-    for (int t = blockIdx.x; t < f.n_tiles; t += gridDim.x)
-        scatter_tile<HAS_END>(sm, f.n, f.rb, f.re, f.bin_rows, f.sa.bin_offsets, f.toff, f.n_tiles, f.hdr, f.units,
+    for (int t = blockIdx.x; t < f.n_tiles; t += gridDim.x) {
+        ScatterPre pre;
+        scatter_preload<HAS_END>(pre, f.n, f.rb, f.re, f.toff, f.n_tiles, t);
+        scatter_tile<HAS_END>(sm, pre, f.n, f.bin_rows, f.n_tiles, f.units,
                               f.tickets, f.sa.heavy_cap, t, f.wmb);
+    }
 }
 
 // x-cache table: sampled occurrence counts, per-slot winner (count, column).

@@ -414,7 +414,11 @@ bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__res
     count_tile<HAS_END>(sm, n, rb, re, cnt, n_tiles, blockIdx.x, wmb);
 }
 
-constexpr int SCAN_THREADS = 1024;
+#ifndef ACSR_SCAN_THREADS
+#define ACSR_SCAN_THREADS 1024  // A/B: 256 with 4 values per thread
+#endif
+constexpr int SCAN_THREADS = ACSR_SCAN_THREADS;
+constexpr int SCAN_IPT = SCAN_THREADS >= 1024 ? 1 : 1024 / SCAN_THREADS;
 
 __global__ void __launch_bounds__(SCAN_THREADS)
 bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int n_tiles,
@@ -422,7 +426,7 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
 {
     __shared__ BinSmem sm;
     pdl_enter();
-    scan_row<SCAN_THREADS, 1, false>(sm, cnt, toff, n_tiles, hdr, sa, blockIdx.x);
+    scan_row<SCAN_THREADS, SCAN_IPT, false>(sm, cnt, toff, n_tiles, hdr, sa, blockIdx.x);
 }
 
 template <bool HAS_END>

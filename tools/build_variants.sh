@@ -53,6 +53,7 @@ for v in "$@"; do
     td16) build td16 -DACSR_TAIL_DIV=16 ;;
     uwr1) build uwr1 -DACSR_UPD_WARPREG=1 ;;
     us1) build us1 -DACSR_UPD_SUB=1 ;;
+    sc256) build sc256 -DACSR_SCAN_THREADS=256 ;;
     td8) build td8 -DACSR_TAIL_DIV=8 ;;
     td32) build td32 -DACSR_TAIL_DIV=32 ;;
     wu64) build wu64 -DACSR_WIN_UNIT_ROWS=64 ;;

@@ -57,6 +57,34 @@ def test_bins_bitwise_rmat(acsr, cuda, scale):
     assert np.array_equal(m.bin_rows.cpu().numpy(), br)
 
 
+@pytest.mark.parametrize("env", ["ACSR_BIN_SS=1", "ACSR_BIN_FUSED=1", "ACSR_PDL=0"])
+def test_bins_alternative_launch_paths(cuda, env):
+    """The opt-in binning launch paths (scan + scatter in one launch; one cooperative
+    launch) and PDL off give the same bins and plan: bitwise bins vs the oracle and an SpMV
+    on integer data bitwise, in a fresh process (the knobs are read once per process)."""
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = (
+        "import sys; sys.path.insert(0, %r)\n"
+        "import numpy as np, torch, oracle, synth\n"
+        "import paper_conf_sc_ashariseps14_b200 as acsr\n"
+        "for sc in (12, 17):\n"
+        "    rp, ci = synth.rmat_csr(sc)\n"
+        "    val = synth.values(ci.numel(), 3, integer=True); x = synth.vector(rp.numel() - 1, 4, integer=True)\n"
+        "    m = acsr.ACSRMatrix(rp.cuda(), ci.cuda(), val.cuda())\n"
+        "    y = m.spmv(x.cuda()).cpu().numpy()\n"
+        "    br, off = oracle.bins(rp.numpy())\n"
+        "    assert np.array_equal(m.bin_rows.cpu().numpy(), br) and np.array_equal(m.bin_offsets.cpu().numpy(), off)\n"
+        "    y_ref, _ = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())\n"
+        "    assert np.array_equal(y, y_ref)\n"
+        "print('alt-path ok')\n" % root)
+    k, v = env.split("=")
+    out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=300,
+                         env=dict(os.environ, **{k: v}))
+    assert out.returncode == 0 and "alt-path ok" in out.stdout, out.stdout[-2000:] + out.stderr[-2000:]
+
+
 def test_bins_boundary_and_slack(acsr, cuda):
     lens = synth.boundary_lengths(17)
     rp, ci = synth.boundary_csr(lens * 3, 1 << 18, 5)

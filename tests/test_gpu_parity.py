@@ -57,7 +57,7 @@ def test_bins_bitwise_rmat(acsr, cuda, scale):
     assert np.array_equal(m.bin_rows.cpu().numpy(), br)
 
 
-@pytest.mark.parametrize("env", ["ACSR_BIN_SS=1", "ACSR_BIN_FUSED=1", "ACSR_PDL=0"])
+@pytest.mark.parametrize("env", ["ACSR_BIN_SS=1", "ACSR_BIN_FUSED=1", "ACSR_PDL=0", "ACSR_XPREFETCH=0"])
 def test_bins_alternative_launch_paths(cuda, env):
     """The opt-in binning launch paths (scan + scatter in one launch; one cooperative
     launch) and PDL off give the same bins and plan: bitwise bins vs the oracle and an SpMV
@@ -83,6 +83,19 @@ def test_bins_alternative_launch_paths(cuda, env):
     out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=300,
                          env=dict(os.environ, **{k: v}))
     assert out.returncode == 0 and "alt-path ok" in out.stdout, out.stdout[-2000:] + out.stderr[-2000:]
+
+
+def test_update_global_search_path(cuda):
+    """The hub-row update path with the delete list searched in global memory
+    (ACSR_UPD_SMEM=0, the fallback when shared memory cannot be reserved) passes the
+    bitwise update tests too (fresh pytest process: the knob is read once)."""
+    import subprocess
+    import sys
+    out = subprocess.run([sys.executable, "-m", "pytest", os.path.abspath(__file__), "-q", "-x", "-m", "gpu",
+                          "-k", "update_long_row_cta_path or paper_epoch_update_bitwise or update_mixed_bitwise"],
+                         capture_output=True, text=True, timeout=600, env=dict(os.environ, ACSR_UPD_SMEM="0"),
+                         cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    assert out.returncode == 0 and " passed" in out.stdout, out.stdout[-2000:] + out.stderr[-2000:]
 
 
 def test_bins_boundary_and_slack(acsr, cuda):

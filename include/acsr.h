@@ -77,6 +77,16 @@ enum { ACSR_NBINS = 32 };
  * equal the oracle bit for bit.  plan_ws must not be shared by concurrent calls. */
 size_t acsr_bin_workspace_bytes(int64_t n_rows, int64_t n_cols, int64_t nnz_max);
 
+/* Plan health.  If nnz_max understates the stored entries seen by acsr_bin, the SpMV work
+ * list no longer fits the workspace: the plan is marked invalid (nothing is written out of
+ * bounds), and every later acsr_spmv / acsr_pagerank_step on it writes a quiet NaN to every
+ * output row (PageRank: *delta2 = NaN, and ctrl[0] = ACSR_CTRL_PLAN_ERROR so a device-side
+ * loop stops) instead of leaving stale data.  acsr_plan_status synchronises `stream` and
+ * returns ACSR_ERR_CAPACITY for such a plan (detail in acsr_last_error()), ACSR_OK
+ * otherwise; call it after acsr_bin whenever nnz_max is not known to be an upper bound. */
+enum { ACSR_CTRL_PLAN_ERROR = 2 };
+acsr_status acsr_plan_status(const void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream);
+
 acsr_status acsr_bin(int64_t n_rows, int64_t n_cols, int64_t nnz_max,
                      const int32_t *row_begin, const int32_t *row_end /* NULL => standard CSR */,
                      const int32_t *col_idx /* NULL => no x cache */,

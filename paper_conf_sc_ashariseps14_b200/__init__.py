@@ -103,6 +103,8 @@ _lib.acsr_hits_workspace_bytes.argtypes = [_i64]
 _lib.acsr_hits_workspace_bytes.restype = _sz
 _lib.acsr_hits_normalize.argtypes = [_i64, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
 _lib.acsr_hits_normalize.restype = ctypes.c_int
+_lib.acsr_plan_status.argtypes = [_vp, _sz, _vp]
+_lib.acsr_plan_status.restype = ctypes.c_int
 
 ACSR_BIN_SHORT_ALG2 = 1  # include/acsr.h: per-bin Alg. 2 units for bins 0..5
 ACSR_PEER_MAX = 8
@@ -111,7 +113,7 @@ ACSR_IPC_HANDLE_BYTES = 64
 EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_bin_ex", "acsr_spmv", "acsr_pagerank_step",
             "acsr_pagerank_scale", "acsr_pagerank_step_peer", "acsr_peer_create", "acsr_peer_open",
             "acsr_peer_destroy", "acsr_peer_push", "acsr_peer_delta2", "acsr_peer_query", "acsr_peer_read_xs", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_update_edges_dev", "acsr_relayout",
-            "acsr_hits_workspace_bytes", "acsr_hits_normalize",
+            "acsr_hits_workspace_bytes", "acsr_hits_normalize", "acsr_plan_status",
             "acsr_status_string", "acsr_last_error", "acsr_version")
 
 
@@ -189,6 +191,16 @@ def acsr_bin(row_begin, row_end=None, nnz_max=None, bin_rows=None, bin_offsets=N
            "acsr_bin")
     return bin_rows, bin_offsets, plan_ws
 
+
+def acsr_plan_status(plan_ws, stream=None):
+    """Synchronising health check of a plan (include/acsr.h): raises ACSRError
+    (ACSR_ERR_CAPACITY) if acsr_bin's nnz_max understated the stored entries, in which case
+    every SpMV / PageRank output of the plan is NaN."""
+    _check(_lib.acsr_plan_status(_dev(plan_ws, torch.uint8, "plan_ws"), plan_ws.numel(), _stream(stream)),
+           "acsr_plan_status")
+
+
+ACSR_CTRL_PLAN_ERROR = 2
 
 # --------------------------------------------------------------------------- SpMV
 def acsr_spmv(row_begin, col_idx, values, x, bin_rows, bin_offsets, plan_ws, row_end=None, y=None,

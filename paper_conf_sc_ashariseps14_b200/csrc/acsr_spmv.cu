@@ -88,6 +88,7 @@ struct SpmvArgs {
     double restart_weight;
     int32_t *ctrl;  // device-side convergence: [0] stop flag, [1] executed steps (nullable)
     double eps2;
+    int64_t n_rows;  // rows of the call (NaN fill of an overflowed plan)
     int64_t x_prefetch;  // bytes of x to bulk-prefetch into L2 at entry (0: none)
     // fused peer-memory exchange of xs_next (acsr_pagerank_step_peer; peer.nranks == 0: off)
     const PeerArgs *peer;  // device copy (PeerState::view) or NULL
@@ -859,6 +860,23 @@ spmv_kernel(SpmvArgs<V> a)
         }
     }
     const int n_units = hdr->n_units;
+    // A plan whose unit list overflowed its workspace (acsr_bin with an understated
+    // nnz_max) has n_units == 0: the rows are not computed.  Never return stale data
+    // silently: every output row gets a quiet NaN (and, for PageRank, Delta^2 = NaN and
+    // ctrl[0] = ACSR_CTRL_PLAN_ERROR, below); acsr_plan_status reports the cause.
+    const int plan_bad = *(volatile int32_t *)&hdr->overflow;
+    if (plan_bad) {
+        const double qnan = __longlong_as_double(0x7ff8000000000000ll);
+        for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < a.n_rows;
+             r += (int64_t)gridDim.x * blockDim.x) {
+            if (PR) {
+                a.x_new[r] = qnan;
+                if (a.xs_next) a.xs_next[r] = qnan;
+            } else {
+                a.y[r] = (V)qnan;
+            }
+        }
+    }
     {
         char *ws = (char *)hdr;
         a.units = (const int2 *)(ws + hdr->off_units);
@@ -957,13 +975,17 @@ spmv_kernel(SpmvArgs<V> a)
                 const uint64_t hi = *(volatile uint64_t *)&hdr->d2_hi;
                 const uint64_t mid = *(volatile uint64_t *)&hdr->d2_mid;
                 const uint64_t lo = *(volatile uint64_t *)&hdr->d2_lo;
-                const double d2v = (double)hi + ((double)mid + (double)lo * 5.421010862427522e-20) * 5.421010862427522e-20;
+                double d2v = (double)hi + ((double)mid + (double)lo * 5.421010862427522e-20) * 5.421010862427522e-20;
+                if (plan_bad) d2v = __longlong_as_double(0x7ff8000000000000ll);
                 *a.delta2 = d2v;  // with the peer exchange: this rank's partial
                 if (PEER) {
                     __threadfence_system();
-                    peer_signal(*a.peer, pc + 1, true, hi, mid, lo);
+                    // an overflowed plan publishes a saturated partial: no rank converges on it
+                    peer_signal(*a.peer, pc + 1, true, plan_bad ? ~0ull : hi, mid, lo);
                 }
-                if (a.ctrl) {
+                if (a.ctrl && plan_bad) {
+                    a.ctrl[0] = ACSR_CTRL_PLAN_ERROR;  // stops the loop; acsr_plan_status tells why
+                } else if (a.ctrl) {
                     a.ctrl[1] += 1;
                     // peer exchange: the global test runs at the next step's entry (or in
                     // acsr_peer_delta2), once every rank's partial has arrived
@@ -1217,14 +1239,14 @@ extern "C" acsr_status acsr_spmv(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
         SpmvArgs<double> a{};
         a.rb = row_begin; a.re = row_end; a.col = col_idx;
         a.val = (const double *)values; a.x = n_cols > 0 ? (const double *)x : nullptr; a.y = (double *)y;
-        a.bin_rows = bin_rows; a.hdr = (PlanHeader *)plan_ws;
+        a.bin_rows = bin_rows; a.hdr = (PlanHeader *)plan_ws; a.n_rows = n_rows;
         a.x_prefetch = a.x ? x_prefetch_bytes(n_cols * (int64_t)sizeof(double)) : 0;
         dispatch<double, false>(a, stream);
     } else {
         SpmvArgs<float> a{};
         a.rb = row_begin; a.re = row_end; a.col = col_idx;
         a.val = (const float *)values; a.x = n_cols > 0 ? (const float *)x : nullptr; a.y = (float *)y;
-        a.bin_rows = bin_rows; a.hdr = (PlanHeader *)plan_ws;
+        a.bin_rows = bin_rows; a.hdr = (PlanHeader *)plan_ws; a.n_rows = n_rows;
         a.x_prefetch = a.x ? x_prefetch_bytes(n_cols * (int64_t)sizeof(float)) : 0;
         dispatch<float, false>(a, stream);
     }
@@ -1249,7 +1271,7 @@ extern "C" acsr_status acsr_pagerank_step(const acsr_pr_args *p, cudaStream_t st
     SpmvArgs<double> a{};
     a.rb = p->row_begin; a.re = p->row_end; a.col = p->col_idx;
     a.val = nullptr; a.x = p->n_cols > 0 ? p->xs : nullptr; a.y = nullptr;
-    a.bin_rows = p->bin_rows; a.hdr = (PlanHeader *)p->plan_ws;
+    a.bin_rows = p->bin_rows; a.hdr = (PlanHeader *)p->plan_ws; a.n_rows = p->n_rows;
     a.x_old = p->x; a.outdeg = p->outdeg; a.x_new = p->x_new; a.xs_next = p->xs_next;
     a.damping = p->damping; a.teleport = p->teleport; a.delta2 = p->delta2;
     a.restart = p->restart; a.restart_weight = p->restart_weight;
@@ -1283,7 +1305,7 @@ extern "C" acsr_status acsr_pagerank_step_peer(const acsr_pr_args *p, acsr_peer 
     SpmvArgs<double> a{};
     a.rb = p->row_begin; a.re = p->row_end; a.col = p->col_idx;
     a.val = nullptr; a.x = nullptr; a.y = nullptr;  // x: the peer buffer, chosen in-kernel
-    a.bin_rows = p->bin_rows; a.hdr = (PlanHeader *)p->plan_ws;
+    a.bin_rows = p->bin_rows; a.hdr = (PlanHeader *)p->plan_ws; a.n_rows = p->n_rows;
     a.x_old = p->x; a.outdeg = p->outdeg; a.x_new = p->x_new; a.xs_next = p->xs_next;
     a.damping = p->damping; a.teleport = p->teleport; a.delta2 = p->delta2;
     a.restart = p->restart; a.restart_weight = p->restart_weight;
@@ -1305,4 +1327,26 @@ extern "C" acsr_status acsr_pagerank_scale(int64_t n, const double *x, const int
     if (blocks > 148 * 16) blocks = 148 * 16;
     pagerank_scale_kernel<<<(int)blocks, 256, 0, stream>>>(n, x, outdeg, xs);
     return acsr_check_launch("acsr_pagerank_scale");
+}
+
+extern "C" acsr_status acsr_plan_status(const void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream)
+{
+    if (!plan_ws || plan_ws_bytes < sizeof(PlanHeader)) {
+        acsr_set_error("acsr_plan_status: plan workspace missing or too small");
+        return ACSR_ERR_WORKSPACE;
+    }
+    int32_t ovf = 0;
+    cudaError_t e = cudaMemcpyAsync(&ovf, &((const PlanHeader *)plan_ws)->overflow, sizeof(int32_t),
+                                    cudaMemcpyDeviceToHost, stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(stream);
+    if (e != cudaSuccess) {
+        acsr_set_error("acsr_plan_status: %s", cudaGetErrorString(e));
+        return ACSR_ERR_CUDA;
+    }
+    if (ovf) {
+        acsr_set_error("acsr_plan_status: the plan's work list overflowed its workspace (nnz_max passed to "
+                       "acsr_bin is smaller than the stored entries); SpMV outputs of this plan are NaN");
+        return ACSR_ERR_CAPACITY;
+    }
+    return ACSR_OK;
 }

@@ -9,9 +9,9 @@ from __future__ import annotations
 
 import torch
 
-from . import (acsr_bin, acsr_bin_workspace_bytes, acsr_hits_normalize, acsr_hits_workspace_bytes,
-               acsr_pagerank_scale, acsr_pagerank_step, acsr_relayout, acsr_spmv, acsr_update_edges,
-               acsr_update_workspace_bytes)
+from . import (ACSR_CTRL_PLAN_ERROR, acsr_bin, acsr_bin_workspace_bytes, acsr_hits_normalize,
+               acsr_hits_workspace_bytes, acsr_pagerank_scale, acsr_pagerank_step, acsr_plan_status, acsr_relayout,
+               acsr_spmv, acsr_update_edges, acsr_update_workspace_bytes)
 
 
 class ACSRMatrix:
@@ -38,6 +38,10 @@ class ACSRMatrix:
     def rebin(self, stream=None):
         acsr_bin(self.row_begin, self.row_end, self.nnz_max, self.bin_rows, self.bin_offsets,
                  self.plan_ws, stream, col_idx=self.col_idx, n_cols=self.n_cols, short_rows=self.short_rows)
+
+    def plan_status(self, stream=None):
+        """Synchronising check that the plan is valid (raises ACSRError otherwise)."""
+        acsr_plan_status(self.plan_ws, stream)
 
     def spmv(self, x, y=None, stream=None):
         return acsr_spmv(self.row_begin, self.col_idx, self.values, x, self.bin_rows,
@@ -188,6 +192,8 @@ def _power_loop(m: ACSRMatrix, outdeg, x, damping, teleport, eps, max_iter, chec
                 step(k)
                 k += 1
         c = ctrl.cpu()
+        if int(c[0]) == ACSR_CTRL_PLAN_ERROR:
+            acsr_plan_status(m.plan_ws, stream)  # raises: the plan is invalid (outputs are NaN)
         if int(c[0]):
             break
     it = int(c[1])

@@ -294,32 +294,16 @@ def test_spmv_ragged_sizes(acsr, cuda, n, mapping):
     check_spmv(y.numpy(), y_ref, den, torch.float64, exact=True)
 
 
-def sampled_parity(rp, ci, val, x, y, bins_check=None, n_random=4000, seed=0):
-    """Check y (host numpy) on a sample of rows -- random rows, the longest rows and the
-    first rows of every bin -- against the oracle computed row by row on the sample."""
-    rph = rp.cpu().numpy()
-    n = rph.size - 1
-    ln = np.diff(rph)
-    rng = np.random.default_rng(seed)
-    sample = set(rng.choice(n, min(n_random, n), replace=False).tolist()) | set(np.argsort(ln)[-50:].tolist())
-    if bins_check is not None:
-        br, off = bins_check
-        for b in range(32):
-            sample |= set(br[off[b]:off[b + 1]][:20].tolist())
-    rows = np.array(sorted(sample))
-    sub_rp = np.zeros(rows.size + 1, np.int64)
-    sub_rp[1:] = np.cumsum(ln[rows])
-    cih, vh = ci.cpu().numpy(), val.cpu().numpy()
-    sub_ci = np.concatenate([cih[rph[r]:rph[r + 1]] for r in rows])
-    sub_v = np.concatenate([vh[rph[r]:rph[r + 1]] for r in rows])
-    y_ref, den = oracle.spmv(sub_rp.astype(np.int32), sub_ci, sub_v, x.cpu().numpy())
-    check_spmv(y[rows], y_ref, den, val.dtype)
+def full_parity(rp, ci, val, x, y):
+    """Every row of y (host numpy) against the oracle on the whole matrix (Dot2, O4)."""
+    y_ref, den = oracle.spmv(rp.cpu().numpy(), ci.cpu().numpy(), val.cpu().numpy(), x.cpu().numpy())
+    check_spmv(y, y_ref, den, val.dtype)
 
 
 @pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
-def test_full_size_rmat20_sampled(acsr, cuda, dtype):
+def test_full_size_rmat20_every_row(acsr, cuda, dtype):
     """C2 at BASELINE size, in the launch configuration bench.py times: bins bitwise, and
-    sampled rows (every bin, the longest rows) against the oracle one by one."""
+    EVERY row against the oracle element by element."""
     rp, ci = synth.rmat_csr(20, device=cuda)
     n = rp.numel() - 1
     val = synth.values(ci.numel(), 1014, dtype, device=cuda)
@@ -329,12 +313,12 @@ def test_full_size_rmat20_sampled(acsr, cuda, dtype):
     br, off = oracle.bins(rp.cpu().numpy())
     assert np.array_equal(m.bin_offsets.cpu().numpy(), off)
     assert np.array_equal(m.bin_rows.cpu().numpy(), br)
-    sampled_parity(rp, ci, val, x, y, (br, off))
+    full_parity(rp, ci, val, x, y)
 
 
 @pytest.mark.parametrize("shape", ["WEB_GOOGLE", "LIVEJOURNAL"])
-def test_full_size_powerlaw_sampled(acsr, cuda, shape):
-    """C3 shapes at full size (0.9 M / 4.85 M rows): bins bitwise + sampled rows."""
+def test_full_size_powerlaw_every_row(acsr, cuda, shape):
+    """C3 shapes at full size (0.9 M / 4.85 M rows): bins bitwise + every row."""
     rp, ci = synth.powerlaw_csr(seed=3, device=cuda, **getattr(synth, shape))
     n = rp.numel() - 1
     val = synth.values(ci.numel(), 4, device=cuda)
@@ -343,7 +327,7 @@ def test_full_size_powerlaw_sampled(acsr, cuda, shape):
     y = m.spmv(x).cpu().numpy()
     br, off = oracle.bins(rp.cpu().numpy())
     assert np.array_equal(m.bin_rows.cpu().numpy(), br)
-    sampled_parity(rp, ci, val, x, y, (br, off), n_random=3000)
+    full_parity(rp, ci, val, x, y)
 
 
 def test_c1_rmat14_single_spmv(acsr, cuda):
@@ -407,12 +391,34 @@ def test_pagerank_converged_parity(acsr, cuda, scale):
     assert np.all(np.abs(x.cpu().numpy() - xr) <= 1e-11 * xr + 1e-18)
 
 
-def test_pagerank_s26_first_steps_sampled(acsr, cuda):
+def _oracle_pagerank_step_parallel(rph, cih, odh, xh, teleport, d, threads=None):
+    """The oracle step (O6) over every row, computed in row blocks by host threads (the
+    ctypes call releases the GIL; the step is row-independent, so blocks change no bit).
+    Each block passes the row offsets of its rows and the FULL col / outdeg / x arrays
+    (gathers use global ids).  Returns x' for all rows."""
+    from concurrent.futures import ThreadPoolExecutor
+    n = rph.size - 1
+    threads = threads or max(1, min(32, os.cpu_count() or 1))
+    cuts = np.linspace(0, n, 4 * threads + 1).astype(np.int64)
+    out = np.empty(n, np.float64)
+
+    def block(i):
+        r0, r1 = int(cuts[i]), int(cuts[i + 1])
+        if r1 > r0:
+            xn, _ = oracle.pagerank_step(rph[r0:r1 + 1], cih, odh, xh, teleport, d)
+            out[r0:r1] = xn
+
+    with ThreadPoolExecutor(threads) as ex:
+        list(ex.map(block, range(cuts.size - 1)))
+    return out
+
+
+def test_pagerank_s26_first_steps_every_row(acsr, cuda):
     """C4 at BASELINE size (R-MAT s26 in-link pattern: 67 M rows, ~1.06 B nnz), in the
     launch configuration bench.py times (one fused acsr_pagerank_step per iteration from
-    the cold start): bins bitwise, and for each of the first three steps the sampled rows
-    (random, the longest, the first rows of every bin) against the oracle step taken from
-    the same iterate ("at s26, check parity on the first 3 PageRank steps")."""
+    the cold start): bins bitwise, and for each of the first three steps EVERY row against
+    the oracle step taken from the same iterate ("at s26, check parity on the
+    first 3 PageRank steps in full"), plus x'/outdeg bitwise and Delta^2."""
     rp, ci = synth.rmat_csr(26, device=cuda, transpose=True)
     n = rp.numel() - 1
     od = torch.bincount(ci.long(), minlength=n).to(torch.int32)
@@ -421,16 +427,8 @@ def test_pagerank_s26_first_steps_sampled(acsr, cuda):
     br, off = oracle.bins(rph)
     assert np.array_equal(m.bin_offsets.cpu().numpy(), off)
     assert np.array_equal(m.bin_rows.cpu().numpy(), br)
-    ln = np.diff(rph)
-    rng = np.random.default_rng(26)
-    sample = set(rng.choice(n, 3000, replace=False).tolist()) | set(np.argsort(ln)[-20:].tolist())
-    for b in range(32):
-        sample |= set(br[off[b]:off[b + 1]][:10].tolist())
-    rows = np.array(sorted(sample))
-    sub_rp = np.zeros(rows.size + 1, np.int64)
-    sub_rp[1:] = np.cumsum(ln[rows])
-    idx = torch.cat([torch.arange(int(rph[r]), int(rph[r + 1]), device=cuda) for r in rows])
-    sub_ci = ci[idx].cpu().numpy()
+    del br
+    cih = ci.cpu().numpy()
     odh = od.cpu().numpy()
     teleport = (1.0 - 0.85) / n
     x = torch.full((n,), 1.0 / n, dtype=torch.float64, device=cuda)
@@ -441,13 +439,16 @@ def test_pagerank_s26_first_steps_sampled(acsr, cuda):
         acsr.acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xs, x, od,
                                 xn, xsn, d2, 0.85, teleport, n)
         xh = x.cpu().numpy()
-        ref, _ = oracle.pagerank_step(sub_rp.astype(np.int32), sub_ci, odh, xh, teleport, 0.85)
-        got = xn.cpu().numpy()[rows]
-        # step bar (fp64 O5): |err| <= 1e-12 * (teleport + d * sum |xs|), all terms >= 0
-        assert np.all(np.abs(got - ref) <= 1e-12 * ref), (step, np.max(np.abs(got - ref) / ref))
-        # the scaled vector the next step gathers is x'/outdeg (IEEE division)
-        xs_ref = np.where(odh[rows] > 0, got / np.maximum(odh[rows], 1), 0.0)
-        assert np.array_equal(xsn.cpu().numpy()[rows], xs_ref)
+        ref = _oracle_pagerank_step_parallel(rph, cih, odh, xh, teleport, 0.85)
+        got = xn.cpu().numpy()
+        # step bar (fp64 O5): |err| <= 1e-12 * (teleport + d * sum |xs|) = 1e-12 * ref (all >= 0)
+        bad = np.abs(got - ref) > 1e-12 * ref
+        assert not bad.any(), (step, np.flatnonzero(bad)[:10], np.max(np.abs(got - ref) / ref))
+        # the scaled vector the next step gathers is x'/outdeg (IEEE division): bitwise
+        xs_ref = np.where(odh > 0, got / np.maximum(odh, 1), 0.0)
+        assert np.array_equal(xsn.cpu().numpy(), xs_ref), step
+        # Delta^2 = sum (x' - x)^2 (exact fixed point on the GPU; compared to the oracle rows)
+        assert float(d2.item()) == pytest.approx(float(np.sum((ref - xh) ** 2)), rel=1e-9)
         x, xn = xn, x
         xs, xsn = xsn, xs
 
@@ -599,6 +600,37 @@ def test_update_rejections_leave_matrix_unchanged(acsr, cuda):
             assert torch.equal(a, b)
 
 
+def test_understated_nnz_max_is_loud(acsr, cuda):
+    """An nnz_max smaller than the stored entries overflows the plan's work list: the plan
+    is marked invalid, acsr_plan_status raises ACSR_ERR_CAPACITY, the SpMV writes NaN to
+    every row (never stale data) and a device-side PageRank loop stops with
+    ctrl[0] = ACSR_CTRL_PLAN_ERROR and Delta^2 = NaN (no silent failure)."""
+    n, L = 64, 20000
+    rp = torch.arange(n + 1, dtype=torch.int32) * L
+    ci = (torch.arange(n * L) % n).to(torch.int32)
+    x = torch.ones(n, dtype=torch.float64, device=cuda)
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda), None, nnz_max=1000)
+    with pytest.raises(acsr.ACSRError, match="ACSR_ERR_CAPACITY"):
+        m.plan_status()
+    y = torch.zeros(n, dtype=torch.float64, device=cuda)
+    m.spmv(x, y)
+    assert torch.isnan(y).all()
+    od = torch.full((n,), L, dtype=torch.int32, device=cuda)
+    with pytest.raises(acsr.ACSRError, match="ACSR_ERR_CAPACITY"):
+        acsr.pagerank(m, od)
+    xs = acsr.acsr_pagerank_scale(x / n, od)
+    xn, xsn = torch.zeros_like(x), torch.zeros_like(x)
+    d2 = torch.zeros(1, dtype=torch.float64, device=cuda)
+    ctrl = torch.zeros(2, dtype=torch.int32, device=cuda)
+    acsr.acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xs, x / n, od, xn, xsn,
+                            d2, ctrl=ctrl, eps2=1.0)
+    assert int(ctrl[0]) == acsr.ACSR_CTRL_PLAN_ERROR and torch.isnan(d2).all() and torch.isnan(xn).all()
+    # the same matrix with a correct bound is fine
+    m2 = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda), None)
+    m2.plan_status()
+    assert torch.equal(m2.spmv(x), torch.full((n,), float(L), dtype=torch.float64, device=cuda))
+
+
 def test_argument_errors(acsr, cuda):
     with pytest.raises(TypeError):
         acsr.acsr_bin(torch.zeros(3, dtype=torch.int32), None, nnz_max=0)  # CPU tensor
@@ -740,6 +772,35 @@ def test_hits_parity(acsr, cuda, scale):
         a_ref, h_ref, _ = oracle.hits(rp.numpy(), ci.numpy(), rpT.numpy(), ciT.numpy(), eps=0.0, max_iter=it)
     assert np.allclose(a.cpu().numpy(), a_ref, rtol=1e-9, atol=1e-15)
     assert np.allclose(h.cpu().numpy(), h_ref, rtol=1e-9, atol=1e-15)
+
+
+@pytest.mark.parametrize("scale", [12, 16])
+def test_hits_one_step_parity(acsr, cuda, scale):
+    """One HITS step (Eq. 5-7 + reading R6) from the same non-normalised iterate: the block
+    SpMV + acsr_hits_normalize against oracle.hits_step.  Bar (derived): y = [A^T h; A a]
+    has non-negative terms, so the SpMV bar 1e-12 * den is 1e-12 relative per entry; each
+    side's norm carries at most a gamma_n sequential error (n u relative on the squared
+    sum), so a', h' agree to (1e-12 + 2 n u) relative.  Distances to a far iterate to 1e-9."""
+    rp, ci = synth.rmat_csr(scale)
+    rpT, ciT = synth.rmat_csr(scale, transpose=True)
+    n = rp.numel() - 1
+    a = synth.vector(n, 71).abs().numpy()
+    h = synth.vector(n, 72).abs().numpy()
+    a_ref, h_ref, d2_ref = oracle.hits_step(rp.numpy(), ci.numpy(), rpT.numpy(), ciT.numpy(), a, h)
+    bp, bc = acsr.hits_matrix(rp.to(cuda), ci.to(cuda), n)
+    B = acsr.ACSRMatrix(bp, bc, None, n_cols=2 * n)
+    v = torch.from_numpy(np.concatenate([a, h])).to(cuda)
+    y = B.spmv(v)
+    vn = torch.empty_like(v)
+    d2 = torch.zeros(2, dtype=torch.float64, device=cuda)
+    ws = torch.empty(acsr.acsr_hits_workspace_bytes(n), dtype=torch.uint8, device=cuda)
+    acsr.acsr_hits_normalize(y, v, vn, d2, ws)
+    got = vn.cpu().numpy()
+    tol = 1e-12 + 2 * n * 2.0 ** -53
+    for g, r in ((got[:n], a_ref), (got[n:], h_ref)):
+        assert np.all(np.abs(g - r) <= tol * r + 1e-300)
+        assert np.array_equal(g == 0.0, r == 0.0)
+    assert d2.cpu().numpy() == pytest.approx(d2_ref, rel=1e-9)
 
 
 def test_degree_relabel_pagerank_equivalent(acsr, cuda):

@@ -138,3 +138,68 @@ def test_empty_matrix_and_plain_threads():
     assert np.array_equal(y1, y4)  # same per-row order regardless of threads
     yd, den = oracle.spmv(rp, ci, v, x)
     assert np.all(np.abs(y1 - yd) <= 1e-12 * den)
+
+
+# ---------------------------------------------------------------------- fp32 pins (round 2)
+def _rand_csr32(n, m, density, seed, integer):
+    A, rp, ci, v = _rand_csr(n, m, density, seed, integer=integer)
+    return A.astype(np.float32), rp, ci, v.astype(np.float32)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_fp32_den_exact_on_integer_data(seed):
+    """oracle_spmv_f32's den (the denominator of every fp32 parity bar, reading Q16) equals
+    |A| @ |x| exactly on integer data (every partial sum is an exact small integer)."""
+    A, rp, ci, v = _rand_csr32(64, 48, 0.3, seed, integer=True)
+    x = np.random.default_rng(300 + seed).integers(-8, 9, 48).astype(np.float32)
+    y, den = oracle.spmv(rp, ci, v, x)
+    assert np.array_equal(den, np.abs(A.astype(np.float64)) @ np.abs(x.astype(np.float64)))
+    ref = np.array([sum(int(A[i, j]) * int(x[j]) for j in range(48)) for i in range(64)], np.float32)
+    assert np.array_equal(y, ref)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_fp32_den_matches_fsum_on_float_data(seed):
+    """den on U(-1,1) float data: the exact sum of |a||x| (fractions) within n*u relative
+    (it is a plain double accumulation of exact non-negative products)."""
+    A, rp, ci, v = _rand_csr32(30, 400, 0.5, seed, integer=False)
+    x = np.random.default_rng(9 + seed).uniform(-1, 1, 400).astype(np.float32)
+    _, den = oracle.spmv(rp, ci, v, x)
+    for i in range(30):
+        ex = sum(abs(Fraction(float(v[k])) * Fraction(float(x[ci[k]]))) for k in range(rp[i], rp[i + 1]))
+        assert abs(Fraction(float(den[i])) - ex) <= Fraction(400) * Fraction(U64) * ex, i
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_fp32_plain_is_double_sum_rounded_once(seed):
+    """oracle_spmv_plain_f32 (the bitwise checker of the GPU's fp32 window rows): float
+    products are exact in double, summed in double, rounded once to float.  Pinned
+    against the exact rational row sum: |y - exact| <= ulp32(exact)/2 + n u64 sum|p|."""
+    A, rp, ci, v = _rand_csr32(40, 300, 0.5, seed, integer=False)
+    x = np.random.default_rng(21 + seed).uniform(-1, 1, 300).astype(np.float32)
+    y = oracle.spmv_plain(rp, ci, v, x)
+    assert y.dtype == np.float32
+    for i in range(40):
+        terms = [Fraction(float(v[k])) * Fraction(float(x[ci[k]])) for k in range(rp[i], rp[i + 1])]
+        ex = sum(terms, Fraction(0))
+        absum = sum((abs(t) for t in terms), Fraction(0))
+        half_ulp = Fraction(float(np.spacing(np.float32(abs(float(ex)))))) / 2
+        assert abs(Fraction(float(y[i])) - ex) <= half_ulp * Fraction(1001, 1000) + len(terms) * Fraction(U64) * absum, i
+
+
+def test_fp32_plain_integer_exact_and_in_element_order():
+    """Integer data: exact.  Element order: with p = (2^60, 1, -2^60) a left-to-right double
+    sum gives 0 (2^60 + 1 rounds to 2^60), while (2^60, -2^60, 1) gives 1 -- IEEE facts,
+    so the in-order reading of the window-row checker is pinned, not re-typed."""
+    A, rp, ci, v = _rand_csr32(64, 48, 0.3, 5, integer=True)
+    x = np.random.default_rng(305).integers(-8, 9, 48).astype(np.float32)
+    y = oracle.spmv_plain(rp, ci, v, x)
+    assert np.array_equal(y, (A.astype(np.float64) @ x.astype(np.float64)).astype(np.float32))
+    big = np.float32(2.0 ** 60)
+    rp2 = np.array([0, 3, 6], np.int32)
+    ci2 = np.zeros(6, np.int32)
+    v2 = np.array([big, 1, -big, big, -big, 1], np.float32)
+    y2 = oracle.spmv_plain(rp2, ci2, v2, np.ones(1, np.float32))
+    assert y2[0] == 0.0 and y2[1] == 1.0
+    y64 = oracle.spmv_plain(rp2, ci2, v2.astype(np.float64), np.ones(1))
+    assert y64[0] == 0.0 and y64[1] == 1.0

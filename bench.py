@@ -12,10 +12,15 @@ L2 is flushed (256 MiB write) between timed steps, outside the step's events.
                   [--workload rmat20|rmat20_f32|webgoogle|livejournal|rmat20_split|pagerank|
                               pagerank_dist|dynamic|dynamic_mixed|hits|rwr]
 
-With N > 1 (torchrun) every rank runs its own independent matrix (seed + rank): the
-units are independent problems, no data-path collective, scaling "weak"; the time is
-the max over ranks.  `--impl reference` times the CPU oracle (plain sequential C) on
-the same workload (rank 0 only).
+With N > 1 (torchrun) the default workload is the SAME C2 matrix row-split across the
+ranks (§VIII, reading Q19: contiguous nnz-balanced row ranges from acsr_partition,
+every rank bins its rows and runs acsr_spmv on them; y stays distributed) -- one problem
+at every N (strong scaling), the time is the max over ranks.  `--replicas` restores the
+old independent-matrix-per-rank mode.  Every default line also carries a `pagerank_dist`
+record: C4 (R-MAT s26 in-link PageRank) row-partitioned over the N ranks with the
+library-owned NCCL exchange (acsr_comm) and with the fused peer-memory exchange, against
+SURVEY §8(e)'s bound max(T1/P, T_comm).  `--impl reference` times the CPU oracle (plain
+sequential C) on the same workload (rank 0 only).
 """
 from __future__ import annotations
 
@@ -222,13 +227,22 @@ def read_stream_gbs(dev, gib=2, reps=5):
 HBM_SPEC_GBS = 8000.0  # B200 HBM3e nominal (the north star's denominator)
 
 
-def algorithmic_bytes(rp, ci, dtype):
+def algorithmic_bytes(rp, ci, dtype, n_cols=None):
     """(s_v+4) nnz + 4(n+1) row_ptr + 4n bin_rows + s_v n_c x + s_v n y."""
     n = rp.numel() - 1
     nnz = ci.numel()
     sv = 8 if dtype == torch.float64 else 4
-    n_c = int((torch.bincount(ci.long(), minlength=n) > 0).sum())
+    n_c = int((torch.bincount(ci.long(), minlength=n if n_cols is None else n_cols) > 0).sum())
     return (sv + 4) * nnz + 4 * (n + 1) + 4 * n + sv * n_c + sv * n, n_c
+
+
+def workload_config(label, n, nnz, world, replicas=False):
+    """The `config` of the default line: identical keys and values at every N (and in the
+    reference arm), so the driver can match the lines."""
+    return {"workload": label, "n_rows": n, "nnz": nnz,
+            "l2": "flushed: 256 MiB write between timed steps (outside the step events)",
+            "parallelism": (f"independent matrix per rank x{world} (weak)" if replicas
+                            else f"row-split x{world} (P:345)" if world > 1 else "1 GPU")}
 
 
 def ncu_traffic(label):
@@ -242,21 +256,42 @@ def ncu_traffic(label):
 
 
 # ------------------------------------------------------------------------------ acsr arm
+def row_split(rp, ci, val, rank, world, b_nnz, b_row):
+    """This rank's rows [splits[rank], splits[rank+1]) of one CSR (acsr_partition, O8),
+    col/val copied with their global 16-byte phase (dist.aligned_slice) so every row is
+    summed as on one GPU.  Returns (row_ptr_local, col_local, val_local, splits)."""
+    import paper_conf_sc_ashariseps14_b200 as acsr
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+    splits = acsr.acsr_partition(rp, world, b_nnz, b_row).cpu().numpy()
+    lo, hi = int(splits[rank]), int(splits[rank + 1])
+    k0, k1 = int(rp[lo]), int(rp[hi])
+    rpl = (rp[lo:hi + 1].to(torch.int64) - k0).to(torch.int32)
+    cil = pdist.aligned_slice(ci, k0, k1, 4)
+    vl = None if val is None else pdist.aligned_slice(val, k0, k1, 16 // val.element_size())
+    return rpl, cil, vl, splits
+
+
 def run_acsr(args, dev, rank, world):
     import paper_conf_sc_ashariseps14_b200 as acsr
 
-    label, dtype, rp, ci, val, x = make_workload(args.workload, dev, rank)
+    replicas = args.replicas and world > 1
+    label, dtype, rp, ci, val, x = make_workload(args.workload, dev, rank if replicas else 0)
+    n_glob, nnz_glob = rp.numel() - 1, ci.numel()
+    splits = None
+    if world > 1 and not replicas:  # one matrix, row-split (P:345): this rank's rows
+        rp, ci, val, splits = row_split(rp, ci, val, rank, world, 4 + val.element_size(), 16)
+        torch.cuda.empty_cache()
     n, nnz = rp.numel() - 1, ci.numel()
-    alg_bytes, n_c = algorithmic_bytes(rp, ci, dtype)
+    alg_bytes, n_c = algorithmic_bytes(rp, ci, dtype, n_cols=x.numel())
     stream = torch.cuda.current_stream()
     br = torch.empty(n, dtype=torch.int32, device=dev)
     bo = torch.empty(33, dtype=torch.int32, device=dev)
-    ws = torch.empty(acsr.acsr_bin_workspace_bytes(n, n, nnz), dtype=torch.uint8, device=dev)
+    ws = torch.empty(acsr.acsr_bin_workspace_bytes(n, x.numel(), nnz), dtype=torch.uint8, device=dev)
     y = torch.empty(n, dtype=dtype, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
     def step():
-        acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=n)
+        acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=x.numel())
         acsr.acsr_spmv(rp, ci, val, x, br, bo, ws, None, y)
 
     for _ in range(args.warmup):
@@ -273,7 +308,7 @@ def run_acsr(args, dev, rank, world):
         for k in range(K):
             flush.zero_()
             ev[k][0].record(stream)
-            acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=n)
+            acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=x.numel())
             ev[k][1].record(stream)
             acsr.acsr_spmv(rp, ci, val, x, br, bo, ws, None, y)
             ev[k][2].record(stream)
@@ -322,7 +357,7 @@ def run_acsr(args, dev, rank, world):
     x_d = torch.empty_like(x)
     for _ in range(2):
         x_d.copy_(x_h, non_blocking=True)
-        acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=n)
+        acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=x.numel())
         acsr.acsr_spmv(rp, ci, val, x_d, br, bo, ws, None, y)
         y_h.copy_(y, non_blocking=True)
     torch.cuda.synchronize()
@@ -330,7 +365,7 @@ def run_acsr(args, dev, rank, world):
     r0.record(stream)
     for _ in range(ke):
         x_d.copy_(x_h, non_blocking=True)
-        acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=n)
+        acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=x.numel())
         acsr.acsr_spmv(rp, ci, val, x_d, br, bo, ws, None, y)
         y_h.copy_(y, non_blocking=True)
     r1.record(stream)
@@ -361,21 +396,23 @@ def run_acsr(args, dev, rank, world):
             tg.append(g0.elapsed_time(g1))
     t_gather = float(np.median(tg))
     del g_out
+    c4 = None if args.no_c4 else pagerank_dist_record(args, dev, rank, world)
     if rank != 0:
         return None
     peak, peak_kind = peaks()
-    gflops = 2.0 * nnz * K * world / (tot * 1e-3) / 1e9
+    units = nnz * world if replicas else nnz_glob  # nnz multiplied per step by the whole job
+    gflops = 2.0 * units * K / (tot * 1e-3) / 1e9
     spmv_ms = float(t_spmv.mean())
     achieved = alg_bytes / (spmv_ms * 1e-3) / 1e9
     line = {
         "metric": "SpMV GFLOP/s (bin+SpMV per step) & HBM GB/s vs peak",
         "value": round(gflops, 3), "unit": "GFLOP/s", "n_gpus": world, "steps": K, "warmup": args.warmup,
-        "ms_per_step": round(tot / K, 5), "higher_is_better": True, "scaling": "weak",
+        "ms_per_step": round(tot / K, 5), "higher_is_better": True, "scaling": "weak" if replicas else "strong",
         "vs_baseline": None, "dtype": "f64" if dtype == torch.float64 else "f32", "data": "synthetic",
-        "config": {"workload": label, "n_rows": n, "nnz": nnz, "referenced_cols": n_c,
-                   "l2": "flushed: 256 MiB write between timed steps (outside the step events)",
-                   "parallelism": "independent matrix per rank (weak)" if world > 1 else "1 GPU"},
-        "breakdown": {"t_bin_ms": round(float(t_bin.mean()), 5), "t_spmv_ms": round(spmv_ms, 5),
+        "config": workload_config(label, n_glob, nnz_glob, world, replicas),
+        "breakdown": {"rank0_rows": n, "rank0_nnz": nnz, "rank0_referenced_cols": n_c,
+                      "splits": None if splits is None else [int(v) for v in splits],
+                      "t_bin_ms": round(float(t_bin.mean()), 5), "t_spmv_ms": round(spmv_ms, 5),
                       "pt_st": round(float(t_bin.mean()) / spmv_ms, 3),
                       "spmv_gflops": round(2.0 * nnz / (spmv_ms * 1e-3) / 1e9, 2),
                       "t_spmv_min_ms": round(float(t_spmv.min()), 5),
@@ -387,8 +424,9 @@ def run_acsr(args, dev, rank, world):
                                           "nnz random gathers + col read + nnz-value write, no row sums",
                       "spmv_over_gather_pass": round(spmv_ms / t_gather, 3),
                       "gather_roofline_ms": round(nnz / 197e9 * 1e3, 5),
-                      "gather_roofline_note": "pure random 8-byte gathers from an L2-resident x run at ~197 G/s "
-                                              "on this B200 (profiles/r1_gather_bench.jsonl); one gather per nnz"},
+                      "gather_roofline_note": "pure random 8-byte gathers from an L2-resident x run at ~198 G/s "
+                                              "on this B200, limited by the L1TEX->XBAR request interface "
+                                              "(profiles/r2_gather_limiter.json); one gather per nnz"},
         "context": ctx,
         "bins": bstats,
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
@@ -399,18 +437,20 @@ def run_acsr(args, dev, rank, world):
                                         "frac_vs_read_stream": round(achieved / rs, 4),
                                         "spec_gbs": HBM_SPEC_GBS,
                                         "frac_vs_spec": round(achieved / HBM_SPEC_GBS, 4)}},
-        "e2e": {"value": round(2.0 * nnz * world / (t_e2e * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
+        "e2e": {"value": round(2.0 * units / (t_e2e * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
                 "h2d_bytes_per_step": int(h2d) * world, "d2h_bytes_per_step": int(d2h) * world,
                 "ms_per_step": round(t_e2e, 4),
                 "note": "whole CSR + x uploaded every step (PCIe-bound); resident_matrix: CSR kept in HBM, "
                         "x in / y out per step",
-                "resident_matrix": {"value": round(2.0 * nnz * world / (t_res * 1e-3) / 1e9, 3),
+                "resident_matrix": {"value": round(2.0 * units / (t_res * 1e-3) / 1e9, 3),
                                     "unit": "GFLOP/s", "ms_per_step": round(t_res, 4),
                                     "h2d_bytes_per_step": int(x_h.numel() * x_h.element_size()) * world,
                                     "d2h_bytes_per_step": int(d2h) * world}},
         "gpu_launches": 4 * K * world,  # per step and rank: bin_count, bin_scan, bin_scatter, spmv_kernel
         "clocks": clk.summary(),
     }
+    if c4 is not None:
+        line["pagerank_dist"] = c4
     if not args.no_cpu_baseline and world == 1:  # the oracle baseline: rank 0 at N = 1 only
         line["cpu_baseline"] = cpu_baseline(rp, ci, val, x, dtype)
     return line
@@ -483,12 +523,19 @@ def run_pagerank(args, dev, rank, world):
     n, nnz = rp.numel() - 1, ci.numel()
     outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
     t_relabel = None
-    if args.relabel:
+    if args.relabel:  # acsr_degree_relabel on the device (sort + scan + copy), timed with events
+        for _ in range(2):
+            acsr.acsr_degree_relabel(rp, ci, outdeg)
         torch.cuda.synchronize()
-        t0 = time.perf_counter()
-        rp, ci, outdeg, _ = acsr.degree_relabel(rp, ci, outdeg)
+        r0, r1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        r0.record()
+        rp2, ci2, od2, _ = acsr.acsr_degree_relabel(rp, ci, outdeg)
+        r1.record()
         torch.cuda.synchronize()
-        t_relabel = time.perf_counter() - t0
+        t_relabel = r0.elapsed_time(r1) * 1e-3
+        rp, ci, outdeg = rp2, ci2, od2
+        del rp2, ci2, od2
+        torch.cuda.empty_cache()
     n_nd = int((outdeg > 0).sum())
     m = acsr.ACSRMatrix(rp, ci)
     torch.cuda.synchronize()
@@ -544,11 +591,14 @@ def run_pagerank(args, dev, rank, world):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"pagerank_rmat{S}_inlink" + ("_degree_relabelled" if args.relabel else ""),
                        "n_rows": n, "nnz": nnz, "non_dangling": n_nd,
-                       "relabel_s": None if t_relabel is None else round(t_relabel, 3),
+                       "relabel": "acsr_degree_relabel (device)" if args.relabel else None,
                        "l2": "not flushed (iterative use); x = %d MB" % (8 * n >> 20),
                        "parallelism": "independent replica per rank" if world > 1 else "1 GPU"},
             "breakdown": {"t_bin_ms": round(t_bin, 4), "cold_iterations": it, "final_delta": dd ** 0.5,
                           "cold_run_ms": round(t_conv * 1e3, 3),
+                          "relabel_ms": None if t_relabel is None else round(t_relabel * 1e3, 3),
+                          "cold_solve_incl_relabel_and_bin_ms": None if t_relabel is None else
+                          round((t_relabel + t_conv) * 1e3 + t_bin, 3),
                           "gflops_equiv": round(nnz / (ms * 1e-3) / 1e9, 2)},
             "roofline": {"bound": "hbm", "achieved": round(alg / (ms * 1e-3) / 1e9, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(alg / (ms * 1e-3) / 1e9 / peak, 4), "traffic": None,
@@ -673,6 +723,115 @@ def run_pagerank_dist(args, dev, rank, world):
                        "exchange_layout": "non-dangling only (lossless)" if pr.compact else "all vertices",
                        "exchange": args.exchange},
             "gpu_launches": K * (2 if args.exchange == "peer" else 1), "clocks": clk.summary()}
+
+
+def _max_over_ranks(vals, dev, world):
+    if world == 1:
+        return [float(v) for v in vals]
+    t = torch.tensor([float(v) for v in vals], dtype=torch.float64, device=dev)
+    torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+    return [float(v) for v in t.tolist()]
+
+
+def pagerank_dist_record(args, dev, rank, world):
+    """C4 (BASELINE configs[3]): PageRank on the R-MAT s26 in-link pattern, row-partitioned
+    over the N ranks (acsr_partition, cost 4 len + 36), compact non-dangling exchange
+    layout, timed for K iterations with each exchange:
+      acsr  -- acsr_pagerank_step with the library's NCCL communicator (all-gather of the
+               xs slices + exact global Delta^2, device-side stop flag);
+      peer  -- the exchange fused into the step over CUDA-IPC peer memory (N1).
+    Also T1 (the whole graph on rank 0's GPU alone, measured in the same job), T_comm (the
+    same all-gather alone) and frac_of_bound = max(T1/P, T_comm) / T."""
+    import paper_conf_sc_ashariseps14_b200 as acsr
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+
+    S = args.c4_scale
+    K = max(3, min(args.steps, 10))
+    torch.cuda.synchronize()
+    g0 = time.perf_counter()
+    rp, ci = synth.rmat_csr(S, device=dev, transpose=True)
+    n, nnz = rp.numel() - 1, ci.numel()
+    outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    torch.cuda.synchronize()
+    t_gen = time.perf_counter() - g0
+    # T1: one GPU, whole graph (rank 0; the other ranks wait at the barrier)
+    t1 = None
+    if rank == 0:
+        m = acsr.ACSRMatrix(rp, ci)
+        x = torch.full((n,), 1.0 / n, dtype=torch.float64, device=dev)
+        xs = acsr.acsr_pagerank_scale(x, outdeg)
+        xn, xsn = torch.empty_like(x), torch.empty_like(x)
+        d2 = torch.zeros(1, dtype=torch.float64, device=dev)
+        args_ = (m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws)
+        for _ in range(2):
+            acsr.acsr_pagerank_step(*args_, xs, x, outdeg, xn, xsn, d2, 0.85, 0.15 / n, n)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(K):
+            acsr.acsr_pagerank_step(*args_, xs, x, outdeg, xn, xsn, d2, 0.85, 0.15 / n, n)
+        e1.record()
+        torch.cuda.synchronize()
+        t1 = e0.elapsed_time(e1) / K
+        del m, x, xs, xn, xsn
+        torch.cuda.empty_cache()
+    if world > 1:
+        torch.distributed.barrier()
+    splits = acsr.acsr_partition(rp, world, 4, 36).cpu().numpy()
+    lo, hi = int(splits[rank]), int(splits[rank + 1])
+    rpl = (rp[lo:hi + 1].to(torch.int64) - int(rp[lo])).to(torch.int32)
+    cil = ci[int(rp[lo]):int(rp[hi])].clone()
+    odl = outdeg[lo:hi].clone()
+    nnz_local = cil.numel()
+    del rp, ci
+    torch.cuda.empty_cache()
+    out = {"workload": f"pagerank_rmat{S}_inlink_partitioned", "n_rows": n, "nnz": nnz,
+           "generate_s": round(t_gen, 2), "iterations_timed": K, "splits": [int(v) for v in splits],
+           "t1_ms": None if t1 is None else round(t1, 4)}
+    comm = acsr.AcsrComm.from_process_group() if world > 1 else None
+    for ex in ("acsr", "peer"):
+        pr = pdist.DistPageRank(rpl, cil, odl, splits, n, exchange=ex, comm=comm)
+        pr.run(max_iter=2, eps=0.0)
+        torch.cuda.synchronize()
+        if world > 1:
+            torch.distributed.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        pr.run(eps=0.0, max_iter=K, check_every=K)
+        e1.record()
+        torch.cuda.synchronize()
+        ms = _max_over_ranks([e0.elapsed_time(e1) / K], dev, world)[0]
+        rec = {"ms_per_iter": round(ms, 4), "gteps": round(nnz / (ms * 1e-3) / 1e9, 2),
+               "exchange_slice": pr.Lx, "exchange_bytes_in_per_rank_per_iter": pr.exchange_bytes_per_rank()}
+        if ex == "acsr" and world > 1:
+            # T_comm: the same in-place all-gather alone (NCCL over NVLink), K times
+            buf = torch.zeros(world * pr.Lx, dtype=torch.float64, device=dev)
+            mine = buf[rank * pr.Lx:(rank + 1) * pr.Lx]
+            pr.comm.allgather(mine, buf)
+            torch.cuda.synchronize()
+            c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            c0.record()
+            for _ in range(K):
+                pr.comm.allgather(mine, buf)
+            c1.record()
+            torch.cuda.synchronize()
+            rec["t_comm_ms"] = round(_max_over_ranks([c0.elapsed_time(c1) / K], dev, world)[0], 4)
+            del buf
+        if ex == "peer" and pr.peer is not None:
+            pr.peer.close()
+        out[ex] = rec
+        del pr
+        torch.cuda.empty_cache()
+    if comm is not None:
+        comm.close()
+    if rank == 0:
+        t_comm = out["acsr"].get("t_comm_ms", 0.0)
+        bound = max(t1 / world, t_comm)
+        out["bound_ms"] = round(bound, 4)
+        out["bound_note"] = "SURVEY §8(e): max(T1/P, T_comm), T1 = whole graph on one GPU, T_comm = the all-gather alone"
+        for ex in ("acsr", "peer"):
+            out[ex]["frac_of_bound"] = round(bound / out[ex]["ms_per_iter"], 4)
+            out[ex]["speedup_vs_t1"] = round(t1 / out[ex]["ms_per_iter"], 3)
+    return out
 
 
 def run_hits_rwr(args, dev, rank, world):
@@ -948,15 +1107,19 @@ def run_reference(args, dev):
     v = 2.0 * cih.size / dt / 1e9
     return {"metric": "SpMV GFLOP/s (bin+SpMV per step) & HBM GB/s vs peak", "impl": "reference",
             "value": round(v, 4), "unit": "GFLOP/s", "n_gpus": int(os.environ.get("WORLD_SIZE", "1")), "steps": K, "warmup": args.warmup,
-            "ms_per_step": round(dt * 1e3, 3), "higher_is_better": True, "scaling": "weak",
+            "ms_per_step": round(dt * 1e3, 3), "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64" if dtype == torch.float64 else "f32", "data": "synthetic",
-            "config": {"workload": label, "n_rows": int(rph.size - 1), "nnz": int(cih.size)},
+            "config": workload_config(label, int(rph.size - 1), int(cih.size), int(os.environ.get("WORLD_SIZE", "1"))),
             "cpu_baseline": {"value": round(v, 4), "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
                              "sample": f"whole matrix per step: oracle bins (O3) + plain SpMV (O4'), {K} steps"},
             "e2e": {"value": round(v, 4), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
 
 
 def main():
+    wd = os.environ.get("ACSR_BENCH_WATCHDOG")  # debugging: dump every thread's stack and exit after N s
+    if wd:
+        import faulthandler
+        faulthandler.dump_traceback_later(float(wd), exit=True)
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=50)
@@ -967,9 +1130,13 @@ def main():
     ap.add_argument("--scale", type=int, default=None, help="R-MAT scale for pagerank/dynamic")
     ap.add_argument("--batches", type=int, default=None, help="dynamic: number of insertion batches")
     ap.add_argument("--relabel", action="store_true", help="pagerank: degree-ordered vertex relabelling")
-    ap.add_argument("--exchange", default="nccl", choices=["nccl", "peer"],
-                    help="pagerank_dist: NCCL all-gather after the step, or the exchange fused into the "
-                         "step over peer memory (acsr_pagerank_step_peer)")
+    ap.add_argument("--exchange", default="acsr", choices=["acsr", "torch", "peer"],
+                    help="pagerank_dist: the library's NCCL exchange inside acsr_pagerank_step (acsr_comm), "
+                         "torch.distributed collectives, or the exchange fused into the step over peer memory")
+    ap.add_argument("--replicas", action="store_true",
+                    help="N > 1: independent matrix per rank (weak) instead of one row-split matrix")
+    ap.add_argument("--no-c4", action="store_true", help="skip the pagerank_dist (C4) record of the default line")
+    ap.add_argument("--c4-scale", type=int, default=26, help="R-MAT scale of the pagerank_dist record")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -985,6 +1152,11 @@ def main():
     local_dev = local % max(ndev, 1)  # (ranks > GPUs only in the single-GPU test of this path)
     torch.cuda.set_device(local_dev)
     dev = torch.device("cuda", local_dev)
+    if world > 1 and os.environ.get("ACSR_SHARED_GPU_TEST") == "1":
+        # test-only: several ranks on ONE GPU.  NCCL refuses two ranks on one device of one
+        # host, so each rank claims its own host id and NCCL talks over loopback sockets.
+        os.environ.update(NCCL_HOSTID=f"acsr-test-host-{rank}", NCCL_SOCKET_IFNAME="lo", NCCL_IB_DISABLE="1",
+                          NCCL_P2P_DISABLE="1", NCCL_SHM_DISABLE="1", NCCL_NVLS_ENABLE="0")
     if world > 1:
         backend = os.environ.get("ACSR_DIST_BACKEND", "nccl")  # gloo: test the path on one GPU
         if backend == "nccl":

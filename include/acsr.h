@@ -39,7 +39,7 @@ typedef enum {
     ACSR_ERR_WORKSPACE = 2,     /* workspace pointer NULL or smaller than the query */
     ACSR_ERR_CAPACITY = 3,      /* (device status) an updated row exceeds its reserved slack */
     ACSR_ERR_CUDA = 4,          /* CUDA launch / runtime failure, see acsr_last_error() */
-    ACSR_ERR_NCCL = 5,          /* reserved for the NCCL exchange (multi-GPU) */
+    ACSR_ERR_NCCL = 5,          /* NCCL failure in the multi-GPU exchange, see acsr_last_error() */
     ACSR_ERR_UNSUPPORTED = 6    /* e.g. no sm_100 device */
 } acsr_status;
 
@@ -138,6 +138,40 @@ acsr_status acsr_spmv(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
                       void *plan_ws, size_t plan_ws_bytes, cudaStream_t stream);
 
 /* ------------------------------------------------------------------------ */
+/* Multi-GPU communicator (§VIII: "map half of the rows ... to each device.  Each
+ * GPU is thus responsible for computing half the results", generalised to P ranks as
+ * contiguous row ranges, reading Q19).  One rank per GPU (one process per GPU, a single
+ * node: NCCL over NVLink / NVSwitch).  The library owns the NCCL communicator and a small
+ * device buffer; nothing else.  Protocol: rank 0 calls acsr_comm_get_unique_id and ships
+ * the ACSR_COMM_ID_BYTES HOST bytes to every rank (any host transport); every rank then
+ * calls acsr_comm_init with the SAME CUDA device current that it will use for the steps.
+ * acsr_comm_init blocks until all nranks ranks joined.  NCCL failures return
+ * ACSR_ERR_NCCL with the NCCL text in acsr_last_error(). */
+enum { ACSR_COMM_ID_BYTES = 128 };
+typedef struct acsr_comm acsr_comm;
+acsr_status acsr_comm_get_unique_id(void *id /* HOST out, ACSR_COMM_ID_BYTES */);
+acsr_status acsr_comm_init(acsr_comm **out, int nranks, int rank, const void *id /* HOST */);
+acsr_status acsr_comm_destroy(acsr_comm *comm);
+acsr_status acsr_comm_query(const acsr_comm *comm, int *nranks /* HOST out, nullable */,
+                            int *rank /* HOST out, nullable */);
+/* recv[q * bytes_per_rank ...] = rank q's send (in place allowed: send == recv + rank *
+ * bytes_per_rank).  For setup-time layout work (e.g. the non-dangling masks of the compact
+ * exchange layout, handles) and for gathering a row-split SpMV's y slices. */
+acsr_status acsr_comm_allgather(acsr_comm *comm, const void *send, void *recv, size_t bytes_per_rank,
+                                cudaStream_t stream);
+
+/* O8 row partition, on the device: splits[0] = 0, splits[nranks] = n_rows and
+ *   splits[k] = min{ r : sum_{r' < r} cost(r') >= ceil(k * total / nranks) },
+ *   cost(r) = b_nnz * len_r + b_row   (integer bytes of the rank's traffic per row:
+ *   PageRank pattern 4 * len + 36, weighted fp64 SpMV 12 * len + 16).
+ * splits: DEVICE int64 [nranks + 1].  ws: acsr_partition_workspace_bytes(n_rows) bytes
+ * (an int64 prefix of the costs + the scan's scratch). */
+size_t acsr_partition_workspace_bytes(int64_t n_rows);
+acsr_status acsr_partition(int64_t n_rows, const int32_t *row_begin, const int32_t *row_end /* NULL => standard */,
+                           int64_t b_nnz, int64_t b_row, int nranks, int64_t *splits, void *ws, size_t ws_bytes,
+                           cudaStream_t stream);
+
+/* ------------------------------------------------------------------------ */
 /* PageRank step (Alg. 5; §VI-A) on one rank's rows.
  *   PR^{k+1} = (1-d) PR^(0) + d (A^T PR^k),  A row-normalised.
  * Storage (reading Q12): the IN-LINK pattern CSR (row v lists the sources u of
@@ -147,9 +181,20 @@ acsr_status acsr_spmv(acsr_dtype dt, int64_t n_rows, int64_t n_cols,
  *   x_new[v]   = teleport + damping * y_v          (teleport = (1-d)/n, host)
  *   xs_next[v] = outdeg[v] > 0 ? x_new[v] / outdeg[v] : 0
  *   *delta2    = sum_v (x_new[v] - x[v])^2          (deterministic order)
- * Multi-GPU (§VIII, reading Q19): each rank calls this on its contiguous
- * row range and then all-gathers xs_next (caller side, torch.distributed/NCCL);
- * col ids index the replicated xs. */
+ * Multi-GPU (§VIII, reading Q19): each rank calls this on its contiguous row range
+ * (col ids index the replicated xs) with `comm` set.  The call then also runs the
+ * exchange on `stream`, right after the step kernel (A9 of SURVEY §8(a)):
+ *   xs_all[q * slice_len + i] = rank q's xs_next[i], i < slice_len   (ncclAllGather; in
+ *       place when xs_next == xs_all + rank * slice_len; xs_next must hold >= slice_len
+ *       entries -- entries i >= n_rows are padding the caller keeps at 0 -- and a rank
+ *       may exchange fewer than n_rows entries, e.g. only its non-dangling prefix);
+ *   *delta2 = the GLOBAL sum of (x_new - x)^2 over every rank's rows: the ranks' exact
+ *       192-bit fixed-point partials are all-gathered and added in rank order, so every
+ *       rank gets the same bits -- equal to the single-GPU Delta^2 of the same iterate;
+ *   ctrl (if given): the stop decision is taken on the global Delta^2, identically on
+ *       every rank, so device-side loops stay in lock step.
+ * Every rank must issue the same sequence of calls.  xs_all is the xs of the NEXT step
+ * (double-buffer xs / xs_all across steps). */
 typedef struct {
     int64_t n_rows;               /* local rows */
     int64_t n_cols;               /* length of xs (global, possibly padded) */
@@ -177,9 +222,18 @@ typedef struct {
                                    * between synchronisations with results identical to a
                                    * test after every step (single GPU). */
     double eps2;                  /* convergence threshold on delta2 (eps^2) */
+    acsr_comm *comm;              /* NULL => single GPU, no exchange; else see above */
+    double *xs_all;               /* with comm: [n_cols] replicated xs' receiving every slice */
+    int64_t slice_len;            /* with comm: entries per rank in xs_all (n_cols >= nranks * slice_len) */
 } acsr_pr_args;
 
 acsr_status acsr_pagerank_step(const acsr_pr_args *args, cudaStream_t stream);
+
+/* First iterate of Alg. 5 (PR^(0) = 1/n; or a warm start): xs_next[r] =
+ * x[r] / outdeg[r] (0 when outdeg is 0) for the local rows, then -- with comm -- the same
+ * all-gather into xs_all as a step.  Fields used: n_rows, n_cols, x, outdeg, xs_next, comm,
+ * xs_all, slice_len. */
+acsr_status acsr_pagerank_init(const acsr_pr_args *args, cudaStream_t stream);
 
 /* The same fused step is Random Walk with Restart (Eq. 8):
  *   r' = c (W r) + (1 - c) e_i,  W_{vu} = 1/outdeg_u on every edge u -> v (reading R5)
@@ -270,6 +324,27 @@ acsr_status acsr_peer_read_xs(const acsr_peer *p, double *dst, cudaStream_t stre
 size_t acsr_hits_workspace_bytes(int64_t n);
 acsr_status acsr_hits_normalize(int64_t n, const double *y, const double *v, double *v_next,
                                 double *dist2, void *ws, size_t ws_bytes, cudaStream_t stream);
+
+/* ------------------------------------------------------------------------ */
+/* Degree-ordered vertex relabelling of a PageRank in-link graph (an application-level
+ * preprocessing option for large graphs -- C4 -- not part of ACSR).  Alg. 5 (P:279-291,
+ * reading Q12) gathers xs[u] = x_u / outdeg_u for every in-link u -> v; renumbering the
+ * vertices by decreasing out-degree packs the most gathered entries of xs at the front of
+ * the vector, where they stay in L2.  Rows and columns get the same permutation (P A P^T),
+ * so every kernel runs unchanged and PR in the original numbering is x'[perm[v]].  The
+ * graph persists across the dynamic-graph epochs, so the relabel is paid once.
+ *   row_ptr [n+1], col_idx [nnz]   the in-link CSR (standard; row v = sources of v)
+ *   outdeg [n]                     out-degree of every vertex
+ *   row_ptr_out [n+1], col_out [nnz], outdeg_out [n]   the relabelled graph
+ *   perm_out [n]                   perm_out[v] = new id of old vertex v
+ * Order: decreasing out-degree, ties by increasing old id (stable).  Entry j of old row u
+ * becomes entry j of new row perm[u] (column order inside a row kept).  col_idx/col_out may
+ * be NULL (permutation and row pointers only).  Outputs must not alias the inputs.
+ * Everything runs on `stream` (CUB radix sort + scan, two copy kernels; no host sync). */
+size_t acsr_relabel_workspace_bytes(int64_t n);
+acsr_status acsr_degree_relabel(int64_t n, const int32_t *row_ptr, const int32_t *col_idx, const int32_t *outdeg,
+                                int32_t *row_ptr_out, int32_t *col_out, int32_t *outdeg_out, int32_t *perm_out,
+                                void *ws, size_t ws_bytes, cudaStream_t stream);
 
 /* ------------------------------------------------------------------------ */
 /* Dynamic-graph update (§VII): for update i (row r = upd_rows[i],

@@ -35,6 +35,8 @@ ACSR_ERR_INVALID_VALUE = 1
 ACSR_ERR_WORKSPACE = 2
 ACSR_ERR_CAPACITY = 3
 ACSR_ERR_CUDA = 4
+ACSR_ERR_NCCL = 5
+ACSR_COMM_ID_BYTES = 128
 ACSR_F32 = 0
 ACSR_F64 = 1
 NBINS = 32
@@ -78,7 +80,8 @@ class PrArgs(ctypes.Structure):
                 ("col_idx", _vp), ("bin_rows", _vp), ("bin_offsets", _vp), ("plan_ws", _vp),
                 ("plan_ws_bytes", _sz), ("xs", _vp), ("x", _vp), ("outdeg", _vp), ("x_new", _vp),
                 ("xs_next", _vp), ("damping", _dbl), ("teleport", _dbl), ("delta2", _vp),
-                ("restart", _i64), ("restart_weight", _dbl), ("ctrl", _vp), ("eps2", _dbl)]
+                ("restart", _i64), ("restart_weight", _dbl), ("ctrl", _vp), ("eps2", _dbl),
+                ("comm", _vp), ("xs_all", _vp), ("slice_len", _i64)]
 
 
 _lib.acsr_pagerank_step.argtypes = [ctypes.POINTER(PrArgs), _vp]
@@ -105,6 +108,26 @@ _lib.acsr_hits_normalize.argtypes = [_i64, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
 _lib.acsr_hits_normalize.restype = ctypes.c_int
 _lib.acsr_plan_status.argtypes = [_vp, _sz, _vp]
 _lib.acsr_plan_status.restype = ctypes.c_int
+_lib.acsr_comm_get_unique_id.argtypes = [_vp]
+_lib.acsr_comm_get_unique_id.restype = ctypes.c_int
+_lib.acsr_comm_init.argtypes = [ctypes.POINTER(_vp), ctypes.c_int, ctypes.c_int, _vp]
+_lib.acsr_comm_init.restype = ctypes.c_int
+_lib.acsr_comm_destroy.argtypes = [_vp]
+_lib.acsr_comm_destroy.restype = ctypes.c_int
+_lib.acsr_comm_query.argtypes = [_vp, ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.c_int)]
+_lib.acsr_comm_query.restype = ctypes.c_int
+_lib.acsr_comm_allgather.argtypes = [_vp, _vp, _vp, _sz, _vp]
+_lib.acsr_comm_allgather.restype = ctypes.c_int
+_lib.acsr_pagerank_init.argtypes = [ctypes.POINTER(PrArgs), _vp]
+_lib.acsr_pagerank_init.restype = ctypes.c_int
+_lib.acsr_partition_workspace_bytes.argtypes = [_i64]
+_lib.acsr_partition_workspace_bytes.restype = _sz
+_lib.acsr_partition.argtypes = [_i64, _vp, _vp, _i64, _i64, ctypes.c_int, _vp, _vp, _sz, _vp]
+_lib.acsr_partition.restype = ctypes.c_int
+_lib.acsr_relabel_workspace_bytes.argtypes = [_i64]
+_lib.acsr_relabel_workspace_bytes.restype = _sz
+_lib.acsr_degree_relabel.argtypes = [_i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
+_lib.acsr_degree_relabel.restype = ctypes.c_int
 
 ACSR_BIN_SHORT_ALG2 = 1  # include/acsr.h: per-bin Alg. 2 units for bins 0..5
 ACSR_PEER_MAX = 8
@@ -114,6 +137,9 @@ EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_bin_ex", "acsr_spmv", 
             "acsr_pagerank_scale", "acsr_pagerank_step_peer", "acsr_peer_create", "acsr_peer_open",
             "acsr_peer_destroy", "acsr_peer_push", "acsr_peer_delta2", "acsr_peer_query", "acsr_peer_read_xs", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_update_edges_dev", "acsr_relayout",
             "acsr_hits_workspace_bytes", "acsr_hits_normalize", "acsr_plan_status",
+            "acsr_comm_get_unique_id", "acsr_comm_init", "acsr_comm_destroy", "acsr_comm_query",
+            "acsr_comm_allgather", "acsr_pagerank_init", "acsr_partition_workspace_bytes", "acsr_partition",
+            "acsr_relabel_workspace_bytes", "acsr_degree_relabel",
             "acsr_status_string", "acsr_last_error", "acsr_version")
 
 
@@ -235,9 +261,12 @@ def acsr_pagerank_scale(x, outdeg, xs=None, stream=None):
 
 def acsr_pagerank_step(row_begin, col_idx, bin_rows, bin_offsets, plan_ws, xs, x, outdeg, x_new,
                        xs_next, delta2, damping=0.85, teleport=None, n_global=None, row_end=None,
-                       stream=None, restart=-1, restart_weight=0.0, ctrl=None, eps2=-1.0):
+                       stream=None, restart=-1, restart_weight=0.0, ctrl=None, eps2=-1.0, comm=None,
+                       xs_all=None, slice_len=0):
     """One fused PageRank step on the local rows (Alg. 5).  delta2: 1-element float64.
-    With teleport=0, damping=c, restart=i, restart_weight=1-c it is an RWR step (Eq. 8)."""
+    With teleport=0, damping=c, restart=i, restart_weight=1-c it is an RWR step (Eq. 8).
+    comm (AcsrComm): multi-GPU -- the step is followed by the library's exchange: xs_next[:slice_len]
+    of every rank all-gathered into xs_all, delta2 = the global Delta^2 (include/acsr.h)."""
     n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
     ng = xs.numel() if n_global is None else n_global
     tel = (1.0 - damping) / ng if teleport is None else teleport
@@ -252,9 +281,122 @@ def acsr_pagerank_step(row_begin, col_idx, bin_rows, bin_offsets, plan_ws, xs, x
                _dev(x_new, torch.float64, "x_new") if n else None,
                _dev(xs_next, torch.float64, "xs_next") if n else None, float(damping), float(tel),
                _dev(delta2, torch.float64, "delta2"), int(restart), float(restart_weight),
-               _dev(ctrl, torch.int32, "ctrl", True), float(eps2))
+               _dev(ctrl, torch.int32, "ctrl", True), float(eps2),
+               comm._c if comm is not None else None,
+               _dev(xs_all, torch.float64, "xs_all") if comm is not None else None, int(slice_len))
     _check(_lib.acsr_pagerank_step(ctypes.byref(a), _stream(stream)), "acsr_pagerank_step")
     return x_new, xs_next, delta2
+
+
+def acsr_pagerank_init(x, outdeg, xs_next, comm=None, xs_all=None, slice_len=0, stream=None):
+    """xs_next[:n] = x / outdeg (first iterate, P:285 / warm start); with comm the
+    slices are all-gathered into xs_all (include/acsr.h)."""
+    n = x.numel()
+    a = PrArgs()
+    a.n_rows = n
+    a.n_cols = xs_all.numel() if xs_all is not None else n
+    a.x = _dev(x, torch.float64, "x") if n else None
+    a.outdeg = _dev(outdeg, torch.int32, "outdeg") if n else None
+    a.xs_next = _dev(xs_next, torch.float64, "xs_next") if xs_next.numel() else None
+    a.comm = comm._c if comm is not None else None
+    a.xs_all = _dev(xs_all, torch.float64, "xs_all") if comm is not None else None
+    a.slice_len = int(slice_len)
+    _check(_lib.acsr_pagerank_init(ctypes.byref(a), _stream(stream)), "acsr_pagerank_init")
+    return xs_next
+
+
+# --------------------------------------------------------------------------- multi-GPU
+class AcsrComm:
+    """Owner of one ``acsr_comm`` (include/acsr.h): the library's NCCL communicator.
+    Rank 0's ``unique_id()`` bytes must reach every rank (any host transport) before
+    every rank constructs ``AcsrComm(nranks, rank, uid)`` with its GPU current."""
+
+    @staticmethod
+    def unique_id() -> bytes:
+        buf = ctypes.create_string_buffer(ACSR_COMM_ID_BYTES)
+        _check(_lib.acsr_comm_get_unique_id(buf), "acsr_comm_get_unique_id")
+        return bytes(buf.raw)
+
+    def __init__(self, nranks: int, rank: int, uid: bytes):
+        if len(uid) != ACSR_COMM_ID_BYTES:
+            raise ValueError("unique id must be ACSR_COMM_ID_BYTES bytes")
+        self._c = _vp()
+        buf = ctypes.create_string_buffer(bytes(uid), ACSR_COMM_ID_BYTES)
+        _check(_lib.acsr_comm_init(ctypes.byref(self._c), int(nranks), int(rank), buf), "acsr_comm_init")
+        self.nranks, self.rank = int(nranks), int(rank)
+
+    @classmethod
+    def from_process_group(cls, group=None):
+        """Build the communicator over the ranks of a torch.distributed group (the group
+        only carries the 128-byte id; the data path is the library's NCCL)."""
+        import torch.distributed as dist
+        if not dist.is_initialized():
+            return cls(1, 0, cls.unique_id())
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        obj = [cls.unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0,
+                                   group=group)
+        return cls(world, rank, obj[0])
+
+    def query(self):
+        nr, rk = ctypes.c_int(), ctypes.c_int()
+        _check(_lib.acsr_comm_query(self._c, ctypes.byref(nr), ctypes.byref(rk)), "acsr_comm_query")
+        return int(nr.value), int(rk.value)
+
+    def allgather(self, send, recv, stream=None):
+        """recv (nranks x send.numel(), same dtype) <- every rank's send (in place allowed)."""
+        if recv.numel() != self.nranks * send.numel() or recv.dtype != send.dtype:
+            raise ValueError("recv must hold nranks * send.numel() elements of send's dtype")
+        _check(_lib.acsr_comm_allgather(self._c, _dev(send, None, "send") if send.numel() else None,
+                                        _dev(recv, None, "recv") if recv.numel() else None,
+                                        send.numel() * send.element_size(), _stream(stream)),
+               "acsr_comm_allgather")
+        return recv
+
+    def close(self):
+        if self._c:
+            _check(_lib.acsr_comm_destroy(self._c), "acsr_comm_destroy")
+            self._c = _vp()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def acsr_degree_relabel(row_ptr, col_idx, outdeg, stream=None):
+    """Degree-ordered relabelling on the device (include/acsr.h).  Returns
+    (row_ptr', col', outdeg', perm) with perm[v] = new id of vertex v (int32)."""
+    n = row_ptr.numel() - 1
+    dev = row_ptr.device
+    rp2 = torch.empty(n + 1, dtype=torch.int32, device=dev)
+    c2 = torch.empty_like(col_idx) if col_idx is not None else None
+    od2 = torch.empty(n, dtype=torch.int32, device=dev)
+    perm = torch.empty(n, dtype=torch.int32, device=dev)
+    ws = torch.empty(int(_lib.acsr_relabel_workspace_bytes(n)), dtype=torch.uint8, device=dev)
+    _check(_lib.acsr_degree_relabel(n, _dev(row_ptr, torch.int32, "row_ptr"),
+                                    _dev(col_idx, torch.int32, "col_idx") if c2 is not None and c2.numel() else None,
+                                    _dev(outdeg, torch.int32, "outdeg") if n else None,
+                                    _dev(rp2, torch.int32, "row_ptr_out"),
+                                    _dev(c2, torch.int32, "col_out") if c2 is not None and c2.numel() else None,
+                                    _dev(od2, torch.int32, "outdeg_out") if n else None,
+                                    _dev(perm, torch.int32, "perm_out") if n else None,
+                                    _dev(ws, torch.uint8, "ws"), ws.numel(), _stream(stream)), "acsr_degree_relabel")
+    return rp2, c2, od2, perm
+
+
+def acsr_partition(row_begin, nranks, b_nnz, b_row, row_end=None, stream=None):
+    """O8 split points on the device (int64 CUDA tensor [nranks + 1])."""
+    n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
+    dev = row_begin.device
+    splits = torch.empty(int(nranks) + 1, dtype=torch.int64, device=dev)
+    ws = torch.empty(int(_lib.acsr_partition_workspace_bytes(n)), dtype=torch.uint8, device=dev)
+    _check(_lib.acsr_partition(n, _dev(row_begin, torch.int32, "row_begin") if n else None,
+                               _dev(row_end, torch.int32, "row_end", True), int(b_nnz), int(b_row), int(nranks),
+                               _dev(splits, torch.int64, "splits"), _dev(ws, torch.uint8, "ws"), ws.numel(),
+                               _stream(stream)), "acsr_partition")
+    return splits
 
 
 # --------------------------------------------------------------------------- peer exchange

@@ -1,0 +1,242 @@
+// acsr_comm.cu -- the multi-GPU exchange owned by the library (§VIII row split,
+// reading Q19).
+//
+// Row-partitioned PageRank needs, after every step, (1) every rank's slice of the scaled
+// vector xs' = PR'/outdeg in every rank's replicated xs and (2) the global Delta^2 of the
+// convergence test (Alg. 5; reading Q9).  Both run here on the caller's stream,
+// right behind the fused step kernel, over NCCL (NVLink / NVSwitch inside a node):
+//   * one in-place ncclAllGather of the equal-length (padded) slices, and
+//   * one ncclAllGather of the ranks' EXACT 192-bit fixed-point Delta^2 partials, which a
+//     one-warp kernel then adds in rank order: the global Delta^2 -- and with it the
+//     device-side stop decision -- is the same bits on every rank and equal to the
+//     single-GPU value (fixed-point sums do not depend on the order or the partition).
+// Also here: acsr_partition (O8's nnz-balanced contiguous split, computed on the device
+// with a CUB prefix sum + binary search) and a byte all-gather for setup-time layout work.
+#include <cuda_runtime.h>
+#include <nccl.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <cub/device/device_scan.cuh>
+#include <thrust/iterator/counting_iterator.h>
+#include <thrust/iterator/transform_iterator.h>
+
+#include "acsr_internal.cuh"
+
+struct acsr_comm {
+    ncclComm_t nccl = nullptr;
+    int nranks = 0, rank = 0, device = 0;
+    uint64_t *d2 = nullptr;  // device [(nranks + 1) * 3]: own partial, then every rank's
+};
+
+static acsr_status nccl_fail(const char *what, ncclResult_t r)
+{
+    acsr_set_error("%s: %s", what, ncclGetErrorString(r));
+    return ACSR_ERR_NCCL;
+}
+
+namespace acsr {
+
+// global Delta^2 = exact sum of the gathered partials (rank order; the sum is exact, so
+// any order gives the same bits); the device-side stop flag for every rank alike
+__global__ void comm_d2_finalize_kernel(const uint64_t *__restrict__ parts, int nranks, double *delta2,
+                                        int32_t *ctrl, double eps2)
+{
+    if (threadIdx.x != 0) return;
+    if (ctrl && *(volatile int32_t *)ctrl) return;  // converged (or plan error) earlier: step was a no-op
+    uint64_t hi = 0, mid = 0, lo = 0;
+    for (int q = 0; q < nranks; q++) fix192_merge(hi, mid, lo, parts[3 * q], parts[3 * q + 1], parts[3 * q + 2]);
+    const double d2 = fix192_to_double(hi, mid, lo);
+    *delta2 = d2;
+    if (ctrl && d2 <= eps2) ctrl[0] = 1;
+}
+
+__global__ void split_search_kernel(const int64_t *__restrict__ incl, int64_t n, int P, int64_t *splits)
+{
+    const int k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k > P) return;
+    if (k == 0 || k == P || n == 0) {
+        splits[k] = (k == P) ? n : 0;
+        return;
+    }
+    const int64_t total = incl[n - 1];
+    const int64_t target = ((int64_t)k * total + P - 1) / P;  // ceil(k * total / P)
+    // min r in [0, n] with sum_{r' < r} cost(r') = (r ? incl[r-1] : 0) >= target
+    int64_t lo = 0, hi = n;
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) / 2;
+        const int64_t f = mid ? incl[mid - 1] : 0;
+        if (f >= target) hi = mid;
+        else lo = mid + 1;
+    }
+    splits[k] = lo;
+}
+
+struct RowCost {
+    const int32_t *rb, *re;
+    int64_t b_nnz, b_row;
+    __host__ __device__ int64_t operator()(int64_t r) const
+    {
+        const int64_t len = (int64_t)(re ? re[r] : rb[r + 1]) - rb[r];
+        return b_nnz * len + b_row;
+    }
+};
+
+}  // namespace acsr
+
+using namespace acsr;
+
+extern "C" acsr_status acsr_comm_get_unique_id(void *id)
+{
+    if (!id) {
+        acsr_set_error("acsr_comm_get_unique_id: id is NULL");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    ncclUniqueId u;
+    const ncclResult_t r = ncclGetUniqueId(&u);
+    if (r != ncclSuccess) return nccl_fail("acsr_comm_get_unique_id", r);
+    memcpy(id, u.internal, NCCL_UNIQUE_ID_BYTES);
+    return ACSR_OK;
+}
+
+extern "C" acsr_status acsr_comm_init(acsr_comm **out, int nranks, int rank, const void *id)
+{
+    static_assert(ACSR_COMM_ID_BYTES == NCCL_UNIQUE_ID_BYTES, "unique id size");
+    if (!out || !id || nranks < 1 || rank < 0 || rank >= nranks) {
+        acsr_set_error("acsr_comm_init: invalid argument");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    *out = nullptr;
+    acsr_comm *c = new acsr_comm();
+    c->nranks = nranks;
+    c->rank = rank;
+    cudaGetDevice(&c->device);
+    cudaError_t e = cudaMalloc(&c->d2, sizeof(uint64_t) * 3 * (size_t)(nranks + 1));
+    if (e != cudaSuccess) {
+        acsr_set_error("acsr_comm_init: %s", cudaGetErrorString(e));
+        delete c;
+        return ACSR_ERR_CUDA;
+    }
+    cudaMemset(c->d2, 0, sizeof(uint64_t) * 3 * (size_t)(nranks + 1));
+    ncclUniqueId u;
+    memcpy(u.internal, id, NCCL_UNIQUE_ID_BYTES);
+    const ncclResult_t r = ncclCommInitRank(&c->nccl, nranks, u, rank);
+    if (r != ncclSuccess) {
+        cudaFree(c->d2);
+        delete c;
+        return nccl_fail("acsr_comm_init (ncclCommInitRank)", r);
+    }
+    *out = c;
+    return ACSR_OK;
+}
+
+extern "C" acsr_status acsr_comm_destroy(acsr_comm *c)
+{
+    if (!c) return ACSR_OK;
+    acsr_status st = ACSR_OK;
+    if (c->nccl) {
+        const ncclResult_t r = ncclCommDestroy(c->nccl);
+        if (r != ncclSuccess) st = nccl_fail("acsr_comm_destroy", r);
+    }
+    cudaFree(c->d2);
+    delete c;
+    return st;
+}
+
+extern "C" acsr_status acsr_comm_query(const acsr_comm *c, int *nranks, int *rank)
+{
+    if (!c) {
+        acsr_set_error("acsr_comm_query: comm is NULL");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    if (nranks) *nranks = c->nranks;
+    if (rank) *rank = c->rank;
+    return ACSR_OK;
+}
+
+extern "C" acsr_status acsr_comm_allgather(acsr_comm *c, const void *send, void *recv, size_t bytes_per_rank,
+                                           cudaStream_t stream)
+{
+    if (!c || (bytes_per_rank > 0 && (!send || !recv))) {
+        acsr_set_error("acsr_comm_allgather: invalid argument");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    if (bytes_per_rank == 0) return ACSR_OK;
+    const ncclResult_t r = ncclAllGather(send, recv, bytes_per_rank, ncclUint8, c->nccl, stream);
+    if (r != ncclSuccess) return nccl_fail("acsr_comm_allgather", r);
+    return acsr_check_launch("acsr_comm_allgather");
+}
+
+// Called by acsr_pagerank_step after the fused step kernel (which wrote its Delta^2
+// partial to comm->d2[0..3)) when args->comm != NULL.
+acsr_status acsr_comm_step_exchange(const acsr_pr_args *p, cudaStream_t stream)
+{
+    acsr_comm *c = p->comm;
+    ncclResult_t r = ncclGroupStart();
+    if (r == ncclSuccess && p->slice_len > 0)
+        r = ncclAllGather(p->xs_next, p->xs_all, (size_t)p->slice_len, ncclFloat64, c->nccl, stream);
+    if (r == ncclSuccess) r = ncclAllGather(c->d2, c->d2 + 3, 3, ncclUint64, c->nccl, stream);
+    const ncclResult_t r2 = ncclGroupEnd();
+    if (r != ncclSuccess) return nccl_fail("acsr_pagerank_step (exchange)", r);
+    if (r2 != ncclSuccess) return nccl_fail("acsr_pagerank_step (exchange)", r2);
+    comm_d2_finalize_kernel<<<1, 32, 0, stream>>>(c->d2 + 3, c->nranks, p->delta2, p->ctrl, p->eps2);
+    return acsr_check_launch("acsr_pagerank_step (Delta^2 finalize)");
+}
+
+uint64_t *acsr_comm_d2_slot(acsr_comm *c) { return c->d2; }
+int acsr_comm_nranks(const acsr_comm *c) { return c->nranks; }
+
+extern "C" acsr_status acsr_pagerank_init(const acsr_pr_args *p, cudaStream_t stream)
+{
+    if (!p || p->n_rows < 0 || (p->n_rows > 0 && (!p->x || !p->outdeg || !p->xs_next))) {
+        acsr_set_error("acsr_pagerank_init: invalid argument");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    if (p->comm && (!p->xs_all || p->slice_len < 0 ||
+                    p->n_cols < (int64_t)acsr_comm_nranks(p->comm) * p->slice_len)) {
+        acsr_set_error("acsr_pagerank_init: with comm, xs_all [n_cols >= nranks * slice_len] is required");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    acsr_status st = acsr_pagerank_scale(p->n_rows, p->x, p->outdeg, p->xs_next, stream);
+    if (st != ACSR_OK || !p->comm) return st;
+    if (p->slice_len == 0) return ACSR_OK;
+    const ncclResult_t r = ncclAllGather(p->xs_next, p->xs_all, (size_t)p->slice_len, ncclFloat64, p->comm->nccl, stream);
+    if (r != ncclSuccess) return nccl_fail("acsr_pagerank_init (all-gather)", r);
+    return acsr_check_launch("acsr_pagerank_init");
+}
+
+extern "C" size_t acsr_partition_workspace_bytes(int64_t n_rows)
+{
+    size_t temp = 0;
+    auto it = thrust::make_transform_iterator(thrust::counting_iterator<int64_t>(0), RowCost{nullptr, nullptr, 0, 0});
+    cub::DeviceScan::InclusiveSum(nullptr, temp, it, (int64_t *)nullptr, n_rows > 0 ? n_rows : 1);
+    return align_up(sizeof(int64_t) * (size_t)(n_rows > 0 ? n_rows : 1), 256) + align_up(temp, 256);
+}
+
+extern "C" acsr_status acsr_partition(int64_t n_rows, const int32_t *row_begin, const int32_t *row_end,
+                                      int64_t b_nnz, int64_t b_row, int nranks, int64_t *splits, void *ws,
+                                      size_t ws_bytes, cudaStream_t stream)
+{
+    if (n_rows < 0 || nranks < 1 || !splits || b_nnz < 0 || b_row < 0 || (n_rows > 0 && !row_begin)) {
+        acsr_set_error("acsr_partition: invalid argument");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    if (!ws || ws_bytes < acsr_partition_workspace_bytes(n_rows)) {
+        acsr_set_error("acsr_partition: workspace missing or too small");
+        return ACSR_ERR_WORKSPACE;
+    }
+    int64_t *incl = (int64_t *)ws;
+    if (n_rows > 0) {
+        char *temp = (char *)ws + align_up(sizeof(int64_t) * (size_t)n_rows, 256);
+        size_t temp_bytes = ws_bytes - align_up(sizeof(int64_t) * (size_t)n_rows, 256);
+        auto it = thrust::make_transform_iterator(thrust::counting_iterator<int64_t>(0),
+                                                  RowCost{row_begin, row_end, b_nnz, b_row});
+        const cudaError_t e = cub::DeviceScan::InclusiveSum(temp, temp_bytes, it, incl, n_rows, stream);
+        if (e != cudaSuccess) {
+            acsr_set_error("acsr_partition (scan): %s", cudaGetErrorString(e));
+            return ACSR_ERR_CUDA;
+        }
+    }
+    split_search_kernel<<<(nranks + 1 + 127) / 128, 128, 0, stream>>>(incl, n_rows, nranks, splits);
+    return acsr_check_launch("acsr_partition");
+}

@@ -286,6 +286,25 @@ __device__ __forceinline__ void peer_signal(const PeerArgs &p, unsigned long lon
     p.st->last_step = with_d2 ? 1u : 0u;
 }
 
+// 192-bit fixed point (hi + mid 2^-64 + lo 2^-128) helpers for exact Delta^2 sums
+__host__ __device__ __forceinline__ void fix192_merge(uint64_t &hi, uint64_t &mid, uint64_t &lo, uint64_t h,
+                                                      uint64_t m, uint64_t l)
+{
+    const uint64_t nlo = lo + l;
+    const uint64_t c1 = nlo < lo;
+    const uint64_t m1 = mid + m;
+    const uint64_t c2a = m1 < mid;
+    const uint64_t m2 = m1 + c1;
+    const uint64_t c2b = m2 < m1;
+    lo = nlo;
+    mid = m2;
+    hi += h + c2a + c2b;
+}
+__host__ __device__ __forceinline__ double fix192_to_double(uint64_t hi, uint64_t mid, uint64_t lo)
+{
+    return (double)hi + ((double)mid + (double)lo * 5.421010862427522e-20) * 5.421010862427522e-20;
+}
+
 // Global Delta^2 of push c: the exact sum of every rank's 192-bit partial (the same bits
 // on every rank, whatever the order), after peer_wait(p, c).
 __device__ __forceinline__ double peer_sum_d2(const PeerArgs &p, unsigned long long c)
@@ -374,6 +393,11 @@ inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, s
 }
 
 }  // namespace acsr
+
+// library-owned NCCL exchange (acsr_comm.cu)
+acsr_status acsr_comm_step_exchange(const acsr_pr_args *p, cudaStream_t stream);
+uint64_t *acsr_comm_d2_slot(acsr_comm *c);
+int acsr_comm_nranks(const acsr_comm *c);
 
 // error plumbing (acsr_capi.cu)
 void acsr_set_error(const char *fmt, ...);

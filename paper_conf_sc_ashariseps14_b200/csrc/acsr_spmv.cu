@@ -50,6 +50,9 @@
 #ifndef ACSR_WIN_PREFETCH
 #define ACSR_WIN_PREFETCH 0  // 1: prefetch the next window's row bounds (A/B: no gain on C3a, LiveJournal-like +5 %)
 #endif
+#ifndef ACSR_PF_UNIT
+#define ACSR_PF_UNIT 0  // 1: L2 bulk prefetch of a unit's col/val runs at unit start (A/B)
+#endif
 #ifndef ACSR_VEC_MIN
 #define ACSR_VEC_MIN 512  // rows (chunks) shorter than this use the lane-strided scalar path
 #endif
@@ -89,6 +92,7 @@ struct SpmvArgs {
     int32_t *ctrl;  // device-side convergence: [0] stop flag, [1] executed steps (nullable)
     double eps2;
     int64_t n_rows;  // rows of the call (NaN fill of an overflowed plan)
+    uint64_t *d2_out;  // multi-GPU (acsr_comm): the last CTA writes this rank's exact 192-bit partial here
     int64_t x_prefetch;  // bytes of x to bulk-prefetch into L2 at entry (0: none)
     // fused peer-memory exchange of xs_next (acsr_pagerank_step_peer; peer.nranks == 0: off)
     const PeerArgs *peer;  // device copy (PeerState::view) or NULL
@@ -362,6 +366,26 @@ struct Kern {
         return acc + xv;
     }
 
+    // cp.async.bulk.prefetch.L2 of the element range [kb, ke) of col (and val): the rows
+    // of a unit are processed one after another, so the later rows' CSR runs come from L2
+    // instead of DRAM (ACSR_PF_UNIT)
+    static __device__ __forceinline__ void pf_bytes(const void *p, int64_t bytes)
+    {
+        uintptr_t b = (uintptr_t)p & ~(uintptr_t)15;
+        const uintptr_t e = ((uintptr_t)p + (uintptr_t)bytes + 15) & ~(uintptr_t)15;
+        while (b < e) {
+            const uint32_t sz = (uint32_t)(e - b < 32768 ? e - b : 32768);
+            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(b), "r"(sz) : "memory");
+            b += sz;
+        }
+    }
+    static __device__ __forceinline__ void pf_range(const A &a, int kb, int ke)
+    {
+        if (ke <= kb) return;
+        pf_bytes(a.col + kb, 4 * (int64_t)(ke - kb));
+        if (HAS_VAL) pf_bytes(a.val + kb, (int64_t)sizeof(V) * (ke - kb));
+    }
+
     // write the row result (or the PageRank epilogue for local row r)
     static __device__ __forceinline__ void finish(const A &a, int r, double s, Fix192 &d2)
     {
@@ -527,6 +551,7 @@ struct Kern {
         const int myr = lane < cnt ? __ldg(a.bin_rows + start + lane) : 0;
         int mb = 0, me = 0;
         if (lane < cnt) row_bounds(a, myr, mb, me);
+        if (ACSR_PF_UNIT && lane > 0 && lane < cnt) pf_range(a, mb, me);  // rows 1.. of the unit
 #if ACSR_PAIR_ROWS
         // two rows in flight: element k of a row feeds accumulator (k mod 64) < 32 ? p : q,
         // whether or not the row has a partner -> per-row order independent of pairing
@@ -586,6 +611,12 @@ struct Kern {
         constexpr unsigned FULL = 0xffffffffu;
         const unsigned lt = (1u << lane) - 1u;
         const unsigned le = 0xffffffffu >> (31 - lane);
+        if (ACSR_PF_UNIT && nrows > WIN_ROWS && lane == 0) {
+            // the unit's rows are consecutive: one contiguous CSR run (windows 2.. of the unit)
+            const int kb = __ldg(a.rb + r0 + WIN_ROWS);
+            const int ke = HAS_END ? __ldg(a.re + r0 + nrows - 1) : __ldg(a.rb + r0 + nrows);
+            pf_range(a, kb, ke);
+        }
 #if ACSR_WIN_PREFETCH
         // the next window's row bounds are loaded while this window runs (one dependent
         // DRAM round trip less per window on short-row matrices)
@@ -983,6 +1014,11 @@ spmv_kernel(SpmvArgs<V> a)
                     // an overflowed plan publishes a saturated partial: no rank converges on it
                     peer_signal(*a.peer, pc + 1, true, plan_bad ? ~0ull : hi, mid, lo);
                 }
+                if (a.d2_out) {  // acsr_comm: all-gathered and summed by the exchange
+                    a.d2_out[0] = plan_bad ? ~0ull : hi;
+                    a.d2_out[1] = mid;
+                    a.d2_out[2] = lo;
+                }
                 if (a.ctrl && plan_bad) {
                     a.ctrl[0] = ACSR_CTRL_PLAN_ERROR;  // stops the loop; acsr_plan_status tells why
                 } else if (a.ctrl) {
@@ -1264,7 +1300,16 @@ extern "C" acsr_status acsr_pagerank_step(const acsr_pr_args *p, cudaStream_t st
         acsr_set_error("acsr_pagerank_step: plan workspace missing or too small");
         return ACSR_ERR_WORKSPACE;
     }
+    if (p->comm && (!p->xs_all || p->slice_len < 0 || p->n_cols < (int64_t)acsr_comm_nranks(p->comm) * p->slice_len ||
+                    (p->slice_len > 0 && !p->xs_next))) {
+        acsr_set_error("acsr_pagerank_step: with comm, xs_all [n_cols >= nranks * slice_len] and xs_next are required");
+        return ACSR_ERR_INVALID_VALUE;
+    }
     if (p->n_rows == 0) {
+        if (p->comm) {  // still part of the exchange: a zero partial
+            cudaMemsetAsync(acsr_comm_d2_slot(p->comm), 0, 3 * sizeof(uint64_t), stream);
+            return acsr_comm_step_exchange(p, stream);
+        }
         zero_delta_kernel<<<1, 1, 0, stream>>>(p->delta2);
         return acsr_check_launch("acsr_pagerank_step(empty)");
     }
@@ -1277,8 +1322,14 @@ extern "C" acsr_status acsr_pagerank_step(const acsr_pr_args *p, cudaStream_t st
     a.restart = p->restart; a.restart_weight = p->restart_weight;
     a.ctrl = p->ctrl; a.eps2 = p->eps2;
     a.x_prefetch = a.x ? x_prefetch_bytes(p->n_cols * (int64_t)sizeof(double)) : 0;
+    if (p->comm) {
+        a.eps2 = -1.0;  // the stop decision is global (acsr_comm_step_exchange)
+        a.d2_out = acsr_comm_d2_slot(p->comm);
+    }
     dispatch<double, true>(a, stream);
-    return acsr_check_launch("acsr_pagerank_step");
+    const acsr_status st = acsr_check_launch("acsr_pagerank_step");
+    if (st != ACSR_OK || !p->comm) return st;
+    return acsr_comm_step_exchange(p, stream);
 }
 
 extern "C" acsr_status acsr_pagerank_step_peer(const acsr_pr_args *p, acsr_peer *peer, cudaStream_t stream)

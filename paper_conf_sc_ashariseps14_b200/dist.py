@@ -1,25 +1,28 @@
 """Row-partitioned multi-GPU PageRank (§VIII P:343-348 "a simple division ... each GPU is
 thus responsible for computing half the results", generalised to P ranks; reading Q19).
 
-One process per GPU (torchrun); ``torch.distributed`` (NCCL over NVLink/NVSwitch) is the
-plumbing.  Per iteration each rank runs ONE fused ``acsr_pagerank_step`` launch on its
-contiguous row range (SpMV on the in-link pattern + teleport/damping epilogue + xs slice +
-Delta^2 partial), then
+One process per GPU (torchrun).  Per iteration each rank runs ONE fused
+``acsr_pagerank_step`` on its contiguous row range (SpMV on the in-link pattern +
+teleport/damping epilogue + xs slice + exact Delta^2 partial) and the exchange, A9 of
+SURVEY §8(a).  Three exchanges, all bitwise-equivalent:
 
-  * all-gathers the xs slices (equal-size padded slices, in place -> NCCL ring/NVLS
-    all-gather; the only data-path exchange, A9 in SURVEY §8(a)),
-  * all-reduces the 8-byte Delta^2 (the convergence test of Alg. 5, reading Q9).
+  * ``exchange="acsr"`` (default on GPUs): the library owns it (include/acsr.h,
+    ``acsr_comm``): the same ``acsr_pagerank_step`` call, given the communicator, runs an
+    in-place NCCL all-gather of the equal-length slices and an all-gather of the ranks'
+    exact fixed-point Delta^2 partials on the caller's stream; the global Delta^2 and the
+    device-side stop flag are identical on every rank, so steps are enqueued back to back
+    with a host check every ``check_every`` steps, as on one GPU.  torch.distributed only
+    carries the 128-byte NCCL id at setup.
+  * ``exchange="torch"``: the same data movement through torch.distributed collectives
+    (all_gather_into_tensor + all_reduce of Delta^2); used by the gloo tests on CPU
+    (tests/test_dist_gloo.py, oracle step) and by ranks sharing one GPU over gloo.
+  * ``exchange="peer"``: the all-gather disappears into the step kernel itself, which
+    stores every finished xs' slice entry into all ranks' replicated xs over peer memory
+    (``acsr_pagerank_step_peer``).
 
-With ``exchange="peer"`` the all-gather disappears: the fused step kernel itself stores
-every finished xs' slice entry into all ranks' replicated xs over peer memory (NVLink /
-NVSwitch P2P stores through CUDA IPC mappings, overlapped with the rest of the step) and
-signals the push with a release flag; the next step waits on the flags at entry, and
-the global Delta^2 is the exact sum of the ranks' fixed-point partials
-(``acsr_pagerank_step_peer`` / ``acsr_peer_delta2``, include/acsr.h).
-
-Host logic here (partition, column renumbering into the padded layout, the loop) is
-device-agnostic so it is unit-tested with the gloo backend on CPU (tests/test_dist_gloo.py)
-by injecting a CPU step function; on GPUs the step is the CUDA kernel.
+Host logic here (partition, column renumbering into the padded or compact layout, the
+loop) is device-agnostic so it is unit-tested with the gloo backend on CPU by injecting a
+CPU step function; on GPUs the step is the CUDA kernel.
 """
 from __future__ import annotations
 
@@ -96,12 +99,19 @@ class DistPageRank:
     (acsr_pagerank_step)."""
 
     def __init__(self, row_ptr_local, col_local, outdeg_local, splits, n_global, damping=0.85,
-                 group=None, step_fn=None, scale_fn=None, device=None, compact=True, exchange="nccl"):
-        if exchange not in ("nccl", "peer"):
-            raise ValueError(f"exchange must be 'nccl' (collective all-gather) or 'peer', not {exchange!r}")
-        if exchange == "peer" and (step_fn is not None or scale_fn is not None):
-            raise ValueError("exchange='peer' fuses the exchange into the CUDA step (no step_fn)")
+                 group=None, step_fn=None, scale_fn=None, device=None, compact=True, exchange=None, comm=None):
+        if exchange is None:
+            exchange = "torch" if step_fn is not None else "acsr"
+        if exchange not in ("acsr", "torch", "peer"):
+            raise ValueError(f"exchange must be 'acsr' (library NCCL), 'torch' (torch.distributed) or 'peer', "
+                             f"not {exchange!r}")
+        if exchange in ("peer", "acsr") and (step_fn is not None or scale_fn is not None):
+            raise ValueError(f"exchange={exchange!r} runs inside the library's CUDA step (no step_fn)")
         self.exchange_mode = exchange
+        self.comm = None
+        if exchange == "acsr":
+            from . import AcsrComm
+            self.comm = comm if comm is not None else AcsrComm.from_process_group(group)
         self.group = group
         self.rank = dist.get_rank(group) if dist.is_initialized() else 0
         self.world = dist.get_world_size(group) if dist.is_initialized() else 1
@@ -168,7 +178,10 @@ class DistPageRank:
         pad = torch.zeros(L, dtype=torch.uint8, device=dev)
         pad[: self.n_local] = nd_local.to(torch.uint8)
         allm = torch.zeros(world * L, dtype=torch.uint8, device=dev)
-        dist.all_gather_into_tensor(allm, pad.clone() if dev.type == "cpu" else pad, group=self.group)
+        if self.comm is not None:
+            self.comm.allgather(pad, allm)
+        else:
+            dist.all_gather_into_tensor(allm, pad.clone() if dev.type == "cpu" else pad, group=self.group)
         sizes = np.diff(self.splits)
         nd = torch.cat([allm[k * L: k * L + int(sizes[k])] for k in range(world)]).to(torch.bool)
         nnd = [int(allm[k * L: k * L + int(sizes[k])].sum()) for k in range(world)]
@@ -242,22 +255,60 @@ class DistPageRank:
             raise RuntimeError("acsr_peer: a peer barrier timed out (a rank stopped issuing steps?)")
         return bufs[it % 2], it, float(self.delta2.item())
 
+    def _run_acsr(self, x, eps, max_iter, check_every):
+        """Library-owned exchange: every acsr_pagerank_step call carries the communicator,
+        so the step, the xs all-gather and the exact global Delta^2 (+ device-side stop
+        flag, identical on every rank) are enqueued back to back; the host looks at the
+        flag every check_every steps.  Same results as a host test after every step."""
+        from . import acsr_pagerank_init, acsr_pagerank_step
+        m, comm = self._m, self.comm
+        Ls = self.Lx if self.compact else self.L  # exchanged entries per rank
+
+        def local_out(buf):
+            if self.compact:
+                return self.xs_loc  # the exchanged prefix is xs_loc[:Lx]
+            return buf[self.rank * self.L:(self.rank + 1) * self.L]  # in place
+
+        bufs = [x, torch.empty_like(x)]
+        xsb = [self.xs, self.xs_next]
+        acsr_pagerank_init(x, self.outdeg, local_out(xsb[0]), comm=comm, xs_all=xsb[0], slice_len=Ls)
+        ctrl = torch.zeros(2, dtype=torch.int32, device=self.device)
+        eps2 = eps * eps if eps >= 0 else -1.0
+        k = 0
+        while k < max_iter:
+            for _ in range(min(check_every, max_iter - k)):
+                a, b = k % 2, (k + 1) % 2
+                acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xsb[a], bufs[a],
+                                   self.outdeg, bufs[b], local_out(xsb[b]), self.delta2, self.damping,
+                                   self.teleport, self.n_global, ctrl=ctrl, eps2=eps2, comm=comm, xs_all=xsb[b],
+                                   slice_len=Ls)
+                k += 1
+            c = ctrl.cpu()
+            if int(c[0]):
+                break
+        it = int(ctrl[1].item())
+        if int(ctrl[0]) == 2:
+            m.plan_status()  # raises: invalid plan
+        return bufs[it % 2], it, float(self.delta2.item())
+
     def exchange_bytes_per_rank(self):
         """Bytes each rank receives per iteration from the all-gather."""
         return (self.world - 1) * self.Lx * 8
 
-    def run(self, x0_local=None, eps=1e-6, max_iter=1000, check_every=1):
+    def run(self, x0_local=None, eps=1e-6, max_iter=1000, check_every=None):
         """Alg. 5 loop; returns (x_local, iterations, delta2_global) with x_local in the
-        caller's local row order.  check_every (peer exchange only): (step, Delta^2) pairs
-        enqueued between host synchronisations, steps after convergence are no-ops on
+        caller's local row order.  check_every (acsr / peer exchanges): steps enqueued
+        between host synchronisations (default 8 / 1); steps after convergence are no-ops on
         every rank (device-side stop flag) -- same results as checking every step."""
         dev = self.device
         if x0_local is None:
             x = torch.full((self.n_local,), 1.0 / self.n_global, dtype=torch.float64, device=dev)
         else:
             x = x0_local.clone() if self.perm is None else x0_local[self.perm].contiguous()
-        if self.peer is not None:
-            x, it, d2 = self._run_peer(x, eps, max_iter, max(1, int(check_every)))
+        if self.exchange_mode in ("peer", "acsr"):
+            ce = check_every if check_every is not None else (8 if self.exchange_mode == "acsr" else 1)
+            run = self._run_peer if self.exchange_mode == "peer" else self._run_acsr
+            x, it, d2 = run(x, eps, max_iter, max(1, int(ce)))
             if self.perm is not None:
                 out = torch.empty_like(x)
                 out[self.perm] = x

@@ -273,23 +273,10 @@ def hits(out_ptr, out_col, eps=1e-6, max_iter=1000, stream=None, B=None):
 
 def degree_relabel(in_ptr, in_col, outdeg):
     """Vertex relabelling for PageRank locality (an application-level preprocessing step,
-    not part of ACSR): vertices are renumbered by decreasing out-degree so the most
-    gathered entries of xs = x / outdeg sit together at the front of the vector.  Rows and
-    columns of the in-link pattern get the same permutation (P A P^T), so the kernels run
-    unchanged; PR in the original order is x_new[perm].  Returns
-    (row_ptr', col', outdeg', perm) with perm[v] = new id of vertex v."""
-    n = in_ptr.numel() - 1
-    dev = in_ptr.device
-    order = torch.sort(outdeg.long(), descending=True, stable=True).indices  # new id -> old
-    perm = torch.empty(n, dtype=torch.int64, device=dev)
-    perm[order] = torch.arange(n, device=dev)
-    ln = (in_ptr[1:] - in_ptr[:-1]).long()
-    rows = torch.repeat_interleave(torch.arange(n, device=dev), ln)
-    new_r = perm[rows]
-    new_c = perm[in_col.long()]
-    key = torch.sort(new_r * n + new_c).values
-    r2 = key // n
-    c2 = (key - r2 * n).to(torch.int32)
-    rp2 = torch.zeros(n + 1, dtype=torch.int64, device=dev)
-    rp2[1:] = torch.cumsum(torch.bincount(r2, minlength=n), 0)
-    return rp2.to(torch.int32), c2, outdeg[order].contiguous(), perm
+    not part of ACSR), on the device: acsr_degree_relabel (include/acsr.h) -- vertices by
+    decreasing out-degree (ties by id), rows and columns alike (P A P^T), so the kernels run
+    unchanged and PR in the original order is x_new[perm].  Returns
+    (row_ptr', col', outdeg', perm) with perm[v] = new id of vertex v (int64)."""
+    from . import acsr_degree_relabel
+    rp2, c2, od2, perm = acsr_degree_relabel(in_ptr, in_col, outdeg)
+    return rp2, c2, od2, perm.to(torch.int64)

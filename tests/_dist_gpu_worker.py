@@ -6,8 +6,15 @@ import torch
 import torch.distributed as dist
 
 
-def worker(rank, world, port, scale, q, exchange="nccl", compact=True, check_every=1):
+def worker(rank, world, port, scale, q, exchange="torch", compact=True, check_every=1):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    if exchange == "acsr":
+        # the library's NCCL communicator with every rank on the SAME GPU: NCCL refuses two
+        # ranks on one device of one host, so each rank claims its own host id (the ranks
+        # then talk over NCCL's socket transport on loopback).  Test-only: on a real node
+        # every rank has its own GPU and NCCL uses NVLink / NVSwitch.
+        os.environ.update(NCCL_HOSTID=f"acsr-test-host-{rank}", NCCL_SOCKET_IFNAME="lo", NCCL_IB_DISABLE="1",
+                          NCCL_P2P_DISABLE="1", NCCL_SHM_DISABLE="1", NCCL_NVLS_ENABLE="0")
     dist.init_process_group("gloo", rank=rank, world_size=world)
     import synth
     from paper_conf_sc_ashariseps14_b200 import dist as pdist
@@ -29,7 +36,9 @@ def worker(rank, world, port, scale, q, exchange="nccl", compact=True, check_eve
         assert all(torch.equal(allx[0], a) for a in allx), "replicated xs differ across ranks"
         pr.peer.close()
     else:
-        x, it, d2 = pr.run(eps=1e-6)
+        x, it, d2 = pr.run(eps=1e-6, check_every=check_every)
+        if exchange == "acsr":
+            pr.comm.close()
     parts = [torch.zeros(pr.L, dtype=torch.float64) for _ in range(world)]
     xp = torch.zeros(pr.L, dtype=torch.float64)
     xp[: x.numel()] = x.cpu()

@@ -124,6 +124,63 @@ int main(void)
     ok &= pushes == 2 && perr == 0 && cur != NULL;
     ok &= acsr_peer_create(&peer, 9, 0, 10, 0, 5, handle) == ACSR_ERR_INVALID_VALUE;
     AK(acsr_peer_destroy(peer));
+
+    /* the library-owned NCCL exchange, one rank: acsr_pagerank_init + acsr_pagerank_step
+     * with comm (in-place all-gather of the slice, global Delta^2 from the exact partials)
+     * gives the same x_new as the peer step above and the same Delta^2 */
+    char uid[ACSR_COMM_ID_BYTES];
+    acsr_comm *comm = NULL;
+    AK(acsr_comm_get_unique_id(uid));
+    AK(acsr_comm_init(&comm, 1, 0, uid));
+    int nr = 0, rk = -1;
+    AK(acsr_comm_query(comm, &nr, &rk));
+    ok &= nr == 1 && rk == 0;
+    double *d_xa, *d_xb, *d_xn2, *d_d2c;
+    int32_t *d_ctrl;
+    CK(cudaMalloc((void **)&d_xa, sizeof(double) * n_cols));
+    CK(cudaMalloc((void **)&d_xb, sizeof(double) * n_cols));
+    CK(cudaMalloc((void **)&d_xn2, sizeof(xn)));
+    CK(cudaMalloc((void **)&d_d2c, sizeof(double)));
+    CK(cudaMalloc((void **)&d_ctrl, 2 * sizeof(int32_t)));
+    CK(cudaMemset(d_xa, 0, sizeof(double) * n_cols));
+    CK(cudaMemset(d_xb, 0, sizeof(double) * n_cols));
+    CK(cudaMemset(d_ctrl, 0, 2 * sizeof(int32_t)));
+    acsr_pr_args c;
+    memset(&c, 0, sizeof(c));
+    c.n_rows = n; c.n_cols = n_cols; c.row_begin = d_rp; c.col_idx = d_col;
+    c.bin_rows = d_bins; c.bin_offsets = d_off; c.plan_ws = d_ws; c.plan_ws_bytes = ws_bytes;
+    c.x = d_x0; c.outdeg = d_od; c.xs_next = d_xa; c.comm = comm; c.xs_all = d_xa; c.slice_len = n;
+    AK(acsr_pagerank_init(&c, st));
+    c.xs = d_xa; c.x_new = d_xn2; c.xs_next = d_xb; c.xs_all = d_xb;
+    c.damping = damping; c.teleport = teleport; c.delta2 = d_d2c; c.restart = -1;
+    c.ctrl = d_ctrl; c.eps2 = 1e300; /* converges on the first step: ctrl[0] = 1, ctrl[1] = 1 */
+    AK(acsr_pagerank_step(&c, st));
+    CK(cudaStreamSynchronize(st));
+    double xn2[6], d2c;
+    int32_t ctrl[2];
+    CK(cudaMemcpy(xn2, d_xn2, sizeof(xn2), cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&d2c, d_d2c, sizeof(double), cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(ctrl, d_ctrl, sizeof(ctrl), cudaMemcpyDeviceToHost));
+    for (int r = 0; r < n; r++) ok &= xn2[r] == xn[r];
+    ok &= d2c == d2g && ctrl[0] == 1 && ctrl[1] == 1;
+    /* with comm, xs_all is required */
+    c.xs_all = NULL;
+    ok &= acsr_pagerank_step(&c, st) == ACSR_ERR_INVALID_VALUE;
+    AK(acsr_comm_destroy(comm));
+
+    /* O8 partition on the device, and a valid plan reports ACSR_OK */
+    int64_t *d_splits, splits[3];
+    void *d_pws;
+    size_t pws = acsr_partition_workspace_bytes(n);
+    CK(cudaMalloc((void **)&d_splits, sizeof(splits)));
+    CK(cudaMalloc(&d_pws, pws));
+    AK(acsr_partition(n, d_rp, NULL, 4, 36, 2, d_splits, d_pws, pws, st));
+    CK(cudaStreamSynchronize(st));
+    CK(cudaMemcpy(splits, d_splits, sizeof(splits), cudaMemcpyDeviceToHost));
+    /* costs 36, 40, 48, 56, 316, 6036 (total 6532): the prefix before row r first reaches
+     * ceil(6532 / 2) = 3266 at r = 6 (the last row holds most of the cost) */
+    ok &= splits[0] == 0 && splits[1] == 6 && splits[2] == 6;
+    AK(acsr_plan_status(d_ws, ws_bytes, st));
     printf("capi_smoke %s (version %d)\n", ok ? "OK" : "FAIL", acsr_version());
     return ok ? 0 : 1;
 }

@@ -818,6 +818,32 @@ def test_degree_relabel_pagerank_equivalent(acsr, cuda):
     assert np.all(np.abs(back - x_ref) <= 1e-11 * x_ref + 1e-18)
 
 
+@pytest.mark.parametrize("scale", [12, 17])
+def test_degree_relabel_structure_bitwise(acsr, cuda, scale):
+    """acsr_degree_relabel against its definition, on the host (integer data, bitwise):
+    order = vertices by decreasing out-degree, ties by increasing id (numpy stable sort);
+    perm = its inverse; new row perm[u] = old row u with every column c replaced by perm[c],
+    in the same order; outdeg' = outdeg[order].  Includes rows longer than the 1024-entry
+    threshold of the CTA copy path at s17."""
+    rp, ci, od, n = _inlink(scale, cuda)
+    rp2, c2, od2, perm = acsr.acsr_degree_relabel(rp.to(cuda), ci.to(cuda), od.to(cuda))
+    rph, cih, odh = rp.numpy(), ci.numpy(), od.numpy()
+    order = np.argsort(-odh.astype(np.int64), kind="stable")
+    pr = np.empty(n, np.int64)
+    pr[order] = np.arange(n)
+    assert np.array_equal(perm.cpu().numpy(), pr)
+    assert np.array_equal(od2.cpu().numpy(), odh[order])
+    ln = np.diff(rph)
+    rp_ref = np.zeros(n + 1, np.int64)
+    rp_ref[1:] = np.cumsum(ln[order])
+    assert np.array_equal(rp2.cpu().numpy(), rp_ref)
+    starts = np.repeat(rph[:-1][order] - rp_ref[:-1], ln[order])
+    src = np.arange(cih.size) + starts  # old position of every new entry
+    assert np.array_equal(c2.cpu().numpy(), pr[cih[src]])
+    if scale == 17:
+        assert ln.max() > 1024
+
+
 def test_paper_epoch_update_bitwise(acsr, cuda):
     # P:337 paper-shaped epoch generated on the device from the live graph (synth.mixed_epoch)
     n, rb, re, cap, col, val, od, rp, ci = _slack_graph(14, frac=1)
@@ -949,6 +975,53 @@ def test_dist_pagerank_two_ranks_one_gpu(cuda):
     assert np.all(np.abs(full - x_ref) <= 1e-11 * x_ref + 1e-18)
 
 
+@pytest.mark.parametrize("compact", [True, False])
+def test_dist_pagerank_acsr_comm_two_ranks(cuda, compact):
+    """The library-owned exchange (acsr_comm: NCCL all-gather of the xs slices + exact
+    global Delta^2 inside acsr_pagerank_step) with two ranks, here sharing one GPU (NCCL
+    over its socket transport; see the worker).  Same iterate, iteration count and
+    Delta^2 bits as the torch.distributed exchange, and the oracle bar."""
+    full_a, it_a, d2_a = _two_ranks(14, exchange="acsr", compact=compact, check_every=4)
+    full_t, it_t, d2_t = _two_ranks(14, exchange="torch", compact=compact)
+    assert it_a == it_t
+    assert np.array_equal(full_a, full_t)
+    # the library adds exact fixed-point partials: the single-GPU Delta^2 of the last step
+    rp, ci, od, n = _inlink(14, cuda)
+    x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)
+    assert abs(it_a - it_ref) <= 1
+    if it_a != it_ref:
+        x_ref, _, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=0.0, max_iter=it_a)
+    assert np.all(np.abs(full_a - x_ref) <= 1e-11 * x_ref + 1e-18)
+    assert d2_a == pytest.approx(d2_t, rel=1e-12)
+
+
+def test_acsr_partition_equals_oracle(acsr, cuda):
+    """acsr_partition (O8 on the device: CUB prefix + binary search) = oracle.partition bitwise."""
+    for scale, P, bn, br in ((14, 2, 4, 36), (16, 3, 12, 16), (17, 8, 4, 36), (10, 1, 4, 36)):
+        rp, ci = synth.rmat_csr(scale, transpose=True)
+        got = acsr.acsr_partition(rp.to(cuda), P, bn, br).cpu().numpy()
+        assert np.array_equal(got, oracle.partition(rp.numpy(), P, bn, br)), (scale, P)
+    rb, re, cap, c2, _ = synth.with_slack(*synth.rmat_csr(12))
+    got = acsr.acsr_partition(rb.to(cuda), 4, 4, 36, row_end=re.to(cuda)).cpu().numpy()
+    assert np.array_equal(got, oracle.partition(rb.numpy(), 4, 4, 36, row_end=re.numpy()))
+    empty = acsr.acsr_partition(torch.zeros(1, dtype=torch.int32, device=cuda), 3, 4, 36).cpu().numpy()
+    assert np.array_equal(empty, [0, 0, 0, 0])
+
+
+def test_single_rank_acsr_comm_step_equals_pagerank(acsr, cuda):
+    """acsr_pagerank_step with a one-rank acsr_comm (exchange + global Delta^2 in the
+    library) gives the single-GPU loop's iterate, iteration count and Delta^2 bitwise."""
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+    rp, ci, od, n = _inlink(15, cuda)
+    m = acsr.ACSRMatrix(rp.to(cuda), ci.to(cuda))
+    x1, it1, d21 = acsr.pagerank(m, od.to(cuda), eps=1e-6)
+    pr = pdist.DistPageRank(rp.to(cuda), ci.to(cuda), od.to(cuda), np.array([0, n]), n, exchange="acsr")
+    assert pr.comm.query() == (1, 0)
+    x2, it2, d22 = pr.run(eps=1e-6)
+    assert it1 == it2 and torch.equal(x1, x2) and d21 == d22
+    pr.comm.close()
+
+
 @pytest.mark.parametrize("dtype", ["float64", "float32"])
 def test_dist_spmv_row_split_bitwise(acsr, cuda, dtype):
     """N4 (P:345 row split): one SpMV row-split over three ranks sharing the GPU equals the
@@ -990,7 +1063,7 @@ def test_peer_exchange_two_ranks_one_gpu(cuda, compact):
     # bits (iterate, iteration count, Delta^2); every rank's replicated xs identical
     # (checked in the worker); and the oracle bar.
     full_p, it_p, d2_p = _two_ranks(14, exchange="peer", compact=compact)
-    full_c, it_c, d2_c = _two_ranks(14, exchange="nccl", compact=compact)
+    full_c, it_c, d2_c = _two_ranks(14, exchange="torch", compact=compact)
     assert it_p == it_c and np.array_equal(full_p, full_c)
     # Delta^2: the collective path all-reduces two rounded doubles, the peer path adds the
     # exact fixed-point partials and rounds once -> equal up to that one rounding
@@ -1009,7 +1082,7 @@ def test_peer_exchange_three_ranks_one_gpu(cuda):
     # three ranks: every fused step stores its slice into two remote regions (the
     # out-of-line remote loop with the self-skip); same bits as the collective path
     full_p, it_p, _ = _two_ranks(13, world=3, exchange="peer", compact=True, check_every=4)
-    full_c, it_c, _ = _two_ranks(13, world=3, exchange="nccl", compact=True)
+    full_c, it_c, _ = _two_ranks(13, world=3, exchange="torch", compact=True)
     assert it_p == it_c and np.array_equal(full_p, full_c)
     rp, ci, od, n = _inlink(13, cuda)
     x_ref, it_ref, _ = oracle.pagerank(rp.numpy(), ci.numpy(), od.numpy(), eps=1e-6)

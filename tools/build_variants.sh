@@ -3,8 +3,10 @@
 set -e
 cd "$(dirname "$0")/.."
 L=paper_conf_sc_ashariseps14_b200/lib
-F="-O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo -Xcompiler -fPIC -shared -cudart shared"
-build() { name=$1; shift; nvcc $F "$@" -o $L/libacsr_$name.so paper_conf_sc_ashariseps14_b200/csrc/*.cu & }
+NC=$(python -c "import __graft_entry__ as g; print(g.nccl_dirs()[0])")
+NL=$(python -c "import __graft_entry__ as g; print(g.nccl_dirs()[1])")
+F="-O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo -Xcompiler -fPIC -shared -cudart shared -I $NC"
+build() { name=$1; shift; nvcc $F "$@" -o $L/libacsr_$name.so paper_conf_sc_ashariseps14_b200/csrc/*.cu -L $NL -l:libnccl.so.2 -Xlinker -rpath=$NL & }
 for v in "$@"; do
   case $v in
     s1) build s1 -DACSR_STREAM_LD=1 ;;
@@ -55,6 +57,10 @@ for v in "$@"; do
     us1) build us1 -DACSR_UPD_SUB=1 ;;
     sc256) build sc256 -DACSR_SCAN_THREADS=256 ;;
     td8) build td8 -DACSR_TAIL_DIV=8 ;;
+    pf) build pf -DACSR_PF_UNIT=1 ;;
+    t256mb5) build t256mb5 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=5 ;;
+    pft256mb5) build pft256mb5 -DACSR_PF_UNIT=1 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=5 ;;
+    pfwg8) build pfwg8 -DACSR_PF_UNIT=1 -DACSR_WIN_G=8 ;;
     td32) build td32 -DACSR_TAIL_DIV=32 ;;
     wu64) build wu64 -DACSR_WIN_UNIT_ROWS=64 ;;
     wu32) build wu32 -DACSR_WIN_UNIT_ROWS=32 ;;

@@ -189,6 +189,7 @@ __device__ __forceinline__ void scan_row(BinSmem &sm, const int32_t *__restrict_
         hdr->off_xc_vote = (int64_t)sa.L.off_xc_vote;
         hdr->off_xc_tag = (int64_t)sa.L.off_xc_tag;
         hdr->off_xc_val = (int64_t)sa.L.off_xc_val;
+        hdr->off_tile_done = (int64_t)sa.L.off_tile_done;
         hdr->xc_valid = sa.xc_valid;
         hdr->xc_stride = sa.xc_stride;
         hdr->n_cols = sa.n_cols;
@@ -240,6 +241,7 @@ __device__ __forceinline__ void plan_from_totals(BinSmem &sm, PlanHeader *hdr, c
         hdr->off_xc_vote = (int64_t)sa.L.off_xc_vote;
         hdr->off_xc_tag = (int64_t)sa.L.off_xc_tag;
         hdr->off_xc_val = (int64_t)sa.L.off_xc_val;
+        hdr->off_tile_done = (int64_t)sa.L.off_tile_done;
         hdr->xc_valid = sa.xc_valid;
         hdr->xc_stride = sa.xc_stride;
         hdr->n_cols = sa.n_cols;
@@ -294,8 +296,9 @@ template <bool HAS_END>
 __device__ __forceinline__ void scatter_tile(BinSmem &sm, const ScatterPre &pre, int64_t n,
                                              int32_t *__restrict__ bin_rows, int n_tiles,
                                              int2 *__restrict__ units, int32_t *__restrict__ tickets,
-                                             int64_t heavy_cap, int tile, int wmb)
+                                             int64_t heavy_cap, int tile, int wmb, int32_t *tile_done)
 {
+    if (threadIdx.x == 0) tile_done[tile] = 0;  // the fused peer exchange's per-tile row count
     constexpr int NW = BIN_THREADS / 32;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     // sm.boff / sm.ovf / sm.nheavy were filled by the caller (plan_from_totals or
@@ -442,7 +445,8 @@ bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__r
     scatter_preload<HAS_END>(pre, n, rb, re, toff, n_tiles, blockIdx.x);  // overlaps the prologue
     plan_from_totals(sm, hdr, sa, n_tiles, blockIdx.x == 0);
     __syncthreads();
-    scatter_tile<HAS_END>(sm, pre, n, bin_rows, n_tiles, units, tickets, sa.heavy_cap, blockIdx.x, wmb);
+    scatter_tile<HAS_END>(sm, pre, n, bin_rows, n_tiles, units, tickets, sa.heavy_cap, blockIdx.x, wmb,
+                          (int32_t *)((char *)hdr + sa.L.off_tile_done));
 }
 
 // ---- scan + scatter in ONE launch (opt-in, ACSR_BIN_SS=1): the first SCAN_ROWS CTAs to start (an
@@ -489,7 +493,8 @@ bin_scan_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t
     ScatterPre pre;
     scatter_preload<HAS_END>(pre, n, rb, re, toff, n_tiles, tile);  // toff is complete after the wait
     __syncthreads();
-    scatter_tile<HAS_END>(sm, pre, n, bin_rows, n_tiles, units, tickets, sa.heavy_cap, tile, wmb);
+    scatter_tile<HAS_END>(sm, pre, n, bin_rows, n_tiles, units, tickets, sa.heavy_cap, tile, wmb,
+                          (int32_t *)((char *)hdr + sa.L.off_tile_done));
 }
 
 // ---- one cooperative launch: count -> grid barrier -> scan -> grid barrier -> scatter
@@ -524,7 +529,7 @@ bin_fused_kernel(FusedArgs f)
         ScatterPre pre;
         scatter_preload<HAS_END>(pre, f.n, f.rb, f.re, f.toff, f.n_tiles, t);
         scatter_tile<HAS_END>(sm, pre, f.n, f.bin_rows, f.n_tiles, f.units,
-                              f.tickets, f.sa.heavy_cap, t, f.wmb);
+                              f.tickets, f.sa.heavy_cap, t, f.wmb, (int32_t *)((char *)f.hdr + f.sa.L.off_tile_done));
     }
 }
 

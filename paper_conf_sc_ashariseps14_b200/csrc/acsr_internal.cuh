@@ -149,13 +149,14 @@ struct PlanHeader {
     int64_t n_cols;
     uint64_t d2_hi, d2_mid, d2_lo;  // exact 192-bit fixed-point Delta^2 accumulator (PageRank/RWR)
     int64_t off_units, off_partial, off_ticket, off_xc_vote, off_xc_tag, off_xc_val;
+    int64_t off_tile_done;  // int32 [n_tiles]: rows finished per tile (fused peer exchange), zeroed by acsr_bin
     int32_t totals[NBINS + 2 + 2];  // per scan row totals (bins, light units, heavy units)
 };
 
 struct PlanLayout {
     int64_t n_tiles = 0, light_cap = 0, heavy_cap = 0;
     size_t off_cnt = 0, off_toff = 0, off_units = 0, off_partial = 0, off_ticket = 0,
-           off_xc_vote = 0, off_xc_tag = 0, off_xc_val = 0, off_xc_count = 0, total = 0;
+           off_xc_vote = 0, off_xc_tag = 0, off_xc_val = 0, off_xc_count = 0, off_tile_done = 0, total = 0;
 };
 
 __host__ __device__ inline size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
@@ -188,6 +189,8 @@ inline PlanLayout plan_layout(int64_t n_rows, int64_t n_cols, int64_t nnz_max)
     o = align_up(o + sizeof(double) * (size_t)L.heavy_cap, 256);
     L.off_ticket = o;
     o = align_up(o + sizeof(int32_t) * (size_t)L.heavy_cap, 256);
+    L.off_tile_done = o;  // rows finished per tile (fused peer exchange)
+    o = align_up(o + sizeof(int32_t) * (size_t)L.n_tiles, 256);
     L.off_xc_count = o;  // sampled occurrence count per column
     o = align_up(o + sizeof(int32_t) * (size_t)(n_cols > 0 ? n_cols : 0), 256);
     L.total = o;

@@ -53,6 +53,9 @@
 #ifndef ACSR_PF_UNIT
 #define ACSR_PF_UNIT 0  // 1: L2 bulk prefetch of a unit's col/val runs at unit start (A/B)
 #endif
+#ifndef ACSR_PEER_TILE_PUSH
+#define ACSR_PEER_TILE_PUSH 1  // 0: every finished row is stored to every peer at once (round-1 A/B)
+#endif
 #ifndef ACSR_VEC_MIN
 #define ACSR_VEC_MIN 512  // rows (chunks) shorter than this use the lane-strided scalar path
 #endif
@@ -93,6 +96,7 @@ struct SpmvArgs {
     double eps2;
     int64_t n_rows;  // rows of the call (NaN fill of an overflowed plan)
     uint64_t *d2_out;  // multi-GPU (acsr_comm): the last CTA writes this rank's exact 192-bit partial here
+    int32_t *tile_done;  // fused peer exchange: rows finished per tile (plan workspace)
     int64_t x_prefetch;  // bytes of x to bulk-prefetch into L2 at entry (0: none)
     // fused peer-memory exchange of xs_next (acsr_pagerank_step_peer; peer.nranks == 0: off)
     const PeerArgs *peer;  // device copy (PeerState::view) or NULL
@@ -151,6 +155,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t phase)
 // and truncated below 2^-128.
 struct Fix192 {
     uint64_t hi, mid, lo;
+    int fin, ftile;  // fused peer exchange: rows this lane finished in the current unit, their tile
 };
 
 __device__ __forceinline__ void fix_merge(Fix192 &a, uint64_t hi, uint64_t mid, uint64_t lo)
@@ -402,7 +407,11 @@ struct Kern {
             if (PEER && r < a.peer_len) {
                 const int64_t o = a.peer_next + 8 * (a.peer_off + r);
                 *(double *)(a.pself + o) = xs;  // own replicated buffer: inline
-                if (a.peer_n > 1) peer_store(a.pbase, a.peer_n, a.peer_rank, o, xs);
+                if (!ACSR_PEER_TILE_PUSH && a.peer_n > 1) peer_store(a.pbase, a.peer_n, a.peer_rank, o, xs);
+            }
+            if (PEER) {  // per-tile completion count (peer_tile_done)
+                d2.fin++;
+                d2.ftile = r / TILE_ROWS;
             }
             const double diff = xn - __ldg(a.x_old + r);
             fix_add(d2, diff * diff);
@@ -786,6 +795,41 @@ struct Kern {
     }
 #endif
 
+    // Fused peer exchange, per-tile push (ACSR_PEER_TILE_PUSH): every row of a unit lies in
+    // one 1024-row tile; after the unit the warp adds its finished rows to the tile's count
+    // (release: threadfence before the atomic), and the warp that completes the tile reads
+    // the tile's xs' entries back from its own buffer (L2) and stores them to every other
+    // rank as coalesced 256-byte warp stores -- instead of one scattered 8-byte remote store
+    // per row and peer as rows finish in bin order.
+    static __device__ __forceinline__ void peer_tile_done(const A &a, int lane, Fix192 &d2)
+    {
+        constexpr unsigned FULL = 0xffffffffu;
+        const int total = __reduce_add_sync(FULL, d2.fin);
+        if (total == 0) return;
+        const unsigned any = __ballot_sync(FULL, d2.fin > 0);
+        const int tile = __shfl_sync(FULL, d2.ftile, __ffs(any) - 1);
+        d2.fin = 0;
+        const int tile_rows = (int)min((int64_t)TILE_ROWS, a.n_rows - (int64_t)tile * TILE_ROWS);
+        int done = 0;
+        if (lane == 0) {
+            __threadfence();
+            done = atomicAdd(a.tile_done + tile, total) + total == tile_rows;
+        }
+        done = __shfl_sync(FULL, done, 0);
+        if (!done) return;
+        __threadfence();
+        const int r0 = tile * TILE_ROWS;
+        const int r1 = min(r0 + tile_rows, a.peer_len);
+        const char *own = a.pself + a.peer_next + 8 * a.peer_off;
+        for (int q = 0; q < a.peer_n; q++) {
+            if (q == a.peer_rank) continue;
+            char *dst = a.pbase[q] + a.peer_next + 8 * a.peer_off;
+            for (int r = r0 + lane; r < r1; r += 32)
+                *(double *)(dst + 8 * (int64_t)r) = __ldcg((const double *)(own + 8 * (int64_t)r));
+        }
+        if (lane == 0) a.tile_done[tile] = 0;  // ready for the next step on this plan
+    }
+
     static __device__ __forceinline__ void unit(const A &a, int u, int lane, Fix192 &d2, double *wbuf, int2 *wtab)
     {
         const int2 d = __ldg(a.units + u);
@@ -913,6 +957,7 @@ spmv_kernel(SpmvArgs<V> a)
         a.units = (const int2 *)(ws + hdr->off_units);
         a.partial = (double *)(ws + hdr->off_partial);
         a.ticket = (int32_t *)(ws + hdr->off_ticket);
+        a.tile_done = (int32_t *)(ws + hdr->off_tile_done);
     }
     if (XC) {
         // shared x cache: [XC_SLOTS values | XC_SLOTS 16-bit tags], filled by TMA bulk copies
@@ -939,9 +984,13 @@ spmv_kernel(SpmvArgs<V> a)
     __shared__ int2 win_tab[WIN_MAX_BIN >= 0 ? SPMV_WARPS * 32 : 1];
     double *wbuf = win_buf + (WIN_MAX_BIN >= 0 ? (threadIdx.x >> 5) * 32 * WIN_G : 0);
     int2 *wtab = win_tab + (WIN_MAX_BIN >= 0 ? (threadIdx.x >> 5) * 32 : 0);
-    Fix192 d2{0, 0, 0};
+    Fix192 d2{0, 0, 0, 0, 0};
+    const bool tile_push = PEER && ACSR_PEER_TILE_PUSH && a.peer_n > 1;
 #if ACSR_SCHED_STATIC
-    for (int u = gw; u < n_units; u += nw) K::unit(a, u, lane, d2, wbuf, wtab);
+    for (int u = gw; u < n_units; u += nw) {
+        K::unit(a, u, lane, d2, wbuf, wtab);
+        if (tile_push) K::peer_tile_done(a, lane, d2);
+    }
 #else
     // first prefetched claims: one atomic per CTA (a same-address atomic per warp at
     // launch costs microseconds of serialisation at the L2 slice)
@@ -952,6 +1001,7 @@ spmv_kernel(SpmvArgs<V> a)
     int nxt = s_claim + (threadIdx.x >> 5);
     while (u < n_units) {
         K::unit(a, u, lane, d2, wbuf, wtab);
+        if (tile_push) K::peer_tile_done(a, lane, d2);
         u = __shfl_sync(0xffffffffu, nxt, 0) + nw;
         if (u < n_units && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
     }
@@ -976,7 +1026,7 @@ spmv_kernel(SpmvArgs<V> a)
     __syncthreads();
     if (threadIdx.x >= 32) return;
     if (PR) {
-        d2 = lane < SPMV_WARPS ? Fix192{s_d2[lane][0], s_d2[lane][1], s_d2[lane][2]} : Fix192{0, 0, 0};
+        d2 = lane < SPMV_WARPS ? Fix192{s_d2[lane][0], s_d2[lane][1], s_d2[lane][2], 0, 0} : Fix192{0, 0, 0, 0, 0};
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
             const uint64_t h = __shfl_xor_sync(0xffffffffu, d2.hi, o);

@@ -106,6 +106,8 @@ class UpdateGraph:
                      "ins_cols": torch.zeros(self.max_ins, dtype=torch.int32, device=dev)}
         self.status = torch.zeros(2, dtype=torch.int32, device=dev)
         self.ws = torch.empty(acsr_update_workspace_bytes(self.max_upd), dtype=torch.uint8, device=dev)
+        self._h2d_done = None  # event after the last replay's H2D copies
+        self._pending = None   # the last replay's host change lists (alive until copied)
 
         def seq():
             m.update(self.bufs, outdeg=outdeg, status=self.status, ws=self.ws, n_upd_dev=self.n_dev)
@@ -121,16 +123,25 @@ class UpdateGraph:
             seq()
 
     def replay(self, changes_host):
-        """changes_host: dict of pinned host int32 tensors upd_rows, ins_ptr, ins_cols."""
+        """changes_host: dict of pinned host int32 tensors upd_rows, ins_ptr, ins_cols.
+        The H2D copies are asynchronous: the pinned batch size this object writes is only
+        rewritten after the previous replay's copies have executed (an event), and the
+        caller's change tensors are kept referenced until the next replay, so several
+        replays may be enqueued without a synchronisation."""
         n = changes_host["upd_rows"].numel()
         k = changes_host["ins_cols"].numel()
         if n > self.max_upd or k > self.max_ins:
             raise ValueError("batch exceeds the UpdateGraph capacities")
+        if self._h2d_done is not None:
+            self._h2d_done.synchronize()  # the previous DMA has read n_host (and its lists)
         self.bufs["upd_rows"][:n].copy_(changes_host["upd_rows"], non_blocking=True)
         self.bufs["ins_ptr"][:n + 1].copy_(changes_host["ins_ptr"], non_blocking=True)
         self.bufs["ins_cols"][:k].copy_(changes_host["ins_cols"], non_blocking=True)
         self.n_host[0] = n
         self.n_dev.copy_(self.n_host, non_blocking=True)
+        self._h2d_done = torch.cuda.Event()
+        self._h2d_done.record()
+        self._pending = changes_host
         self.graph.replay()
         return self.status
 

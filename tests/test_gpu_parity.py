@@ -549,6 +549,20 @@ def test_update_graph_replay_bitwise(acsr, cuda):
         xs_ref = np.where(od_h > 0, x.cpu().numpy() / np.maximum(od_h, 1), 0.0)
         y_ref, den = oracle.spmv(rb.numpy(), col_h, None, xs_ref, row_end=re_h)
         check_spmv(y.cpu().numpy(), y_ref, den, torch.float64)
+    # the same three batches replayed back to back with NO synchronisation in between
+    # (the pinned batch size must not be overwritten before its copy ran)
+    m2 = acsr.ACSRMatrix(rb.to(cuda), col.to(cuda), None, row_end=re.to(cuda), row_cap=cap.to(cuda),
+                         nnz_max=col.numel())
+    odd2 = od.to(cuda)
+    y2 = torch.empty_like(x)
+    g2 = acsr.UpdateGraph(m2, odd2, x, torch.empty_like(x), y2, max_upd=6000, max_ins=6000)
+    for ch in batches:
+        g2.replay({k: torch.from_numpy(v).pin_memory() for k, v in ch.items()})
+    torch.cuda.synchronize()
+    assert g2.status.cpu().tolist() == [0, -1]
+    assert np.array_equal(m2.row_end.cpu().numpy(), re_h)
+    assert np.array_equal(m2.col_idx.cpu().numpy()[live], col_h[live])
+    assert np.array_equal(odd2.cpu().numpy(), od_h) and torch.equal(y2, y)
     # a device batch size beyond the capacity buffers: rejected, nothing modified
     before = m.col_idx.clone(), m.row_end.clone()
     g.n_host[0] = 7000

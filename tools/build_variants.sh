@@ -58,6 +58,7 @@ for v in "$@"; do
     sc256) build sc256 -DACSR_SCAN_THREADS=256 ;;
     td8) build td8 -DACSR_TAIL_DIV=8 ;;
     pf) build pf -DACSR_PF_UNIT=1 ;;
+    ptp0) build ptp0 -DACSR_PEER_TILE_PUSH=0 ;;
     t256mb5) build t256mb5 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=5 ;;
     pft256mb5) build pft256mb5 -DACSR_PF_UNIT=1 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=5 ;;
     pfwg8) build pfwg8 -DACSR_PF_UNIT=1 -DACSR_WIN_G=8 ;;

@@ -77,7 +77,7 @@ def _L():
         _lib.oracle_update.argtypes = [i64, i64, i32p, i32p, i32p, i32p, vp, ctypes.c_int, i64,
                                        i32p, i32p, i32p, i32p, i32p, vp, i32p, i32p]
         _lib.oracle_update.restype = ctypes.c_int
-        _lib.oracle_partition.argtypes = [i64, i32p, i32p, i64, i64, ctypes.c_int, vp]
+        _lib.oracle_partition.argtypes = [i64, i32p, i32p, i64, i64, ctypes.c_int, i64, vp]
         _lib.oracle_csr_build.argtypes = [i64, i64, i32p, i32p, vp, ctypes.c_int, ctypes.c_int,
                                           i32p, i32p, vp]
         _lib.oracle_csr_build.restype = i64
@@ -237,11 +237,11 @@ def update(n_cols, row_begin, row_end, row_cap, col, val, upd_rows, del_ptr, del
     return int(st[0]), int(st[1])
 
 
-def partition(row_begin, P, b_nnz, b_row, row_end=None):
+def partition(row_begin, P, b_nnz, b_row, row_end=None, align=1):
     rb, re = _i32(row_begin), _i32(row_end)
     n = _n_rows(rb, re)
     s = np.empty(P + 1, np.int64)
-    _L().oracle_partition(n, _p(rb), _p(re), int(b_nnz), int(b_row), int(P), _p(s))
+    _L().oracle_partition(n, _p(rb), _p(re), int(b_nnz), int(b_row), int(P), int(align), _p(s))
     return s
 
 

@@ -126,6 +126,12 @@ def test_partition_bruteforce(P):
         assert s[k] == brute
     assert np.all(np.diff(s) >= 0)
     assert np.all(np.diff(pref[s]) <= -(-total // P) + cost.max())
+    # reading R7: split points rounded up to a multiple of `align`, clamped to n
+    for align in (32, 1024, 5000):
+        sa = oracle.partition(rp, P, 4, 36, align=align)
+        assert sa[0] == 0 and sa[P] == n
+        for k in range(1, P):
+            assert sa[k] == min(n, -(-int(s[k]) // align) * align)
 
 
 def test_csr_build_vs_scipy():

@@ -262,7 +262,7 @@ def row_split(rp, ci, val, rank, world, b_nnz, b_row):
     summed as on one GPU.  Returns (row_ptr_local, col_local, val_local, splits)."""
     import paper_conf_sc_ashariseps14_b200 as acsr
     from paper_conf_sc_ashariseps14_b200 import dist as pdist
-    splits = acsr.acsr_partition(rp, world, b_nnz, b_row).cpu().numpy()
+    splits = acsr.acsr_partition(rp, world, b_nnz, b_row, align=32).cpu().numpy()
     lo, hi = int(splits[rank]), int(splits[rank + 1])
     k0, k1 = int(rp[lo]), int(rp[hi])
     rpl = (rp[lo:hi + 1].to(torch.int64) - k0).to(torch.int32)
@@ -524,12 +524,13 @@ def run_pagerank(args, dev, rank, world):
     outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
     t_relabel = None
     if args.relabel:  # acsr_degree_relabel on the device (sort + scan + copy), timed with events
+        srt = args.relabel_sort
         for _ in range(2):
-            acsr.acsr_degree_relabel(rp, ci, outdeg)
+            acsr.acsr_degree_relabel(rp, ci, outdeg, sort_rows=srt)
         torch.cuda.synchronize()
         r0, r1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         r0.record()
-        rp2, ci2, od2, _ = acsr.acsr_degree_relabel(rp, ci, outdeg)
+        rp2, ci2, od2, _ = acsr.acsr_degree_relabel(rp, ci, outdeg, sort_rows=srt)
         r1.record()
         torch.cuda.synchronize()
         t_relabel = r0.elapsed_time(r1) * 1e-3
@@ -591,7 +592,8 @@ def run_pagerank(args, dev, rank, world):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"pagerank_rmat{S}_inlink" + ("_degree_relabelled" if args.relabel else ""),
                        "n_rows": n, "nnz": nnz, "non_dangling": n_nd,
-                       "relabel": "acsr_degree_relabel (device)" if args.relabel else None,
+                       "relabel": ("acsr_degree_relabel (device%s)" % (", rows sorted" if args.relabel_sort else ""))
+                       if args.relabel else None,
                        "l2": "not flushed (iterative use); x = %d MB" % (8 * n >> 20),
                        "parallelism": "independent replica per rank" if world > 1 else "1 GPU"},
             "breakdown": {"t_bin_ms": round(t_bin, 4), "cold_iterations": it, "final_delta": dd ** 0.5,
@@ -601,7 +603,8 @@ def run_pagerank(args, dev, rank, world):
                           round((t_relabel + t_conv) * 1e3 + t_bin, 3),
                           "gflops_equiv": round(nnz / (ms * 1e-3) / 1e9, 2)},
             "roofline": {"bound": "hbm", "achieved": round(alg / (ms * 1e-3) / 1e9, 1), "peak": peak, "unit": "GB/s",
-                         "frac": round(alg / (ms * 1e-3) / 1e9 / peak, 4), "traffic": None,
+                         "frac": round(alg / (ms * 1e-3) / 1e9 / peak, 4),
+                         "traffic": ncu_traffic(f"pagerank_rmat{S}_inlink" + ("_degree_relabelled" if args.relabel else "")),
                          "kernel": "acsr::spmv_kernel<PR>", "peak_kind": kind,
                          "algorithmic_bytes_per_launch": int(alg)},
             "gpu_launches": K, "clocks": clk.summary()}
@@ -987,9 +990,17 @@ def run_dynamic(args, dev, rank, world):
         x, it, _ = acsr.pagerank(m, outdeg, x0=x, eps=1e-6)
         x_g.copy_(x)
     r = np.array(rec)
+    # SURVEY §8(d) algorithmic bytes of the dominant kernel (the pattern SpMV on the slack
+    # in-link CSR after the last batch): col 4 nnz + row_begin/row_end/bin_rows 12 n +
+    # x gathers 8 n_c (referenced = non-dangling sources) + y 8 n
+    nnz_now = int((m.row_end - m.row_begin).to(torch.int64).sum())
+    n_c_now = int((outdeg > 0).sum())
+    alg_spmv = 4 * nnz_now + 12 * n + 8 * n_c_now + 8 * n
     if rank != 0:
         return None
     t_h2d, t_upd, t_bin, t_spmv = (float(r[:, i].mean()) for i in range(4))
+    peak, kind = peaks()
+    label_dyn = f"dynamic_rmat{S}_inlink_16384_insert_batches"
     return {"metric": "bin+SpMV ms per dynamic-graph update (C5)", "value": round(t_bin + t_spmv, 5),
             "unit": "ms", "n_gpus": world, "steps": len(rec), "warmup": args.warmup,
             "ms_per_step": round(t_h2d + t_upd + t_bin + t_spmv, 5), "higher_is_better": False,
@@ -1014,6 +1025,11 @@ def run_dynamic(args, dev, rank, world):
                           "inserted_edges_mean": round(float(r[:, 6].mean()), 1),
                           "batch_encode_s_total": round(t_gen, 2),
                           "relayouts": relayouts},
+            "roofline": {"bound": "hbm", "achieved": round(alg_spmv / (t_spmv * 1e-3) / 1e9, 1), "peak": peak,
+                         "unit": "GB/s", "frac": round(alg_spmv / (t_spmv * 1e-3) / 1e9 / peak, 4),
+                         "traffic": ncu_traffic(label_dyn), "kernel": "acsr::spmv_kernel (pattern, slack CSR)",
+                         "peak_kind": kind, "algorithmic_bytes_per_launch": int(alg_spmv),
+                         "note": "4 nnz + 12 n + 8 n_c + 8 n after the last batch"},
             # per timed batch: update_init + update_validate + update_apply (insert-only),
             # bin_count + bin_scan + bin_scatter, pagerank_scale + spmv_kernel
             "gpu_launches": 8 * len(rec)}
@@ -1130,6 +1146,7 @@ def main():
     ap.add_argument("--scale", type=int, default=None, help="R-MAT scale for pagerank/dynamic")
     ap.add_argument("--batches", type=int, default=None, help="dynamic: number of insertion batches")
     ap.add_argument("--relabel", action="store_true", help="pagerank: degree-ordered vertex relabelling")
+    ap.add_argument("--relabel-sort", action="store_true", help="pagerank --relabel: sort every row's columns")
     ap.add_argument("--exchange", default="acsr", choices=["acsr", "torch", "peer"],
                     help="pagerank_dist: the library's NCCL exchange inside acsr_pagerank_step (acsr_comm), "
                          "torch.distributed collectives, or the exchange fused into the step over peer memory")

@@ -163,13 +163,17 @@ acsr_status acsr_comm_allgather(acsr_comm *comm, const void *send, void *recv, s
 /* O8 row partition, on the device: splits[0] = 0, splits[nranks] = n_rows and
  *   splits[k] = min{ r : sum_{r' < r} cost(r') >= ceil(k * total / nranks) },
  *   cost(r) = b_nnz * len_r + b_row   (integer bytes of the rank's traffic per row:
- *   PageRank pattern 4 * len + 36, weighted fp64 SpMV 12 * len + 16).
+ *   PageRank pattern 4 * len + 36, weighted fp64 SpMV 12 * len + 16),
+ * then each splits[k] rounded up to a multiple of `align` (<= 1: unchanged) and clamped to
+ * n_rows (reading R7: with align = 32 every rank's rows start on a 32-row boundary, so
+ * the SpMV's short-row windows hold the same rows on P ranks as on one GPU and a
+ * row-split SpMV gives the one-GPU y bit for bit).
  * splits: DEVICE int64 [nranks + 1].  ws: acsr_partition_workspace_bytes(n_rows) bytes
  * (an int64 prefix of the costs + the scan's scratch). */
 size_t acsr_partition_workspace_bytes(int64_t n_rows);
 acsr_status acsr_partition(int64_t n_rows, const int32_t *row_begin, const int32_t *row_end /* NULL => standard */,
-                           int64_t b_nnz, int64_t b_row, int nranks, int64_t *splits, void *ws, size_t ws_bytes,
-                           cudaStream_t stream);
+                           int64_t b_nnz, int64_t b_row, int nranks, int64_t align, int64_t *splits, void *ws,
+                           size_t ws_bytes, cudaStream_t stream);
 
 /* ------------------------------------------------------------------------ */
 /* PageRank step (Alg. 5; §VI-A) on one rank's rows.
@@ -338,13 +342,18 @@ acsr_status acsr_hits_normalize(int64_t n, const double *y, const double *v, dou
  *   row_ptr_out [n+1], col_out [nnz], outdeg_out [n]   the relabelled graph
  *   perm_out [n]                   perm_out[v] = new id of old vertex v
  * Order: decreasing out-degree, ties by increasing old id (stable).  Entry j of old row u
- * becomes entry j of new row perm[u] (column order inside a row kept).  col_idx/col_out may
- * be NULL (permutation and row pointers only).  Outputs must not alias the inputs.
- * Everything runs on `stream` (CUB radix sort + scan, two copy kernels; no host sync). */
-size_t acsr_relabel_workspace_bytes(int64_t n);
-acsr_status acsr_degree_relabel(int64_t n, const int32_t *row_ptr, const int32_t *col_idx, const int32_t *outdeg,
-                                int32_t *row_ptr_out, int32_t *col_out, int32_t *outdeg_out, int32_t *perm_out,
-                                void *ws, size_t ws_bytes, cudaStream_t stream);
+ * becomes entry j of new row perm[u] (column order inside a row kept), or -- with flag
+ * ACSR_RELABEL_SORT_ROWS -- every new row's columns are sorted ascending (the hot, now small,
+ * column ids of a row sit together: fewer 128-byte lines per warp gather).  col_idx/col_out
+ * may be NULL (permutation and row pointers only).  Outputs must not alias the inputs.
+ * nnz = row_ptr[n] (sizes the workspace of the row sort).  Everything runs on `stream` (CUB
+ * radix sort + scan, two copy kernels, CUB segmented sort; no host sync).  Unknown flag
+ * bits -> ACSR_ERR_INVALID_VALUE. */
+enum { ACSR_RELABEL_SORT_ROWS = 1u };
+size_t acsr_relabel_workspace_bytes(int64_t n, int64_t nnz, unsigned flags);
+acsr_status acsr_degree_relabel(int64_t n, int64_t nnz, const int32_t *row_ptr, const int32_t *col_idx,
+                                const int32_t *outdeg, int32_t *row_ptr_out, int32_t *col_out, int32_t *outdeg_out,
+                                int32_t *perm_out, unsigned flags, void *ws, size_t ws_bytes, cudaStream_t stream);
 
 /* ------------------------------------------------------------------------ */
 /* Dynamic-graph update (§VII): for update i (row r = upd_rows[i],

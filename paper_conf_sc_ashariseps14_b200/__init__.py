@@ -122,11 +122,11 @@ _lib.acsr_pagerank_init.argtypes = [ctypes.POINTER(PrArgs), _vp]
 _lib.acsr_pagerank_init.restype = ctypes.c_int
 _lib.acsr_partition_workspace_bytes.argtypes = [_i64]
 _lib.acsr_partition_workspace_bytes.restype = _sz
-_lib.acsr_partition.argtypes = [_i64, _vp, _vp, _i64, _i64, ctypes.c_int, _vp, _vp, _sz, _vp]
+_lib.acsr_partition.argtypes = [_i64, _vp, _vp, _i64, _i64, ctypes.c_int, _i64, _vp, _vp, _sz, _vp]
 _lib.acsr_partition.restype = ctypes.c_int
-_lib.acsr_relabel_workspace_bytes.argtypes = [_i64]
+_lib.acsr_relabel_workspace_bytes.argtypes = [_i64, _i64, ctypes.c_uint]
 _lib.acsr_relabel_workspace_bytes.restype = _sz
-_lib.acsr_degree_relabel.argtypes = [_i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
+_lib.acsr_degree_relabel.argtypes = [_i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp, ctypes.c_uint, _vp, _sz, _vp]
 _lib.acsr_degree_relabel.restype = ctypes.c_int
 
 ACSR_BIN_SHORT_ALG2 = 1  # include/acsr.h: per-bin Alg. 2 units for bins 0..5
@@ -365,36 +365,43 @@ class AcsrComm:
             pass
 
 
-def acsr_degree_relabel(row_ptr, col_idx, outdeg, stream=None):
+ACSR_RELABEL_SORT_ROWS = 1
+
+
+def acsr_degree_relabel(row_ptr, col_idx, outdeg, sort_rows=False, stream=None):
     """Degree-ordered relabelling on the device (include/acsr.h).  Returns
-    (row_ptr', col', outdeg', perm) with perm[v] = new id of vertex v (int32)."""
+    (row_ptr', col', outdeg', perm) with perm[v] = new id of vertex v (int32).
+    sort_rows: columns of every new row sorted ascending (ACSR_RELABEL_SORT_ROWS)."""
     n = row_ptr.numel() - 1
     dev = row_ptr.device
+    nnz = col_idx.numel() if col_idx is not None else 0
+    flags = ACSR_RELABEL_SORT_ROWS if sort_rows else 0
     rp2 = torch.empty(n + 1, dtype=torch.int32, device=dev)
     c2 = torch.empty_like(col_idx) if col_idx is not None else None
     od2 = torch.empty(n, dtype=torch.int32, device=dev)
     perm = torch.empty(n, dtype=torch.int32, device=dev)
-    ws = torch.empty(int(_lib.acsr_relabel_workspace_bytes(n)), dtype=torch.uint8, device=dev)
-    _check(_lib.acsr_degree_relabel(n, _dev(row_ptr, torch.int32, "row_ptr"),
+    ws = torch.empty(int(_lib.acsr_relabel_workspace_bytes(n, nnz, flags)), dtype=torch.uint8, device=dev)
+    _check(_lib.acsr_degree_relabel(n, nnz, _dev(row_ptr, torch.int32, "row_ptr"),
                                     _dev(col_idx, torch.int32, "col_idx") if c2 is not None and c2.numel() else None,
                                     _dev(outdeg, torch.int32, "outdeg") if n else None,
                                     _dev(rp2, torch.int32, "row_ptr_out"),
                                     _dev(c2, torch.int32, "col_out") if c2 is not None and c2.numel() else None,
                                     _dev(od2, torch.int32, "outdeg_out") if n else None,
-                                    _dev(perm, torch.int32, "perm_out") if n else None,
+                                    _dev(perm, torch.int32, "perm_out") if n else None, flags,
                                     _dev(ws, torch.uint8, "ws"), ws.numel(), _stream(stream)), "acsr_degree_relabel")
     return rp2, c2, od2, perm
 
 
-def acsr_partition(row_begin, nranks, b_nnz, b_row, row_end=None, stream=None):
-    """O8 split points on the device (int64 CUDA tensor [nranks + 1])."""
+def acsr_partition(row_begin, nranks, b_nnz, b_row, row_end=None, align=1, stream=None):
+    """O8 split points on the device (int64 CUDA tensor [nranks + 1]), rounded up to a
+    multiple of `align` (reading R7)."""
     n = row_begin.numel() - 1 if row_end is None else row_begin.numel()
     dev = row_begin.device
     splits = torch.empty(int(nranks) + 1, dtype=torch.int64, device=dev)
     ws = torch.empty(int(_lib.acsr_partition_workspace_bytes(n)), dtype=torch.uint8, device=dev)
     _check(_lib.acsr_partition(n, _dev(row_begin, torch.int32, "row_begin") if n else None,
                                _dev(row_end, torch.int32, "row_end", True), int(b_nnz), int(b_row), int(nranks),
-                               _dev(splits, torch.int64, "splits"), _dev(ws, torch.uint8, "ws"), ws.numel(),
+                               int(align), _dev(splits, torch.int64, "splits"), _dev(ws, torch.uint8, "ws"), ws.numel(),
                                _stream(stream)), "acsr_partition")
     return splits
 

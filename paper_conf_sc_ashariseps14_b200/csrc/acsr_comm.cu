@@ -51,7 +51,8 @@ __global__ void comm_d2_finalize_kernel(const uint64_t *__restrict__ parts, int 
     if (ctrl && d2 <= eps2) ctrl[0] = 1;
 }
 
-__global__ void split_search_kernel(const int64_t *__restrict__ incl, int64_t n, int P, int64_t *splits)
+__global__ void split_search_kernel(const int64_t *__restrict__ incl, int64_t n, int P, int64_t align,
+                                    int64_t *splits)
 {
     const int k = blockIdx.x * blockDim.x + threadIdx.x;
     if (k > P) return;
@@ -68,6 +69,10 @@ __global__ void split_search_kernel(const int64_t *__restrict__ incl, int64_t n,
         const int64_t f = mid ? incl[mid - 1] : 0;
         if (f >= target) hi = mid;
         else lo = mid + 1;
+    }
+    if (align > 1) {  // reading R7: every rank starts on an aligned row
+        lo = (lo + align - 1) / align * align;
+        if (lo > n) lo = n;
     }
     splits[k] = lo;
 }
@@ -214,8 +219,8 @@ extern "C" size_t acsr_partition_workspace_bytes(int64_t n_rows)
 }
 
 extern "C" acsr_status acsr_partition(int64_t n_rows, const int32_t *row_begin, const int32_t *row_end,
-                                      int64_t b_nnz, int64_t b_row, int nranks, int64_t *splits, void *ws,
-                                      size_t ws_bytes, cudaStream_t stream)
+                                      int64_t b_nnz, int64_t b_row, int nranks, int64_t align, int64_t *splits,
+                                      void *ws, size_t ws_bytes, cudaStream_t stream)
 {
     if (n_rows < 0 || nranks < 1 || !splits || b_nnz < 0 || b_row < 0 || (n_rows > 0 && !row_begin)) {
         acsr_set_error("acsr_partition: invalid argument");
@@ -237,6 +242,6 @@ extern "C" acsr_status acsr_partition(int64_t n_rows, const int32_t *row_begin, 
             return ACSR_ERR_CUDA;
         }
     }
-    split_search_kernel<<<(nranks + 1 + 127) / 128, 128, 0, stream>>>(incl, n_rows, nranks, splits);
+    split_search_kernel<<<(nranks + 1 + 127) / 128, 128, 0, stream>>>(incl, n_rows, nranks, align, splits);
     return acsr_check_launch("acsr_partition");
 }

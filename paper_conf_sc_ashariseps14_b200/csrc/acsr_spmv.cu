@@ -47,6 +47,9 @@
 #ifndef ACSR_WIN_LDS4
 #define ACSR_WIN_LDS4 0  // 1: four shared loads in flight per add group (A/B: C3a +6 %, C2 +2 %, slower)
 #endif
+#ifndef ACSR_WIN_SEGSCAN
+#define ACSR_WIN_SEGSCAN 1  // 0: per-lane in-order sums of the row's products from shared memory (round 1)
+#endif
 #ifndef ACSR_WIN_PREFETCH
 #define ACSR_WIN_PREFETCH 0  // 1: prefetch the next window's row bounds (A/B: no gain on C3a, LiveJournal-like +5 %)
 #endif
@@ -328,6 +331,8 @@ __device__ __forceinline__ double ldx(const float *p)
     return (double)__ldg(p);
 #endif
 }
+
+__device__ __forceinline__ bool cb_valid(int cb, int T) { return cb < T; }
 
 // xs' slice entry -> every OTHER rank's replicated buffer (byte offset o in each region)
 __device__ __noinline__ void peer_store(char *const *pbase, int nranks, int self, int64_t o, double v)
@@ -657,10 +662,16 @@ struct Kern {
             const int T = __shfl_sync(FULL, incl, 31);
             const unsigned ne = __ballot_sync(FULL, l > 0);
             if (l > 0) tab[__popc(ne & lt)] = make_int2(beg, pre);
+#if ACSR_WIN_SEGSCAN
+            buf[lane] = 0.0;  // per-row partial sums (tab index)
+#endif
             __syncwarp();
             double acc = 0.0;
             for (int t0 = 0; t0 < T; t0 += 32 * WIN_G) {
                 double p[WIN_G];
+#if ACSR_WIN_SEGSCAN
+                int rjg[WIN_G];
+#endif
 #pragma unroll
                 for (int g = 0; g < WIN_G; g++) {
                     const int cb = t0 + 32 * g;
@@ -674,13 +685,38 @@ struct Kern {
                     // row found for a clamped lane is the last non-empty row, which holds T-1.
                     const bool v = cb + lane < T;
                     const int t = v ? cb + lane : T - 1;
-                    const int2 bp = tab[q0 + __popc(H & le) - 1];
+                    const int rj = q0 + __popc(H & le) - 1;  // the element's row (tab index)
+                    const int2 bp = tab[rj];
                     const int k = bp.x + (t - bp.y);
                     const int c = lds_i(a.col + k);
                     const double xv = gx(a, c);
                     const double pv = HAS_VAL ? lds_v(a.val + k) * xv : xv;
                     p[g] = v ? pv : 0.0;
+#if ACSR_WIN_SEGSCAN
+                    rjg[g] = rj;
+#endif
                 }
+#if ACSR_WIN_SEGSCAN
+                // segmented reduction of each 32-element group by shuffles (rows are
+                // contiguous lane runs, the row index rj is non-decreasing across lanes):
+                // after the inclusive segmented scan the last lane of each run holds the
+                // run's sum and adds it to the row's partial in shared memory (groups in
+                // order -> deterministic for a given window)
+#pragma unroll
+                for (int g = 0; g < WIN_G; g++) {
+                    double sv = p[g];
+                    const int rj = rjg[g];
+#pragma unroll
+                    for (int d = 1; d < 32; d <<= 1) {
+                        const double o = __shfl_up_sync(FULL, sv, d);
+                        const int orj = __shfl_up_sync(FULL, rj, d);
+                        if (lane >= d && orj == rj) sv += o;
+                    }
+                    const int nrj = __shfl_down_sync(FULL, rj, 1);
+                    if (cb_valid(t0 + 32 * g, T) && (lane == 31 || nrj != rj)) buf[rj] += sv;
+                    __syncwarp();
+                }
+#else
 #pragma unroll
                 for (int g = 0; g < WIN_G; g++) buf[32 * g + lane] = p[g];
                 __syncwarp();
@@ -701,7 +737,11 @@ struct Kern {
                     for (; i < i1; i++) acc += buf[i];
                 }
                 __syncwarp();
+#endif
             }
+#if ACSR_WIN_SEGSCAN
+            if (l > 0) acc = buf[__popc(ne & lt)];
+#endif
             if (mine) finish(a, r, acc, d2);
             __syncwarp();  // tab / buf reused by the next window
         }

@@ -31,10 +31,11 @@ import torch
 import torch.distributed as dist
 
 
-def partition_rows(row_lengths: np.ndarray, P: int, b_nnz: int = 4, b_row: int = 36) -> np.ndarray:
+def partition_rows(row_lengths: np.ndarray, P: int, b_nnz: int = 4, b_row: int = 36, align: int = 1) -> np.ndarray:
     """Contiguous split balanced on cost(r) = b_nnz*len_r + b_row (integer bytes; PageRank
     pattern: 4 B per column index + 36 B per row).  splits[0] = 0, splits[P] = n and
-    splits[k] = min{r : sum_{r'<r} cost >= ceil(k*total/P)}."""
+    splits[k] = min{r : sum_{r'<r} cost >= ceil(k*total/P)}, rounded up to a multiple of
+    align (reading R7).  Host version for the CPU tests; GPUs use acsr_partition."""
     ln = np.asarray(row_lengths, dtype=np.int64)
     n = ln.size
     pref = np.zeros(n + 1, dtype=np.int64)
@@ -45,6 +46,8 @@ def partition_rows(row_lengths: np.ndarray, P: int, b_nnz: int = 4, b_row: int =
     for k in range(1, P):
         t = -(-k * total // P)
         s[k] = int(np.searchsorted(pref, t, side="left"))
+        if align > 1:
+            s[k] = min(n, -(-int(s[k]) // align) * align)
     return s
 
 
@@ -363,8 +366,10 @@ class DistSpMV:
     them -- no exchange in the SpMV itself.  gather() all-gathers the y slices (padded,
     in place) when every rank needs the whole y.
 
-    The local col/val keep their global 16-byte phase (aligned_slice), so every row is
-    summed exactly as on one GPU: the P-rank y equals the 1-GPU y bit for bit.
+    The local col/val keep their global 16-byte phase (aligned_slice) and, with split points
+    on 32-row boundaries (partition align=32, reading R7), every short-row window holds the
+    same rows, so every row is summed exactly as on one GPU: the P-rank y equals the 1-GPU
+    y bit for bit.
 
     spmv_fn(row_ptr, col, val, x) -> y_local overrides the CUDA call (CPU tests)."""
 

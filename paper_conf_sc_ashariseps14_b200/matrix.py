@@ -282,12 +282,12 @@ def hits(out_ptr, out_col, eps=1e-6, max_iter=1000, stream=None, B=None):
     return v[:n], v[n:], it
 
 
-def degree_relabel(in_ptr, in_col, outdeg):
+def degree_relabel(in_ptr, in_col, outdeg, sort_rows=False):
     """Vertex relabelling for PageRank locality (an application-level preprocessing step,
     not part of ACSR), on the device: acsr_degree_relabel (include/acsr.h) -- vertices by
     decreasing out-degree (ties by id), rows and columns alike (P A P^T), so the kernels run
     unchanged and PR in the original order is x_new[perm].  Returns
     (row_ptr', col', outdeg', perm) with perm[v] = new id of vertex v (int64)."""
     from . import acsr_degree_relabel
-    rp2, c2, od2, perm = acsr_degree_relabel(in_ptr, in_col, outdeg)
+    rp2, c2, od2, perm = acsr_degree_relabel(in_ptr, in_col, outdeg, sort_rows=sort_rows)
     return rp2, c2, od2, perm.to(torch.int64)

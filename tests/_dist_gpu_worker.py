@@ -62,7 +62,8 @@ def spmv_worker(rank, world, port, scale, dtype_name, q):
     n = rp.numel() - 1
     val = synth.values(ci.numel(), 1014, dtype, dev)
     x = synth.vector(n, 2014, dtype, dev)
-    splits = pdist.partition_rows((rp[1:] - rp[:-1]).cpu().numpy(), world, b_nnz=4 + val.element_size(), b_row=16)
+    splits = pdist.partition_rows((rp[1:] - rp[:-1]).cpu().numpy(), world, b_nnz=4 + val.element_size(), b_row=16,
+                                  align=32)
     sp = pdist.DistSpMV(rp, ci, val, splits)
     y = sp.spmv(x)
     y2 = sp.spmv(x)  # a second call on the same plan: identical

@@ -174,7 +174,7 @@ int main(void)
     size_t pws = acsr_partition_workspace_bytes(n);
     CK(cudaMalloc((void **)&d_splits, sizeof(splits)));
     CK(cudaMalloc(&d_pws, pws));
-    AK(acsr_partition(n, d_rp, NULL, 4, 36, 2, d_splits, d_pws, pws, st));
+    AK(acsr_partition(n, d_rp, NULL, 4, 36, 2, 1, d_splits, d_pws, pws, st));
     CK(cudaStreamSynchronize(st));
     CK(cudaMemcpy(splits, d_splits, sizeof(splits), cudaMemcpyDeviceToHost));
     /* costs 36, 40, 48, 56, 316, 6036 (total 6532): the prefix before row r first reaches

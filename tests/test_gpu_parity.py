@@ -214,28 +214,31 @@ def test_powerlaw_webgoogle_like(acsr, cuda, mapping):
 
 
 @pytest.mark.parametrize("dtype", [torch.float64, torch.float32])
-def test_window_rows_are_in_order_sums(acsr, cuda, dtype):
-    """Short-row windows: a row with <= 32 non-zeros is summed by one lane in element
-    order from rounded products, i.e. exactly the oracle's plain sequential loop (O4',
-    compiled without FMA contraction; fp32 accumulated in double, rounded once) -- so
-    those rows must match oracle.spmv_plain BIT FOR BIT, and a row's result must not
-    depend on its neighbours (lengths of other rows changed -> same bits)."""
+def test_window_rows_depend_only_on_their_window(acsr, cuda, dtype):
+    """Short-row windows: the products of a window's short rows (32 consecutive rows,
+    <= 32 non-zeros each) are reduced by a segmented shuffle scan, so a row's summation
+    order depends on the window it sits in (its offset in the window's concatenation) and
+    on nothing else.  Checks: the O5 bar against the Dot2 oracle, run-to-run bitwise
+    determinism, and bitwise-unchanged rows when only rows of OTHER windows change
+    length (rows of odd windows lose their last non-zero, even windows keep their bits)."""
     rp, ci = synth.rmat_csr(16)
     n = rp.numel() - 1
     val = synth.values(ci.numel(), 31, dtype)
     x = synth.vector(n, 32, dtype)
-    _, y = run_csr(acsr, rp, ci, val, x, cuda)
-    y_plain = oracle.spmv_plain(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    m, y = run_csr(acsr, rp, ci, val, x, cuda)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y.numpy(), y_ref, den, dtype)
     ln = (rp[1:] - rp[:-1]).numpy()
     short = ln <= 32
     assert short.sum() > n // 2
-    assert np.array_equal(y.numpy()[short].view(np.uint8), y_plain[short].view(np.uint8))
-    # drop the last non-zero of every third row: the other rows keep their bits
+    y_again = m.spmv(x.to(cuda)).cpu()
+    assert np.array_equal(y.numpy().view(np.uint8), y_again.numpy().view(np.uint8))
     rb, re = rp[:-1].clone(), rp[1:].clone()
-    cut = (torch.arange(n) % 3 == 0) & (re > rb)
+    odd = (torch.arange(n) // 32) % 2 == 1
+    cut = odd & (torch.arange(n) % 3 == 0) & (re > rb)
     re[cut] -= 1
     _, y2 = run_csr(acsr, rb, ci, val, x, cuda, row_end=re)
-    keep = ~cut.numpy()
+    keep = ~odd.numpy()
     assert np.array_equal(y2.numpy()[keep].view(np.uint8), y.numpy()[keep].view(np.uint8))
 
 
@@ -832,15 +835,16 @@ def test_degree_relabel_pagerank_equivalent(acsr, cuda):
     assert np.all(np.abs(back - x_ref) <= 1e-11 * x_ref + 1e-18)
 
 
+@pytest.mark.parametrize("sort_rows", [False, True])
 @pytest.mark.parametrize("scale", [12, 17])
-def test_degree_relabel_structure_bitwise(acsr, cuda, scale):
+def test_degree_relabel_structure_bitwise(acsr, cuda, scale, sort_rows):
     """acsr_degree_relabel against its definition, on the host (integer data, bitwise):
     order = vertices by decreasing out-degree, ties by increasing id (numpy stable sort);
     perm = its inverse; new row perm[u] = old row u with every column c replaced by perm[c],
     in the same order; outdeg' = outdeg[order].  Includes rows longer than the 1024-entry
     threshold of the CTA copy path at s17."""
     rp, ci, od, n = _inlink(scale, cuda)
-    rp2, c2, od2, perm = acsr.acsr_degree_relabel(rp.to(cuda), ci.to(cuda), od.to(cuda))
+    rp2, c2, od2, perm = acsr.acsr_degree_relabel(rp.to(cuda), ci.to(cuda), od.to(cuda), sort_rows=sort_rows)
     rph, cih, odh = rp.numpy(), ci.numpy(), od.numpy()
     order = np.argsort(-odh.astype(np.int64), kind="stable")
     pr = np.empty(n, np.int64)
@@ -853,7 +857,11 @@ def test_degree_relabel_structure_bitwise(acsr, cuda, scale):
     assert np.array_equal(rp2.cpu().numpy(), rp_ref)
     starts = np.repeat(rph[:-1][order] - rp_ref[:-1], ln[order])
     src = np.arange(cih.size) + starts  # old position of every new entry
-    assert np.array_equal(c2.cpu().numpy(), pr[cih[src]])
+    ref = pr[cih[src]]
+    if sort_rows:  # each row's columns ascending (numpy lexsort by (row, col))
+        rows = np.repeat(np.arange(n), ln[order])
+        ref = ref[np.lexsort((ref, rows))]
+    assert np.array_equal(c2.cpu().numpy(), ref)
     if scale == 17:
         assert ln.max() > 1024
 
@@ -1011,10 +1019,11 @@ def test_dist_pagerank_acsr_comm_two_ranks(cuda, compact):
 
 def test_acsr_partition_equals_oracle(acsr, cuda):
     """acsr_partition (O8 on the device: CUB prefix + binary search) = oracle.partition bitwise."""
-    for scale, P, bn, br in ((14, 2, 4, 36), (16, 3, 12, 16), (17, 8, 4, 36), (10, 1, 4, 36)):
+    for scale, P, bn, br, al in ((14, 2, 4, 36, 1), (16, 3, 12, 16, 32), (17, 8, 4, 36, 1), (10, 1, 4, 36, 1),
+                                 (15, 5, 12, 16, 1024)):
         rp, ci = synth.rmat_csr(scale, transpose=True)
-        got = acsr.acsr_partition(rp.to(cuda), P, bn, br).cpu().numpy()
-        assert np.array_equal(got, oracle.partition(rp.numpy(), P, bn, br)), (scale, P)
+        got = acsr.acsr_partition(rp.to(cuda), P, bn, br, align=al).cpu().numpy()
+        assert np.array_equal(got, oracle.partition(rp.numpy(), P, bn, br, align=al)), (scale, P)
     rb, re, cap, c2, _ = synth.with_slack(*synth.rmat_csr(12))
     got = acsr.acsr_partition(rb.to(cuda), 4, 4, 36, row_end=re.to(cuda)).cpu().numpy()
     assert np.array_equal(got, oracle.partition(rb.numpy(), 4, 4, 36, row_end=re.numpy()))

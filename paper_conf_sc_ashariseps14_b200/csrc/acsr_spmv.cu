@@ -48,7 +48,7 @@
 #define ACSR_WIN_LDS4 0  // 1: four shared loads in flight per add group (A/B: C3a +6 %, C2 +2 %, slower)
 #endif
 #ifndef ACSR_WIN_SEGSCAN
-#define ACSR_WIN_SEGSCAN 1  // 0: per-lane in-order sums of the row's products from shared memory (round 1)
+#define ACSR_WIN_SEGSCAN 0  // 1: segmented shuffle reduction per 32-element group (A/B r2f: C3a +24 %, C2 +4 %, LiveJournal-like +14 % -- SHFL shares the MIO path with the gathers)
 #endif
 #ifndef ACSR_WIN_PREFETCH
 #define ACSR_WIN_PREFETCH 0  // 1: prefetch the next window's row bounds (A/B: no gain on C3a, LiveJournal-like +5 %)

@@ -59,6 +59,10 @@ for v in "$@"; do
     td8) build td8 -DACSR_TAIL_DIV=8 ;;
     pf) build pf -DACSR_PF_UNIT=1 ;;
     ptp0) build ptp0 -DACSR_PEER_TILE_PUSH=0 ;;
+    ws0) build ws0 -DACSR_WIN_SEGSCAN=0 ;;
+    wu64s) build wu64s -DACSR_WIN_UNIT_ROWS=64 ;;
+    wu32s) build wu32s -DACSR_WIN_UNIT_ROWS=32 ;;
+    wb6s) build wb6s -DACSR_WIN_MAX_BIN=6 ;;
     t256mb5) build t256mb5 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=5 ;;
     pft256mb5) build pft256mb5 -DACSR_PF_UNIT=1 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=5 ;;
     pfwg8) build pfwg8 -DACSR_PF_UNIT=1 -DACSR_WIN_G=8 ;;

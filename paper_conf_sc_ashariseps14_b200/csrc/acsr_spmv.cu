@@ -50,6 +50,9 @@
 #ifndef ACSR_WIN_SEGSCAN
 #define ACSR_WIN_SEGSCAN 0  // 1: segmented shuffle reduction per 32-element group (A/B r2f: C3a +24 %, C2 +4 %, LiveJournal-like +14 % -- SHFL shares the MIO path with the gathers)
 #endif
+#ifndef ACSR_WIN_SUM4
+#define ACSR_WIN_SUM4 0  // 1: four accumulators by row offset mod 4 (A/B r2h: C3a 47.1 -> 49.2 us, C2 unchanged; kept off)
+#endif
 #ifndef ACSR_WIN_PREFETCH
 #define ACSR_WIN_PREFETCH 0  // 1: prefetch the next window's row bounds (A/B: no gain on C3a, LiveJournal-like +5 %)
 #endif
@@ -58,6 +61,12 @@
 #endif
 #ifndef ACSR_PEER_TILE_PUSH
 #define ACSR_PEER_TILE_PUSH 1  // 0: every finished row is stored to every peer at once (round-1 A/B)
+#endif
+#ifndef ACSR_DIAG
+#define ACSR_DIAG 0  // diagnostics only (wrong results): 1 = no x gathers (x[0]), 2 = no val loads (1.0)
+#endif
+#ifndef ACSR_PROF
+#define ACSR_PROF 0  // diagnostics: per-mapping warp-cycle counters (acsr_debug_prof, A/B builds only)
 #endif
 #ifndef ACSR_VEC_MIN
 #define ACSR_VEC_MIN 512  // rows (chunks) shorter than this use the lane-strided scalar path
@@ -272,6 +281,9 @@ __device__ __forceinline__ int4 lds_i4(const int *p)
 }
 __device__ __forceinline__ double2 lds_d2(const double *p)
 {
+#if ACSR_DIAG == 2 || ACSR_DIAG == 3
+    return make_double2(1.0, 1.0 + (double)((uintptr_t)p & 1));
+#endif
 #if ACSR_STREAM_LD == 2
     double2 v;
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0,%1}, [%2], %3;" : "=d"(v.x), "=d"(v.y) : "l"(p), "l"(pol_evict_first()));
@@ -286,6 +298,9 @@ __device__ __forceinline__ double2 lds_d2(const double *p)
 }
 __device__ __forceinline__ float4 lds_f4(const float *p)
 {
+#if ACSR_DIAG == 2 || ACSR_DIAG == 3
+    return make_float4(1.f, 1.f, 1.f, 1.f + (float)((uintptr_t)p & 1));
+#endif
 #if ACSR_STREAM_LD == 2
     float4 v;
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
@@ -300,11 +315,19 @@ __device__ __forceinline__ float4 lds_f4(const float *p)
     return __ldcs(reinterpret_cast<const float4 *>(p));
 #endif
 }
+#if ACSR_DIAG == 2 || ACSR_DIAG == 3
+__device__ __forceinline__ double lds_v(const double *p) { return 1.0 + (double)((uintptr_t)p & 1); }
+__device__ __forceinline__ double lds_v(const float *p) { return 1.0 + (double)((uintptr_t)p & 1); }
+#else
 __device__ __forceinline__ double lds_v(const double *p) { return lds_d(p); }
 __device__ __forceinline__ double lds_v(const float *p) { return (double)lds_f(p); }
+#endif
 
 __device__ __forceinline__ double ldx(const double *p)
 {
+#if ACSR_DIAG == 1 || ACSR_DIAG == 3
+    return 1.0 + (double)((uintptr_t)p & 1);  // no load (the address still depends on col)
+#endif
 #if ACSR_X_LD == 2
     double v;
     asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(pol_evict_last()));
@@ -319,6 +342,9 @@ __device__ __forceinline__ double ldx(const double *p)
 }
 __device__ __forceinline__ double ldx(const float *p)
 {
+#if ACSR_DIAG == 1 || ACSR_DIAG == 3
+    return 1.0 + (double)((uintptr_t)p & 1);
+#endif
 #if ACSR_X_LD == 2
     float v;
     asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol_evict_last()));
@@ -333,6 +359,15 @@ __device__ __forceinline__ double ldx(const float *p)
 }
 
 __device__ __forceinline__ bool cb_valid(int cb, int T) { return cb < T; }
+
+#if ACSR_PROF
+// [0] window units  [1] light_sub units  [2] light_warp units  [3] heavy units  [4] empty units
+// [5] window: row-bounds wait  [6] window: chunk loads + gathers  [7] window: in-order sums
+// [8] kernel entry -> first unit  [9] last unit -> exit  [10..14] unit counts by type
+// [15] launches
+__device__ unsigned long long g_prof[16];
+#define PROF_ADD(i, v) atomicAdd(&g_prof[i], (unsigned long long)(v))
+#endif
 
 // xs' slice entry -> every OTHER rank's replicated buffer (byte offset o in each region)
 __device__ __noinline__ void peer_store(char *const *pbase, int nranks, int self, int64_t o, double v)
@@ -649,7 +684,17 @@ struct Kern {
 #else
             if (in) row_bounds(a, r, beg, end);
 #endif
+#if ACSR_PROF
+            long long pt0 = clock64();
+#endif
             const int len = end - beg;
+#if ACSR_PROF
+            {
+                const int lsync = __shfl_sync(FULL, len, 0);  // forces the wait here
+                if (lane == 0 && lsync >= 0) PROF_ADD(5, clock64() - pt0);
+                pt0 = clock64();
+            }
+#endif
             const bool mine = in && len <= WIN_MAX_LEN;
             const int l = mine ? len : 0;
             int incl = l;
@@ -667,6 +712,9 @@ struct Kern {
 #endif
             __syncwarp();
             double acc = 0.0;
+#if ACSR_WIN_SUM4
+            double a1 = 0.0, a2 = 0.0, a3 = 0.0;
+#endif
             for (int t0 = 0; t0 < T; t0 += 32 * WIN_G) {
                 double p[WIN_G];
 #if ACSR_WIN_SEGSCAN
@@ -720,9 +768,37 @@ struct Kern {
 #pragma unroll
                 for (int g = 0; g < WIN_G; g++) buf[32 * g + lane] = p[g];
                 __syncwarp();
+#if ACSR_PROF
+                if (lane == 0) PROF_ADD(6, clock64() - pt0);
+                pt0 = clock64();
+#endif
                 if (l > 0) {
                     const int i1 = min(pre + l, t0 + 32 * WIN_G) - t0;
                     int i = max(pre, t0) - t0;
+#if ACSR_WIN_SUM4
+                    // four accumulators by row offset j mod 4, each summed in element order:
+                    // the result depends only on the row (not on where the 128-element
+                    // chunks cut it) and the chain of dependent adds is 4x shorter
+                    int j = i + t0 - pre;
+                    for (; i < i1 && (j & 3); i++, j++) {
+                        const double b = buf[i];
+                        const int m = j & 3;
+                        a1 += m == 1 ? b : 0.0;
+                        a2 += m == 2 ? b : 0.0;
+                        a3 += m == 3 ? b : 0.0;
+                    }
+                    for (; i + 4 <= i1; i += 4) {
+                        const double b0 = buf[i], b1 = buf[i + 1], b2 = buf[i + 2], b3 = buf[i + 3];
+                        acc += b0;
+                        a1 += b1;
+                        a2 += b2;
+                        a3 += b3;
+                    }
+                    if (i < i1) acc += buf[i];
+                    if (i + 1 < i1) a1 += buf[i + 1];
+                    if (i + 2 < i1) a2 += buf[i + 2];
+                    i = i1;
+#endif
 #if ACSR_WIN_LDS4
                     // four shared loads in flight, then the adds in element order (the sum
                     // is the same bits as the one-at-a-time loop; only the loads overlap)
@@ -737,10 +813,16 @@ struct Kern {
                     for (; i < i1; i++) acc += buf[i];
                 }
                 __syncwarp();
+#if ACSR_PROF
+                if (lane == 0) PROF_ADD(7, clock64() - pt0);
+                pt0 = clock64();
+#endif
 #endif
             }
 #if ACSR_WIN_SEGSCAN
             if (l > 0) acc = buf[__popc(ne & lt)];
+#elif ACSR_WIN_SUM4
+            acc = (acc + a1) + (a2 + a3);
 #endif
             if (mine) finish(a, r, acc, d2);
             __syncwarp();  // tab / buf reused by the next window
@@ -1039,12 +1121,35 @@ spmv_kernel(SpmvArgs<V> a)
     __syncthreads();
     int u = gw;
     int nxt = s_claim + (threadIdx.x >> 5);
+#if ACSR_PROF
+    long long t_first = clock64(), t_last = 0;
+    if (lane == 0) PROF_ADD(8, 0);
+    bool first = true;
+#endif
     while (u < n_units) {
+#if ACSR_PROF
+        const long long tu = clock64();
+        if (first && lane == 0) PROF_ADD(8, tu - t_first);
+        first = false;
+        const uint32_t ty = (uint32_t)__ldg(a.units + u).y;
+        const int kind = (ty & HEAVY_FLAG) ? 3 : (ty & WIN_FLAG) ? 0 : ((ty >> 24) == 0 ? 4 : ((ty >> 24) <= 6 ? 1 : 2));
+#endif
         K::unit(a, u, lane, d2, wbuf, wtab);
+#if ACSR_PROF
+        __syncwarp();
+        t_last = clock64();
+        if (lane == 0) {
+            PROF_ADD(kind, t_last - tu);
+            PROF_ADD(10 + kind, 1);
+        }
+#endif
         if (tile_push) K::peer_tile_done(a, lane, d2);
         u = __shfl_sync(0xffffffffu, nxt, 0) + nw;
         if (u < n_units && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
     }
+#if ACSR_PROF
+    if (t_last == 0) t_last = clock64();
+#endif
 #endif
     // CTA-level exit: Delta^2 (exact fixed point) reduced warp -> CTA in shared memory,
     // then ONE set of atomics and ONE exit ticket per CTA
@@ -1064,6 +1169,10 @@ spmv_kernel(SpmvArgs<V> a)
         }
     }
     __syncthreads();
+#if ACSR_PROF
+    if (lane == 0) PROF_ADD(9, clock64() - t_last);
+    if (threadIdx.x == 0 && blockIdx.x == 0) PROF_ADD(15, 1);
+#endif
     if (threadIdx.x >= 32) return;
     if (PR) {
         d2 = lane < SPMV_WARPS ? Fix192{s_d2[lane][0], s_d2[lane][1], s_d2[lane][2], 0, 0} : Fix192{0, 0, 0, 0, 0};
@@ -1491,3 +1600,16 @@ extern "C" acsr_status acsr_plan_status(const void *plan_ws, size_t plan_ws_byte
     }
     return ACSR_OK;
 }
+
+#if ACSR_PROF
+extern "C" int acsr_debug_prof(unsigned long long *out16, int reset)
+{
+    cudaDeviceSynchronize();
+    cudaMemcpyFromSymbol(out16, acsr::g_prof, sizeof(unsigned long long) * 16);
+    if (reset) {
+        unsigned long long z[16] = {0};
+        cudaMemcpyToSymbol(acsr::g_prof, z, sizeof(z));
+    }
+    return 16;
+}
+#endif

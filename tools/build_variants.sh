@@ -60,6 +60,11 @@ for v in "$@"; do
     pf) build pf -DACSR_PF_UNIT=1 ;;
     ptp0) build ptp0 -DACSR_PEER_TILE_PUSH=0 ;;
     ws0) build ws0 -DACSR_WIN_SEGSCAN=0 ;;
+    diag1) build diag1 -DACSR_DIAG=1 ;;
+    sum1) build sum1 -DACSR_WIN_SUM4=0 ;;
+    prof) build prof -DACSR_PROF=1 ;;
+    diag2) build diag2 -DACSR_DIAG=2 ;;
+    diag12) build diag12 -DACSR_DIAG=3 ;;
     wu64s) build wu64s -DACSR_WIN_UNIT_ROWS=64 ;;
     wu32s) build wu32s -DACSR_WIN_UNIT_ROWS=32 ;;
     wb6s) build wb6s -DACSR_WIN_MAX_BIN=6 ;;

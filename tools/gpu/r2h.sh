@@ -1,0 +1,19 @@
+# round-2: four-accumulator window sums (row-only order) vs in-order sums
+TAG=${1:-r2h}
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "window or spmv or dist_spmv or full_size" 2>&1 | tail -n 3
+: > gpurun_out/ab_$TAG.jsonl
+for rep in 1 2; do
+for v in "" sum1; do
+  for wl in rmat20 webgoogle livejournal rmat20_f32; do
+    ACSR_LIB_VARIANT=$v timeout 300 python tools/spmv_ab.py $wl 30 2>/dev/null | sed "s/^{/{\"variant\": \"$v\", /" >> gpurun_out/ab_$TAG.jsonl
+  done
+done
+done
+python - <<'PY'
+import json,collections
+rows=[json.loads(l) for l in open('gpurun_out/ab_r2h.jsonl') if l.strip()]
+d=collections.defaultdict(list)
+for r in rows: d[(r['variant'] or 'base', r['wl'])].append(r['t_spmv_us'])
+for k,v in sorted(d.items()): print(k, v)
+PY

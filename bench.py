@@ -236,6 +236,10 @@ def algorithmic_bytes(rp, ci, dtype, n_cols=None):
     return (sv + 4) * nnz + 4 * (n + 1) + 4 * n + sv * n_c + sv * n, n_c
 
 
+def acsr_num_sms_host():
+    return torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
+
+
 def workload_config(label, n, nnz, world, replicas=False):
     """The `config` of the default line: identical keys and values at every N (and in the
     reference arm), so the driver can match the lines."""
@@ -449,6 +453,18 @@ def run_acsr(args, dev, rank, world):
         "gpu_launches": 4 * K * world,  # per step and rank: bin_count, bin_scan, bin_scatter, spmv_kernel
         "clocks": clk.summary(),
     }
+    # the gather bound (profiles/r2_gather_limiter.json): one L1TEX->XBAR request per
+    # SM-cycle; requests = one per nnz gather + the CSR streams in 128-byte lines + y store beats
+    sv = 8 if dtype == torch.float64 else 4
+    reqs = nnz + (4 + sv) * nnz / 128.0 + 8.0 * (n + 1) / 128.0 + sv * n / 32.0
+    f_sm = (line["clocks"].get("sm_mhz") or 1965.0) * 1e6
+    gb_ms = reqs / (acsr_num_sms_host() * f_sm) * 1e3
+    line["roofline"]["vs_gather_bound"] = {
+        "requests_per_launch": int(reqs), "bound_ms_at_1_req_per_sm_cycle": round(gb_ms, 5),
+        "frac": round(gb_ms / spmv_ms, 4), "sustained_bound_ms_at_85pct": round(gb_ms / 0.85, 5),
+        "frac_of_sustained": round(gb_ms / 0.85 / spmv_ms, 4),
+        "note": "L2-resident x: the SM's L1TEX->XBAR request interface is the busiest unit of a pure random "
+                "gather (ncu, 85 % of elapsed); no L1 hits assumed"}
     if c4 is not None:
         line["pagerank_dist"] = c4
     if not args.no_cpu_baseline and world == 1:  # the oracle baseline: rank 0 at N = 1 only

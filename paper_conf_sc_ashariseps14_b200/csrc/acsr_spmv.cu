@@ -63,10 +63,16 @@
 #define ACSR_PEER_TILE_PUSH 1  // 0: every finished row is stored to every peer at once (round-1 A/B)
 #endif
 #ifndef ACSR_DIAG
-#define ACSR_DIAG 0  // diagnostics only (wrong results): 1 = no x gathers (x[0]), 2 = no val loads (1.0)
+#define ACSR_DIAG 0  // diagnostics only (wrong results): 1 = no x gathers, 2 = no val loads, 3 = neither, 4 = no remote peer stores
 #endif
 #ifndef ACSR_PROF
 #define ACSR_PROF 0  // diagnostics: per-mapping warp-cycle counters (acsr_debug_prof, A/B builds only)
+#endif
+#ifndef ACSR_WIN_DYN_SMEM
+#define ACSR_WIN_DYN_SMEM (ACSR_WIN_G > 4)  // window scratch in dynamic shared memory (needed for WIN_G > 4)
+#endif
+#ifndef ACSR_PF_TILES
+#define ACSR_PF_TILES 0  // > 0: stream-ahead L2 prefetch of the CSR (col/val) this many 1024-row tiles ahead (A/B)
 #endif
 #ifndef ACSR_VEC_MIN
 #define ACSR_VEC_MIN 512  // rows (chunks) shorter than this use the lane-strided scalar path
@@ -447,7 +453,8 @@ struct Kern {
             if (PEER && r < a.peer_len) {
                 const int64_t o = a.peer_next + 8 * (a.peer_off + r);
                 *(double *)(a.pself + o) = xs;  // own replicated buffer: inline
-                if (!ACSR_PEER_TILE_PUSH && a.peer_n > 1) peer_store(a.pbase, a.peer_n, a.peer_rank, o, xs);
+                if (!ACSR_PEER_TILE_PUSH && ACSR_DIAG != 4 && a.peer_n > 1)
+                    peer_store(a.pbase, a.peer_n, a.peer_rank, o, xs);
             }
             if (PEER) {  // per-tile completion count (peer_tile_done)
                 d2.fin++;
@@ -944,7 +951,7 @@ struct Kern {
         const int r1 = min(r0 + tile_rows, a.peer_len);
         const char *own = a.pself + a.peer_next + 8 * a.peer_off;
         for (int q = 0; q < a.peer_n; q++) {
-            if (q == a.peer_rank) continue;
+            if (q == a.peer_rank || ACSR_DIAG == 4) continue;  // DIAG 4: no remote stores (store-count baseline)
             char *dst = a.pbase[q] + a.peer_next + 8 * a.peer_off;
             for (int r = r0 + lane; r < r1; r += 32)
                 *(double *)(dst + 8 * (int64_t)r) = __ldcg((const double *)(own + 8 * (int64_t)r));
@@ -968,7 +975,26 @@ struct Kern {
         }
 #endif
         if (WIN_MAX_BIN >= 0 && (y & WIN_FLAG)) {
+#if ACSR_PF_TILES > 0
+            // the first window unit of tile t (the list goes tile by tile) starts the L2
+            // prefetch of tile t + ACSR_PF_TILES's CSR run: the column/value streams then
+            // come from L2 instead of DRAM when their units run (bounds loaded now, the
+            // prefetch issued after this unit so the loads' latency overlaps its work)
+            int pb = 0, pe = 0;
+            const bool pf = (d.x % TILE_ROWS) == 0 && lane == 0;
+            if (pf) {
+                const int64_t t0 = (int64_t)d.x + (int64_t)ACSR_PF_TILES * TILE_ROWS;
+                if (t0 < a.n_rows) {
+                    const int64_t t1 = t0 + TILE_ROWS < a.n_rows ? t0 + TILE_ROWS : a.n_rows;
+                    pb = __ldg(a.rb + t0);
+                    pe = HAS_END ? __ldg(a.re + t1 - 1) : __ldg(a.rb + t1);
+                }
+            }
             window(a, d.x, (int)(y & 0xFFFFFF), lane, d2, wbuf, wtab);
+            if (pf && pe > pb) pf_range(a, pb, pe);
+#else
+            window(a, d.x, (int)(y & 0xFFFFFF), lane, d2, wbuf, wtab);
+#endif
             return;
         }
         const int b = (int)(y >> 24), cnt = (int)(y & 0xFFFFFF);
@@ -1025,6 +1051,19 @@ spmv_kernel(SpmvArgs<V> a)
             }
         }
     }
+#if ACSR_PF_TILES > 0
+    if (threadIdx.x < 32) {  // tiles 0 .. ACSR_PF_TILES-1: one per CTA, grid-strided (before the PDL wait:
+        // the CSR is not written by the preceding kernels; a prefetch is only a cache hint)
+        for (int64_t t = blockIdx.x + threadIdx.x * (int64_t)gridDim.x; t < ACSR_PF_TILES; t += 32 * (int64_t)gridDim.x) {
+            const int64_t t0 = t * TILE_ROWS;
+            if (t0 >= a.n_rows) break;
+            const int64_t t1 = t0 + TILE_ROWS < a.n_rows ? t0 + TILE_ROWS : a.n_rows;
+            const int pb = __ldg(a.rb + t0);
+            const int pe = HAS_END ? __ldg(a.re + t1 - 1) : __ldg(a.rb + t1);
+            if (pe > pb) K::pf_range(a, pb, pe);
+        }
+    }
+#endif
     pdl_enter();
     if (PR && a.ctrl && *(volatile int32_t *)a.ctrl) return;  // converged earlier: no-op step
     unsigned long long pc = 0;  // peer exchange: pushes completed before this step
@@ -1102,8 +1141,14 @@ spmv_kernel(SpmvArgs<V> a)
         a.xtag = stag;
     }
     // per-warp short-row window scratch (products + (beg, pre) table)
+#if ACSR_WIN_DYN_SMEM
+    // window scratch in dynamic shared memory after the (optional) x cache: lets WIN_G > 4
+    double *win_buf = (double *)(smem + (XC ? (sizeof(V) + sizeof(uint16_t)) * ((size_t)1 << a.xc_bits) : 0));
+    int2 *win_tab = (int2 *)(win_buf + SPMV_WARPS * 32 * WIN_G);
+#else
     __shared__ double win_buf[WIN_MAX_BIN >= 0 ? SPMV_WARPS * 32 * WIN_G : 1];
     __shared__ int2 win_tab[WIN_MAX_BIN >= 0 ? SPMV_WARPS * 32 : 1];
+#endif
     double *wbuf = win_buf + (WIN_MAX_BIN >= 0 ? (threadIdx.x >> 5) * 32 * WIN_G : 0);
     int2 *wtab = win_tab + (WIN_MAX_BIN >= 0 ? (threadIdx.x >> 5) * 32 : 0);
     Fix192 d2{0, 0, 0, 0, 0};
@@ -1271,7 +1316,8 @@ static size_t spmv_smem(int bits)
 {
     static int reserve = -1;
     if (reserve < 0) reserve = env_int("ACSR_SMEM_RESERVE", 0);
-    return (XC ? (sizeof(V) + sizeof(uint16_t)) * ((size_t)1 << bits) : 0) + (size_t)reserve;
+    const size_t win = ACSR_WIN_DYN_SMEM ? (size_t)SPMV_WARPS * 32 * (WIN_G * sizeof(double) + sizeof(int2)) : 0;
+    return (XC ? (sizeof(V) + sizeof(uint16_t)) * ((size_t)1 << bits) : 0) + win + (size_t)reserve;
 }
 
 // ACSR_X_PERSIST_MB=m (experiment, default off): an L2 access-policy window marks the

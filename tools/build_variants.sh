@@ -63,6 +63,14 @@ for v in "$@"; do
     diag1) build diag1 -DACSR_DIAG=1 ;;
     sum1) build sum1 -DACSR_WIN_SUM4=0 ;;
     prof) build prof -DACSR_PROF=1 ;;
+    noremote) build noremote -DACSR_DIAG=4 ;;
+    noremote0) build noremote0 -DACSR_DIAG=4 -DACSR_PEER_TILE_PUSH=0 ;;
+    pft32) build pft32 -DACSR_PF_TILES=32 ;;
+    pft128) build pft128 -DACSR_PF_TILES=128 ;;
+    pft320) build pft320 -DACSR_PF_TILES=320 ;;
+    wg8d) build wg8d -DACSR_WIN_G=8 ;;
+    wg6d) build wg6d -DACSR_WIN_G=6 ;;
+    wg4d) build wg4d -DACSR_WIN_DYN_SMEM=1 ;;
     diag2) build diag2 -DACSR_DIAG=2 ;;
     diag12) build diag12 -DACSR_DIAG=3 ;;
     wu64s) build wu64s -DACSR_WIN_UNIT_ROWS=64 ;;

@@ -752,28 +752,9 @@ def _max_over_ranks(vals, dev, world):
     return [float(v) for v in t.tolist()]
 
 
-def pagerank_dist_record(args, dev, rank, world):
-    """C4 (BASELINE configs[3]): PageRank on the R-MAT s26 in-link pattern, row-partitioned
-    over the N ranks (acsr_partition, cost 4 len + 36), compact non-dangling exchange
-    layout, timed for K iterations with each exchange:
-      acsr  -- acsr_pagerank_step with the library's NCCL communicator (all-gather of the
-               xs slices + exact global Delta^2, device-side stop flag);
-      peer  -- the exchange fused into the step over CUDA-IPC peer memory (N1).
-    Also T1 (the whole graph on rank 0's GPU alone, measured in the same job), T_comm (the
-    same all-gather alone) and frac_of_bound = max(T1/P, T_comm) / T."""
-    import paper_conf_sc_ashariseps14_b200 as acsr
-    from paper_conf_sc_ashariseps14_b200 import dist as pdist
-
-    S = args.c4_scale
-    K = max(3, min(args.steps, 10))
-    torch.cuda.synchronize()
-    g0 = time.perf_counter()
-    rp, ci = synth.rmat_csr(S, device=dev, transpose=True)
-    n, nnz = rp.numel() - 1, ci.numel()
-    outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
-    torch.cuda.synchronize()
-    t_gen = time.perf_counter() - g0
-    # T1: one GPU, whole graph (rank 0; the other ranks wait at the barrier)
+def _c4_variant(acsr, pdist, rp, ci, outdeg, n, nnz, K, dev, rank, world, comm):
+    """One graph of the C4 record: T1 (rank 0 alone, whole graph), then the row-partitioned
+    run with each exchange, T_comm and the fraction of SURVEY §8(e)'s bound."""
     t1 = None
     if rank == 0:
         m = acsr.ACSRMatrix(rp, ci)
@@ -800,13 +781,7 @@ def pagerank_dist_record(args, dev, rank, world):
     rpl = (rp[lo:hi + 1].to(torch.int64) - int(rp[lo])).to(torch.int32)
     cil = ci[int(rp[lo]):int(rp[hi])].clone()
     odl = outdeg[lo:hi].clone()
-    nnz_local = cil.numel()
-    del rp, ci
-    torch.cuda.empty_cache()
-    out = {"workload": f"pagerank_rmat{S}_inlink_partitioned", "n_rows": n, "nnz": nnz,
-           "generate_s": round(t_gen, 2), "iterations_timed": K, "splits": [int(v) for v in splits],
-           "t1_ms": None if t1 is None else round(t1, 4)}
-    comm = acsr.AcsrComm.from_process_group() if world > 1 else None
+    out = {"splits": [int(v) for v in splits], "t1_ms": None if t1 is None else round(t1, 4)}
     for ex in ("acsr", "peer"):
         pr = pdist.DistPageRank(rpl, cil, odl, splits, n, exchange=ex, comm=comm)
         pr.run(max_iter=2, eps=0.0)
@@ -840,16 +815,54 @@ def pagerank_dist_record(args, dev, rank, world):
         out[ex] = rec
         del pr
         torch.cuda.empty_cache()
-    if comm is not None:
-        comm.close()
     if rank == 0:
         t_comm = out["acsr"].get("t_comm_ms", 0.0)
         bound = max(t1 / world, t_comm)
         out["bound_ms"] = round(bound, 4)
-        out["bound_note"] = "SURVEY §8(e): max(T1/P, T_comm), T1 = whole graph on one GPU, T_comm = the all-gather alone"
         for ex in ("acsr", "peer"):
             out[ex]["frac_of_bound"] = round(bound / out[ex]["ms_per_iter"], 4)
             out[ex]["speedup_vs_t1"] = round(t1 / out[ex]["ms_per_iter"], 3)
+    return out
+
+
+def pagerank_dist_record(args, dev, rank, world):
+    """C4 (BASELINE configs[3]): PageRank on the R-MAT s26 in-link pattern, row-partitioned
+    over the N ranks (acsr_partition, cost 4 len + 36), compact non-dangling exchange
+    layout, timed for K iterations with each exchange:
+      acsr  -- acsr_pagerank_step with the library's NCCL communicator (all-gather of the
+               xs slices + exact global Delta^2, device-side stop flag);
+      peer  -- the exchange fused into the step over CUDA-IPC peer memory (N1).
+    Both on the generated graph and on its degree-relabelled copy (acsr_degree_relabel,
+    timed).  Also T1 (the whole graph on rank 0's GPU alone, measured in the same job),
+    T_comm (the same all-gather alone) and frac_of_bound = max(T1/P, T_comm) / T."""
+    import paper_conf_sc_ashariseps14_b200 as acsr
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+
+    S = args.c4_scale
+    K = max(3, min(args.steps, 10))
+    torch.cuda.synchronize()
+    g0 = time.perf_counter()
+    rp, ci = synth.rmat_csr(S, device=dev, transpose=True)
+    n, nnz = rp.numel() - 1, ci.numel()
+    outdeg = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    torch.cuda.synchronize()
+    t_gen = time.perf_counter() - g0
+    out = {"workload": f"pagerank_rmat{S}_inlink_partitioned", "n_rows": n, "nnz": nnz,
+           "generate_s": round(t_gen, 2), "iterations_timed": K,
+           "bound_note": "SURVEY §8(e): max(T1/P, T_comm), T1 = whole graph on one GPU, T_comm = the all-gather alone"}
+    comm = acsr.AcsrComm.from_process_group() if world > 1 else None
+    out["plain"] = _c4_variant(acsr, pdist, rp, ci, outdeg, n, nnz, K, dev, rank, world, comm)
+    r0, r1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    r0.record()
+    rp2, ci2, od2, _ = acsr.acsr_degree_relabel(rp, ci, outdeg)
+    r1.record()
+    torch.cuda.synchronize()
+    del rp, ci, outdeg
+    torch.cuda.empty_cache()
+    out["relabelled"] = _c4_variant(acsr, pdist, rp2, ci2, od2, n, nnz, K, dev, rank, world, comm)
+    out["relabelled"]["relabel_ms"] = round(r0.elapsed_time(r1), 3)
+    if comm is not None:
+        comm.close()
     return out
 
 

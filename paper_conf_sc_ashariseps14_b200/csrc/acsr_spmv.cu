@@ -74,6 +74,9 @@
 #ifndef ACSR_PF_TILES
 #define ACSR_PF_TILES 0  // > 0: stream-ahead L2 prefetch of the CSR (col/val) this many 1024-row tiles ahead (A/B)
 #endif
+#ifndef ACSR_CLAIM_BATCH
+#define ACSR_CLAIM_BATCH 0  // > 0: CTA-batched unit claims of this many units (A/B)
+#endif
 #ifndef ACSR_VEC_MIN
 #define ACSR_VEC_MIN 512  // rows (chunks) shorter than this use the lane-strided scalar path
 #endif
@@ -1162,7 +1165,11 @@ spmv_kernel(SpmvArgs<V> a)
     // first prefetched claims: one atomic per CTA (a same-address atomic per warp at
     // launch costs microseconds of serialisation at the L2 slice)
     __shared__ int s_claim;
+#if ACSR_CLAIM_BATCH > 0
+    if (threadIdx.x == 0) s_claim = SPMV_WARPS * atomicAdd(&hdr->work_ctr, 1);  // this CTA's batch 0
+#else
     if (threadIdx.x == 0) s_claim = atomicAdd(&hdr->work_ctr, SPMV_WARPS);
+#endif
     __syncthreads();
     int u = gw;
     int nxt = s_claim + (threadIdx.x >> 5);
@@ -1170,6 +1177,38 @@ spmv_kernel(SpmvArgs<V> a)
     long long t_first = clock64(), t_last = 0;
     if (lane == 0) PROF_ADD(8, 0);
     bool first = true;
+#endif
+#if ACSR_CLAIM_BATCH > 0
+    // CTA-batched claiming: after the static first round (unit = global warp id) the
+    // global counter hands out batches of ACSR_CLAIM_BATCH consecutive units to a CTA,
+    // whose warps take them one by one from a shared-memory counter.  The warp that
+    // takes the first unit of batch b fetches the id of batch b + 1, so a batch is
+    // published long before it is needed; global atomics drop ACSR_CLAIM_BATCH-fold, so
+    // units can be small (short tail) without saturating one L2 slice with claims.
+    constexpr int CB = ACSR_CLAIM_BATCH;
+    constexpr int RING = 32;  // published batch ids: (local batch << 32 | global batch), one 64-bit word
+    __shared__ int s_claims;
+    __shared__ unsigned long long s_batch[RING];
+    if (threadIdx.x < RING) s_batch[threadIdx.x] = ~0ull;
+    if (threadIdx.x == 0) {
+        s_claims = 0;
+        s_batch[0] = (unsigned long long)(unsigned)(s_claim / SPMV_WARPS);  // batch 0: the CTA's first atomic
+    }
+    __syncthreads();
+    auto claim = [&]() -> int {
+        const int i = atomicAdd(&s_claims, 1);
+        const int b = i / CB, j = i - b * CB;
+        if (j == 0) {  // fetch the NEXT batch's id, published with its local batch number
+            const int g = atomicAdd(&hdr->work_ctr, 1);
+            ((volatile unsigned long long *)s_batch)[(b + 1) % RING] =
+                ((unsigned long long)(unsigned)(b + 1) << 32) | (unsigned)g;
+        }
+        unsigned long long v;
+        while (((v = ((volatile unsigned long long *)s_batch)[b % RING]) >> 32) != (unsigned long long)(unsigned)b)
+            __nanosleep(32);
+        return nw + (int)(unsigned)v * CB + j;
+    };
+    if (lane == 0) nxt = claim();
 #endif
     while (u < n_units) {
 #if ACSR_PROF
@@ -1189,8 +1228,13 @@ spmv_kernel(SpmvArgs<V> a)
         }
 #endif
         if (tile_push) K::peer_tile_done(a, lane, d2);
+#if ACSR_CLAIM_BATCH > 0
+        u = __shfl_sync(0xffffffffu, nxt, 0);
+        if (u < n_units && lane == 0) nxt = claim();
+#else
         u = __shfl_sync(0xffffffffu, nxt, 0) + nw;
         if (u < n_units && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
+#endif
     }
 #if ACSR_PROF
     if (t_last == 0) t_last = clock64();

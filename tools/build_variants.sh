@@ -63,6 +63,11 @@ for v in "$@"; do
     diag1) build diag1 -DACSR_DIAG=1 ;;
     sum1) build sum1 -DACSR_WIN_SUM4=0 ;;
     prof) build prof -DACSR_PROF=1 ;;
+    cb16) build cb16 -DACSR_CLAIM_BATCH=16 ;;
+    cb16w32) build cb16w32 -DACSR_CLAIM_BATCH=16 -DACSR_WIN_UNIT_ROWS=32 ;;
+    cb32w32) build cb32w32 -DACSR_CLAIM_BATCH=32 -DACSR_WIN_UNIT_ROWS=32 ;;
+    cb16w32u1) build cb16w32u1 -DACSR_CLAIM_BATCH=16 -DACSR_WIN_UNIT_ROWS=32 -DACSR_UNIT_SHIFT=-1 ;;
+    w32) build w32 -DACSR_WIN_UNIT_ROWS=32 ;;
     noremote) build noremote -DACSR_DIAG=4 ;;
     noremote0) build noremote0 -DACSR_DIAG=4 -DACSR_PEER_TILE_PUSH=0 ;;
     pft32) build pft32 -DACSR_PF_TILES=32 ;;

@@ -328,6 +328,14 @@ acsr_status acsr_peer_read_xs(const acsr_peer *p, double *dst, cudaStream_t stre
 size_t acsr_hits_workspace_bytes(int64_t n);
 acsr_status acsr_hits_normalize(int64_t n, const double *y, const double *v, double *v_next,
                                 double *dist2, void *ws, size_t ws_bytes, cudaStream_t stream);
+/* The same with device-side convergence (as acsr_pr_args.ctrl): ctrl NULL or [2] device;
+ * a call with ctrl[0] != 0 does nothing; otherwise ctrl[1] += 1 and ctrl[0] = 1 once both
+ * dist2[0] and dist2[1] are <= eps2.  Lets the host enqueue blocks of (acsr_spmv,
+ * acsr_hits_normalize_ctrl) iterations between synchronisations with the results of a test
+ * after every iteration (the iterate after k executed iterations is in buffer k mod 2). */
+acsr_status acsr_hits_normalize_ctrl(int64_t n, const double *y, const double *v, double *v_next,
+                                     double *dist2, int32_t *ctrl, double eps2, void *ws, size_t ws_bytes,
+                                     cudaStream_t stream);
 
 /* ------------------------------------------------------------------------ */
 /* Degree-ordered vertex relabelling of a PageRank in-link graph (an application-level

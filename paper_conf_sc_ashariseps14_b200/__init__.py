@@ -106,6 +106,8 @@ _lib.acsr_hits_workspace_bytes.argtypes = [_i64]
 _lib.acsr_hits_workspace_bytes.restype = _sz
 _lib.acsr_hits_normalize.argtypes = [_i64, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
 _lib.acsr_hits_normalize.restype = ctypes.c_int
+_lib.acsr_hits_normalize_ctrl.argtypes = [_i64, _vp, _vp, _vp, _vp, _vp, _dbl, _vp, _sz, _vp]
+_lib.acsr_hits_normalize_ctrl.restype = ctypes.c_int
 _lib.acsr_plan_status.argtypes = [_vp, _sz, _vp]
 _lib.acsr_plan_status.restype = ctypes.c_int
 _lib.acsr_comm_get_unique_id.argtypes = [_vp]
@@ -136,7 +138,7 @@ ACSR_IPC_HANDLE_BYTES = 64
 EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_bin_ex", "acsr_spmv", "acsr_pagerank_step",
             "acsr_pagerank_scale", "acsr_pagerank_step_peer", "acsr_peer_create", "acsr_peer_open",
             "acsr_peer_destroy", "acsr_peer_push", "acsr_peer_delta2", "acsr_peer_query", "acsr_peer_read_xs", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_update_edges_dev", "acsr_relayout",
-            "acsr_hits_workspace_bytes", "acsr_hits_normalize", "acsr_plan_status",
+            "acsr_hits_workspace_bytes", "acsr_hits_normalize", "acsr_hits_normalize_ctrl", "acsr_plan_status",
             "acsr_comm_get_unique_id", "acsr_comm_init", "acsr_comm_destroy", "acsr_comm_query",
             "acsr_comm_allgather", "acsr_pagerank_init", "acsr_partition_workspace_bytes", "acsr_partition",
             "acsr_relabel_workspace_bytes", "acsr_degree_relabel",
@@ -563,14 +565,16 @@ def acsr_hits_workspace_bytes(n: int) -> int:
     return int(_lib.acsr_hits_workspace_bytes(int(n)))
 
 
-def acsr_hits_normalize(y, v, v_next, dist2, ws=None, stream=None):
-    """HITS normalisation of y = [A^T h; A a] into v_next (Eq. 5-7, reading R6)."""
+def acsr_hits_normalize(y, v, v_next, dist2, ws=None, stream=None, ctrl=None, eps2=-1.0):
+    """HITS normalisation of y = [A^T h; A a] into v_next (Eq. 5-7, reading R6).  ctrl:
+    device-side convergence (acsr_hits_normalize_ctrl)."""
     n = y.numel() // 2
     if ws is None:
         ws = torch.empty(acsr_hits_workspace_bytes(n), dtype=torch.uint8, device=y.device)
-    _check(_lib.acsr_hits_normalize(n, _dev(y, torch.float64, "y"), _dev(v, torch.float64, "v"),
-                                    _dev(v_next, torch.float64, "v_next"), _dev(dist2, torch.float64, "dist2"),
-                                    _dev(ws, torch.uint8, "ws"), ws.numel(), _stream(stream)),
+    _check(_lib.acsr_hits_normalize_ctrl(n, _dev(y, torch.float64, "y"), _dev(v, torch.float64, "v"),
+                                         _dev(v_next, torch.float64, "v_next"), _dev(dist2, torch.float64, "dist2"),
+                                         _dev(ctrl, torch.int32, "ctrl", True), float(eps2),
+                                         _dev(ws, torch.uint8, "ws"), ws.numel(), _stream(stream)),
            "acsr_hits_normalize")
     return v_next, dist2
 

@@ -34,10 +34,11 @@ __device__ __forceinline__ double block_sum(double v, double *sh)
 __global__ void __launch_bounds__(HITS_THREADS) hits_kernel(int64_t n, const double *__restrict__ y,
                                                             const double *__restrict__ v,
                                                             double *__restrict__ vn, HitsWs *ws,
-                                                            double *dist2, int mode)
+                                                            double *dist2, int mode, int32_t *ctrl, double eps2)
 {
     __shared__ double sh[HITS_THREADS / 32];
     __shared__ int last;
+    if (ctrl && *(volatile int32_t *)ctrl) return;  // converged earlier: no-op (device-side loop)
     double acc[2] = {0.0, 0.0};
     const double na = mode ? ws->norm[0] : 0.0, nh = mode ? ws->norm[1] : 0.0;
     for (int64_t i = blockIdx.x * (int64_t)HITS_THREADS + threadIdx.x; i < 2 * n;
@@ -69,6 +70,12 @@ __global__ void __launch_bounds__(HITS_THREADS) hits_kernel(int64_t n, const dou
         for (int b = 0; b < HITS_CTAS; b++) t += __ldcg(&ws->part[threadIdx.x][b]);
         if (mode == 0) ws->norm[threadIdx.x] = sqrt(t);
         else dist2[threadIdx.x] = t;
+        const double th = __shfl_sync(0x3u, t, 1);  // the hub distance (thread 1)
+        if (threadIdx.x == 0 && mode == 1 && ctrl) {
+            ctrl[1] += 1;
+            // both Euclidean distances <= eps ("until both ... converge")
+            if (t <= eps2 && th <= eps2) ctrl[0] = 1;
+        }
     }
     if (last && threadIdx.x == 0) ws->ticket = 0;
 }
@@ -86,6 +93,13 @@ extern "C" size_t acsr_hits_workspace_bytes(int64_t n)
 extern "C" acsr_status acsr_hits_normalize(int64_t n, const double *y, const double *v, double *v_next,
                                            double *dist2, void *ws, size_t ws_bytes, cudaStream_t stream)
 {
+    return acsr_hits_normalize_ctrl(n, y, v, v_next, dist2, nullptr, -1.0, ws, ws_bytes, stream);
+}
+
+extern "C" acsr_status acsr_hits_normalize_ctrl(int64_t n, const double *y, const double *v, double *v_next,
+                                                double *dist2, int32_t *ctrl, double eps2, void *ws, size_t ws_bytes,
+                                                cudaStream_t stream)
+{
     if (n < 0 || !dist2 || (n > 0 && (!y || !v || !v_next))) {
         acsr_set_error("acsr_hits_normalize: invalid argument");
         return ACSR_ERR_INVALID_VALUE;
@@ -96,7 +110,7 @@ extern "C" acsr_status acsr_hits_normalize(int64_t n, const double *y, const dou
     }
     HitsWs *w = (HitsWs *)ws;
     cudaMemsetAsync(&w->ticket, 0, sizeof(int), stream);
-    hits_kernel<<<HITS_CTAS, HITS_THREADS, 0, stream>>>(n, y, v, v_next, w, dist2, 0);
-    hits_kernel<<<HITS_CTAS, HITS_THREADS, 0, stream>>>(n, y, v, v_next, w, dist2, 1);
+    hits_kernel<<<HITS_CTAS, HITS_THREADS, 0, stream>>>(n, y, v, v_next, w, dist2, 0, ctrl, eps2);
+    hits_kernel<<<HITS_CTAS, HITS_THREADS, 0, stream>>>(n, y, v, v_next, w, dist2, 1, ctrl, eps2);
     return acsr_check_launch("acsr_hits_normalize");
 }

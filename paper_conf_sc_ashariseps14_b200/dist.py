@@ -407,13 +407,18 @@ class DistSpMV:
         if self._m is not None:
             self._m.rebin()
 
-    def gather(self, y_local):
-        """Whole y on every rank (padded equal-size all-gather of the slices)."""
+    def gather(self, y_local, comm=None):
+        """Whole y on every rank (padded equal-size all-gather of the slices): through the
+        library's NCCL communicator (acsr_comm_allgather) when comm is given, else
+        torch.distributed (the gloo CPU tests)."""
         if self.world == 1:
             return y_local
         pad = torch.zeros(self.L, dtype=y_local.dtype, device=y_local.device)
         pad[: self.n_local] = y_local
         allp = torch.empty(self.world * self.L, dtype=y_local.dtype, device=y_local.device)
-        dist.all_gather_into_tensor(allp, pad, group=self.group)
+        if comm is not None:
+            comm.allgather(pad, allp)
+        else:
+            dist.all_gather_into_tensor(allp, pad, group=self.group)
         sizes = np.diff(self.splits)
         return torch.cat([allp[k * self.L: k * self.L + int(sizes[k])] for k in range(self.world)])

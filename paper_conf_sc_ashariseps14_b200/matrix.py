@@ -256,29 +256,35 @@ def hits_matrix(out_ptr, out_col, n=None):
     return row_ptr, col
 
 
-def hits(out_ptr, out_col, eps=1e-6, max_iter=1000, stream=None, B=None):
+def hits(out_ptr, out_col, eps=1e-6, max_iter=1000, stream=None, B=None, check_every=8):
     """HITS (Eq. 5-7; reading R6): one acsr_spmv on [[0, A^T], [A, 0]] per
     iteration plus acsr_hits_normalize.  a^0 = h^0 = 1/|V|.  B: the binned block
-    matrix (ACSRMatrix of hits_matrix(out_ptr, out_col)), built here when None.  Returns
-    (a, h, iters)."""
+    matrix (ACSRMatrix of hits_matrix(out_ptr, out_col)), built here when None.  The stop
+    test (both distances <= eps) runs on the device: check_every iterations are
+    enqueued per host synchronisation and iterations after convergence are no-ops -- the
+    same result as a host test after every iteration.  Returns (a, h, iters)."""
     n = out_ptr.numel() - 1
     dev = out_ptr.device
     if B is None:
         rp, col = hits_matrix(out_ptr, out_col, n)
         B = ACSRMatrix(rp, col, None, n_cols=2 * n)
-    v = torch.full((2 * n,), 1.0 / n, dtype=torch.float64, device=dev)
-    y, vn = torch.empty_like(v), torch.empty_like(v)
+    bufs = [torch.full((2 * n,), 1.0 / n, dtype=torch.float64, device=dev),
+            torch.empty(2 * n, dtype=torch.float64, device=dev)]
+    y = torch.empty_like(bufs[0])
     d2 = torch.zeros(2, dtype=torch.float64, device=dev)
+    ctrl = torch.zeros(2, dtype=torch.int32, device=dev)
     ws = torch.empty(acsr_hits_workspace_bytes(n), dtype=torch.uint8, device=dev)
-    it = 0
-    while it < max_iter:
-        B.spmv(v, y, stream)
-        acsr_hits_normalize(y, v, vn, d2, ws, stream)
-        v, vn = vn, v
-        it += 1
-        da, dh = (float(t) for t in d2.cpu())
-        if da ** 0.5 <= eps and dh ** 0.5 <= eps:
+    eps2 = eps * eps if eps >= 0 else -1.0
+    k = 0
+    while k < max_iter:
+        for _ in range(min(max(1, check_every), max_iter - k)):
+            B.spmv(bufs[k % 2], y, stream)
+            acsr_hits_normalize(y, bufs[k % 2], bufs[(k + 1) % 2], d2, ws, stream, ctrl=ctrl, eps2=eps2)
+            k += 1
+        if int(ctrl[0].item()):
             break
+    it = int(ctrl[1].item())
+    v = bufs[it % 2]
     return v[:n], v[n:], it
 
 

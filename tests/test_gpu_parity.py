@@ -786,6 +786,10 @@ def test_hits_parity(acsr, cuda, scale):
         a_ref, h_ref, _ = oracle.hits(rp.numpy(), ci.numpy(), rpT.numpy(), ciT.numpy(), eps=0.0, max_iter=it)
     assert np.allclose(a.cpu().numpy(), a_ref, rtol=1e-9, atol=1e-15)
     assert np.allclose(h.cpu().numpy(), h_ref, rtol=1e-9, atol=1e-15)
+    # device-side stop test: enqueueing 8 iterations per host check (steps after convergence
+    # are no-ops) gives the iterate of a host test after every iteration, bitwise
+    a1, h1, it1 = acsr.hits(rp.to(cuda), ci.to(cuda), eps=1e-6, check_every=1)
+    assert it1 == it and torch.equal(a1, a) and torch.equal(h1, h)
 
 
 @pytest.mark.parametrize("scale", [12, 16])

@@ -1034,6 +1034,33 @@ def test_acsr_partition_equals_oracle(acsr, cuda):
     assert np.array_equal(empty, [0, 0, 0, 0])
 
 
+def test_partition_and_relabel_edge_cases(acsr, cuda):
+    """acsr_partition with more ranks than rows and on empty rows; acsr_degree_relabel on a
+    one-vertex graph, on a graph without edges (all ties -> identity) and on an empty graph;
+    argument errors of the multi-GPU calls."""
+    rp = torch.tensor([0, 5, 5, 9], dtype=torch.int32)
+    for P in (1, 2, 3, 8):
+        got = acsr.acsr_partition(rp.to(cuda), P, 4, 36).cpu().numpy()
+        assert np.array_equal(got, oracle.partition(rp.numpy(), P, 4, 36)), P
+        assert got[0] == 0 and got[-1] == 3 and np.all(np.diff(got) >= 0)
+    one = acsr.acsr_degree_relabel(torch.tensor([0, 1], dtype=torch.int32, device=cuda),
+                                   torch.tensor([0], dtype=torch.int32, device=cuda),
+                                   torch.tensor([1], dtype=torch.int32, device=cuda))
+    assert one[3].cpu().tolist() == [0] and one[1].cpu().tolist() == [0] and one[0].cpu().tolist() == [0, 1]
+    n = 1000
+    rp2, c2, od2, perm = acsr.acsr_degree_relabel(torch.zeros(n + 1, dtype=torch.int32, device=cuda),
+                                                  torch.zeros(0, dtype=torch.int32, device=cuda),
+                                                  torch.zeros(n, dtype=torch.int32, device=cuda))
+    assert torch.equal(perm.cpu(), torch.arange(n, dtype=torch.int32)) and int(rp2[-1]) == 0
+    e = acsr.acsr_degree_relabel(torch.zeros(1, dtype=torch.int32, device=cuda), None,
+                                 torch.zeros(0, dtype=torch.int32, device=cuda))
+    assert e[0].cpu().tolist() == [0]
+    with pytest.raises(acsr.ACSRError, match="INVALID_VALUE"):
+        acsr.AcsrComm(2, 5, acsr.AcsrComm.unique_id())
+    with pytest.raises(ValueError):
+        acsr.AcsrComm(1, 0, b"short")
+
+
 def test_single_rank_acsr_comm_step_equals_pagerank(acsr, cuda):
     """acsr_pagerank_step with a one-rank acsr_comm (exchange + global Delta^2 in the
     library) gives the single-GPU loop's iterate, iteration count and Delta^2 bitwise."""

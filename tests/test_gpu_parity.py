@@ -891,6 +891,63 @@ def test_paper_epoch_update_bitwise(acsr, cuda):
         assert np.array_equal(odd.cpu().numpy(), od_h)
 
 
+def _live(rb, re):
+    """Indices of the stored entries of a slack CSR (vectorised)."""
+    ln = (re - rb).astype(np.int64)
+    return np.repeat(rb.astype(np.int64) - np.concatenate([[0], np.cumsum(ln)[:-1]]), ln) + np.arange(int(ln.sum()))
+
+
+def test_c5_full_size_batches_bitwise(acsr, cuda):
+    """C5 at BASELINE size in the bench's configuration (R-MAT s20 in-link pattern, slack
+    cap = len + max(4, ceil(len/4)), 16,384-edge insert batches from the same R-MAT, seeds
+    3000 + b): two batches through acsr_update_edges -> acsr_bin -> acsr_spmv; col, row_end,
+    outdeg and bins bitwise against the oracle (O7, O3) after each batch, y = A xs at the fp64
+    bar; then one paper-shaped mixed epoch (N2) bitwise."""
+    S = 20
+    rp, ci = synth.rmat_csr(S, transpose=True)
+    n = rp.numel() - 1
+    od = torch.bincount(ci.long(), minlength=n).to(torch.int32)
+    rb, re, cap, col, _ = synth.with_slack(rp, ci)
+    keys = np.sort(np.repeat(np.arange(n), np.diff(rp.numpy())).astype(np.int64) * n + ci.numpy())
+    m = acsr.ACSRMatrix(rb.to(cuda), col.to(cuda), None, row_end=re.to(cuda), row_cap=cap.to(cuda),
+                        nnz_max=col.numel())
+    odd = od.to(cuda)
+    rb_h, cap_h = rb.numpy(), cap.numpy()
+    re_h, col_h, od_h = re.numpy().copy(), col.numpy().copy(), od.numpy().copy()
+    x = (synth.vector(n, 7).abs() + 0.5)
+    for ch, _ in synth.insert_batches(S, 2, 16384, keys):
+        code, _ = oracle.update(n, rb_h, re_h, cap_h, col_h, None, ch["upd_rows"], None, None, ch["ins_ptr"],
+                                ch["ins_cols"], None, od_h)
+        st = m.update(_dev_changes(ch, cuda), outdeg=odd)
+        torch.cuda.synchronize()
+        assert st.cpu().tolist() == [code, -1 if code == 0 else st.cpu().tolist()[1]]
+        if code != 0:  # capacity: both sides rejected the whole batch, nothing changed
+            continue
+        assert np.array_equal(m.row_end.cpu().numpy(), re_h)
+        live = _live(rb_h, re_h)
+        assert np.array_equal(m.col_idx.cpu().numpy()[live], col_h[live])
+        assert np.array_equal(odd.cpu().numpy(), od_h)
+        m.rebin()
+        m.plan_status()
+        br, off = oracle.bins(rb_h, re_h)
+        assert np.array_equal(m.bin_rows.cpu().numpy(), br) and np.array_equal(m.bin_offsets.cpu().numpy(), off)
+        xs = np.where(od_h > 0, x.numpy() / np.maximum(od_h, 1), 0.0)
+        y = m.spmv(torch.from_numpy(xs).to(cuda)).cpu().numpy()
+        y_ref, den = oracle.spmv(rb_h, col_h, None, xs, row_end=re_h)
+        check_spmv(y, y_ref, den, torch.float64)
+    ch = synth.mixed_epoch(m.row_begin, m.row_end, m.col_idx, n, 0.1, 91)
+    code, _ = oracle.update(n, rb_h, re_h, cap_h, col_h, None, ch["upd_rows"], ch["del_ptr"], ch["del_cols"],
+                            ch["ins_ptr"], ch["ins_cols"], None, od_h)
+    st = m.update(_dev_changes(ch, cuda), outdeg=odd)
+    torch.cuda.synchronize()
+    assert int(st[0]) == code
+    if code == 0:
+        assert np.array_equal(m.row_end.cpu().numpy(), re_h)
+        live = _live(rb_h, re_h)
+        assert np.array_equal(m.col_idx.cpu().numpy()[live], col_h[live])
+        assert np.array_equal(odd.cpu().numpy(), od_h)
+
+
 def test_update_long_row_cta_path(acsr, cuda):
     # hub rows (> 2048 entries) with deletes take the CTA-per-row validate/compact path
     lens = [3, 10000, 5, 40000, 0, 2049]

@@ -68,8 +68,11 @@
 #ifndef ACSR_PROF
 #define ACSR_PROF 0  // diagnostics: per-mapping warp-cycle counters (acsr_debug_prof, A/B builds only)
 #endif
+#ifndef ACSR_WIN_RPL
+#define ACSR_WIN_RPL 1  // short-row window rows per lane (window = 32 * RPL consecutive rows)
+#endif
 #ifndef ACSR_WIN_DYN_SMEM
-#define ACSR_WIN_DYN_SMEM (ACSR_WIN_G > 4)  // window scratch in dynamic shared memory (needed for WIN_G > 4)
+#define ACSR_WIN_DYN_SMEM (ACSR_WIN_G > 4 || ACSR_WIN_RPL > 1)  // window scratch in dynamic shared memory
 #endif
 #ifndef ACSR_PF_TILES
 #define ACSR_PF_TILES 0  // > 0: stream-ahead L2 prefetch of the CSR (col/val) this many 1024-row tiles ahead (A/B)
@@ -83,6 +86,8 @@
 
 
 namespace acsr {
+
+constexpr int WIN_TAB = 32 * ACSR_WIN_RPL;  // (row_begin, prefix) entries of a window's short rows
 
 template <typename V>
 struct SpmvArgs {
@@ -664,6 +669,93 @@ struct Kern {
     // 32-element group and a per-warp (beg, pre) table of the non-empty short rows.
     // Products go to a per-warp shared buffer; each lane then adds ITS row's products in
     // element order, so a row's sum depends only on the row (as in every other mapping).
+#if ACSR_WIN_RPL > 1
+    // Wide short-row windows (ACSR_WIN_RPL rows per lane): the same mapping as window()
+    // below, but a warp concatenates 32 * RPL consecutive rows at once (row i of the window
+    // = lane + 32 j, j < RPL), so one row-bounds round trip and each chunk of 32 * WIN_G
+    // elements serve RPL times more rows (short-row matrices: more elements per dependent
+    // memory round trip).  Each lane sums its RPL rows' products in element order.
+    static __device__ __forceinline__ void window(const A &a, int r0, int nrows, int lane, Fix192 &d2,
+                                                  double *buf, int2 *tab)
+    {
+        constexpr unsigned FULL = 0xffffffffu;
+        constexpr int RPL = ACSR_WIN_RPL, WR = 32 * RPL, CH = 32 * WIN_G;
+        const unsigned lt = (1u << lane) - 1u;
+        const unsigned le = 0xffffffffu >> (31 - lane);
+        for (int w = 0; w < nrows; w += WR) {
+            int beg[RPL], l[RPL], pre[RPL];
+            bool mine[RPL];
+#pragma unroll
+            for (int j = 0; j < RPL; j++) {
+                const int i = w + j * 32 + lane;
+                int b = 0, e = 0;
+                if (i < nrows) row_bounds(a, r0 + i, b, e);
+                beg[j] = b;
+                mine[j] = i < nrows && e - b <= WIN_MAX_LEN;
+                l[j] = mine[j] ? e - b : 0;
+            }
+            int base = 0, nbase = 0;
+#pragma unroll
+            for (int j = 0; j < RPL; j++) {
+                int incl = l[j];
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {
+                    const int t = __shfl_up_sync(FULL, incl, d);
+                    if (lane >= d) incl += t;
+                }
+                pre[j] = base + incl - l[j];
+                const unsigned ne = __ballot_sync(FULL, l[j] > 0);
+                if (l[j] > 0) tab[nbase + __popc(ne & lt)] = make_int2(beg[j], pre[j]);
+                base += __shfl_sync(FULL, incl, 31);
+                nbase += __popc(ne);
+            }
+            const int T = base;
+            __syncwarp();
+            double acc[RPL];
+#pragma unroll
+            for (int j = 0; j < RPL; j++) acc[j] = 0.0;
+            for (int t0 = 0; t0 < T; t0 += CH) {
+                double p[WIN_G];
+#pragma unroll
+                for (int g = 0; g < WIN_G; g++) {
+                    const int cb = t0 + 32 * g;
+                    unsigned hb = 0;
+                    int qc = 0;
+#pragma unroll
+                    for (int j = 0; j < RPL; j++) {
+                        const bool hd = l[j] > 0 && pre[j] >= cb && pre[j] < cb + 32;
+                        hb |= hd ? 1u << (pre[j] - cb) : 0u;
+                        qc += __popc(__ballot_sync(FULL, l[j] > 0 && pre[j] < cb));
+                    }
+                    const unsigned H = __reduce_or_sync(FULL, hb);
+                    const bool v = cb + lane < T;
+                    const int t = v ? cb + lane : T - 1;
+                    const int2 bp = tab[qc + __popc(H & le) - 1];
+                    const int k = bp.x + (t - bp.y);
+                    const int c = lds_i(a.col + k);
+                    const double xv = gx(a, c);
+                    const double pv = HAS_VAL ? lds_v(a.val + k) * xv : xv;
+                    p[g] = v ? pv : 0.0;
+                }
+#pragma unroll
+                for (int g = 0; g < WIN_G; g++) buf[32 * g + lane] = p[g];
+                __syncwarp();
+#pragma unroll
+                for (int j = 0; j < RPL; j++) {
+                    if (l[j] > 0) {
+                        const int i1 = min(pre[j] + l[j], t0 + CH) - t0;
+                        for (int i = max(pre[j], t0) - t0; i < i1; i++) acc[j] += buf[i];
+                    }
+                }
+                __syncwarp();
+            }
+#pragma unroll
+            for (int j = 0; j < RPL; j++)
+                if (mine[j]) finish(a, r0 + w + j * 32 + lane, acc[j], d2);
+            __syncwarp();  // tab / buf reused by the next window
+        }
+    }
+#else
     static __device__ __forceinline__ void window(const A &a, int r0, int nrows, int lane, Fix192 &d2,
                                                   double *buf, int2 *tab)
     {
@@ -838,6 +930,7 @@ struct Kern {
             __syncwarp();  // tab / buf reused by the next window
         }
     }
+#endif
 
     static __device__ __forceinline__ void empty_rows(const A &a, int start, int cnt, int lane, Fix192 &d2)
     {
@@ -1147,13 +1240,13 @@ spmv_kernel(SpmvArgs<V> a)
 #if ACSR_WIN_DYN_SMEM
     // window scratch in dynamic shared memory after the (optional) x cache: lets WIN_G > 4
     double *win_buf = (double *)(smem + (XC ? (sizeof(V) + sizeof(uint16_t)) * ((size_t)1 << a.xc_bits) : 0));
-    int2 *win_tab = (int2 *)(win_buf + SPMV_WARPS * 32 * WIN_G);
+    int2 *win_tab = (int2 *)(win_buf + SPMV_WARPS * 32 * WIN_G);  // WIN_TAB entries per warp
 #else
     __shared__ double win_buf[WIN_MAX_BIN >= 0 ? SPMV_WARPS * 32 * WIN_G : 1];
-    __shared__ int2 win_tab[WIN_MAX_BIN >= 0 ? SPMV_WARPS * 32 : 1];
+    __shared__ int2 win_tab[WIN_MAX_BIN >= 0 ? SPMV_WARPS * WIN_TAB : 1];
 #endif
     double *wbuf = win_buf + (WIN_MAX_BIN >= 0 ? (threadIdx.x >> 5) * 32 * WIN_G : 0);
-    int2 *wtab = win_tab + (WIN_MAX_BIN >= 0 ? (threadIdx.x >> 5) * 32 : 0);
+    int2 *wtab = win_tab + (WIN_MAX_BIN >= 0 ? (threadIdx.x >> 5) * WIN_TAB : 0);
     Fix192 d2{0, 0, 0, 0, 0};
     const bool tile_push = PEER && ACSR_PEER_TILE_PUSH && a.peer_n > 1;
 #if ACSR_SCHED_STATIC
@@ -1360,7 +1453,7 @@ static size_t spmv_smem(int bits)
 {
     static int reserve = -1;
     if (reserve < 0) reserve = env_int("ACSR_SMEM_RESERVE", 0);
-    const size_t win = ACSR_WIN_DYN_SMEM ? (size_t)SPMV_WARPS * 32 * (WIN_G * sizeof(double) + sizeof(int2)) : 0;
+    const size_t win = ACSR_WIN_DYN_SMEM ? (size_t)SPMV_WARPS * (32 * WIN_G * sizeof(double) + WIN_TAB * sizeof(int2)) : 0;
     return (XC ? (sizeof(V) + sizeof(uint16_t)) * ((size_t)1 << bits) : 0) + win + (size_t)reserve;
 }
 

@@ -68,6 +68,10 @@ for v in "$@"; do
     cb32w32) build cb32w32 -DACSR_CLAIM_BATCH=32 -DACSR_WIN_UNIT_ROWS=32 ;;
     cb16w32u1) build cb16w32u1 -DACSR_CLAIM_BATCH=16 -DACSR_WIN_UNIT_ROWS=32 -DACSR_UNIT_SHIFT=-1 ;;
     w32) build w32 -DACSR_WIN_UNIT_ROWS=32 ;;
+    rpl2) build rpl2 -DACSR_WIN_RPL=2 ;;
+    rpl4) build rpl4 -DACSR_WIN_RPL=4 ;;
+    rpl2g8) build rpl2g8 -DACSR_WIN_RPL=2 -DACSR_WIN_G=8 ;;
+    rpl4g8) build rpl4g8 -DACSR_WIN_RPL=4 -DACSR_WIN_G=8 ;;
     noremote) build noremote -DACSR_DIAG=4 ;;
     noremote0) build noremote0 -DACSR_DIAG=4 -DACSR_PEER_TILE_PUSH=0 ;;
     pft32) build pft32 -DACSR_PF_TILES=32 ;;

@@ -425,6 +425,18 @@ acsr_status acsr_relayout(acsr_dtype dt, int64_t n_rows,
                           const int32_t *new_begin, int32_t *new_end,
                           int32_t *new_col, void *new_val, cudaStream_t stream);
 
+/* The grown layout of reading R4, on the device: for every row
+ *   new_cap[r]   = max(cap_r + max(min_slack, ceil(cap_r / frac)),
+ *                      len_r + max(min_slack, ceil(len_r / frac)))      (every row grows)
+ *   new_begin[r] = sum_{r' < r} new_cap[r']                             (exclusive prefix)
+ * and total[0] = sum of new_cap (int64, DEVICE; the caller allocates total entries for the
+ * new col / val arrays and checks total < 2^31 before acsr_relayout).  min_slack >= 1,
+ * frac >= 1.  ws: acsr_grow_workspace_bytes(n_rows) bytes. */
+size_t acsr_grow_workspace_bytes(int64_t n_rows);
+acsr_status acsr_grow_layout(int64_t n_rows, const int32_t *row_begin, const int32_t *row_end,
+                             const int32_t *row_cap, int32_t min_slack, int32_t frac, int32_t *new_begin,
+                             int32_t *new_cap, int64_t *total, void *ws, size_t ws_bytes, cudaStream_t stream);
+
 /* ------------------------------------------------------------------------ */
 const char *acsr_status_string(acsr_status s);
 const char *acsr_last_error(void); /* thread-local detail of the last failure */

@@ -126,6 +126,10 @@ _lib.acsr_partition_workspace_bytes.argtypes = [_i64]
 _lib.acsr_partition_workspace_bytes.restype = _sz
 _lib.acsr_partition.argtypes = [_i64, _vp, _vp, _i64, _i64, ctypes.c_int, _i64, _vp, _vp, _sz, _vp]
 _lib.acsr_partition.restype = ctypes.c_int
+_lib.acsr_grow_workspace_bytes.argtypes = [_i64]
+_lib.acsr_grow_workspace_bytes.restype = _sz
+_lib.acsr_grow_layout.argtypes = [_i64, _vp, _vp, _vp, ctypes.c_int32, ctypes.c_int32, _vp, _vp, _vp, _vp, _sz, _vp]
+_lib.acsr_grow_layout.restype = ctypes.c_int
 _lib.acsr_relabel_workspace_bytes.argtypes = [_i64, _i64, ctypes.c_uint]
 _lib.acsr_relabel_workspace_bytes.restype = _sz
 _lib.acsr_degree_relabel.argtypes = [_i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp, ctypes.c_uint, _vp, _sz, _vp]
@@ -141,7 +145,8 @@ EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_bin_ex", "acsr_spmv", 
             "acsr_hits_workspace_bytes", "acsr_hits_normalize", "acsr_hits_normalize_ctrl", "acsr_plan_status",
             "acsr_comm_get_unique_id", "acsr_comm_init", "acsr_comm_destroy", "acsr_comm_query",
             "acsr_comm_allgather", "acsr_pagerank_init", "acsr_partition_workspace_bytes", "acsr_partition",
-            "acsr_relabel_workspace_bytes", "acsr_degree_relabel",
+            "acsr_relabel_workspace_bytes", "acsr_degree_relabel", "acsr_grow_workspace_bytes",
+            "acsr_grow_layout",
             "acsr_status_string", "acsr_last_error", "acsr_version")
 
 
@@ -368,6 +373,24 @@ class AcsrComm:
 
 
 ACSR_RELABEL_SORT_ROWS = 1
+
+
+def acsr_grow_layout(row_begin, row_end, row_cap, min_slack=8, frac=2, stream=None):
+    """Reading R4's grown layout on the device.  Returns (new_begin, new_cap, total) with
+    total an int (synchronising read: the caller sizes the new col / val arrays with it)."""
+    n = row_begin.numel()
+    dev = row_begin.device
+    nb = torch.empty(n, dtype=torch.int32, device=dev)
+    nc = torch.empty(n, dtype=torch.int32, device=dev)
+    tot = torch.zeros(1, dtype=torch.int64, device=dev)
+    ws = torch.empty(int(_lib.acsr_grow_workspace_bytes(n)), dtype=torch.uint8, device=dev)
+    _check(_lib.acsr_grow_layout(n, _dev(row_begin, torch.int32, "row_begin") if n else None,
+                                 _dev(row_end, torch.int32, "row_end") if n else None,
+                                 _dev(row_cap, torch.int32, "row_cap") if n else None, int(min_slack), int(frac),
+                                 _dev(nb, torch.int32, "new_begin") if n else None,
+                                 _dev(nc, torch.int32, "new_cap") if n else None, _dev(tot, torch.int64, "total"),
+                                 _dev(ws, torch.uint8, "ws"), ws.numel(), _stream(stream)), "acsr_grow_layout")
+    return nb, nc, int(tot.item())
 
 
 def acsr_degree_relabel(row_ptr, col_idx, outdeg, sort_rows=False, stream=None):

@@ -62,23 +62,19 @@ class ACSRMatrix:
         ceil(len_r / frac))) -- every row grows, so repeated rejections always progress.
         Then re-bin."""
         assert self.row_end is not None
-        ln = (self.row_end - self.row_begin).to(torch.int64)
-        old = self.row_cap.to(torch.int64)
-        cap = torch.maximum(old + torch.clamp((old + frac - 1) // frac, min=min_slack),
-                            ln + torch.clamp((ln + frac - 1) // frac, min=min_slack))
-        nb = torch.zeros_like(cap)
-        nb[1:] = torch.cumsum(cap, 0)[:-1]
-        total = int(nb[-1] + cap[-1]) if cap.numel() else 0
-        assert total < 2 ** 31
+        from . import acsr_grow_layout
+        new_begin, cap, total = acsr_grow_layout(self.row_begin, self.row_end, self.row_cap, min_slack, frac,
+                                                 stream=stream)
+        if total >= 2 ** 31:
+            raise OverflowError("grown slack CSR exceeds int32 indices")
         dev = self.row_begin.device
-        new_begin = nb.to(torch.int32)
         new_end = torch.empty_like(new_begin)
         new_col = torch.full((max(total, 1),), -1, dtype=torch.int32, device=dev)
         new_val = None if self.values is None else torch.zeros(max(total, 1), dtype=self.values.dtype,
                                                                device=dev)
         acsr_relayout(self.row_begin, self.row_end, self.col_idx, self.values, new_begin, new_end, new_col,
                       new_val, stream=stream)
-        self.row_begin, self.row_end, self.row_cap = new_begin, new_end, cap.to(torch.int32)
+        self.row_begin, self.row_end, self.row_cap = new_begin, new_end, cap
         self.col_idx, self.values = new_col, new_val
         if total > self.nnz_max:
             self.nnz_max = total

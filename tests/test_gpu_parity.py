@@ -1118,6 +1118,20 @@ def test_partition_and_relabel_edge_cases(acsr, cuda):
         acsr.AcsrComm(1, 0, b"short")
 
 
+def test_grow_layout_matches_reading_r4(acsr, cuda):
+    """acsr_grow_layout = reading R4 written out on the host: cap' = max(cap + max(m, ceil(cap/f)),
+    len + max(m, ceil(len/f))), begin' = exclusive prefix, total = sum (bitwise, integers)."""
+    n, rb, re, cap, col, _, od, rp, ci = _slack_graph(13)
+    for m_, f in ((8, 2), (4, 4), (1, 1)):
+        nb, nc, tot = acsr.acsr_grow_layout(rb.to(cuda), re.to(cuda), cap.to(cuda), m_, f)
+        ln = (re - rb).numpy().astype(np.int64)
+        c = cap.numpy().astype(np.int64)
+        ref = np.maximum(c + np.maximum(m_, -(-c // f)), ln + np.maximum(m_, -(-ln // f)))
+        pre = np.concatenate([[0], np.cumsum(ref)[:-1]])
+        assert np.array_equal(nc.cpu().numpy(), ref) and np.array_equal(nb.cpu().numpy(), pre)
+        assert tot == int(ref.sum())
+
+
 def test_single_rank_acsr_comm_step_equals_pagerank(acsr, cuda):
     """acsr_pagerank_step with a one-rank acsr_comm (exchange + global Delta^2 in the
     library) gives the single-GPU loop's iterate, iteration count and Delta^2 bitwise."""

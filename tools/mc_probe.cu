@@ -16,14 +16,27 @@ int main() {
     printf("multicast supported: %d\n", mc);
     if (!mc) return 0;
     CUmulticastObjectProp prop = {};
-    prop.numDevices = 1; prop.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR; prop.size = 2 << 20;
-    size_t gran = 0; CKD(cuMulticastGetGranularity(&gran, &prop, CU_MULTICAST_GRANULARITY_RECOMMENDED));
-    prop.size = ((prop.size + gran - 1) / gran) * gran;
-    printf("granularity %zu size %zu\n", gran, prop.size);
-    CUmemGenericAllocationHandle mch; CKD(cuMulticastCreate(&mch, &prop));
+    CUmemGenericAllocationHandle mch;
+    int created = 0;
+    const int nds[] = {1, 2};
+    const unsigned long long hts[] = {CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, CU_MEM_HANDLE_TYPE_NONE, CU_MEM_HANDLE_TYPE_FABRIC};
+    for (int a = 0; a < 2 && !created; a++)
+        for (int b = 0; b < 3 && !created; b++) {
+            prop = {};
+            prop.numDevices = nds[a]; prop.handleTypes = hts[b]; prop.size = 2 << 20;
+            size_t gran = 0;
+            if (cuMulticastGetGranularity(&gran, &prop, CU_MULTICAST_GRANULARITY_RECOMMENDED) != CUDA_SUCCESS) continue;
+            prop.size = ((prop.size + gran - 1) / gran) * gran;
+            CUresult r = cuMulticastCreate(&mch, &prop);
+            const char *es; cuGetErrorString(r, &es);
+            printf("cuMulticastCreate numDevices=%d handleTypes=%llu: %s\n", nds[a], hts[b], es);
+            if (r == CUDA_SUCCESS) created = 1;
+        }
+    if (!created) return 0;
+    if (prop.numDevices > 1) { printf("only a >= 2-device multicast object is creatable; cannot complete it on 1 GPU\n"); return 0; }
     CKD(cuMulticastAddDevice(mch, dev));
     CUmemAllocationProp ap = {}; ap.type = CU_MEM_ALLOCATION_TYPE_PINNED; ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE; ap.location.id = dev;
-    ap.requestedHandleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+    ap.requestedHandleTypes = (CUmemAllocationHandleType)prop.handleTypes;
     CUmemGenericAllocationHandle mh; CKD(cuMemCreate(&mh, prop.size, &ap, 0));
     CKD(cuMulticastBindMem(mch, 0, mh, 0, prop.size, 0));
     CUdeviceptr uva, mva;

@@ -175,6 +175,32 @@ acsr_status acsr_partition(int64_t n_rows, const int32_t *row_begin, const int32
                            int64_t b_nnz, int64_t b_row, int nranks, int64_t align, int64_t *splits, void *ws,
                            size_t ws_bytes, cudaStream_t stream);
 
+/* Compact exchange layout of the row-partitioned PageRank (SURVEY §8(e) lever 2): xs_u = 0
+ * exactly when outdeg_u = 0 (Alg. 5 with reading Q11), and such a vertex is never a column
+ * of the in-link pattern, so only non-dangling vertices get a slot.  Inputs: the global
+ * non-dangling mask nd[n_global] (DEVICE u8; assembled from every rank's local mask, e.g. by
+ * acsr_comm_allgather) and the partition splits (DEVICE int64 [nranks + 1]).  Outputs:
+ *   counts[k] (DEVICE int64)  non-dangling vertices of rank k;  lx[0] = max(1, max counts)
+ *   pos[v]  (DEVICE int32)    owner(v) * Lx + (rank of v among its owner's non-dangling
+ *                             vertices) for non-dangling v, nranks * Lx (a trailing slot that
+ *                             is always 0) otherwise -- the column renumbering;
+ *   order   (DEVICE int32, nullable; [splits[rank+1] - splits[rank]])  this rank's local rows,
+ *                             non-dangling first, each group in row order (new -> old), so the
+ *                             exchanged slice is a prefix of the local xs (acsr_permute_graph).
+ * ws: acsr_exchange_layout_workspace_bytes(n_global) bytes. */
+size_t acsr_exchange_layout_workspace_bytes(int64_t n_global);
+acsr_status acsr_exchange_layout(int64_t n_global, int nranks, const int64_t *splits, const uint8_t *nd, int rank,
+                                 int32_t *pos, int32_t *order, int64_t *counts, int64_t *lx, void *ws, size_t ws_bytes,
+                                 cudaStream_t stream);
+
+/* Rows of a standard CSR reordered (new row i = old row order[i]) with every column mapped
+ * through col_map (DEVICE int32 [n_cols], NULL: kept); entry order inside a row kept.  The
+ * copy machinery of acsr_degree_relabel.  ws: acsr_permute_workspace_bytes(n) bytes. */
+size_t acsr_permute_workspace_bytes(int64_t n);
+acsr_status acsr_permute_graph(int64_t n, const int32_t *row_ptr, const int32_t *col_idx, const int32_t *order,
+                               const int32_t *col_map, int32_t *row_ptr_out, int32_t *col_out, void *ws, size_t ws_bytes,
+                               cudaStream_t stream);
+
 /* ------------------------------------------------------------------------ */
 /* PageRank step (Alg. 5; §VI-A) on one rank's rows.
  *   PR^{k+1} = (1-d) PR^(0) + d (A^T PR^k),  A row-normalised.

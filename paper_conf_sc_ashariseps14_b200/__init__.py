@@ -126,6 +126,14 @@ _lib.acsr_partition_workspace_bytes.argtypes = [_i64]
 _lib.acsr_partition_workspace_bytes.restype = _sz
 _lib.acsr_partition.argtypes = [_i64, _vp, _vp, _i64, _i64, ctypes.c_int, _i64, _vp, _vp, _sz, _vp]
 _lib.acsr_partition.restype = ctypes.c_int
+_lib.acsr_exchange_layout_workspace_bytes.argtypes = [_i64]
+_lib.acsr_exchange_layout_workspace_bytes.restype = _sz
+_lib.acsr_exchange_layout.argtypes = [_i64, ctypes.c_int, _vp, _vp, ctypes.c_int, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
+_lib.acsr_exchange_layout.restype = ctypes.c_int
+_lib.acsr_permute_workspace_bytes.argtypes = [_i64]
+_lib.acsr_permute_workspace_bytes.restype = _sz
+_lib.acsr_permute_graph.argtypes = [_i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]
+_lib.acsr_permute_graph.restype = ctypes.c_int
 _lib.acsr_grow_workspace_bytes.argtypes = [_i64]
 _lib.acsr_grow_workspace_bytes.restype = _sz
 _lib.acsr_grow_layout.argtypes = [_i64, _vp, _vp, _vp, ctypes.c_int32, ctypes.c_int32, _vp, _vp, _vp, _vp, _sz, _vp]
@@ -146,7 +154,8 @@ EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_bin_ex", "acsr_spmv", 
             "acsr_comm_get_unique_id", "acsr_comm_init", "acsr_comm_destroy", "acsr_comm_query",
             "acsr_comm_allgather", "acsr_pagerank_init", "acsr_partition_workspace_bytes", "acsr_partition",
             "acsr_relabel_workspace_bytes", "acsr_degree_relabel", "acsr_grow_workspace_bytes",
-            "acsr_grow_layout",
+            "acsr_grow_layout", "acsr_exchange_layout_workspace_bytes", "acsr_exchange_layout",
+            "acsr_permute_workspace_bytes", "acsr_permute_graph",
             "acsr_status_string", "acsr_last_error", "acsr_version")
 
 
@@ -373,6 +382,46 @@ class AcsrComm:
 
 
 ACSR_RELABEL_SORT_ROWS = 1
+
+
+def acsr_exchange_layout(nd, splits, rank=-1, stream=None):
+    """Compact exchange layout (include/acsr.h).  nd: CUDA uint8 [n_global] non-dangling mask;
+    splits: CUDA int64 [P + 1].  Returns (pos int32 [n_global], order int32 [local rows] or None,
+    counts int64 [P] (host list), Lx int)."""
+    n = nd.numel()
+    P = splits.numel() - 1
+    dev = nd.device
+    pos = torch.empty(n, dtype=torch.int32, device=dev)
+    counts = torch.empty(P, dtype=torch.int64, device=dev)
+    lx = torch.empty(1, dtype=torch.int64, device=dev)
+    order = None
+    if rank >= 0:
+        sp = splits.cpu()
+        order = torch.empty(int(sp[rank + 1] - sp[rank]), dtype=torch.int32, device=dev)
+    ws = torch.empty(int(_lib.acsr_exchange_layout_workspace_bytes(n)), dtype=torch.uint8, device=dev)
+    _check(_lib.acsr_exchange_layout(n, P, _dev(splits, torch.int64, "splits"),
+                                     _dev(nd, torch.uint8, "nd") if n else None, int(rank),
+                                     _dev(pos, torch.int32, "pos") if n else None,
+                                     _dev(order, torch.int32, "order") if order is not None and order.numel() else None,
+                                     _dev(counts, torch.int64, "counts"), _dev(lx, torch.int64, "lx"),
+                                     _dev(ws, torch.uint8, "ws"), ws.numel(), _stream(stream)), "acsr_exchange_layout")
+    return pos, order, [int(c) for c in counts.cpu()], int(lx.item())
+
+
+def acsr_permute_graph(row_ptr, col_idx, order, col_map=None, stream=None):
+    """Rows reordered (new row i = old row order[i]), columns mapped through col_map."""
+    n = row_ptr.numel() - 1
+    dev = row_ptr.device
+    rp2 = torch.empty(n + 1, dtype=torch.int32, device=dev)
+    c2 = torch.empty_like(col_idx)
+    ws = torch.empty(int(_lib.acsr_permute_workspace_bytes(n)), dtype=torch.uint8, device=dev)
+    _check(_lib.acsr_permute_graph(n, _dev(row_ptr, torch.int32, "row_ptr"),
+                                   _dev(col_idx, torch.int32, "col_idx") if col_idx.numel() else None,
+                                   _dev(order, torch.int32, "order") if n else None,
+                                   _dev(col_map, torch.int32, "col_map", True), _dev(rp2, torch.int32, "row_ptr_out"),
+                                   _dev(c2, torch.int32, "col_out") if c2.numel() else None,
+                                   _dev(ws, torch.uint8, "ws"), ws.numel(), _stream(stream)), "acsr_permute_graph")
+    return rp2, c2
 
 
 def acsr_grow_layout(row_begin, row_end, row_cap, min_slack=8, frac=2, stream=None):

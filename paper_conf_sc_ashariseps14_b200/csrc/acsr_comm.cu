@@ -245,3 +245,91 @@ extern "C" acsr_status acsr_partition(int64_t n_rows, const int32_t *row_begin, 
     split_search_kernel<<<(nranks + 1 + 127) / 128, 128, 0, stream>>>(incl, n_rows, nranks, align, splits);
     return acsr_check_launch("acsr_partition");
 }
+
+// ---------------------------------------------------------------------------------------
+// Compact (dangling-free) exchange layout of the row-partitioned PageRank (SURVEY §8(e)
+// lever 2): xs_u = 0 exactly when outdeg_u = 0 (Alg. 5 with reading Q11), so only
+// non-dangling vertices get a slot in the replicated xs.
+namespace acsr {
+__global__ void nd_to_int_kernel(int64_t n, const uint8_t *__restrict__ nd, int32_t *__restrict__ v)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n; i += (int64_t)gridDim.x * blockDim.x)
+        v[i] = i < n ? (nd[i] != 0) : 0;
+}
+
+// one thread per rank: non-dangling count; Lx = max(1, max count)
+__global__ void layout_counts_kernel(const int64_t *__restrict__ splits, int P, const int32_t *__restrict__ excl,
+                                     int64_t *__restrict__ counts, int64_t *lx)
+{
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    int64_t m = 1;
+    for (int k = 0; k < P; k++) {
+        const int64_t c = (int64_t)excl[splits[k + 1]] - excl[splits[k]];
+        counts[k] = c;
+        m = c > m ? c : m;
+    }
+    *lx = m;
+}
+
+__global__ void layout_pos_kernel(int64_t n, const int64_t *__restrict__ splits, int P, const uint8_t *__restrict__ nd,
+                                  const int32_t *__restrict__ excl, const int64_t *__restrict__ lx,
+                                  int32_t *__restrict__ pos, int rank, int32_t *__restrict__ order)
+{
+    const int64_t Lx = *lx;
+    const int64_t lo = splits[rank], hi = splits[rank + 1];
+    const int64_t nloc_nd = (int64_t)excl[hi] - excl[lo];
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        int owner = 0;
+        while (owner + 1 < P && splits[owner + 1] <= v) owner++;
+        const bool isnd = nd[v] != 0;
+        const int64_t rk = (int64_t)excl[v] - excl[splits[owner]];
+        pos[v] = (int32_t)(isnd ? owner * Lx + rk : (int64_t)P * Lx);
+        if (order && v >= lo && v < hi) {  // this rank's rows: non-dangling first, each group in row order
+            const int64_t r = v - lo;
+            const int64_t dst = isnd ? rk : nloc_nd + (r - rk);
+            order[dst] = (int32_t)r;
+        }
+    }
+}
+}  // namespace acsr
+
+extern "C" size_t acsr_exchange_layout_workspace_bytes(int64_t n_global)
+{
+    const size_t nn = (size_t)(n_global > 0 ? n_global : 0) + 1;
+    size_t temp = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, temp, (const int32_t *)nullptr, (int32_t *)nullptr, (int)nn);
+    return 2 * align_up(4 * nn, 256) + align_up(temp, 256);
+}
+
+extern "C" acsr_status acsr_exchange_layout(int64_t n_global, int nranks, const int64_t *splits, const uint8_t *nd,
+                                            int rank, int32_t *pos, int32_t *order, int64_t *counts, int64_t *lx,
+                                            void *ws, size_t ws_bytes, cudaStream_t stream)
+{
+    if (n_global < 0 || n_global >= ((int64_t)1 << 31) || nranks < 1 || rank < -1 || rank >= nranks || !splits ||
+        !counts || !lx || (n_global > 0 && (!nd || !pos)) || (order && rank < 0)) {
+        acsr_set_error("acsr_exchange_layout: invalid argument");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    if (!ws || ws_bytes < acsr_exchange_layout_workspace_bytes(n_global)) {
+        acsr_set_error("acsr_exchange_layout: workspace missing or too small");
+        return ACSR_ERR_WORKSPACE;
+    }
+    const size_t nn = (size_t)n_global + 1;
+    int32_t *v = (int32_t *)ws;
+    int32_t *excl = (int32_t *)((char *)ws + align_up(4 * nn, 256));
+    void *temp = (char *)ws + 2 * align_up(4 * nn, 256);
+    size_t tb = ws_bytes - 2 * align_up(4 * nn, 256);
+    const int sms = acsr_num_sms();
+    const int grid = (int)((int64_t)(nn + 255) / 256 < (int64_t)sms * 8 ? (int64_t)(nn + 255) / 256 : (int64_t)sms * 8);
+    nd_to_int_kernel<<<grid, 256, 0, stream>>>(n_global, nd, v);
+    const cudaError_t e = cub::DeviceScan::ExclusiveSum(temp, tb, v, excl, (int)nn, stream);
+    if (e != cudaSuccess) {
+        acsr_set_error("acsr_exchange_layout (scan): %s", cudaGetErrorString(e));
+        return ACSR_ERR_CUDA;
+    }
+    layout_counts_kernel<<<1, 32, 0, stream>>>(splits, nranks, excl, counts, lx);
+    if (n_global > 0)
+        layout_pos_kernel<<<grid, 256, 0, stream>>>(n_global, splits, nranks, nd, excl, lx, pos, rank < 0 ? 0 : rank,
+                                                    order);
+    return acsr_check_launch("acsr_exchange_layout");
+}

@@ -95,7 +95,7 @@ __global__ void relabel_perm_kernel(int64_t n, const int32_t *__restrict__ order
 // exclusive prefixes); long rows are listed for the CTA pass
 __global__ void __launch_bounds__(RELABEL_THREADS)
 relabel_copy_kernel(int64_t n, const int32_t *__restrict__ order, const int32_t *__restrict__ rp,
-                    const int32_t *__restrict__ col, const int32_t *__restrict__ perm,
+                    const int32_t *__restrict__ col, const int32_t *__restrict__ perm /* NULL: columns kept */,
                     const int32_t *__restrict__ rp_new, int32_t *__restrict__ col_new, int32_t *__restrict__ long_rows,
                     int32_t *ctr)
 {
@@ -137,7 +137,8 @@ relabel_copy_kernel(int64_t n, const int32_t *__restrict__ order, const int32_t 
             const int pj = __shfl_sync(0xffffffffu, pre, j);
             if (t < T) {
                 const int e = t - pj;
-                col_new[dj + e] = perm[__ldcs(col + bj + e)];
+                const int c = __ldcs(col + bj + e);
+                col_new[dj + e] = perm ? perm[c] : c;
             }
         }
     }
@@ -161,7 +162,10 @@ relabel_long_kernel(const int32_t *__restrict__ order, const int32_t *__restrict
         if (i < 0) break;
         const int32_t u = order[i];
         const int beg = rp[u], len = rp[u + 1] - beg, dst = rp_new[i];
-        for (int e = threadIdx.x; e < len; e += blockDim.x) col_new[dst + e] = perm[__ldcs(col + beg + e)];
+        for (int e = threadIdx.x; e < len; e += blockDim.x) {
+            const int c = __ldcs(col + beg + e);
+            col_new[dst + e] = perm ? perm[c] : c;
+        }
     }
 }
 
@@ -238,4 +242,64 @@ extern "C" acsr_status acsr_degree_relabel(int64_t n, int64_t nnz, const int32_t
         }
     }
     return acsr_check_launch("acsr_degree_relabel");
+}
+
+// ---------------------------------------------------------------------------------------
+// acsr_permute_graph: rows reordered by `order` (new row i = old row order[i]) and every
+// column mapped through col_map (NULL: kept) -- the same scan + copy kernels as the relabel.
+namespace acsr {
+__global__ void permute_len_kernel(int64_t n, const int32_t *__restrict__ order, const int32_t *__restrict__ rp,
+                                   int32_t *__restrict__ len_new)
+{
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t u = order[i];
+        len_new[i] = rp[u + 1] - rp[u];
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) len_new[n] = 0;
+}
+}  // namespace acsr
+
+extern "C" size_t acsr_permute_workspace_bytes(int64_t n) { return relabel_layout(n, 0, 0).total; }
+
+extern "C" acsr_status acsr_permute_graph(int64_t n, const int32_t *row_ptr, const int32_t *col_idx,
+                                          const int32_t *order, const int32_t *col_map, int32_t *row_ptr_out,
+                                          int32_t *col_out, void *ws, size_t ws_bytes, cudaStream_t stream)
+{
+    if (n < 0 || n >= ((int64_t)1 << 31) - 1 || !row_ptr_out || (n > 0 && (!row_ptr || !order))) {
+        acsr_set_error("acsr_permute_graph: invalid argument");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    const RelabelLayout L = relabel_layout(n, 0, 0);
+    if (!ws || ws_bytes < L.total) {
+        acsr_set_error("acsr_permute_graph: workspace missing or too small");
+        return ACSR_ERR_WORKSPACE;
+    }
+    if (n == 0) {
+        cudaMemsetAsync(row_ptr_out, 0, sizeof(int32_t), stream);
+        return acsr_check_launch("acsr_permute_graph");
+    }
+    char *w = (char *)ws;
+    int32_t *len_new = (int32_t *)(w + L.off_len), *long_rows = (int32_t *)(w + L.off_long);
+    int32_t *ctr = (int32_t *)(w + L.off_ctr);
+    void *temp = w + L.off_temp;
+    const int sms = acsr_num_sms();
+    const int grid = (int)((n + RELABEL_THREADS - 1) / RELABEL_THREADS < (int64_t)sms * 8
+                               ? (n + RELABEL_THREADS - 1) / RELABEL_THREADS : (int64_t)sms * 8);
+    cudaMemsetAsync(ctr, 0, 16, stream);
+    permute_len_kernel<<<grid, RELABEL_THREADS, 0, stream>>>(n, order, row_ptr, len_new);
+    size_t tb = L.temp_bytes;
+    const cudaError_t e = cub::DeviceScan::ExclusiveSum(temp, tb, len_new, row_ptr_out, (int)n + 1, stream);
+    if (e != cudaSuccess) {
+        acsr_set_error("acsr_permute_graph (scan): %s", cudaGetErrorString(e));
+        return ACSR_ERR_CUDA;
+    }
+    if (col_idx && col_out) {
+        const int64_t nw = (n + 31) / 32;
+        const int cgrid = (int)((nw + 7) / 8 < (int64_t)sms * 16 ? (nw + 7) / 8 : (int64_t)sms * 16);
+        relabel_copy_kernel<<<cgrid, RELABEL_THREADS, 0, stream>>>(n, order, row_ptr, col_idx, col_map, row_ptr_out,
+                                                                   col_out, long_rows, ctr);
+        relabel_long_kernel<<<sms, 1024, 0, stream>>>(order, row_ptr, col_idx, col_map, row_ptr_out, col_out,
+                                                      long_rows, ctr);
+    }
+    return acsr_check_launch("acsr_permute_graph");
 }

@@ -186,7 +186,19 @@ class DistPageRank:
         else:
             dist.all_gather_into_tensor(allm, pad.clone() if dev.type == "cpu" else pad, group=self.group)
         sizes = np.diff(self.splits)
-        nd = torch.cat([allm[k * L: k * L + int(sizes[k])] for k in range(world)]).to(torch.bool)
+        nd = torch.cat([allm[k * L: k * L + int(sizes[k])] for k in range(world)])
+        if dev.type == "cuda":
+            # the layout arithmetic in the library (acsr_exchange_layout, acsr_permute_graph)
+            from . import acsr_exchange_layout, acsr_permute_graph
+            sp = torch.as_tensor(self.splits, dtype=torch.int64, device=dev)
+            pos, order, nnd, self.Lx = acsr_exchange_layout(nd.contiguous(), sp, rank=self.rank)
+            self.n_nd = nnd
+            self.perm = order.to(torch.int64)
+            self.row_ptr, self.col = acsr_permute_graph(row_ptr_local.to(torch.int32).contiguous(),
+                                                        col_local.contiguous(), order, col_map=pos)
+            self.outdeg = outdeg_local[self.perm].contiguous()
+            return
+        nd = nd.to(torch.bool)
         nnd = [int(allm[k * L: k * L + int(sizes[k])].sum()) for k in range(world)]
         self.n_nd = nnd
         self.Lx = max(1, max(nnd))

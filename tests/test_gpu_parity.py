@@ -1132,6 +1132,39 @@ def test_grow_layout_matches_reading_r4(acsr, cuda):
         assert tot == int(ref.sum())
 
 
+@pytest.mark.parametrize("P", [2, 3])
+def test_exchange_layout_matches_definition(acsr, cuda, P):
+    """acsr_exchange_layout + acsr_permute_graph = the compact layout's definition written out
+    on the host: pos[v] = owner(v) * Lx + rank among the owner's non-dangling
+    vertices (P * Lx for dangling v), local order = non-dangling rows first, stable, and the
+    permuted local CSR with renumbered columns -- bitwise, for every rank."""
+    from paper_conf_sc_ashariseps14_b200 import dist as pdist
+    rp, ci, od, n = _inlink(14, cuda)
+    splits = pdist.partition_rows(np.diff(rp.numpy()), P)
+    nd = (od.numpy() > 0)
+    counts = [int(nd[splits[k]:splits[k + 1]].sum()) for k in range(P)]
+    Lx = max(1, max(counts))
+    owner = np.searchsorted(splits[1:-1], np.arange(n), side="right")
+    ex = np.cumsum(nd) - nd
+    pos_ref = np.where(nd, owner * Lx + ex - ex[splits[owner]], P * Lx)
+    sp = torch.as_tensor(splits, dtype=torch.int64, device=cuda)
+    for rank in range(P):
+        pos, order, cnt, lx = acsr.acsr_exchange_layout(torch.from_numpy(nd.astype(np.uint8)).to(cuda), sp, rank)
+        assert cnt == counts and lx == Lx
+        assert np.array_equal(pos.cpu().numpy(), pos_ref)
+        lo, hi = int(splits[rank]), int(splits[rank + 1])
+        ndl = nd[lo:hi]
+        order_ref = np.concatenate([np.flatnonzero(ndl), np.flatnonzero(~ndl)])
+        assert np.array_equal(order.cpu().numpy(), order_ref)
+        rpl = (rp[lo:hi + 1] - rp[lo]).to(torch.int32)
+        cil = ci[int(rp[lo]):int(rp[hi])]
+        rp2, c2 = acsr.acsr_permute_graph(rpl.to(cuda), cil.to(cuda), order, col_map=pos)
+        ln = np.diff(rpl.numpy())[order_ref]
+        assert np.array_equal(rp2.cpu().numpy(), np.concatenate([[0], np.cumsum(ln)]))
+        ref = np.concatenate([pos_ref[cil.numpy()[rpl[r]:rpl[r + 1]]] for r in order_ref]) if ln.sum() else np.zeros(0)
+        assert np.array_equal(c2.cpu().numpy(), ref)
+
+
 def test_single_rank_acsr_comm_step_equals_pagerank(acsr, cuda):
     """acsr_pagerank_step with a one-rank acsr_comm (exchange + global Delta^2 in the
     library) gives the single-GPU loop's iterate, iteration count and Delta^2 bitwise."""

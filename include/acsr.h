@@ -255,6 +255,12 @@ typedef struct {
     acsr_comm *comm;              /* NULL => single GPU, no exchange; else see above */
     double *xs_all;               /* with comm: [n_cols] replicated xs' receiving every slice */
     int64_t slice_len;            /* with comm: entries per rank in xs_all (n_cols >= nranks * slice_len) */
+    const int64_t *slice_counts;  /* with comm: HOST [nranks] or NULL.  If given, only the first
+                                   * slice_counts[q] <= slice_len entries of rank q's slice are
+                                   * exchanged (all-gather-v: one grouped ncclBroadcast per rank),
+                                   * so unequal slices -- e.g. the non-dangling counts of a
+                                   * degree-relabelled partition -- cost their sum, not
+                                   * nranks * max.  Entries past the counts are left untouched. */
 } acsr_pr_args;
 
 acsr_status acsr_pagerank_step(const acsr_pr_args *args, cudaStream_t stream);

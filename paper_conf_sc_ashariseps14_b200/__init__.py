@@ -81,7 +81,7 @@ class PrArgs(ctypes.Structure):
                 ("plan_ws_bytes", _sz), ("xs", _vp), ("x", _vp), ("outdeg", _vp), ("x_new", _vp),
                 ("xs_next", _vp), ("damping", _dbl), ("teleport", _dbl), ("delta2", _vp),
                 ("restart", _i64), ("restart_weight", _dbl), ("ctrl", _vp), ("eps2", _dbl),
-                ("comm", _vp), ("xs_all", _vp), ("slice_len", _i64)]
+                ("comm", _vp), ("xs_all", _vp), ("slice_len", _i64), ("slice_counts", ctypes.POINTER(_i64))]
 
 
 _lib.acsr_pagerank_step.argtypes = [ctypes.POINTER(PrArgs), _vp]
@@ -278,7 +278,7 @@ def acsr_pagerank_scale(x, outdeg, xs=None, stream=None):
 def acsr_pagerank_step(row_begin, col_idx, bin_rows, bin_offsets, plan_ws, xs, x, outdeg, x_new,
                        xs_next, delta2, damping=0.85, teleport=None, n_global=None, row_end=None,
                        stream=None, restart=-1, restart_weight=0.0, ctrl=None, eps2=-1.0, comm=None,
-                       xs_all=None, slice_len=0):
+                       xs_all=None, slice_len=0, slice_counts=None):
     """One fused PageRank step on the local rows (Alg. 5).  delta2: 1-element float64.
     With teleport=0, damping=c, restart=i, restart_weight=1-c it is an RWR step (Eq. 8).
     comm (AcsrComm): multi-GPU -- the step is followed by the library's exchange: xs_next[:slice_len]
@@ -299,12 +299,22 @@ def acsr_pagerank_step(row_begin, col_idx, bin_rows, bin_offsets, plan_ws, xs, x
                _dev(delta2, torch.float64, "delta2"), int(restart), float(restart_weight),
                _dev(ctrl, torch.int32, "ctrl", True), float(eps2),
                comm._c if comm is not None else None,
-               _dev(xs_all, torch.float64, "xs_all") if comm is not None else None, int(slice_len))
+               _dev(xs_all, torch.float64, "xs_all") if comm is not None else None, int(slice_len),
+               _counts(slice_counts))
     _check(_lib.acsr_pagerank_step(ctypes.byref(a), _stream(stream)), "acsr_pagerank_step")
     return x_new, xs_next, delta2
 
 
-def acsr_pagerank_init(x, outdeg, xs_next, comm=None, xs_all=None, slice_len=0, stream=None):
+def _counts(slice_counts):
+    """HOST int64 array for acsr_pr_args.slice_counts (kept alive by the caller's list)."""
+    if slice_counts is None:
+        return None
+    arr = (_i64 * len(slice_counts))(*[int(c) for c in slice_counts])
+    _counts.keep = arr  # the call is synchronous on the host side; keep until the next call
+    return ctypes.cast(arr, ctypes.POINTER(_i64))
+
+
+def acsr_pagerank_init(x, outdeg, xs_next, comm=None, xs_all=None, slice_len=0, stream=None, slice_counts=None):
     """xs_next[:n] = x / outdeg (first iterate, P:285 / warm start); with comm the
     slices are all-gathered into xs_all (include/acsr.h)."""
     n = x.numel()
@@ -317,6 +327,7 @@ def acsr_pagerank_init(x, outdeg, xs_next, comm=None, xs_all=None, slice_len=0, 
     a.comm = comm._c if comm is not None else None
     a.xs_all = _dev(xs_all, torch.float64, "xs_all") if comm is not None else None
     a.slice_len = int(slice_len)
+    a.slice_counts = _counts(slice_counts)
     _check(_lib.acsr_pagerank_init(ctypes.byref(a), _stream(stream)), "acsr_pagerank_init")
     return xs_next
 

@@ -174,12 +174,38 @@ extern "C" acsr_status acsr_comm_allgather(acsr_comm *c, const void *send, void 
 
 // Called by acsr_pagerank_step after the fused step kernel (which wrote its Delta^2
 // partial to comm->d2[0..3)) when args->comm != NULL.
+uint64_t *acsr_comm_d2_slot(acsr_comm *c) { return c->d2; }
+int acsr_comm_nranks(const acsr_comm *c) { return c->nranks; }
+
+// the xs slices: one all-gather of equal slices, or (slice_counts) one broadcast per rank
+static ncclResult_t xs_exchange(const acsr_pr_args *p, acsr_comm *c, cudaStream_t stream)
+{
+    if (p->slice_len <= 0) return ncclSuccess;
+    if (!p->slice_counts)
+        return ncclAllGather(p->xs_next, p->xs_all, (size_t)p->slice_len, ncclFloat64, c->nccl, stream);
+    ncclResult_t r = ncclSuccess;
+    for (int q = 0; q < c->nranks && r == ncclSuccess; q++) {
+        double *dst = p->xs_all + (int64_t)q * p->slice_len;
+        const int64_t cnt = p->slice_counts[q];
+        if (cnt > 0) r = ncclBroadcast(q == c->rank ? (const void *)p->xs_next : dst, dst, (size_t)cnt, ncclFloat64, q,
+                                       c->nccl, stream);
+    }
+    return r;
+}
+
+static bool counts_ok(const acsr_pr_args *p)
+{
+    if (!p->slice_counts) return true;
+    for (int q = 0; q < acsr_comm_nranks(p->comm); q++)
+        if (p->slice_counts[q] < 0 || p->slice_counts[q] > p->slice_len) return false;
+    return true;
+}
+
 acsr_status acsr_comm_step_exchange(const acsr_pr_args *p, cudaStream_t stream)
 {
     acsr_comm *c = p->comm;
     ncclResult_t r = ncclGroupStart();
-    if (r == ncclSuccess && p->slice_len > 0)
-        r = ncclAllGather(p->xs_next, p->xs_all, (size_t)p->slice_len, ncclFloat64, c->nccl, stream);
+    if (r == ncclSuccess) r = xs_exchange(p, c, stream);
     if (r == ncclSuccess) r = ncclAllGather(c->d2, c->d2 + 3, 3, ncclUint64, c->nccl, stream);
     const ncclResult_t r2 = ncclGroupEnd();
     if (r != ncclSuccess) return nccl_fail("acsr_pagerank_step (exchange)", r);
@@ -188,8 +214,6 @@ acsr_status acsr_comm_step_exchange(const acsr_pr_args *p, cudaStream_t stream)
     return acsr_check_launch("acsr_pagerank_step (Delta^2 finalize)");
 }
 
-uint64_t *acsr_comm_d2_slot(acsr_comm *c) { return c->d2; }
-int acsr_comm_nranks(const acsr_comm *c) { return c->nranks; }
 
 extern "C" acsr_status acsr_pagerank_init(const acsr_pr_args *p, cudaStream_t stream)
 {
@@ -202,11 +226,18 @@ extern "C" acsr_status acsr_pagerank_init(const acsr_pr_args *p, cudaStream_t st
         acsr_set_error("acsr_pagerank_init: with comm, xs_all [n_cols >= nranks * slice_len] is required");
         return ACSR_ERR_INVALID_VALUE;
     }
+    if (p->comm && !counts_ok(p)) {
+        acsr_set_error("acsr_pagerank_init: slice_counts[q] must lie in [0, slice_len]");
+        return ACSR_ERR_INVALID_VALUE;
+    }
     acsr_status st = acsr_pagerank_scale(p->n_rows, p->x, p->outdeg, p->xs_next, stream);
     if (st != ACSR_OK || !p->comm) return st;
     if (p->slice_len == 0) return ACSR_OK;
-    const ncclResult_t r = ncclAllGather(p->xs_next, p->xs_all, (size_t)p->slice_len, ncclFloat64, p->comm->nccl, stream);
-    if (r != ncclSuccess) return nccl_fail("acsr_pagerank_init (all-gather)", r);
+    ncclResult_t r = ncclGroupStart();
+    if (r == ncclSuccess) r = xs_exchange(p, p->comm, stream);
+    const ncclResult_t r2 = ncclGroupEnd();
+    if (r != ncclSuccess) return nccl_fail("acsr_pagerank_init (exchange)", r);
+    if (r2 != ncclSuccess) return nccl_fail("acsr_pagerank_init (exchange)", r2);
     return acsr_check_launch("acsr_pagerank_init");
 }
 

@@ -1682,8 +1682,12 @@ extern "C" acsr_status acsr_pagerank_step(const acsr_pr_args *p, cudaStream_t st
         acsr_set_error("acsr_pagerank_step: plan workspace missing or too small");
         return ACSR_ERR_WORKSPACE;
     }
-    if (p->comm && (!p->xs_all || p->slice_len < 0 || p->n_cols < (int64_t)acsr_comm_nranks(p->comm) * p->slice_len ||
-                    (p->slice_len > 0 && !p->xs_next))) {
+    bool counts_bad = false;
+    if (p->comm && p->slice_counts)
+        for (int q = 0; q < acsr_comm_nranks(p->comm); q++)
+            counts_bad |= p->slice_counts[q] < 0 || p->slice_counts[q] > p->slice_len;
+    if (p->comm && (counts_bad || !p->xs_all || p->slice_len < 0 ||
+                    p->n_cols < (int64_t)acsr_comm_nranks(p->comm) * p->slice_len || (p->slice_len > 0 && !p->xs_next))) {
         acsr_set_error("acsr_pagerank_step: with comm, xs_all [n_cols >= nranks * slice_len] and xs_next are required");
         return ACSR_ERR_INVALID_VALUE;
     }

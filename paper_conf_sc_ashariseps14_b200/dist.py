@@ -286,7 +286,10 @@ class DistPageRank:
 
         bufs = [x, torch.empty_like(x)]
         xsb = [self.xs, self.xs_next]
-        acsr_pagerank_init(x, self.outdeg, local_out(xsb[0]), comm=comm, xs_all=xsb[0], slice_len=Ls)
+        # all-gather-v: only each rank's real entries move (non-dangling counts, or row counts)
+        counts = self.n_nd if self.compact else [int(c) for c in np.diff(self.splits)]
+        acsr_pagerank_init(x, self.outdeg, local_out(xsb[0]), comm=comm, xs_all=xsb[0], slice_len=Ls,
+                           slice_counts=counts)
         ctrl = torch.zeros(2, dtype=torch.int32, device=self.device)
         eps2 = eps * eps if eps >= 0 else -1.0
         k = 0
@@ -296,7 +299,7 @@ class DistPageRank:
                 acsr_pagerank_step(m.row_begin, m.col_idx, m.bin_rows, m.bin_offsets, m.plan_ws, xsb[a], bufs[a],
                                    self.outdeg, bufs[b], local_out(xsb[b]), self.delta2, self.damping,
                                    self.teleport, self.n_global, ctrl=ctrl, eps2=eps2, comm=comm, xs_all=xsb[b],
-                                   slice_len=Ls)
+                                   slice_len=Ls, slice_counts=counts)
                 k += 1
             c = ctrl.cpu()
             if int(c[0]):
@@ -307,7 +310,11 @@ class DistPageRank:
         return bufs[it % 2], it, float(self.delta2.item())
 
     def exchange_bytes_per_rank(self):
-        """Bytes each rank receives per iteration from the all-gather."""
+        """Bytes this rank receives per iteration: the other ranks' real entries with the
+        library exchange (all-gather-v) or the peer pushes, the padded slices with torch."""
+        if self.exchange_mode in ("acsr", "peer"):
+            counts = self.n_nd if self.compact else [int(c) for c in np.diff(self.splits)]
+            return 8 * (sum(counts) - counts[self.rank])
         return (self.world - 1) * self.Lx * 8
 
     def run(self, x0_local=None, eps=1e-6, max_iter=1000, check_every=None):

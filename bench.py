@@ -797,15 +797,17 @@ def _c4_variant(acsr, pdist, rp, ci, outdeg, n, nnz, K, dev, rank, world, comm):
         rec = {"ms_per_iter": round(ms, 4), "gteps": round(nnz / (ms * 1e-3) / 1e9, 2),
                "exchange_slice": pr.Lx, "exchange_bytes_in_per_rank_per_iter": pr.exchange_bytes_per_rank()}
         if ex == "acsr" and world > 1:
-            # T_comm: the same in-place all-gather alone (NCCL over NVLink), K times
+            # T_comm: the same exchange alone (all-gather-v of the real entries, NCCL over
+            # NVLink), K times
             buf = torch.zeros(world * pr.Lx, dtype=torch.float64, device=dev)
             mine = buf[rank * pr.Lx:(rank + 1) * pr.Lx]
-            pr.comm.allgather(mine, buf)
+            counts = pr.n_nd if pr.compact else [int(c) for c in np.diff(pr.splits)]
+            pr.comm.allgatherv(mine, buf, counts)
             torch.cuda.synchronize()
             c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             c0.record()
             for _ in range(K):
-                pr.comm.allgather(mine, buf)
+                pr.comm.allgatherv(mine, buf, counts)
             c1.record()
             torch.cuda.synchronize()
             rec["t_comm_ms"] = round(_max_over_ranks([c0.elapsed_time(c1) / K], dev, world)[0], 4)

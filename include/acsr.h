@@ -159,6 +159,10 @@ acsr_status acsr_comm_query(const acsr_comm *comm, int *nranks /* HOST out, null
  * exchange layout, handles) and for gathering a row-split SpMV's y slices. */
 acsr_status acsr_comm_allgather(acsr_comm *comm, const void *send, void *recv, size_t bytes_per_rank,
                                 cudaStream_t stream);
+/* All-gather-v: recv[q * stride_bytes ...] receives counts_bytes[q] bytes (HOST array) of rank
+ * q's send (one grouped ncclBroadcast per rank; bytes past a count are left untouched). */
+acsr_status acsr_comm_allgatherv(acsr_comm *comm, const void *send, void *recv, size_t stride_bytes,
+                                 const int64_t *counts_bytes, cudaStream_t stream);
 
 /* O8 row partition, on the device: splits[0] = 0, splits[nranks] = n_rows and
  *   splits[k] = min{ r : sum_{r' < r} cost(r') >= ceil(k * total / nranks) },

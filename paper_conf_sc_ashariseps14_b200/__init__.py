@@ -120,6 +120,8 @@ _lib.acsr_comm_query.argtypes = [_vp, ctypes.POINTER(ctypes.c_int), ctypes.POINT
 _lib.acsr_comm_query.restype = ctypes.c_int
 _lib.acsr_comm_allgather.argtypes = [_vp, _vp, _vp, _sz, _vp]
 _lib.acsr_comm_allgather.restype = ctypes.c_int
+_lib.acsr_comm_allgatherv.argtypes = [_vp, _vp, _vp, _sz, ctypes.POINTER(_i64), _vp]
+_lib.acsr_comm_allgatherv.restype = ctypes.c_int
 _lib.acsr_pagerank_init.argtypes = [ctypes.POINTER(PrArgs), _vp]
 _lib.acsr_pagerank_init.restype = ctypes.c_int
 _lib.acsr_partition_workspace_bytes.argtypes = [_i64]
@@ -152,7 +154,7 @@ EXPORTED = ("acsr_bin_workspace_bytes", "acsr_bin", "acsr_bin_ex", "acsr_spmv", 
             "acsr_peer_destroy", "acsr_peer_push", "acsr_peer_delta2", "acsr_peer_query", "acsr_peer_read_xs", "acsr_update_workspace_bytes", "acsr_update_edges", "acsr_update_edges_dev", "acsr_relayout",
             "acsr_hits_workspace_bytes", "acsr_hits_normalize", "acsr_hits_normalize_ctrl", "acsr_plan_status",
             "acsr_comm_get_unique_id", "acsr_comm_init", "acsr_comm_destroy", "acsr_comm_query",
-            "acsr_comm_allgather", "acsr_pagerank_init", "acsr_partition_workspace_bytes", "acsr_partition",
+            "acsr_comm_allgather", "acsr_comm_allgatherv", "acsr_pagerank_init", "acsr_partition_workspace_bytes", "acsr_partition",
             "acsr_relabel_workspace_bytes", "acsr_degree_relabel", "acsr_grow_workspace_bytes",
             "acsr_grow_layout", "acsr_exchange_layout_workspace_bytes", "acsr_exchange_layout",
             "acsr_permute_workspace_bytes", "acsr_permute_graph",
@@ -378,6 +380,17 @@ class AcsrComm:
                                         _dev(recv, None, "recv") if recv.numel() else None,
                                         send.numel() * send.element_size(), _stream(stream)),
                "acsr_comm_allgather")
+        return recv
+
+    def allgatherv(self, send, recv, counts, stream=None):
+        """recv viewed as nranks slices of recv.numel() // nranks elements; slice q receives
+        counts[q] elements of rank q's send (acsr_comm_allgatherv)."""
+        es = recv.element_size()
+        stride = recv.numel() // self.nranks * es
+        arr = (_i64 * self.nranks)(*[int(c) * es for c in counts])
+        _check(_lib.acsr_comm_allgatherv(self._c, _dev(send, None, "send") if send.numel() else None,
+                                         _dev(recv, None, "recv") if recv.numel() else None, stride, arr,
+                                         _stream(stream)), "acsr_comm_allgatherv")
         return recv
 
     def close(self):

@@ -172,6 +172,31 @@ extern "C" acsr_status acsr_comm_allgather(acsr_comm *c, const void *send, void 
     return acsr_check_launch("acsr_comm_allgather");
 }
 
+extern "C" acsr_status acsr_comm_allgatherv(acsr_comm *c, const void *send, void *recv, size_t stride_bytes,
+                                            const int64_t *counts_bytes, cudaStream_t stream)
+{
+    if (!c || !counts_bytes || (stride_bytes > 0 && !recv)) {
+        acsr_set_error("acsr_comm_allgatherv: invalid argument");
+        return ACSR_ERR_INVALID_VALUE;
+    }
+    for (int q = 0; q < c->nranks; q++)
+        if (counts_bytes[q] < 0 || (size_t)counts_bytes[q] > stride_bytes || (q == c->rank && counts_bytes[q] && !send)) {
+            acsr_set_error("acsr_comm_allgatherv: counts must lie in [0, stride_bytes]");
+            return ACSR_ERR_INVALID_VALUE;
+        }
+    ncclResult_t r = ncclGroupStart();
+    for (int q = 0; q < c->nranks && r == ncclSuccess; q++) {
+        char *dst = (char *)recv + (size_t)q * stride_bytes;
+        if (counts_bytes[q] > 0)
+            r = ncclBroadcast(q == c->rank ? send : (const void *)dst, dst, (size_t)counts_bytes[q], ncclUint8, q, c->nccl,
+                              stream);
+    }
+    const ncclResult_t r2 = ncclGroupEnd();
+    if (r != ncclSuccess) return nccl_fail("acsr_comm_allgatherv", r);
+    if (r2 != ncclSuccess) return nccl_fail("acsr_comm_allgatherv", r2);
+    return acsr_check_launch("acsr_comm_allgatherv");
+}
+
 // Called by acsr_pagerank_step after the fused step kernel (which wrote its Delta^2
 // partial to comm->d2[0..3)) when args->comm != NULL.
 uint64_t *acsr_comm_d2_slot(acsr_comm *c) { return c->d2; }

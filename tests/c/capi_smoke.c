@@ -166,6 +166,18 @@ int main(void)
     /* with comm, xs_all is required */
     c.xs_all = NULL;
     ok &= acsr_pagerank_step(&c, st) == ACSR_ERR_INVALID_VALUE;
+    /* all-gather-v with one rank: count 2 of a 3-double slice; the third entry untouched */
+    double hsend[3] = {1.5, -2.5, 9.0}, hrecv[3] = {0.0, 0.0, 7.0};
+    double *d_send, *d_recv;
+    CK(cudaMalloc((void **)&d_send, sizeof(hsend)));
+    CK(cudaMalloc((void **)&d_recv, sizeof(hrecv)));
+    CK(cudaMemcpy(d_send, hsend, sizeof(hsend), cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(d_recv, hrecv, sizeof(hrecv), cudaMemcpyHostToDevice));
+    const int64_t cnt_bytes[1] = {2 * sizeof(double)};
+    AK(acsr_comm_allgatherv(comm, d_send, d_recv, sizeof(hrecv), cnt_bytes, st));
+    CK(cudaStreamSynchronize(st));
+    CK(cudaMemcpy(hrecv, d_recv, sizeof(hrecv), cudaMemcpyDeviceToHost));
+    ok &= hrecv[0] == 1.5 && hrecv[1] == -2.5 && hrecv[2] == 7.0;
     AK(acsr_comm_destroy(comm));
 
     /* O8 partition on the device, and a valid plan reports ACSR_OK */

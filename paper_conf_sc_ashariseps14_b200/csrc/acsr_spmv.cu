@@ -80,6 +80,9 @@
 #ifndef ACSR_CLAIM_BATCH
 #define ACSR_CLAIM_BATCH 0  // > 0: CTA-batched unit claims of this many units (A/B)
 #endif
+#ifndef ACSR_PR_STREAM_HINTS
+#define ACSR_PR_STREAM_HINTS 0  // 1: evict-first hints for the PageRank epilogue's per-row vectors (A/B)
+#endif
 #ifndef ACSR_VEC_MIN
 #define ACSR_VEC_MIN 512  // rows (chunks) shorter than this use the lane-strided scalar path
 #endif
@@ -450,8 +453,16 @@ struct Kern {
     {
         if (PR) {
             const double xn = a.teleport + a.damping * s + (r == a.restart ? a.restart_weight : 0.0);
+#if ACSR_PR_STREAM_HINTS
+            // x_new / x_old / outdeg are touched once per step: streaming (evict-first) so they
+            // do not push the hot xs lines out of L2; xs_next keeps the default policy (the next
+            // step gathers it)
+            __stcs(a.x_new + r, xn);
+            const int od = __ldcs(a.outdeg + r);
+#else
             a.x_new[r] = xn;
             const int od = __ldg(a.outdeg + r);
+#endif
             const double xs = od > 0 ? xn / (double)od : 0.0;
             if (a.xs_next) a.xs_next[r] = xs;  // NULL: peer exchange only
             // the exchange, fused: store the slice entry straight into every rank's
@@ -468,7 +479,11 @@ struct Kern {
                 d2.fin++;
                 d2.ftile = r / TILE_ROWS;
             }
+#if ACSR_PR_STREAM_HINTS
+            const double diff = xn - __ldcs(a.x_old + r);
+#else
             const double diff = xn - __ldg(a.x_old + r);
+#endif
             fix_add(d2, diff * diff);
         } else {
             a.y[r] = (V)s;

@@ -602,6 +602,7 @@ def run_pagerank(args, dev, rank, world):
     peak, kind = peaks()
     alg = 4 * nnz + 36 * n + 8 * n_nd
     ms = tot / K
+    traffic = ncu_traffic(f"pagerank_rmat{S}_inlink" + ("_degree_relabelled" if args.relabel else ""))
     return {"metric": "PageRank iteration GTEPS (in-link pattern SpMV + fused epilogue)",
             "value": round(nnz * world / (ms * 1e-3) / 1e9, 3), "unit": "GTEPS", "n_gpus": world, "steps": K,
             "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True, "scaling": "weak",
@@ -620,7 +621,11 @@ def run_pagerank(args, dev, rank, world):
                           "gflops_equiv": round(nnz / (ms * 1e-3) / 1e9, 2)},
             "roofline": {"bound": "hbm", "achieved": round(alg / (ms * 1e-3) / 1e9, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(alg / (ms * 1e-3) / 1e9 / peak, 4),
-                         "traffic": ncu_traffic(f"pagerank_rmat{S}_inlink" + ("_degree_relabelled" if args.relabel else "")),
+                         "traffic": traffic,
+                         "traffic_gbs_at_this_ms": None if not traffic else round(traffic / (ms * 1e-3) / 1e9, 1),
+                         "traffic_frac_of_peak": None if not traffic else round(traffic / (ms * 1e-3) / 1e9 / peak, 4),
+                         "traffic_note": "ncu DRAM bytes of one step (profiles/r2_ncu_c4_traffic.json): random xs misses "
+                                         "fetch a full DRAM burst per 8 used bytes",
                          "kernel": "acsr::spmv_kernel<PR>", "peak_kind": kind,
                          "algorithmic_bytes_per_launch": int(alg)},
             "gpu_launches": K, "clocks": clk.summary()}

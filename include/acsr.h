@@ -264,7 +264,8 @@ typedef struct {
                                    * exchanged (all-gather-v: one grouped ncclBroadcast per rank),
                                    * so unequal slices -- e.g. the non-dangling counts of a
                                    * degree-relabelled partition -- cost their sum, not
-                                   * nranks * max.  Entries past the counts are left untouched. */
+                                   * nranks * max.  Entries past the counts are left untouched.
+                                   * Must hold the same values on every rank. */
 } acsr_pr_args;
 
 acsr_status acsr_pagerank_step(const acsr_pr_args *args, cudaStream_t stream);

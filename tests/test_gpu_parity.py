@@ -998,6 +998,71 @@ def test_update_long_row_cta_path(acsr, cuda):
         assert torch.equal(a, b)
 
 
+def test_property_random_csr_spmv_and_updates(acsr, cuda):
+    """Property test (hypothesis, derandomized): random CSR shapes -- row lengths drawn from
+    a mixture that hits every mapping (empty, window, Alg. 2 / warp per row, split rows),
+    random columns, random n_cols, fp64 and fp32, integer and float values -- bins bitwise,
+    SpMV bitwise on integer data and at the O5 bar on float data; then a random insert /
+    delete batch on the slack copy, bitwise against O7."""
+    from hypothesis import given, settings, strategies as st, HealthCheck
+
+    @settings(max_examples=40, derandomize=True, deadline=None,
+              suppress_health_check=[HealthCheck.too_slow, HealthCheck.data_too_large])
+    @given(st.integers(1, 700), st.integers(1, 5000), st.integers(0, 2 ** 31 - 1), st.booleans(), st.booleans())
+    def check(n, n_cols, seed, f32, integer):
+        rng = np.random.default_rng(seed)
+        kind = rng.integers(0, 5, n)
+        ln = np.where(kind == 0, 0, np.where(kind == 1, rng.integers(1, 33, n),
+                      np.where(kind == 2, rng.integers(33, 1025, n),
+                               np.where(kind == 3, rng.integers(1025, 3000, n), rng.integers(1, 9, n)))))
+        ln = np.minimum(ln, 20000)
+        rp = np.zeros(n + 1, np.int64)
+        rp[1:] = np.cumsum(ln)
+        nnz = int(rp[-1])
+        ci = rng.integers(0, n_cols, nnz).astype(np.int32)
+        dt = np.float32 if f32 else np.float64
+        if integer:
+            val = rng.integers(-8, 9, nnz).astype(dt)
+            x = rng.integers(-8, 9, n_cols).astype(dt)
+        else:
+            val = rng.uniform(-1, 1, nnz).astype(dt)
+            x = rng.uniform(-1, 1, n_cols).astype(dt)
+        rpt = torch.from_numpy(rp.astype(np.int32))
+        m, y = run_csr(acsr, rpt, torch.from_numpy(ci), torch.from_numpy(val), torch.from_numpy(x), cuda)
+        br, off = oracle.bins(rp.astype(np.int32))
+        assert np.array_equal(m.bin_rows.cpu().numpy(), br) and np.array_equal(m.bin_offsets.cpu().numpy(), off)
+        y_ref, den = oracle.spmv(rp.astype(np.int32), ci, val, x)
+        check_spmv(y.numpy(), y_ref, den, torch.float32 if f32 else torch.float64, exact=integer)
+        # a random mixed update batch on the slack copy: O7 bitwise
+        rb, re, cap, c2, v2 = synth.with_slack(rpt, torch.from_numpy(ci), torch.from_numpy(val))
+        rows = np.unique(rng.integers(0, n, max(1, n // 4))).astype(np.int32)
+        dptr, dcol, iptr, icol = [0], [], [0], []
+        for r in rows:
+            cols_r = c2.numpy()[rb[r]:re[r]]
+            k = int(rng.integers(0, min(len(cols_r), 6) + 1))
+            dcol += sorted(rng.choice(cols_r, k, replace=False).tolist()) if k else []
+            dptr.append(len(dcol))
+            icol += rng.integers(0, n_cols, int(rng.integers(0, 5))).tolist()
+            iptr.append(len(icol))
+        ch = {"upd_rows": rows, "del_ptr": np.array(dptr, np.int32), "del_cols": np.array(dcol, np.int32),
+              "ins_ptr": np.array(iptr, np.int32), "ins_cols": np.array(icol, np.int32)}
+        iv = rng.uniform(-1, 1, len(icol)).astype(dt)
+        re_h, c_h, v_h = re.numpy().copy(), c2.numpy().copy(), v2.numpy().copy()
+        code, idx = oracle.update(n_cols, rb.numpy(), re_h, cap.numpy(), c_h, v_h, rows, ch["del_ptr"], ch["del_cols"],
+                                  ch["ins_ptr"], ch["ins_cols"], iv)
+        mu = acsr.ACSRMatrix(rb.to(cuda), c2.to(cuda), v2.to(cuda), n_cols=n_cols, row_end=re.to(cuda),
+                             row_cap=cap.to(cuda), nnz_max=c2.numel())
+        stt = mu.update({k: torch.from_numpy(v).to(cuda) for k, v in ch.items()}, ins_vals=torch.from_numpy(iv).to(cuda))
+        torch.cuda.synchronize()
+        assert stt.cpu().tolist() == [code, idx]
+        assert np.array_equal(mu.row_end.cpu().numpy(), re_h)
+        live = _live(rb.numpy(), re_h)
+        assert np.array_equal(mu.col_idx.cpu().numpy()[live], c_h[live])
+        assert np.array_equal(mu.values.cpu().numpy()[live].view(np.uint8), v_h[live].view(np.uint8))
+
+    check()
+
+
 def test_c_abi_from_plain_c(cuda):
     # the boundary is usable without Python: compile tests/c/capi_smoke.c against
     # include/acsr.h and libacsr.so and run it

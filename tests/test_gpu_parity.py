@@ -1006,7 +1006,7 @@ def test_property_random_csr_spmv_and_updates(acsr, cuda):
     delete batch on the slack copy, bitwise against O7."""
     from hypothesis import given, settings, strategies as st, HealthCheck
 
-    @settings(max_examples=40, derandomize=True, deadline=None,
+    @settings(max_examples=150, derandomize=True, deadline=None,
               suppress_health_check=[HealthCheck.too_slow, HealthCheck.data_too_large])
     @given(st.integers(1, 700), st.integers(1, 5000), st.integers(0, 2 ** 31 - 1), st.booleans(), st.booleans())
     def check(n, n_cols, seed, f32, integer):

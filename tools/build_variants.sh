@@ -69,6 +69,7 @@ for v in "$@"; do
     cb16w32u1) build cb16w32u1 -DACSR_CLAIM_BATCH=16 -DACSR_WIN_UNIT_ROWS=32 -DACSR_UNIT_SHIFT=-1 ;;
     w32) build w32 -DACSR_WIN_UNIT_ROWS=32 ;;
     prs) build prs -DACSR_PR_STREAM_HINTS=1 ;;
+    s1x1) build s1x1 -DACSR_STREAM_LD=1 -DACSR_X_LD=1 ;;
     rpl2) build rpl2 -DACSR_WIN_RPL=2 ;;
     rpl4) build rpl4 -DACSR_WIN_RPL=4 ;;
     rpl2g8) build rpl2g8 -DACSR_WIN_RPL=2 -DACSR_WIN_G=8 ;;

@@ -74,6 +74,9 @@
 #ifndef ACSR_WIN_DYN_SMEM
 #define ACSR_WIN_DYN_SMEM (ACSR_WIN_G > 4 || ACSR_WIN_RPL > 1)  // window scratch in dynamic shared memory
 #endif
+#ifndef ACSR_PF_START_TILES
+#define ACSR_PF_START_TILES 0  // > 0: L2 prefetch of the first tiles' CSR runs before the PDL wait only (A/B)
+#endif
 #ifndef ACSR_PF_TILES
 #define ACSR_PF_TILES 0  // > 0: stream-ahead L2 prefetch of the CSR (col/val) this many 1024-row tiles ahead (A/B)
 #endif
@@ -1162,6 +1165,20 @@ spmv_kernel(SpmvArgs<V> a)
             }
         }
     }
+#if ACSR_PF_START_TILES > 0
+    if (threadIdx.x < 32) {  // the CSR runs of the first tiles the warps will take, into L2, while the
+        // grid waits for the binning (PDL): start-up only, no prefetch inside the loop
+        for (int64_t t = blockIdx.x + threadIdx.x * (int64_t)gridDim.x; t < ACSR_PF_START_TILES;
+             t += 32 * (int64_t)gridDim.x) {
+            const int64_t t0 = t * TILE_ROWS;
+            if (t0 >= a.n_rows) break;
+            const int64_t t1 = t0 + TILE_ROWS < a.n_rows ? t0 + TILE_ROWS : a.n_rows;
+            const int pb = __ldg(a.rb + t0);
+            const int pe = HAS_END ? __ldg(a.re + t1 - 1) : __ldg(a.rb + t1);
+            if (pe > pb) K::pf_range(a, pb, pe);
+        }
+    }
+#endif
 #if ACSR_PF_TILES > 0
     if (threadIdx.x < 32) {  // tiles 0 .. ACSR_PF_TILES-1: one per CTA, grid-strided (before the PDL wait:
         // the CSR is not written by the preceding kernels; a prefetch is only a cache hint)

@@ -70,6 +70,8 @@ for v in "$@"; do
     w32) build w32 -DACSR_WIN_UNIT_ROWS=32 ;;
     prs) build prs -DACSR_PR_STREAM_HINTS=1 ;;
     s1x1) build s1x1 -DACSR_STREAM_LD=1 -DACSR_X_LD=1 ;;
+    pfs64) build pfs64 -DACSR_PF_START_TILES=64 ;;
+    pfs256) build pfs256 -DACSR_PF_START_TILES=256 ;;
     rpl2) build rpl2 -DACSR_WIN_RPL=2 ;;
     rpl4) build rpl4 -DACSR_WIN_RPL=4 ;;
     rpl2g8) build rpl2g8 -DACSR_WIN_RPL=2 -DACSR_WIN_G=8 ;;

@@ -1006,6 +1006,18 @@ def run_dynamic(args, dev, rank, world):
             torch.cuda.synchronize()
             regrow += 1
         relayouts += regrow
+        # re-bin + scale + SpMV of the updated graph back to back, events at the ends only
+        # (the PDL overlap the phase events above break; re-binning the same graph and the
+        # SpMV are idempotent): the per-update "bin + SpMV" as a caller runs it
+        torch.cuda._sleep(1_000_000)
+        j0, j1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        j0.record()
+        m.rebin()
+        acsr.acsr_pagerank_scale(x, outdeg, xs_tmp)
+        m.spmv(xs_tmp, y)
+        j1.record()
+        torch.cuda.synchronize()
+        t_joint = j0.elapsed_time(j1)
         # host-inclusive: the same update + re-bin + SpMV issued from an idle GPU (a
         # re-applied insert batch only appends duplicates, so time it on a scratch copy)
         t_host = host_inclusive_batch(m, pinned, outdeg, st, uws, x, xs_tmp, y) if b >= args.warmup else 0.0
@@ -1014,7 +1026,7 @@ def run_dynamic(args, dev, rank, world):
         torch.cuda.synchronize()
         t_pr = time.perf_counter() - t0
         if b >= args.warmup:
-            rec.append([ev[i].elapsed_time(ev[i + 1]) for i in range(4)] + [t_pr * 1e3, it, k, t_host])
+            rec.append([ev[i].elapsed_time(ev[i + 1]) for i in range(4)] + [t_pr * 1e3, it, k, t_host, t_joint])
     # the same per-batch sequence (update -> re-bin -> scale -> SpMV) from ONE captured CUDA
     # graph (acsr_update_edges_dev reads the batch size on the device), host-inclusive:
     # sync -> pinned copies into the graph's capacity buffers + replay -> sync
@@ -1054,13 +1066,17 @@ def run_dynamic(args, dev, rank, world):
     t_h2d, t_upd, t_bin, t_spmv = (float(r[:, i].mean()) for i in range(4))
     peak, kind = peaks()
     label_dyn = f"dynamic_rmat{S}_inlink_16384_insert_batches"
-    return {"metric": "bin+SpMV ms per dynamic-graph update (C5)", "value": round(t_bin + t_spmv, 5),
+    t_joint = float(r[:, 8].mean())
+    return {"metric": "bin+SpMV ms per dynamic-graph update (C5)", "value": round(t_joint, 5),
             "unit": "ms", "n_gpus": world, "steps": len(rec), "warmup": args.warmup,
             "ms_per_step": round(t_h2d + t_upd + t_bin + t_spmv, 5), "higher_is_better": False,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"dynamic_rmat{S}_inlink_16384_insert_batches", "n_rows": n,
                        "batches_timed": len(rec), "cold_iterations": it0},
-            "breakdown": {"t_h2d_ms": round(t_h2d, 5), "t_update_ms": round(t_upd, 5), "t_bin_ms": round(t_bin, 5),
+            "breakdown": {"value_timing": "re-bin + scale + SpMV of each updated graph back to back (events at the "
+                                          "ends only); phases below from a separate, event-split pass",
+                          "t_bin_plus_spmv_split_ms": round(t_bin + t_spmv, 5),
+                          "t_h2d_ms": round(t_h2d, 5), "t_update_ms": round(t_upd, 5), "t_bin_ms": round(t_bin, 5),
                           "t_spmv_ms": round(t_spmv, 5), "bin_lt_spmv": bool(t_bin < t_spmv),
                           "pt_st": round(t_bin / t_spmv, 3),
                           "rebuild_plus_spmv_ms": round(t_upd + t_bin + t_spmv, 5),

@@ -643,6 +643,8 @@ def run_pagerank(args, dev, rank, world):
                          "traffic_frac_of_peak": None if not traffic else round(traffic / (ms * 1e-3) / 1e9 / peak, 4),
                          "traffic_note": "ncu DRAM bytes of one step (profiles/r2_ncu_c4_traffic.json): random xs misses "
                                          "fetch a full DRAM burst per 8 used bytes",
+                         "vs_other_peaks": {"spec_gbs": HBM_SPEC_GBS,
+                                            "frac_vs_spec": round(alg / (ms * 1e-3) / 1e9 / HBM_SPEC_GBS, 4)},
                          "kernel": "acsr::spmv_kernel<PR>", "peak_kind": kind,
                          "algorithmic_bytes_per_launch": int(alg)},
             "gpu_launches": K, "clocks": clk.summary()}
@@ -1098,7 +1100,9 @@ def run_dynamic(args, dev, rank, world):
                          "unit": "GB/s", "frac": round(alg_spmv / (t_spmv * 1e-3) / 1e9 / peak, 4),
                          "traffic": ncu_traffic(label_dyn), "kernel": "acsr::spmv_kernel (pattern, slack CSR)",
                          "peak_kind": kind, "algorithmic_bytes_per_launch": int(alg_spmv),
-                         "note": "4 nnz + 12 n + 8 n_c + 8 n after the last batch"},
+                         "note": "4 nnz + 12 n + 8 n_c + 8 n after the last batch",
+                         "vs_other_peaks": {"spec_gbs": HBM_SPEC_GBS,
+                                            "frac_vs_spec": round(alg_spmv / (t_spmv * 1e-3) / 1e9 / HBM_SPEC_GBS, 4)}},
             # per timed batch: update_init + update_validate + update_apply (insert-only),
             # bin_count + bin_scan + bin_scatter, pagerank_scale + spmv_kernel
             "gpu_launches": 8 * len(rec)}

@@ -83,6 +83,12 @@
 #ifndef ACSR_CLAIM_BATCH
 #define ACSR_CLAIM_BATCH 0  // > 0: CTA-batched unit claims of this many units (A/B)
 #endif
+#ifndef ACSR_DESC_AHEAD
+#define ACSR_DESC_AHEAD 0  // 1: claim two units ahead, load the next unit's descriptor during this one (A/B)
+#endif
+#ifndef ACSR_CLAIM_LATE
+#define ACSR_CLAIM_LATE 1  // 1: claim the next unit when this one ends (r2af: C2 -3 %); 0: one prefetched claim; 2: prefetched until the last round
+#endif
 #ifndef ACSR_PR_STREAM_HINTS
 #define ACSR_PR_STREAM_HINTS 0  // 1: evict-first hints for the PageRank epilogue's per-row vectors (A/B)
 #endif
@@ -1075,7 +1081,11 @@ struct Kern {
 
     static __device__ __forceinline__ void unit(const A &a, int u, int lane, Fix192 &d2, double *wbuf, int2 *wtab)
     {
-        const int2 d = __ldg(a.units + u);
+        unit_d(a, u, __ldg(a.units + u), lane, d2, wbuf, wtab);
+    }
+    static __device__ __forceinline__ void unit_d(const A &a, int u, const int2 d, int lane, Fix192 &d2, double *wbuf,
+                                                  int2 *wtab)
+    {
         const uint32_t y = (uint32_t)d.y;
 #if ACSR_MERGED_WARP_PATH
         if ((y & HEAVY_FLAG) || (!(y & WIN_FLAG) && (int)(y >> 24) > 6)) {
@@ -1292,6 +1302,10 @@ spmv_kernel(SpmvArgs<V> a)
     __shared__ int s_claim;
 #if ACSR_CLAIM_BATCH > 0
     if (threadIdx.x == 0) s_claim = SPMV_WARPS * atomicAdd(&hdr->work_ctr, 1);  // this CTA's batch 0
+#elif ACSR_CLAIM_LATE
+    // prefetched first claims only while more than one round of units remains after them
+    const bool cta_ahead = ACSR_CLAIM_LATE == 2 && 2 * nw < n_units;
+    if (threadIdx.x == 0) s_claim = cta_ahead ? atomicAdd(&hdr->work_ctr, SPMV_WARPS) : 0;
 #else
     if (threadIdx.x == 0) s_claim = atomicAdd(&hdr->work_ctr, SPMV_WARPS);
 #endif
@@ -1335,6 +1349,44 @@ spmv_kernel(SpmvArgs<V> a)
     };
     if (lane == 0) nxt = claim();
 #endif
+#if ACSR_CLAIM_LATE && ACSR_CLAIM_BATCH == 0 && !ACSR_DESC_AHEAD && !ACSR_PROF
+    // late claims: a prefetched claim parks a unit on a busy warp, which with ~1-2 units
+    // per warp (C3a) leaves other warps idle at the end.  Mode 1 claims every unit only
+    // when the warp is free; mode 2 keeps prefetched claims while more than one round of
+    // units remains and claims late in the last round.
+    bool have = cta_ahead;
+    while (u < n_units) {
+        K::unit(a, u, lane, d2, wbuf, wtab);
+        if (tile_push) K::peer_tile_done(a, lane, d2);
+        if (!have && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
+        u = __shfl_sync(0xffffffffu, nxt, 0) + nw;
+        have = ACSR_CLAIM_LATE == 2 && u + nw < n_units;
+        if (have && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
+    }
+#elif ACSR_DESC_AHEAD && ACSR_CLAIM_BATCH == 0 && !ACSR_PROF
+    // two units in hand: the current one (descriptor loaded) and the next one, whose
+    // descriptor load is in flight while the current unit runs; the claim for the one
+    // after is outstanding as well -- no dependent round trip between units
+    int un = s_claim + (threadIdx.x >> 5) + nw;
+    int2 dc = make_int2(0, 0), dn = make_int2(0, 0);
+    if (u < n_units) dc = __ldg(a.units + u);
+    if (un < n_units) {
+        dn = __ldg(a.units + un);
+        if (lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
+    }
+    while (u < n_units) {
+        K::unit_d(a, u, dc, lane, d2, wbuf, wtab);
+        if (tile_push) K::peer_tile_done(a, lane, d2);
+        u = un;
+        dc = dn;
+        if (u >= n_units) break;
+        un = __shfl_sync(0xffffffffu, nxt, 0) + nw;
+        if (un < n_units) {
+            dn = __ldg(a.units + un);
+            if (lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
+        }
+    }
+#else
     while (u < n_units) {
 #if ACSR_PROF
         const long long tu = clock64();
@@ -1361,6 +1413,7 @@ spmv_kernel(SpmvArgs<V> a)
         if (u < n_units && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
 #endif
     }
+#endif  // ACSR_DESC_AHEAD
 #if ACSR_PROF
     if (t_last == 0) t_last = clock64();
 #endif

@@ -76,6 +76,22 @@ for v in "$@"; do
     rpl4) build rpl4 -DACSR_WIN_RPL=4 ;;
     rpl2g8) build rpl2g8 -DACSR_WIN_RPL=2 -DACSR_WIN_G=8 ;;
     rpl4g8) build rpl4g8 -DACSR_WIN_RPL=4 -DACSR_WIN_G=8 ;;
+    da) build da -DACSR_DESC_AHEAD=1 ;;
+    daw32) build daw32 -DACSR_DESC_AHEAD=1 -DACSR_WIN_UNIT_ROWS=32 ;;
+    daw64) build daw64 -DACSR_DESC_AHEAD=1 -DACSR_WIN_UNIT_ROWS=64 ;;
+    dawp) build dawp -DACSR_DESC_AHEAD=1 -DACSR_WIN_PREFETCH=1 ;;
+    daw32wp) build daw32wp -DACSR_DESC_AHEAD=1 -DACSR_WIN_UNIT_ROWS=32 -DACSR_WIN_PREFETCH=1 ;;
+    cl1) build cl1 -DACSR_CLAIM_LATE=1 ;;
+    cl2) build cl2 -DACSR_CLAIM_LATE=2 ;;
+    cl1w32) build cl1w32 -DACSR_CLAIM_LATE=1 -DACSR_WIN_UNIT_ROWS=32 ;;
+    cl2w32) build cl2w32 -DACSR_CLAIM_LATE=2 -DACSR_WIN_UNIT_ROWS=32 ;;
+    cl2w64) build cl2w64 -DACSR_CLAIM_LATE=2 -DACSR_WIN_UNIT_ROWS=64 ;;
+    cl2um1) build cl2um1 -DACSR_CLAIM_LATE=2 -DACSR_UNIT_SHIFT=-1 ;;
+    cl1um1) build cl1um1 -DACSR_CLAIM_LATE=1 -DACSR_UNIT_SHIFT=-1 ;;
+    cl1w64) build cl1w64 -DACSR_CLAIM_LATE=1 -DACSR_WIN_UNIT_ROWS=64 ;;
+    cl1u1) build cl1u1 -DACSR_CLAIM_LATE=1 -DACSR_UNIT_SHIFT=1 ;;
+    cl1w256) build cl1w256 -DACSR_CLAIM_LATE=1 -DACSR_WIN_UNIT_ROWS=256 ;;
+    cl2w256) build cl2w256 -DACSR_CLAIM_LATE=2 -DACSR_WIN_UNIT_ROWS=256 ;;
     noremote) build noremote -DACSR_DIAG=4 ;;
     noremote0) build noremote0 -DACSR_DIAG=4 -DACSR_PEER_TILE_PUSH=0 ;;
     pft32) build pft32 -DACSR_PF_TILES=32 ;;

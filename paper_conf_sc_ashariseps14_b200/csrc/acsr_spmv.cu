@@ -93,7 +93,7 @@
 #define ACSR_PR_STREAM_HINTS 0  // 1: evict-first hints for the PageRank epilogue's per-row vectors (A/B)
 #endif
 #ifndef ACSR_VEC_MIN
-#define ACSR_VEC_MIN 512  // rows (chunks) shorter than this use the lane-strided scalar path
+#define ACSR_VEC_MIN 1024  // rows (chunks) shorter than this use the lane-strided scalar path (r2ah: 512 -> 1024, C2 fp32 86.0 -> 84.0 us, others equal)
 #endif
 
 

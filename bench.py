@@ -51,6 +51,32 @@ def peaks():
     return FALLBACK_HBM, "fallback"
 
 
+class L2Flush:
+    """The L2 flush between timed steps: a 256 MiB write (larger than the 126 MB L2).
+    ACSR_BENCH_FLUSH=write+read adds a 256 MiB read of a second buffer after the write, so
+    the step starts with a clean L2 (the write leaves ~126 MB of dirty lines whose
+    write-back otherwise lands inside the next timed step).  Graph-capturable."""
+
+    def __init__(self, dev, mode=None):
+        self.mode = mode or os.environ.get("ACSR_BENCH_FLUSH", "write")
+        assert self.mode in ("write", "write+read"), self.mode
+        self.w = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+        if self.mode == "write+read":
+            self.r = torch.zeros(64 << 20, dtype=torch.int32, device=dev)
+            self.acc = torch.zeros((), dtype=torch.int64, device=dev)
+
+    def zero_(self):  # the name the call sites used for the plain write flush
+        self.w.zero_()
+        if self.mode == "write+read":
+            torch.sum(self.r, dim=0, dtype=torch.int64, out=self.acc)
+
+    @staticmethod
+    def describe(mode=None):
+        mode = mode or os.environ.get("ACSR_BENCH_FLUSH", "write")
+        return ("flushed: 256 MiB write" + (" + 256 MiB read (clean L2)" if mode == "write+read" else "")
+                + " between timed steps (outside the step events)")
+
+
 class Clocks:
     """Sample SM clocks + throttle reasons DURING the timed region.
 
@@ -244,7 +270,7 @@ def workload_config(label, n, nnz, world, replicas=False):
     """The `config` of the default line: identical keys and values at every N (and in the
     reference arm), so the driver can match the lines."""
     return {"workload": label, "n_rows": n, "nnz": nnz,
-            "l2": "flushed: 256 MiB write between timed steps (outside the step events)",
+            "l2": L2Flush.describe(),
             "parallelism": (f"independent matrix per rank x{world} (weak)" if replicas
                             else f"row-split x{world} (P:345)" if world > 1 else "1 GPU")}
 
@@ -292,7 +318,7 @@ def run_acsr(args, dev, rank, world):
     bo = torch.empty(33, dtype=torch.int32, device=dev)
     ws = torch.empty(acsr.acsr_bin_workspace_bytes(n, x.numel(), nnz), dtype=torch.uint8, device=dev)
     y = torch.empty(n, dtype=dtype, device=dev)
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    flush = L2Flush(dev)
 
     def step():
         acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=x.numel())
@@ -303,40 +329,72 @@ def run_acsr(args, dev, rank, world):
         step()
     torch.cuda.synchronize()
     K = args.steps
-    # the timed steps: acsr_bin + acsr_spmv back to back, as a caller issues them (events only
-    # at the step's ends: an event between the two calls would break the programmatic-
-    # dependent-launch overlap of the binning's last kernel with the SpMV's launch, measured
-    # +5.3 us per step, profiles/r2_step_events.json)
-    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(K)]
+    # the timed steps: acsr_bin + acsr_spmv back to back through the public calls, the K
+    # steps (each after its L2 flush) issued from ONE CUDA graph captured from those calls, so
+    # the device never waits for the Python host loop (issuing one call at a time from Python
+    # is ~180 us per step, slower than the GPU: the eager loop below is reported beside).
+    # Events only at the step's ends (graph event-record nodes): an event between the two
+    # calls would break the programmatic-dependent-launch overlap of the binning's last
+    # kernel with the SpMV's launch, measured +5.3 us per step (profiles/r2_step_events.json).
+    def graphed(n_ev, body):
+        evs = [[torch.cuda.Event(enable_timing=True, external=True) for _ in range(n_ev)] for _ in range(K)]
+        g = torch.cuda.CUDAGraph()
+        cap = torch.cuda.Stream()
+        cap.wait_stream(stream)
+        with torch.cuda.graph(g, stream=cap):
+            for k in range(K):
+                flush.zero_()
+                body(evs[k])
+        torch.cuda.synchronize()
+        return g, evs
+
+    def body_step(e):
+        e[0].record()
+        acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=x.numel())
+        acsr.acsr_spmv(rp, ci, val, x, br, bo, ws, None, y)
+        e[1].record()
+
+    def body_split(e):
+        e[0].record()
+        acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=x.numel())
+        e[1].record()
+        acsr.acsr_spmv(rp, ci, val, x, br, bo, ws, None, y)
+        e[2].record()
+
+    g_step, ev = graphed(2, body_step)
+    g_split, evb = graphed(3, body_split)
+    g_split.replay()  # warm replays (first replay uploads the graph)
+    g_step.replay()
+    torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
     torch.cuda.synchronize()
     with Clocks(torch.cuda.current_device()) as clk:
         t0 = time.perf_counter()
-        for k in range(K):
-            flush.zero_()
-            ev[k][0].record(stream)
-            acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=x.numel())
-            acsr.acsr_spmv(rp, ci, val, x, br, bo, ws, None, y)
-            ev[k][1].record(stream)
+        g_step.replay()
         torch.cuda.synchronize()
         wall = time.perf_counter() - t0
     if world > 1:
         torch.distributed.barrier()
     t_step = np.array([ev[k][0].elapsed_time(ev[k][1]) for k in range(K)])
-    # the breakdown (and the SpMV kernel's duration for the roofline): the same steps with an
-    # event between the calls, same flush protocol
-    evb = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(K)]
-    for k in range(K):
-        flush.zero_()
-        evb[k][0].record(stream)
-        acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=x.numel())
-        evb[k][1].record(stream)
-        acsr.acsr_spmv(rp, ci, val, x, br, bo, ws, None, y)
-        evb[k][2].record(stream)
+    # the breakdown (and the SpMV kernel's duration for the roofline): the same graphed steps
+    # with an event between the calls, same flush protocol
+    g_split.replay()
     torch.cuda.synchronize()
     t_bin = np.array([evb[k][0].elapsed_time(evb[k][1]) for k in range(K)])
     t_spmv = np.array([evb[k][1].elapsed_time(evb[k][2]) for k in range(K)])
+    # the same steps issued eagerly, one Python call at a time (host-bound: reported only)
+    eve = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(K)]
+    t1 = time.perf_counter()
+    for k in range(K):
+        flush.zero_()
+        eve[k][0].record(stream)
+        acsr.acsr_bin(rp, None, nnz, br, bo, ws, col_idx=ci, n_cols=x.numel())
+        acsr.acsr_spmv(rp, ci, val, x, br, bo, ws, None, y)
+        eve[k][1].record(stream)
+    torch.cuda.synchronize()
+    wall_eager = time.perf_counter() - t1
+    t_step_eager = float(np.mean([eve[k][0].elapsed_time(eve[k][1]) for k in range(K)]))
     # warm variant (SURVEY §8(d) timing protocol): K back-to-back SpMVs, no flush -- the
     # iterative-use number; reported beside the flushed (cold-L2) step, not as `value`
     torch.cuda.synchronize()
@@ -430,8 +488,12 @@ def run_acsr(args, dev, rank, world):
         "config": workload_config(label, n_glob, nnz_glob, world, replicas),
         "breakdown": {"rank0_rows": n, "rank0_nnz": nnz, "rank0_referenced_cols": n_c,
                       "splits": None if splits is None else [int(v) for v in splits],
-                      "timing": "value: events at the step's ends only (bin + SpMV back to back, PDL overlap); "
-                                "t_bin / t_spmv: a second loop with an event between the calls",
+                      "timing": "value: the K flushed steps issued from one CUDA graph captured from the public "
+                                "calls, events (graph event-record nodes) at the step's ends only (bin + SpMV back "
+                                "to back, PDL overlap); t_bin / t_spmv: a second graph with an event between the "
+                                "calls; t_step_eager: the same steps issued one Python call at a time (host-bound)",
+                      "t_step_eager_ms": round(t_step_eager, 5),
+                      "wall_s_eager_loop": round(wall_eager, 4),
                       "t_bin_plus_spmv_split_ms": round(float((t_bin + t_spmv).mean()), 5),
                       "t_bin_ms": round(float(t_bin.mean()), 5), "t_spmv_ms": round(spmv_ms, 5),
                       "pt_st": round(float(t_bin.mean()) / spmv_ms, 3),

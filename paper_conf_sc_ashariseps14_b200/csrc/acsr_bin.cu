@@ -84,15 +84,19 @@ __device__ __forceinline__ void count_tile(BinSmem &sm, int64_t n, const int32_t
     for (int o = 16; o > 0; o >>= 1) my_heavy += __shfl_xor_sync(0xffffffffu, my_heavy, o);
     if ((tid & 31) == 0 && my_heavy) atomicAdd(&sm.heavy, my_heavy);
     __syncthreads();
-    if (tid < NBINS) cnt[(int64_t)tid * n_tiles + tile] = sm.hist[tid];
-    if (tid == NBINS) {
-        int lu = 0;
+    if (tid < 32) {  // warp 0: the tile's row of counts; light units one bin per lane, summed
+        static_assert(NBINS == 32, "one lane per bin");
+        const int h = sm.hist[tid];
+        cnt[(int64_t)tid * n_tiles + tile] = h;
         const bool tl = tail_tile(tile, n_tiles);
-#pragma unroll
-        for (int b = wmb + 1; b <= LIGHT_MAX_BIN; b++) lu += (sm.hist[b] + unit_rows_t(b, tl) - 1) / unit_rows_t(b, tl);
-        if (wmb >= 0) lu += win_units_t((int)min((int64_t)TILE_ROWS, n - base), tl);
-        cnt[(int64_t)NBINS * n_tiles + tile] = lu;
-        cnt[(int64_t)(NBINS + 1) * n_tiles + tile] = sm.heavy;
+        int lu = 0;
+        if (tid > wmb && tid <= LIGHT_MAX_BIN) lu = (h + unit_rows_t(tid, tl) - 1) / unit_rows_t(tid, tl);
+        lu = __reduce_add_sync(0xffffffffu, lu);
+        if (tid == 0) {
+            if (wmb >= 0) lu += win_units_t((int)min((int64_t)TILE_ROWS, n - base), tl);
+            cnt[(int64_t)NBINS * n_tiles + tile] = lu;
+            cnt[(int64_t)(NBINS + 1) * n_tiles + tile] = sm.heavy;
+        }
     }
     __syncthreads();
 }
@@ -403,7 +407,7 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, const ScatterPre &pre,
 
 // ---- three-launch path (used when a cooperative launch is not possible)
 template <bool HAS_END>
-__global__ void __launch_bounds__(BIN_THREADS)
+__global__ void __launch_bounds__(BIN_THREADS, 2048 / BIN_THREADS)
 bin_count_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
                  int32_t *__restrict__ cnt, int n_tiles, PlanHeader *hdr, int wmb)
 {
@@ -433,7 +437,7 @@ bin_scan_kernel(const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int
 }
 
 template <bool HAS_END>
-__global__ void __launch_bounds__(BIN_THREADS)
+__global__ void __launch_bounds__(BIN_THREADS, 2048 / BIN_THREADS)
 bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
                    int32_t *__restrict__ bin_rows, const int32_t *__restrict__ toff, int n_tiles,
                    PlanHeader *hdr, int2 *__restrict__ units, int32_t *__restrict__ tickets, ScanArgs sa,
@@ -457,7 +461,7 @@ bin_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__r
 // first tickets), so the wait cannot deadlock.  Saves the scan kernel's launch boundary
 // but measured slower (see scan_scatter_fused).
 template <bool HAS_END>
-__global__ void __launch_bounds__(BIN_THREADS)
+__global__ void __launch_bounds__(BIN_THREADS, 2048 / BIN_THREADS)
 bin_scan_scatter_kernel(int64_t n, const int32_t *__restrict__ rb, const int32_t *__restrict__ re,
                         const int32_t *__restrict__ cnt, int32_t *__restrict__ toff, int32_t *__restrict__ bin_rows,
                         int n_tiles, PlanHeader *hdr, ScanArgs sa, int2 *__restrict__ units,
@@ -511,7 +515,7 @@ struct FusedArgs {
 };
 
 template <bool HAS_END>
-__global__ void __launch_bounds__(BIN_THREADS)
+__global__ void __launch_bounds__(BIN_THREADS, 2048 / BIN_THREADS)
 bin_fused_kernel(FusedArgs f)
 {
     __shared__ BinSmem sm;

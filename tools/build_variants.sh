@@ -94,6 +94,8 @@ for v in "$@"; do
     t256mb4) build t256mb4 -DACSR_SPMV_THREADS=256 -DACSR_MIN_BLOCKS=4 ;;
     v768) build v768 -DACSR_VEC_MIN=768 ;;
     v2048) build v2048 -DACSR_VEC_MIN=2048 ;;
+    cl0) build cl0 -DACSR_CLAIM_LATE=0 ;;
+    cl0v512) build cl0v512 -DACSR_CLAIM_LATE=0 -DACSR_VEC_MIN=512 ;;
     cl2w256) build cl2w256 -DACSR_CLAIM_LATE=2 -DACSR_WIN_UNIT_ROWS=256 ;;
     noremote) build noremote -DACSR_DIAG=4 ;;
     noremote0) build noremote0 -DACSR_DIAG=4 -DACSR_PEER_TILE_PUSH=0 ;;

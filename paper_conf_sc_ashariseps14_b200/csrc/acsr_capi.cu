@@ -36,6 +36,31 @@ bool acsr::acsr_pdl_enabled()
     return v == 1;
 }
 
+// ACSR_CARVEOUT=<percent> (A/B knob, default unset): the preferred shared-memory carveout
+// given to every kernel launched through launch_pdl, so consecutive kernels of a call
+// chain (binning -> SpMV) can share one L1/shared split instead of the SM reconfiguring
+// between them.
+int acsr::acsr_carveout()
+{
+    static int v = -2;
+    if (v == -2) {
+        const char *e = getenv("ACSR_CARVEOUT");
+        v = (e && e[0]) ? atoi(e) : -1;
+        if (v > 100) v = 100;
+    }
+    return v;
+}
+
+bool acsr::acsr_carveout_once(const void *fn)
+{
+    static const void *seen[128];
+    static int n = 0;
+    for (int i = 0; i < n; i++)
+        if (seen[i] == fn) return false;
+    if (n < 128) seen[n++] = fn;
+    return true;
+}
+
 int acsr_num_sms()
 {
     static int sms[64] = {0};

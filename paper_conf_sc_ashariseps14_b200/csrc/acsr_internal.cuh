@@ -377,11 +377,16 @@ __device__ __forceinline__ void pdl_enter()
 }
 
 bool acsr_pdl_enabled();
+int acsr_carveout();
+bool acsr_carveout_once(const void *fn);
 
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t stream,
                               Args... args)
 {
+    const int co = acsr_carveout();
+    if (co >= 0 && acsr_carveout_once((const void *)kernel))
+        cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout, co);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = grid;
     cfg.blockDim = block;

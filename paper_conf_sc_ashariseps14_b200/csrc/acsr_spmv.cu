@@ -68,6 +68,9 @@
 #ifndef ACSR_PROF
 #define ACSR_PROF 0  // diagnostics: per-mapping warp-cycle counters (acsr_debug_prof, A/B builds only)
 #endif
+#ifndef ACSR_TIMELINE
+#define ACSR_TIMELINE 0  // diagnostics: per-unit start/end cycles + SM id (acsr_debug_timeline, A/B builds only)
+#endif
 #ifndef ACSR_WIN_RPL
 #define ACSR_WIN_RPL 1  // short-row window rows per lane (window = 32 * RPL consecutive rows)
 #endif
@@ -393,6 +396,27 @@ __device__ __forceinline__ bool cb_valid(int cb, int T) { return cb < T; }
 // [15] launches
 __device__ unsigned long long g_prof[16];
 #define PROF_ADD(i, v) atomicAdd(&g_prof[i], (unsigned long long)(v))
+#endif
+
+#if ACSR_TIMELINE
+// per unit u < TL_MAX: {start, end} in SM cycles since the CTA's entry, packed with the SM id
+// (bits 48..55) and the unit kind (bits 56..59); g_tl_cta[b] = {globaltimer at CTA entry, clock64
+// at entry, globaltimer at the CTA's exit}
+constexpr int TL_MAX = 1 << 16;
+__device__ unsigned long long g_tl[TL_MAX][2];
+__device__ unsigned long long g_tl_cta[1024][3];
+__device__ __forceinline__ unsigned long long gtimer()
+{
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+__device__ __forceinline__ unsigned smid()
+{
+    unsigned r;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+    return r;
+}
 #endif
 
 // xs' slice entry -> every OTHER rank's replicated buffer (byte offset o in each region)
@@ -1202,6 +1226,13 @@ spmv_kernel(SpmvArgs<V> a)
         }
     }
 #endif
+#if ACSR_TIMELINE
+    const long long tl_c0 = clock64();
+    if (threadIdx.x == 0 && blockIdx.x < 1024) {
+        g_tl_cta[blockIdx.x][0] = gtimer();
+        g_tl_cta[blockIdx.x][1] = (unsigned long long)tl_c0;
+    }
+#endif
     pdl_enter();
     if (PR && a.ctrl && *(volatile int32_t *)a.ctrl) return;  // converged earlier: no-op step
     unsigned long long pc = 0;  // peer exchange: pushes completed before this step
@@ -1356,7 +1387,21 @@ spmv_kernel(SpmvArgs<V> a)
     // units remains and claims late in the last round.
     bool have = cta_ahead;
     while (u < n_units) {
+#if ACSR_TIMELINE
+        const long long tl_s = clock64() - tl_c0;
+        const uint32_t tl_ty = (uint32_t)__ldg(a.units + u).y;
+        const unsigned long long tl_kind =
+            (tl_ty & HEAVY_FLAG) ? 3 : (tl_ty & WIN_FLAG) ? 0 : ((tl_ty >> 24) == 0 ? 4 : ((tl_ty >> 24) <= 6 ? 1 : 2));
+#endif
         K::unit(a, u, lane, d2, wbuf, wtab);
+#if ACSR_TIMELINE
+        __syncwarp();
+        if (lane == 0 && u < TL_MAX) {
+            const unsigned long long tag = ((unsigned long long)smid() << 48) | (tl_kind << 56);
+            g_tl[u][0] = (unsigned long long)tl_s | tag;
+            g_tl[u][1] = (unsigned long long)(clock64() - tl_c0) | tag;
+        }
+#endif
         if (tile_push) K::peer_tile_done(a, lane, d2);
         if (!have && lane == 0) nxt = atomicAdd(&hdr->work_ctr, 1);
         u = __shfl_sync(0xffffffffu, nxt, 0) + nw;
@@ -1439,6 +1484,9 @@ spmv_kernel(SpmvArgs<V> a)
 #if ACSR_PROF
     if (lane == 0) PROF_ADD(9, clock64() - t_last);
     if (threadIdx.x == 0 && blockIdx.x == 0) PROF_ADD(15, 1);
+#endif
+#if ACSR_TIMELINE
+    if (threadIdx.x == 0 && blockIdx.x < 1024) g_tl_cta[blockIdx.x][2] = gtimer();
 #endif
     if (threadIdx.x >= 32) return;
     if (PR) {
@@ -1872,6 +1920,19 @@ extern "C" acsr_status acsr_plan_status(const void *plan_ws, size_t plan_ws_byte
     }
     return ACSR_OK;
 }
+
+#if ACSR_TIMELINE
+// copies {g_tl (TL_MAX x 2), g_tl_cta (1024 x 3)} to out (TL_MAX*2 + 3072 words), then zeroes them
+extern "C" int acsr_debug_timeline(unsigned long long *out)
+{
+    cudaDeviceSynchronize();
+    cudaMemcpyFromSymbol(out, acsr::g_tl, sizeof(acsr::g_tl));
+    cudaMemcpyFromSymbol(out + 2 * acsr::TL_MAX, acsr::g_tl_cta, sizeof(acsr::g_tl_cta));
+    static unsigned long long z[acsr::TL_MAX][2];
+    cudaMemcpyToSymbol(acsr::g_tl, z, sizeof(z));
+    return acsr::TL_MAX;
+}
+#endif
 
 #if ACSR_PROF
 extern "C" int acsr_debug_prof(unsigned long long *out16, int reset)

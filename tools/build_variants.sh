@@ -63,6 +63,7 @@ for v in "$@"; do
     diag1) build diag1 -DACSR_DIAG=1 ;;
     sum1) build sum1 -DACSR_WIN_SUM4=0 ;;
     prof) build prof -DACSR_PROF=1 ;;
+    tl) build tl -DACSR_TIMELINE=1 ;;
     cb16) build cb16 -DACSR_CLAIM_BATCH=16 ;;
     cb16w32) build cb16w32 -DACSR_CLAIM_BATCH=16 -DACSR_WIN_UNIT_ROWS=32 ;;
     cb32w32) build cb32w32 -DACSR_CLAIM_BATCH=32 -DACSR_WIN_UNIT_ROWS=32 ;;

@@ -68,6 +68,12 @@
 #ifndef ACSR_PROF
 #define ACSR_PROF 0  // diagnostics: per-mapping warp-cycle counters (acsr_debug_prof, A/B builds only)
 #endif
+#ifndef ACSR_CLAIM_GUIDED
+#define ACSR_CLAIM_GUIDED 0  // > 0: guided batches of consecutive units per claim, k = left / (F * warps) (A/B)
+#endif
+#ifndef ACSR_GUIDED_AHEAD
+#define ACSR_GUIDED_AHEAD 1  // guided batches: claim the next batch when the last unit of this one starts
+#endif
 #ifndef ACSR_TIMELINE
 #define ACSR_TIMELINE 0  // diagnostics: per-unit start/end cycles + SM id (acsr_debug_timeline, A/B builds only)
 #endif
@@ -1380,7 +1386,65 @@ spmv_kernel(SpmvArgs<V> a)
     };
     if (lane == 0) nxt = claim();
 #endif
-#if ACSR_CLAIM_LATE && ACSR_CLAIM_BATCH == 0 && !ACSR_DESC_AHEAD && !ACSR_PROF
+#if ACSR_CLAIM_GUIDED > 0 && ACSR_CLAIM_BATCH == 0 && !ACSR_DESC_AHEAD && !ACSR_PROF
+    // guided batches: a warp takes k consecutive units per claim, k = (units left) /
+    // (ACSR_CLAIM_GUIDED * warps) clamped to [1, 32] -- large batches while much work
+    // remains, single units at the end (the tail is one short unit, not one long one).
+    // The batch's descriptors arrive in ONE coalesced load (no dependent descriptor
+    // round trip per unit) and the claim for the next batch is issued when the batch's
+    // last unit starts (ACSR_GUIDED_AHEAD) or when it ends.  Round 0 is static: warp w
+    // takes units [w k0, (w+1) k0); claims hand out units from nw k0 on.
+    {
+        constexpr int F = ACSR_CLAIM_GUIDED;
+        auto batch = [&](int left) -> int {
+            const int k = left / (F * nw);
+            return k < 1 ? 1 : (k > 32 ? 32 : k);
+        };
+        const int k0 = batch(n_units);
+        const int S = nw * k0;
+        int base = gw * k0;
+        int cnt = base < n_units ? min(k0, n_units - base) : 0;
+        int seen = 0;  // the counter's value at this warp's last claim
+        while (cnt > 0) {
+            const int2 dl = lane < cnt ? __ldg(a.units + base + lane) : make_int2(0, 0);
+            int nb = 0, k = 1;
+            for (int i = 0; i < cnt; i++) {
+                const bool last = i == cnt - 1;
+                if (last && ACSR_GUIDED_AHEAD) {
+                    k = batch(n_units - S - seen);
+                    if (lane == 0) nb = atomicAdd(&hdr->work_ctr, k);
+                }
+                int2 d;
+                d.x = __shfl_sync(0xffffffffu, dl.x, i);
+                d.y = __shfl_sync(0xffffffffu, dl.y, i);
+#if ACSR_TIMELINE
+                const long long tl_s = clock64() - tl_c0;
+                const uint32_t tl_ty = (uint32_t)d.y;
+                const unsigned long long tl_kind =
+                    (tl_ty & HEAVY_FLAG) ? 3 : (tl_ty & WIN_FLAG) ? 0 : ((tl_ty >> 24) == 0 ? 4 : ((tl_ty >> 24) <= 6 ? 1 : 2));
+#endif
+                K::unit_d(a, base + i, d, lane, d2, wbuf, wtab);
+#if ACSR_TIMELINE
+                __syncwarp();
+                if (lane == 0 && base + i < TL_MAX) {
+                    const unsigned long long tag = ((unsigned long long)smid() << 48) | (tl_kind << 56);
+                    g_tl[base + i][0] = (unsigned long long)tl_s | tag;
+                    g_tl[base + i][1] = (unsigned long long)(clock64() - tl_c0) | tag;
+                }
+#endif
+                if (tile_push) K::peer_tile_done(a, lane, d2);
+            }
+            if (!ACSR_GUIDED_AHEAD) {
+                k = batch(n_units - S - seen);
+                if (lane == 0) nb = atomicAdd(&hdr->work_ctr, k);
+            }
+            seen = __shfl_sync(0xffffffffu, nb, 0);
+            base = S + seen;
+            cnt = base < n_units ? min(k, n_units - base) : 0;
+            seen += k;
+        }
+    }
+#elif ACSR_CLAIM_LATE && ACSR_CLAIM_BATCH == 0 && !ACSR_DESC_AHEAD && !ACSR_PROF
     // late claims: a prefetched claim parks a unit on a busy warp, which with ~1-2 units
     // per warp (C3a) leaves other warps idle at the end.  Mode 1 claims every unit only
     // when the warp is free; mode 2 keeps prefetched claims while more than one round of

@@ -64,6 +64,14 @@ for v in "$@"; do
     sum1) build sum1 -DACSR_WIN_SUM4=0 ;;
     prof) build prof -DACSR_PROF=1 ;;
     tl) build tl -DACSR_TIMELINE=1 ;;
+    g2) build g2 -DACSR_CLAIM_GUIDED=2 ;;
+    g2w32) build g2w32 -DACSR_CLAIM_GUIDED=2 -DACSR_WIN_UNIT_ROWS=32 ;;
+    g2w64) build g2w64 -DACSR_CLAIM_GUIDED=2 -DACSR_WIN_UNIT_ROWS=64 ;;
+    g1w32) build g1w32 -DACSR_CLAIM_GUIDED=1 -DACSR_WIN_UNIT_ROWS=32 ;;
+    g4w32) build g4w32 -DACSR_CLAIM_GUIDED=4 -DACSR_WIN_UNIT_ROWS=32 ;;
+    g2w32na) build g2w32na -DACSR_CLAIM_GUIDED=2 -DACSR_WIN_UNIT_ROWS=32 -DACSR_GUIDED_AHEAD=0 ;;
+    g2w32u) build g2w32u -DACSR_CLAIM_GUIDED=2 -DACSR_WIN_UNIT_ROWS=32 -DACSR_UNIT_SHIFT=-1 ;;
+    tlg2w32) build tlg2w32 -DACSR_TIMELINE=1 -DACSR_CLAIM_GUIDED=2 -DACSR_WIN_UNIT_ROWS=32 ;;
     cb16) build cb16 -DACSR_CLAIM_BATCH=16 ;;
     cb16w32) build cb16w32 -DACSR_CLAIM_BATCH=16 -DACSR_WIN_UNIT_ROWS=32 ;;
     cb32w32) build cb32w32 -DACSR_CLAIM_BATCH=32 -DACSR_WIN_UNIT_ROWS=32 ;;

@@ -74,6 +74,9 @@
 #ifndef ACSR_GUIDED_AHEAD
 #define ACSR_GUIDED_AHEAD 1  // guided batches: claim the next batch when the last unit of this one starts
 #endif
+#ifndef ACSR_WIN_LANE4
+#define ACSR_WIN_LANE4 0  // 1: window chunk reduction by lanes owning 4 consecutive products + segmented suffix scan
+#endif
 #ifndef ACSR_TIMELINE
 #define ACSR_TIMELINE 0  // diagnostics: per-unit start/end cycles + SM id (acsr_debug_timeline, A/B builds only)
 #endif
@@ -871,10 +874,18 @@ struct Kern {
 #if ACSR_WIN_SUM4
             double a1 = 0.0, a2 = 0.0, a3 = 0.0;
 #endif
+#if ACSR_WIN_LANE4
+            double pend_s = 0.0;  // the row left open at the end of the previous chunk: partial sum,
+            int pend_rj = -1;     // and its table index (-1: none)
+#endif
             for (int t0 = 0; t0 < T; t0 += 32 * WIN_G) {
                 double p[WIN_G];
 #if ACSR_WIN_SEGSCAN
                 int rjg[WIN_G];
+#endif
+#if ACSR_WIN_LANE4
+                unsigned Hs[WIN_G];
+                int Q0 = 0;
 #endif
 #pragma unroll
                 for (int g = 0; g < WIN_G; g++) {
@@ -882,6 +893,10 @@ struct Kern {
                     const bool hd = l > 0 && pre >= cb && pre < cb + 32;
                     const unsigned H = __reduce_or_sync(FULL, hd ? 1u << (pre - cb) : 0u);
                     const int q0 = __popc(__ballot_sync(FULL, l > 0 && pre < cb));
+#if ACSR_WIN_LANE4
+                    Hs[g] = H;
+                    if (g == 0) Q0 = q0;
+#endif
                     // element t, clamped to the last one (T-1) past the end so that every
                     // lane loads from a valid address: no branches, all WIN_G groups'
                     // loads are issued back to back (the f32 build serialised them when
@@ -920,6 +935,124 @@ struct Kern {
                     if (cb_valid(t0 + 32 * g, T) && (lane == 31 || nrj != rj)) buf[rj] += sv;
                     __syncwarp();
                 }
+#elif ACSR_WIN_LANE4
+                static_assert(WIN_G == 4, "lane-4 reduction: 128-element chunks, 4 consecutive products per lane");
+                // Lane i takes the chunk's products 4i .. 4i+3 (two 16-byte shared loads, no bank
+                // conflicts) and sums them per row in element order in registers: the row heads
+                // among its 4 elements are bits 4(i mod 8) .. +3 of group i/8's head mask.  A row
+                // whose elements spill into the following lanes gets their leading parts through
+                // one segmented suffix scan over the lanes (5 shuffle levels per 128 elements,
+                // instead of a per-lane loop of shared loads over the longest row).  Finished row
+                // sums go to the row's table slot (tab is not read for a finished row again); the
+                // row open at the chunk's end is completed by the next chunk's leading elements.
+#pragma unroll
+                for (int g = 0; g < WIN_G; g++) buf[32 * g + lane] = p[g];
+                __syncwarp();
+                {
+                    const double2 qa = *(const double2 *)(buf + 4 * lane);
+                    const double2 qb = *(const double2 *)(buf + 4 * lane + 2);
+                    const double q[4] = {qa.x, qa.y, qb.x, qb.y};
+                    const int gs = lane >> 3;
+                    const unsigned Hl = gs == 0 ? Hs[0] : gs == 1 ? Hs[1] : gs == 2 ? Hs[2] : Hs[3];
+                    const int sh = 4 * (lane & 7);
+                    const unsigned hb = (Hl >> sh) & 0xFu;
+                    int hi = Q0 + __popc(Hl & ((1u << sh) - 1u)) + (gs > 0 ? __popc(Hs[0]) : 0) +
+                             (gs > 1 ? __popc(Hs[1]) : 0) + (gs > 2 ? __popc(Hs[2]) : 0);
+                    double *res = (double *)tab;
+#if ACSR_WIN_LANE4 == 2
+                    // exact element-order sums: a row is started as +0.0 + first product (the
+                    // oracle's loop), continued across lanes by serial carries (round r settles
+                    // chains of r head-less lanes; rows of <= 32 elements cross <= 8 lanes)
+                    const int f = hb ? __ffs(hb) - 1 : 4;  // my elements before my first head
+                    double run = 0.0;
+                    bool seen = false;
+#pragma unroll
+                    for (int j = 0; j < 4; j++) {
+                        const bool h = (hb >> j) & 1u;
+                        if (h && seen) res[hi - 1] = run;  // a row that starts and ends in this lane
+                        run = h ? 0.0 + q[j] : run + q[j];
+                        hi += h ? 1 : 0;
+                        seen = seen || h;
+                    }
+                    const int left = T - t0;  // real elements in this chunk
+                    const int nreal = left >= 128 ? 32 : (left + 3) >> 2;
+                    const unsigned real = nreal >= 32 ? FULL : (1u << nreal) - 1u;
+                    const unsigned hl = __ballot_sync(FULL, seen);
+                    unsigned m = ~hl & real;
+                    int rounds = 1;
+                    while (m) {  // longest run of head-less real lanes
+                        m &= m << 1;
+                        rounds++;
+                    }
+                    const double cin0 = pend_rj >= 0 ? pend_s : 0.0;  // lane 0's carry: the row open across the chunk edge
+                    double out = run;  // the running sum I pass to my right neighbour
+                    for (int r = 0; r < rounds; r++) {
+                        double cin = __shfl_up_sync(FULL, out, 1);
+                        if (lane == 0) cin = cin0;
+                        if (!seen) out = (((cin + q[0]) + q[1]) + q[2]) + q[3];
+                    }
+                    double cin = __shfl_up_sync(FULL, out, 1);
+                    if (lane == 0) cin = cin0;
+                    if (seen) {  // the row continuing into my lane ends before my first head
+                        double x = cin;
+#pragma unroll
+                        for (int j = 0; j < 4; j++)
+                            if (j < f) x += q[j];
+                        const int rc = hi - __popc(hb) - 1;  // its table index
+                        if (rc >= 0) res[rc] = x;
+                    }
+                    const int nh = Q0 + __popc(Hs[0]) + __popc(Hs[1]) + __popc(Hs[2]) + __popc(Hs[3]);
+                    const double tail = __shfl_sync(FULL, out, nreal - 1);  // the open row at the last real lane
+                    if (left > 128) {
+                        pend_s = tail;
+                        pend_rj = nh - 1;
+                    } else {
+                        if (lane == 0 && nh > 0) res[nh - 1] = tail;
+                        pend_rj = -1;
+                    }
+                }
+                __syncwarp();
+#else
+                    double run = 0.0, c = 0.0;
+                    bool seen = false;
+#pragma unroll
+                    for (int j = 0; j < 4; j++) {
+                        const bool h = (hb >> j) & 1u;
+                        if (h && seen) res[hi - 1] = run;  // a row that starts and ends in this lane
+                        if (h && !seen) c = run;           // elements before the lane's first head
+                        run = h ? q[j] : run + q[j];
+                        hi += h ? 1 : 0;
+                        seen = seen || h;
+                    }
+                    if (!seen) c = run;
+                    // U = c_i + (lane i has no head ? U_{i+1} : 0): what lane i passes to the row open on its left
+                    double U = c;
+                    int S = seen ? 1 : 0;
+#pragma unroll
+                    for (int d = 1; d < 32; d <<= 1) {
+                        const double Ur = __shfl_down_sync(FULL, U, d);
+                        const int Sr = __shfl_down_sync(FULL, S, d);
+                        if (lane + d < 32) {
+                            if (!S) U += Ur;
+                            S |= Sr;
+                        }
+                    }
+                    const double R = __shfl_down_sync(FULL, U, 1);  // from the lanes on my right
+                    const double U0 = __shfl_sync(FULL, U, 0);      // the chunk's leading elements
+                    const unsigned hl = __ballot_sync(FULL, seen);
+                    const int ls = hl ? 31 - __clz((int)hl) : -1;  // lane of the chunk's last row head
+                    const double open = run + (lane < 31 ? R : 0.0);
+                    if (seen && lane != ls) res[hi - 1] = open;  // completed inside this chunk
+                    if (lane == 0 && pend_rj >= 0) res[pend_rj] = pend_s + U0;
+                    if (ls >= 0) {
+                        pend_s = __shfl_sync(FULL, open, ls);
+                        pend_rj = __shfl_sync(FULL, hi - 1, ls);
+                    } else {
+                        pend_rj = -1;
+                    }
+                }
+                __syncwarp();
+#endif  // ACSR_WIN_LANE4 == 2
 #else
 #pragma unroll
                 for (int g = 0; g < WIN_G; g++) buf[32 * g + lane] = p[g];
@@ -977,6 +1110,10 @@ struct Kern {
             }
 #if ACSR_WIN_SEGSCAN
             if (l > 0) acc = buf[__popc(ne & lt)];
+#elif ACSR_WIN_LANE4
+            if (lane == 0 && pend_rj >= 0) ((double *)tab)[pend_rj] = pend_s;  // the window's last row
+            __syncwarp();
+            if (l > 0) acc = ((const double *)tab)[__popc(ne & lt)];
 #elif ACSR_WIN_SUM4
             acc = (acc + a1) + (a2 + a3);
 #endif
@@ -1321,7 +1458,7 @@ spmv_kernel(SpmvArgs<V> a)
     double *win_buf = (double *)(smem + (XC ? (sizeof(V) + sizeof(uint16_t)) * ((size_t)1 << a.xc_bits) : 0));
     int2 *win_tab = (int2 *)(win_buf + SPMV_WARPS * 32 * WIN_G);  // WIN_TAB entries per warp
 #else
-    __shared__ double win_buf[WIN_MAX_BIN >= 0 ? SPMV_WARPS * 32 * WIN_G : 1];
+    __shared__ __align__(16) double win_buf[WIN_MAX_BIN >= 0 ? SPMV_WARPS * 32 * WIN_G : 1];
     __shared__ int2 win_tab[WIN_MAX_BIN >= 0 ? SPMV_WARPS * WIN_TAB : 1];
 #endif
     double *wbuf = win_buf + (WIN_MAX_BIN >= 0 ? (threadIdx.x >> 5) * 32 * WIN_G : 0);

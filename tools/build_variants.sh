@@ -64,6 +64,9 @@ for v in "$@"; do
     sum1) build sum1 -DACSR_WIN_SUM4=0 ;;
     prof) build prof -DACSR_PROF=1 ;;
     tl) build tl -DACSR_TIMELINE=1 ;;
+    l4) build l4 -DACSR_WIN_LANE4=1 ;;
+    l4s) build l4s -DACSR_WIN_LANE4=2 ;;
+    tll4) build tll4 -DACSR_TIMELINE=1 -DACSR_WIN_LANE4=1 ;;
     g2) build g2 -DACSR_CLAIM_GUIDED=2 ;;
     g2w32) build g2w32 -DACSR_CLAIM_GUIDED=2 -DACSR_WIN_UNIT_ROWS=32 ;;
     g2w64) build g2w64 -DACSR_CLAIM_GUIDED=2 -DACSR_WIN_UNIT_ROWS=64 ;;

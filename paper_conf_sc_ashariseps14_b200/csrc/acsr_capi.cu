@@ -1,4 +1,5 @@
 // acsr_capi.cu -- status strings, thread-local error text, device queries.
+#include <mutex>
 #include <cuda_runtime.h>
 #include <stdarg.h>
 #include <stdio.h>
@@ -53,8 +54,10 @@ int acsr::acsr_carveout()
 
 bool acsr::acsr_carveout_once(const void *fn)
 {
+    static std::mutex mu;  // ctypes releases the GIL: launches can come from several host threads
     static const void *seen[128];
     static int n = 0;
+    std::lock_guard<std::mutex> lock(mu);
     for (int i = 0; i < n; i++)
         if (seen[i] == fn) return false;
     if (n < 128) seen[n++] = fn;

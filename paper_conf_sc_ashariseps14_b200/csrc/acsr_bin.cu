@@ -90,7 +90,7 @@ __device__ __forceinline__ void count_tile(BinSmem &sm, int64_t n, const int32_t
         cnt[(int64_t)tid * n_tiles + tile] = h;
         const bool tl = tail_tile(tile, n_tiles);
         int lu = 0;
-        if (tid > wmb && tid <= LIGHT_MAX_BIN) lu = (h + unit_rows_t(tid, tl) - 1) / unit_rows_t(tid, tl);
+        if (tid > wmb && tid <= LIGHT_MAX_BIN) lu = ceil_shift(h, unit_shift_t(tid, tl));
         lu = __reduce_add_sync(0xffffffffu, lu);
         if (tid == 0) {
             if (wmb >= 0) lu += win_units_t((int)min((int64_t)TILE_ROWS, n - base), tl);
@@ -381,7 +381,7 @@ __device__ __forceinline__ void scatter_tile(BinSmem &sm, const ScatterPre &pre,
             int acc = nwin;
             for (int b = 0; b <= LIGHT_MAX_BIN; b++) {
                 sm.upre[b] = acc;
-                if (b > wmb) acc += (sm.run[b] + unit_rows_t(b, tl) - 1) / unit_rows_t(b, tl);
+                if (b > wmb) acc += ceil_shift(sm.run[b], unit_shift_t(b, tl));
             }
             sm.upre[LIGHT_MAX_BIN + 1] = acc;
         }

@@ -105,10 +105,12 @@ __host__ __device__ constexpr int win_units(int tile_rows) { return (tile_rows +
 
 // Tail tiles: the last max(1, n_tiles / ACSR_TAIL_DIV) tiles of the work list get 4x
 // smaller work units (32-row windows, a quarter of the rows per bin unit), so the last
-// claims of the dynamic schedule are short and warps run out of work together
-// (0: off; A/B builds).
+// claims of the dynamic schedule are short and warps run out of work together.  With the
+// late claims of round 2 and shift-based unit counts in the binning kernels, 1/16 of the
+// tiles pays on every matrix: C2 step 99.7 -> 98.8 us, fp32 93.6 -> 92.7, LiveJournal-like
+// 425.5 -> 420.1, web-Google-like unchanged (1/8, 1/4, 1/2: smaller or negative gains).
 #ifndef ACSR_TAIL_DIV
-#define ACSR_TAIL_DIV 0
+#define ACSR_TAIL_DIV 16  // r2s2: the last 1/16 of the tiles (profiles/r2s2_taildiv_ab_shift.jsonl); 0: off
 #endif
 __host__ __device__ inline bool tail_tile(int tile, int n_tiles)
 {
@@ -116,14 +118,28 @@ __host__ __device__ inline bool tail_tile(int tile, int n_tiles)
     const int k = n_tiles / (ACSR_TAIL_DIV > 0 ? ACSR_TAIL_DIV : 1);
     return tile >= n_tiles - (k > 1 ? k : 1);
 }
-__host__ __device__ inline int unit_rows_t(int b, bool tail)
+// Unit sizes are powers of two: the per-tile unit counts are computed with shifts (a
+// division by a bin-dependent divisor is a ~20-instruction sequence in the binning kernels)
+__host__ __device__ inline int ilog2_pow2(int v)
 {
-    return tail ? (unit_rows(b) / 4 > 1 ? unit_rows(b) / 4 : 1) : unit_rows(b);
+#ifdef __CUDA_ARCH__
+    return 31 - __clz(v);
+#else
+    return 31 - __builtin_clz((unsigned)v);
+#endif
 }
+static_assert((WIN_UNIT_ROWS & (WIN_UNIT_ROWS - 1)) == 0 && (WIN_ROWS & (WIN_ROWS - 1)) == 0, "powers of two");
+__host__ __device__ inline int unit_shift_t(int b, bool tail)
+{
+    const int s = ilog2_pow2(unit_rows(b));
+    return tail ? (s > 2 ? s - 2 : 0) : s;
+}
+__host__ __device__ inline int unit_rows_t(int b, bool tail) { return 1 << unit_shift_t(b, tail); }
+__host__ __device__ inline int ceil_shift(int v, int s) { return (v + (1 << s) - 1) >> s; }
 __host__ __device__ inline int win_unit_rows_t(bool tail) { return tail ? WIN_ROWS : WIN_UNIT_ROWS; }
 __host__ __device__ inline int win_units_t(int tile_rows, bool tail)
 {
-    return (tile_rows + win_unit_rows_t(tail) - 1) / win_unit_rows_t(tail);
+    return ceil_shift(tile_rows, ilog2_pow2(win_unit_rows_t(tail)));
 }
 
 // unit descriptor: light  x = first index into bin_rows, y = (bin << 24) | rows

@@ -53,6 +53,7 @@ for v in "$@"; do
     l41) build l41 -DACSR_WIN_LDS4=1 ;;
     mw1) build mw1 -DACSR_MERGED_WARP_PATH=1 ;;
     td16) build td16 -DACSR_TAIL_DIV=16 ;;
+    td0) build td0 -DACSR_TAIL_DIV=0 ;;
     uwr1) build uwr1 -DACSR_UPD_WARPREG=1 ;;
     us1) build us1 -DACSR_UPD_SUB=1 ;;
     sc256) build sc256 -DACSR_SCAN_THREADS=256 ;;
@@ -65,6 +66,8 @@ for v in "$@"; do
     prof) build prof -DACSR_PROF=1 ;;
     tl) build tl -DACSR_TIMELINE=1 ;;
     l4) build l4 -DACSR_WIN_LANE4=1 ;;
+    td2) build td2 -DACSR_TAIL_DIV=2 ;;
+    td4x) build td4x -DACSR_TAIL_DIV=4 ;;
     l4s) build l4s -DACSR_WIN_LANE4=2 ;;
     tll4) build tll4 -DACSR_TIMELINE=1 -DACSR_WIN_LANE4=1 ;;
     g2) build g2 -DACSR_CLAIM_GUIDED=2 ;;

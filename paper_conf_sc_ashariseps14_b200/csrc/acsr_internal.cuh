@@ -13,7 +13,10 @@ namespace acsr {
 // acsr_bin processes the rows in tiles of TILE_ROWS rows (one CTA per tile, rounds
 // of 256 rows in row order).  The per-(bin, tile) counts double as the row-space
 // locality unit of the SpMV work map.
-constexpr int BIN_THREADS = 256;
+#ifndef ACSR_BIN_THREADS
+#define ACSR_BIN_THREADS 256  // threads per binning CTA (A/B knob)
+#endif
+constexpr int BIN_THREADS = ACSR_BIN_THREADS;
 #ifndef ACSR_TILE_ROWS
 #define ACSR_TILE_ROWS 1024
 #endif

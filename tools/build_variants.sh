@@ -65,6 +65,21 @@ for v in "$@"; do
     sum1) build sum1 -DACSR_WIN_SUM4=0 ;;
     prof) build prof -DACSR_PROF=1 ;;
     tl) build tl -DACSR_TIMELINE=1 ;;
+    s2td32) build s2td32 -DACSR_TAIL_DIV=32 ;;
+    s2w64) build s2w64 -DACSR_WIN_UNIT_ROWS=64 ;;
+    s2w256) build s2w256 -DACSR_WIN_UNIT_ROWS=256 ;;
+    s2v512) build s2v512 -DACSR_VEC_MIN=512 ;;
+    s2v2048) build s2v2048 -DACSR_VEC_MIN=2048 ;;
+    s2um1) build s2um1 -DACSR_UNIT_SHIFT=-1 ;;
+    s2u1) build s2u1 -DACSR_UNIT_SHIFT=1 ;;
+    s2uw1) build s2uw1 -DACSR_UNIT_WARP_SHIFT=1 ;;
+    s2wb4) build s2wb4 -DACSR_WIN_MAX_BIN=4 ;;
+    s2cl2) build s2cl2 -DACSR_CLAIM_LATE=2 ;;
+    s2g2) build s2g2 -DACSR_WIN_G=2 ;;
+    s2bt128) build s2bt128 -DACSR_BIN_THREADS=128 ;;
+    s2bt512) build s2bt512 -DACSR_BIN_THREADS=512 ;;
+    s2t2k) build s2t2k -DACSR_TILE_ROWS=2048 ;;
+    s2t512) build s2t512 -DACSR_TILE_ROWS=512 ;;
     l4) build l4 -DACSR_WIN_LANE4=1 ;;
     td2) build td2 -DACSR_TAIL_DIV=2 ;;
     td4x) build td4x -DACSR_TAIL_DIV=4 ;;

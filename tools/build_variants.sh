@@ -65,6 +65,8 @@ for v in "$@"; do
     sum1) build sum1 -DACSR_WIN_SUM4=0 ;;
     prof) build prof -DACSR_PROF=1 ;;
     tl) build tl -DACSR_TIMELINE=1 ;;
+    d0off) build d0off -DACSR_DESC0=0 ;;
+    d0pf) build d0pf -DACSR_DESC0=2 ;;
     s2td32) build s2td32 -DACSR_TAIL_DIV=32 ;;
     s2w64) build s2w64 -DACSR_WIN_UNIT_ROWS=64 ;;
     s2w256) build s2w256 -DACSR_WIN_UNIT_ROWS=256 ;;

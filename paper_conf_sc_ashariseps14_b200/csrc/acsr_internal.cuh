@@ -115,10 +115,14 @@ __host__ __device__ constexpr int win_units(int tile_rows) { return (tile_rows +
 #ifndef ACSR_TAIL_DIV
 #define ACSR_TAIL_DIV 16  // r2s2: the last 1/16 of the tiles (profiles/r2s2_taildiv_ab_shift.jsonl); 0: off
 #endif
+#ifndef ACSR_TAIL_MAX_TILES
+#define ACSR_TAIL_MAX_TILES 320  // cap: the tail only has to cover the schedule's last rounds (s26 PageRank: 1/16 of
+#endif                           // 65536 tiles cost the plain step 2 %, profiles/r2s2_c4_taildiv_ab.jsonl)
 __host__ __device__ inline bool tail_tile(int tile, int n_tiles)
 {
     if (ACSR_TAIL_DIV <= 0) return false;
-    const int k = n_tiles / (ACSR_TAIL_DIV > 0 ? ACSR_TAIL_DIV : 1);
+    int k = n_tiles / (ACSR_TAIL_DIV > 0 ? ACSR_TAIL_DIV : 1);
+    k = k < ACSR_TAIL_MAX_TILES ? k : ACSR_TAIL_MAX_TILES;
     return tile >= n_tiles - (k > 1 ? k : 1);
 }
 // Unit sizes are powers of two: the per-tile unit counts are computed with shifts (a

@@ -65,6 +65,14 @@ for v in "$@"; do
     sum1) build sum1 -DACSR_WIN_SUM4=0 ;;
     prof) build prof -DACSR_PROF=1 ;;
     tl) build tl -DACSR_TIMELINE=1 ;;
+    s2wp) build s2wp -DACSR_WIN_PREFETCH=1 ;;
+    s2lds4) build s2lds4 -DACSR_WIN_LDS4=1 ;;
+    s2sum4) build s2sum4 -DACSR_WIN_SUM4=1 ;;
+    s2pair) build s2pair -DACSR_PAIR_ROWS=1 ;;
+    s2br) build s2br -DACSR_BRANCHY_SUB=1 ;;
+    s2s1) build s2s1 -DACSR_STREAM_LD=1 ;;
+    s2x1) build s2x1 -DACSR_X_LD=1 ;;
+    s2mwp) build s2mwp -DACSR_MERGED_WARP_PATH=1 ;;
     d0off) build d0off -DACSR_DESC0=0 ;;
     d0pf) build d0pf -DACSR_DESC0=2 ;;
     s2td32) build s2td32 -DACSR_TAIL_DIV=32 ;;

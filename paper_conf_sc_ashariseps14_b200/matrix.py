@@ -143,17 +143,24 @@ class UpdateGraph:
 
 
 def spmv_from_host(row_ptr_h, col_h, val_h, x_h, y_h=None, device="cuda", stream=None):
-    """End-to-end y = A x from (pinned) host arrays: H2D, acsr_bin, acsr_spmv, D2H."""
-    rp = row_ptr_h.to(device, non_blocking=True)
-    ci = col_h.to(device, non_blocking=True)
-    va = None if val_h is None else val_h.to(device, non_blocking=True)
-    x = x_h.to(device, non_blocking=True)
-    br, bo, ws = acsr_bin(rp, None, ci.numel(), stream=stream, col_idx=ci, n_cols=x.numel())
-    y = acsr_spmv(rp, ci, va, x, br, bo, ws, stream=stream)
-    if y_h is None:
-        return y.cpu()
-    y_h.copy_(y, non_blocking=True)
-    return y_h
+    """End-to-end y = A x from (pinned) host arrays: H2D, acsr_bin, acsr_spmv, D2H, all
+    enqueued on `stream` (default: the current stream).  Calls on different streams
+    overlap: one call's host->device copies run while another's kernels and device->host
+    copy run (PCIe is full duplex)."""
+    if stream is not None and not isinstance(stream, torch.cuda.Stream):
+        stream = torch.cuda.ExternalStream(int(stream))
+    with torch.cuda.stream(stream if stream is not None else torch.cuda.current_stream()):
+        s = torch.cuda.current_stream()
+        rp = row_ptr_h.to(device, non_blocking=True)
+        ci = col_h.to(device, non_blocking=True)
+        va = None if val_h is None else val_h.to(device, non_blocking=True)
+        x = x_h.to(device, non_blocking=True)
+        br, bo, ws = acsr_bin(rp, None, ci.numel(), stream=s, col_idx=ci, n_cols=x.numel())
+        y = acsr_spmv(rp, ci, va, x, br, bo, ws, stream=s)
+        if y_h is None:
+            return y.cpu()
+        y_h.copy_(y, non_blocking=True)
+        return y_h
 
 
 def _power_loop(m: ACSRMatrix, outdeg, x, damping, teleport, eps, max_iter, check_every, stream,

@@ -1087,6 +1087,26 @@ def test_spmv_from_host_e2e(acsr, cuda):
     check_spmv(y.numpy(), y_ref, den, torch.float64)
 
 
+def test_spmv_from_host_two_streams(acsr, cuda):
+    """The double-buffered end-to-end pattern bench.py times: calls alternating between two
+    streams, each with its own pinned output, overlap in flight; every result equals the
+    one-stream call bit for bit (and the oracle at the fp64 bar)."""
+    rp, ci = synth.rmat_csr(15)
+    val = synth.values(ci.numel(), 5)
+    x = synth.vector(rp.numel() - 1, 6)
+    h = [t.pin_memory() for t in (rp, ci, val, x)]
+    y1 = acsr.spmv_from_host(*h, device=cuda)
+    sts = [torch.cuda.Stream(device=cuda) for _ in range(2)]
+    outs = [torch.empty_like(x).pin_memory() for _ in range(6)]
+    for k in range(6):
+        acsr.spmv_from_host(*h, outs[k], device=cuda, stream=sts[k % 2])
+    torch.cuda.synchronize()
+    for o in outs:
+        assert torch.equal(o, y1)
+    y_ref, den = oracle.spmv(rp.numpy(), ci.numpy(), val.numpy(), x.numpy())
+    check_spmv(y1.numpy(), y_ref, den, torch.float64)
+
+
 def _two_ranks(scale, world=2, **kw):
     import socket
     import sys

@@ -471,10 +471,39 @@ def run_acsr(args, dev, rank, world):
     r1.record(stream)
     torch.cuda.synchronize()
     t_res = r0.elapsed_time(r1) / ke
+    # the same steps alternating between two streams, each with its own x / y / plan
+    # buffers (a plan workspace must not be shared by concurrent calls): x in of step k+1
+    # overlaps step k's kernels and y out
+    rbuf = [(torch.empty_like(x), torch.empty_like(y), torch.empty_like(br), torch.empty_like(bo),
+             torch.empty_like(ws), torch.empty(n, dtype=dtype).pin_memory()) for _ in range(2)]
+
+    def res_step(k):
+        xd, yd, brk, bok, wsk, yhk = rbuf[k % 2]
+        with torch.cuda.stream(sts[k % 2]):
+            s_ = sts[k % 2]
+            xd.copy_(x_h, non_blocking=True)
+            acsr.acsr_bin(rp, None, nnz, brk, bok, wsk, col_idx=ci, n_cols=x.numel(), stream=s_)
+            acsr.acsr_spmv(rp, ci, val, xd, brk, bok, wsk, None, yd, stream=s_)
+            yhk.copy_(yd, non_blocking=True)
+
+    for k in range(2):
+        res_step(k)
+    torch.cuda.synchronize()
+    r2, r3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    r2.record(stream)
+    for st in sts:
+        st.wait_event(r2)
+    for k in range(ke):
+        res_step(k)
+    for st in sts:
+        stream.wait_stream(st)
+    r3.record(stream)
+    torch.cuda.synchronize()
+    t_res2 = r2.elapsed_time(r3) / ke
     if world > 1:
-        te = torch.tensor([t_res], dtype=torch.float64, device=dev)
+        te = torch.tensor([t_res, t_res2], dtype=torch.float64, device=dev)
         torch.distributed.all_reduce(te, op=torch.distributed.ReduceOp.MAX)
-        t_res = float(te.item())
+        t_res, t_res2 = float(te[0].item()), float(te[1].item())
     h2d = sum(t.numel() * t.element_size() for t in (rp_h, ci_h, val_h, x_h))
     d2h = y_h.numel() * y_h.element_size()
     ctx = cusparse_context(rp, ci, val, x, n)
@@ -553,10 +582,12 @@ def run_acsr(args, dev, rank, world):
                         "x in / y out per step",
                 "sequential": {"value": round(2.0 * units / (t_e2e_seq * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
                                "ms_per_step": round(t_e2e_seq, 4)},
-                "resident_matrix": {"value": round(2.0 * units / (t_res * 1e-3) / 1e9, 3),
-                                    "unit": "GFLOP/s", "ms_per_step": round(t_res, 4),
+                "resident_matrix": {"value": round(2.0 * units / (t_res2 * 1e-3) / 1e9, 3),
+                                    "unit": "GFLOP/s", "ms_per_step": round(t_res2, 4),
                                     "h2d_bytes_per_step": int(x_h.numel() * x_h.element_size()) * world,
-                                    "d2h_bytes_per_step": int(d2h) * world}},
+                                    "d2h_bytes_per_step": int(d2h) * world,
+                                    "note": "two streams, own x / y / plan per stream; one stream: sequential_ms",
+                                    "sequential_ms": round(t_res, 4)}},
         "gpu_launches": 4 * K * world,  # per step and rank: bin_count, bin_scan, bin_scatter, spmv_kernel
         "clocks": clk.summary(),
     }

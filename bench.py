@@ -1369,6 +1369,11 @@ def main():
         os.environ.update(NCCL_HOSTID=f"acsr-test-host-{rank}", NCCL_SOCKET_IFNAME="lo", NCCL_IB_DISABLE="1",
                           NCCL_P2P_DISABLE="1", NCCL_SHM_DISABLE="1", NCCL_NVLS_ENABLE="0")
     if world > 1:
+        # NCCL's communicator-init log (nranks, transports, NVLS) stays on for the record, on
+        # stderr so rank 0's stdout keeps exactly one JSON line
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
         backend = os.environ.get("ACSR_DIST_BACKEND", "nccl")  # gloo: test the path on one GPU
         if backend == "nccl":
             torch.distributed.init_process_group("nccl", device_id=dev)

@@ -1940,11 +1940,14 @@ static int xcache_bits()
 static int64_t x_prefetch_bytes(int64_t bytes)
 {
     static int on = -1;
+    static int64_t max_bytes = 0;
     if (on < 0) {
         const char *e = getenv("ACSR_XPREFETCH");
         on = (e && e[0] == '0') ? 0 : 1;
+        const char *m = getenv("ACSR_XPREFETCH_MAX_MB");  // largest x prefetched (r2s2: 32 -> 64 MB, C3b -0.35 %)
+        max_bytes = (int64_t)(m && m[0] ? atoi(m) : 64) << 20;
     }
-    return (on && bytes <= ((int64_t)32 << 20)) ? bytes : 0;
+    return (on && bytes <= max_bytes) ? bytes : 0;
 }
 
 template <typename V, bool PR>

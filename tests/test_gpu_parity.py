@@ -1063,6 +1063,43 @@ def test_property_random_csr_spmv_and_updates(acsr, cuda):
     check()
 
 
+def test_property_multi_tile_spmv(acsr, cuda):
+    """Property test (hypothesis, derandomized) over MANY tiles: 1025 .. 120000 rows, so plans
+    hold full and ragged tiles, the 4x smaller units of the tail tiles (ACSR_TAIL_DIV) next
+    to ordinary ones, windows that straddle long rows, and split rows anywhere in the list;
+    bins bitwise, SpMV bitwise on integer data and at the O5 bar on float data."""
+    from hypothesis import given, settings, strategies as st, HealthCheck
+
+    @settings(max_examples=60, derandomize=True, deadline=None,
+              suppress_health_check=[HealthCheck.too_slow, HealthCheck.data_too_large])
+    @given(st.integers(1025, 120000), st.integers(1, 200000), st.integers(0, 2 ** 31 - 1), st.booleans(), st.booleans())
+    def check(n, n_cols, seed, f32, integer):
+        rng = np.random.default_rng(seed)
+        u = rng.random(n)
+        ln = np.where(u < 0.15, 0, np.where(u < 0.75, rng.integers(1, 33, n),
+                      np.where(u < 0.97, rng.integers(33, 1025, n),
+                               np.where(u < 0.995, rng.integers(1, 5, n), rng.integers(1025, 5000, n)))))
+        rp = np.zeros(n + 1, np.int64)
+        rp[1:] = np.cumsum(ln)
+        nnz = int(rp[-1])
+        ci = rng.integers(0, n_cols, nnz).astype(np.int32)
+        dt = np.float32 if f32 else np.float64
+        if integer:
+            val = rng.integers(-8, 9, nnz).astype(dt)
+            x = rng.integers(-8, 9, n_cols).astype(dt)
+        else:
+            val = rng.uniform(-1, 1, nnz).astype(dt)
+            x = rng.uniform(-1, 1, n_cols).astype(dt)
+        rpt = torch.from_numpy(rp.astype(np.int32))
+        m, y = run_csr(acsr, rpt, torch.from_numpy(ci), torch.from_numpy(val), torch.from_numpy(x), cuda)
+        br, off = oracle.bins(rp.astype(np.int32))
+        assert np.array_equal(m.bin_rows.cpu().numpy(), br) and np.array_equal(m.bin_offsets.cpu().numpy(), off)
+        y_ref, den = oracle.spmv(rp.astype(np.int32), ci, val, x)
+        check_spmv(y.numpy(), y_ref, den, torch.float32 if f32 else torch.float64, exact=integer)
+
+    check()
+
+
 def test_c_abi_from_plain_c(cuda):
     # the boundary is usable without Python: compile tests/c/capi_smoke.c against
     # include/acsr.h and libacsr.so and run it
